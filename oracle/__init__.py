@@ -1,0 +1,74 @@
+"""ORACLE: plain CPU implementations of what the HiRace hot path must compute.
+
+TEST INFRASTRUCTURE ONLY.  Only `tests/`, `__graft_entry__.smoke()` and `bench.py`
+(`cpu_baseline` leg and `--impl reference`) may import, call, link or execute anything under
+`oracle/`.  The product package (`paper_conf_sc_jacobsonbg24_b200/`) never imports it and the
+two share no code.
+
+  oracle_d.c  Oracle-D: the race definition, sort + per-level scan, C.
+  brute.py    literal O(n^2) pairwise enumeration of C1, for tiny traces.
+
+Pins (tests/test_oracle_pins.py): brute force on random tiny traces, the paper's listings
+(closed forms, tests/golden/), configs 1/2/4 closed forms, read-only invariants.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "oracle_d.c")
+_SO = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+WARP, BLOCK, GRID = 1, 2, 3
+CLASS_NAMES = {1: "WARP", 2: "BLOCK", 3: "GRID"}
+
+
+def build(force: bool = False) -> str:
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", _SRC, "-o", _SO])
+    return _SO
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        build()
+        lib = ctypes.CDLL(_SO)
+        lib.oracle_races.restype = ctypes.c_int64
+        lib.oracle_races.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                                     ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64]
+        _lib = lib
+    return _lib
+
+
+def races(events: np.ndarray, block_threads: int, warp_size: int):
+    """Oracle-D.  Returns (keys u64[], cls u8[], gstar u8[]) sorted by key."""
+    lib = _load()
+    ev = np.ascontiguousarray(events)
+    n = int(ev.shape[0])
+    cap = max(1024, n)
+    while True:
+        keys = np.empty(cap, np.uint64)
+        cls = np.empty(cap, np.uint8)
+        gs = np.empty(cap, np.uint8)
+        r = lib.oracle_races(ev.ctypes.data if n else None, n, block_threads, warp_size,
+                             keys.ctypes.data, cls.ctypes.data, gs.ctypes.data, cap)
+        if r < 0:
+            raise RuntimeError(f"oracle_races failed ({r})")
+        if r <= cap:
+            return keys[:r], cls[:r], gs[:r]
+        cap = int(r)
+
+
+def races_of(trace):
+    return races(trace.events, trace.block_threads, trace.warp_size)
+
+
+def races_dict(trace) -> dict:
+    k, c, _ = races_of(trace)
+    return {int(a): int(b) for a, b in zip(k, c)}

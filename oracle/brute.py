@@ -1,0 +1,83 @@
+"""Brute-force pairwise race enumeration, literally SURVEY.md §8(c) C1.
+
+TEST INFRASTRUCTURE ONLY (see oracle/__init__.py).  O(n^2) over word-level accesses, for tiny
+traces.  Independent of oracle_d.c (different algorithm, different language) and of the CUDA
+path.
+"""
+from __future__ import annotations
+
+R, W, AB, AG = 0, 1, 2, 3
+WARP, BLOCK, GRID = 1, 2, 3
+SHARED = 1 << 63
+
+
+def accesses(events, block_threads, warp_size):
+    """C1.1: word-level accesses (key, tid, kind, g, b, w, block, warp)."""
+    out = []
+    for e in events:
+        addr, tid, meta = int(e["addr"]), int(e["tid"]), int(e["meta"])
+        kind, size = meta & 3, 1 << ((meta >> 2) & 7)
+        w, b, g = (meta >> 5) & 511, (meta >> 14) & 1023, (meta >> 24) & 255
+        block, warp = tid // block_threads, (tid % block_threads) // warp_size
+        word0 = (addr & ~SHARED) >> 2
+        for k in range(1 if size <= 4 else size // 4):
+            word = word0 + k
+            key = (SHARED | (block << 32) | word) if addr & SHARED else word
+            out.append((key, tid, kind, g, b, w, block, warp))
+    return out
+
+
+def concurrent(a, c):
+    """C1.2."""
+    _, t1, _, g1, b1, w1, blk1, wp1 = a
+    _, t2, _, g2, b2, w2, blk2, wp2 = c
+    if t1 == t2 or g1 != g2:
+        return False
+    if blk1 != blk2:
+        return True
+    if b1 != b2:
+        return False
+    return wp1 != wp2 or w1 == w2
+
+
+def conflict(a, c):
+    """C1.3."""
+    k1, k2 = a[2], c[2]
+    if k1 == R and k2 == R:
+        return False
+    if k1 in (AB, AG) and k2 in (AB, AG):
+        if k1 == AG and k2 == AG:
+            return False
+        return a[6] != c[6]
+    return True
+
+
+def level(a, c):
+    if a[6] != c[6]:
+        return GRID
+    if a[7] != c[7]:
+        return BLOCK
+    return WARP
+
+
+def races(events, block_threads, warp_size):
+    """Returns {key: (class, g*)} by literal enumeration of all pairs (C1.4-C1.6)."""
+    acc = accesses(events, block_threads, warp_size)
+    pairs = {}
+    for i in range(len(acc)):
+        for j in range(i + 1, len(acc)):
+            a, c = acc[i], acc[j]
+            if a[0] == c[0] and concurrent(a, c) and conflict(a, c):
+                # racing pair: record (g, b, level); b is shared by intra-block pairs
+                pairs.setdefault(a[0], []).append((a[3], a[4], level(a, c)))
+    out = {}
+    for key, ps in pairs.items():
+        gstar = min(p[0] for p in ps)
+        in_g = [p for p in ps if p[0] == gstar]
+        if any(p[2] == GRID for p in in_g):
+            out[key] = (GRID, gstar)
+            continue
+        bstar = min(p[1] for p in in_g)
+        in_b = [p for p in in_g if p[1] == bstar]
+        out[key] = (BLOCK if any(p[2] == BLOCK for p in in_b) else WARP, gstar)
+    return out

@@ -1,0 +1,285 @@
+/*
+ * ORACLE-D: a plain, slow, single-threaded CPU implementation of the data-race DEFINITION.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py (its
+ * cpu_baseline leg and `--impl reference`) may load or call this file.  It shares no code,
+ * header, table or constant generator with the CUDA path (paper_conf_sc_jacobsonbg24_b200/):
+ * it does NOT run the HiRace state machine; it evaluates the happens-before race definition
+ * directly, so it can judge the state machine.
+ *
+ * What it computes:
+ *   C1.1  events e = (key, tid, kind, g, b, w); block = tid / blockDim,
+ *         warp = (tid mod blockDim) / warpSize                         PAPER.md L164 (T_bwt), L259
+ *         key: global -> word index; shared -> 1<<63 | block<<32 | word (shared memory is per
+ *         block); 8/16-byte accesses cover 2/4 words, sub-word accesses their
+ *         containing word (per-element shadow; reading R8).
+ *   C1.2  Concurrent(e1,e2) <=> tid1 != tid2 and g1 == g2 and
+ *         [block1 != block2 or (b1 == b2 and (warp1 != warp2 or w1 == w2))]
+ *         (barrier semantics PAPER.md L122, L211-213; grid epoch PAPER.md L221, reading R4)
+ *   C1.3  Conflict: R-R never; atomic-atomic only if not both grid-scope and the two threads
+ *         are in different blocks; every other pair (incl. plain read vs atomic) conflicts
+ *         ("at least one of the accesses is a write", L223-229; readings R2, R3)
+ *   C1.4  racing pair = Concurrent and Conflict; level GRID / BLOCK / WARP
+ *   C1.5  a key is flagged iff it has a racing pair
+ *   C1.6  class: g* = smallest g with a racing pair; GRID if a racing pair of g* is GRID-level;
+ *         otherwise b* = smallest b with a racing pair in g*, BLOCK if a racing pair in
+ *         (g*, b*) is BLOCK-level, else WARP                                 (reading R6)
+ *
+ * Algorithm (C2): expand words, qsort by (key, g, block, b, warp, w, tid), then for every
+ * (key, g) test the three levels with per-group kind masks.  A level has a racing pair iff
+ * two DISTINCT groups (blocks / warps of one (block,b) / threads of one (block,b,warp,w))
+ * hold a conflicting pair of kinds: concurrency at each level is exactly "different group
+ * inside the same enclosing epoch" (C1.2), and conflict depends only on the two kinds and
+ * on whether the blocks are equal (C1.3).
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+typedef struct {
+    uint64_t addr;
+    uint32_t tid;
+    uint32_t meta;
+} oracle_event; /* the 16-byte trace record produced by tracegen */
+
+typedef struct {
+    uint64_t key;
+    uint32_t g, block, b, warp, w, tid, kind;
+} access_t;
+
+enum { K_READ = 0, K_WRITE = 1, K_ATOMIC_BLOCK = 2, K_ATOMIC_GRID = 3 };
+enum { CLS_NONE = 0, CLS_WARP = 1, CLS_BLOCK = 2, CLS_GRID = 3 };
+
+static const uint64_t SHARED = 1ull << 63;
+
+static int is_atomic(uint32_t k) { return k == K_ATOMIC_BLOCK || k == K_ATOMIC_GRID; }
+
+/* C1.3 */
+static int conflict(uint32_t k1, uint32_t k2, int same_block)
+{
+    if (k1 == K_READ && k2 == K_READ)
+        return 0;
+    if (is_atomic(k1) && is_atomic(k2)) {
+        if (k1 == K_ATOMIC_GRID && k2 == K_ATOMIC_GRID)
+            return 0;
+        if (same_block)
+            return 0;
+        return 1;
+    }
+    return 1;
+}
+
+/* exists i != j with kind k1 in masks[i], kind k2 in masks[j], conflict(k1,k2) */
+static int distinct_conflict(const uint8_t *masks, size_t n, int same_block)
+{
+    for (uint32_t k1 = 0; k1 < 4; k1++) {
+        for (uint32_t k2 = 0; k2 < 4; k2++) {
+            if (!conflict(k1, k2, same_block))
+                continue;
+            size_t c1 = 0, c2 = 0, f1 = 0, f2 = 0;
+            for (size_t i = 0; i < n; i++) {
+                if ((masks[i] >> k1) & 1) {
+                    if (c1 == 0)
+                        f1 = i;
+                    c1++;
+                }
+                if ((masks[i] >> k2) & 1) {
+                    if (c2 == 0)
+                        f2 = i;
+                    c2++;
+                }
+            }
+            if (c1 >= 1 && c2 >= 1 && !(c1 == 1 && c2 == 1 && f1 == f2))
+                return 1;
+        }
+    }
+    return 0;
+}
+
+static int cmp_access(const void *pa, const void *pb)
+{
+    const access_t *a = (const access_t *)pa, *b = (const access_t *)pb;
+#define CMP(f)                  \
+    if (a->f != b->f)           \
+        return a->f < b->f ? -1 : 1;
+    CMP(key) CMP(g) CMP(block) CMP(b) CMP(warp) CMP(w) CMP(tid)
+#undef CMP
+    return 0;
+}
+
+/* Growable scratch array of group masks. */
+typedef struct {
+    uint8_t *m;
+    size_t n, cap;
+} masks_t;
+
+static int masks_push(masks_t *s, uint8_t v)
+{
+    if (s->n == s->cap) {
+        size_t nc = s->cap ? 2 * s->cap : 64;
+        uint8_t *p = (uint8_t *)realloc(s->m, nc);
+        if (!p)
+            return -1;
+        s->m = p;
+        s->cap = nc;
+    }
+    s->m[s->n++] = v;
+    return 0;
+}
+
+/*
+ * Returns the number of flagged keys (>= 0; only the first `cap` are written, in increasing
+ * key order), or a negative error: -1 bad argument / out of memory, -2 the definition's
+ * C1.6 premise failed (no GRID pair although >= 2 blocks touched the key in g*; cannot happen
+ * by C1.2/C1.3 and is reported so a test can pin it).
+ * out_g receives g* (the grid epoch of the first racing pair).
+ */
+int64_t oracle_races(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
+                     uint64_t *out_key, uint8_t *out_cls, uint8_t *out_g, uint64_t cap)
+{
+    if (block_threads == 0 || warp_size == 0 || (n && !ev))
+        return -1;
+    /* C1.1: expand to word-level accesses */
+    uint64_t nacc = 0;
+    for (uint64_t i = 0; i < n; i++) {
+        uint32_t sz = 1u << ((ev[i].meta >> 2) & 7);
+        nacc += sz <= 4 ? 1 : sz / 4;
+    }
+    access_t *acc = (access_t *)malloc((nacc ? nacc : 1) * sizeof(access_t));
+    if (!acc)
+        return -1;
+    uint64_t j = 0;
+    for (uint64_t i = 0; i < n; i++) {
+        uint32_t meta = ev[i].meta;
+        uint32_t kind = meta & 3, sz = 1u << ((meta >> 2) & 7);
+        uint32_t w = (meta >> 5) & 511, b = (meta >> 14) & 1023, g = (meta >> 24) & 255;
+        uint32_t tid = ev[i].tid;
+        uint32_t block = tid / block_threads;
+        uint32_t warp = (tid % block_threads) / warp_size;
+        int shared = (ev[i].addr & SHARED) != 0;
+        uint64_t word0 = (ev[i].addr & ~SHARED) >> 2;
+        uint32_t nw = sz <= 4 ? 1 : sz / 4;
+        for (uint32_t k = 0; k < nw; k++) {
+            access_t *a = &acc[j++];
+            uint64_t word = word0 + k;
+            a->key = shared ? (SHARED | ((uint64_t)block << 32) | (word & 0xffffffffull)) : word;
+            a->g = g;
+            a->block = block;
+            a->b = b;
+            a->warp = warp;
+            a->w = w;
+            a->tid = tid;
+            a->kind = kind;
+        }
+    }
+    /* C2.2 */
+    qsort(acc, nacc, sizeof(access_t), cmp_access);
+
+    masks_t blocks = {0}, warps = {0}, threads = {0};
+    int64_t nflag = 0;
+    int err = 0;
+    uint64_t i = 0;
+    while (i < nacc && !err) {
+        uint64_t key = acc[i].key, kend = i;
+        while (kend < nacc && acc[kend].key == key)
+            kend++;
+        int cls = CLS_NONE;
+        uint32_t gstar = 0;
+        /* C2.3: each grid epoch of this key, in increasing g */
+        for (uint64_t gs = i; gs < kend && cls == CLS_NONE;) {
+            uint32_t g = acc[gs].g;
+            uint64_t ge = gs;
+            while (ge < kend && acc[ge].g == g)
+                ge++;
+            /* GRID level: groups = blocks */
+            blocks.n = 0;
+            int has_block_race_at_min_b = 0, have_min_b = 0;
+            uint32_t min_b = 0;
+            for (uint64_t bs = gs; bs < ge;) {
+                uint32_t blk = acc[bs].block;
+                uint64_t be = bs;
+                uint8_t bmask = 0;
+                while (be < ge && acc[be].block == blk)
+                    bmask |= (uint8_t)(1u << acc[be].kind), be++;
+                if (masks_push(&blocks, bmask))
+                    err = -1;
+                /* per block epoch b of this block */
+                for (uint64_t es = bs; es < be;) {
+                    uint32_t b = acc[es].b;
+                    uint64_t ee = es;
+                    while (ee < be && acc[ee].b == b)
+                        ee++;
+                    /* BLOCK level: groups = warps of (block, b) */
+                    warps.n = 0;
+                    int warp_race = 0;
+                    for (uint64_t ws = es; ws < ee;) {
+                        uint32_t wp = acc[ws].warp;
+                        uint64_t we = ws;
+                        uint8_t wmask = 0;
+                        while (we < ee && acc[we].warp == wp)
+                            wmask |= (uint8_t)(1u << acc[we].kind), we++;
+                        if (masks_push(&warps, wmask))
+                            err = -1;
+                        /* WARP level: groups = threads of (block, b, warp, w) */
+                        for (uint64_t xs = ws; xs < we;) {
+                            uint32_t w = acc[xs].w;
+                            uint64_t xe = xs;
+                            while (xe < we && acc[xe].w == w)
+                                xe++;
+                            threads.n = 0;
+                            for (uint64_t ts = xs; ts < xe;) {
+                                uint32_t t = acc[ts].tid;
+                                uint8_t tmask = 0;
+                                while (ts < xe && acc[ts].tid == t)
+                                    tmask |= (uint8_t)(1u << acc[ts].kind), ts++;
+                                if (masks_push(&threads, tmask))
+                                    err = -1;
+                            }
+                            if (distinct_conflict(threads.m, threads.n, 1))
+                                warp_race = 1;
+                            xs = xe;
+                        }
+                        ws = we;
+                    }
+                    int block_race = distinct_conflict(warps.m, warps.n, 1);
+                    if ((block_race || warp_race) && (!have_min_b || b < min_b)) {
+                        have_min_b = 1;
+                        min_b = b;
+                        has_block_race_at_min_b = block_race;
+                    } else if ((block_race || warp_race) && have_min_b && b == min_b && block_race) {
+                        has_block_race_at_min_b = 1;
+                    }
+                    es = ee;
+                }
+                bs = be;
+            }
+            int grid_race = distinct_conflict(blocks.m, blocks.n, 0);
+            if (grid_race) {
+                cls = CLS_GRID;
+            } else if (have_min_b) {
+                if (blocks.n >= 2)
+                    err = -2; /* C1.6 premise: only one block can touch the key in g* */
+                cls = has_block_race_at_min_b ? CLS_BLOCK : CLS_WARP;
+            }
+            gstar = g;
+            gs = ge;
+        }
+        if (cls != CLS_NONE) {
+            if ((uint64_t)nflag < cap) {
+                if (out_key)
+                    out_key[nflag] = key;
+                if (out_cls)
+                    out_cls[nflag] = (uint8_t)cls;
+                if (out_g)
+                    out_g[nflag] = (uint8_t)gstar;
+            }
+            nflag++;
+        }
+        i = kend;
+    }
+    free(blocks.m);
+    free(warps.m);
+    free(threads.m);
+    free(acc);
+    return err ? err : nflag;
+}
