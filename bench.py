@@ -1,0 +1,332 @@
+"""bench.py — checked accesses/s of the B200 HiRace hot path (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl hirace|reference] [--config 2]
+
+One step = one pass of the whole hot path over the workload: shadow reset (a11), replay of
+the full trace through the FSM with CAS updates and race reports (a1-a9), and the device-side
+collection of flagged words (a7).  Default workload = BASELINE.json configs[1] (config 2:
+tiled shared-memory stencil, 1024 blocks x 256 threads, racy-A variant, 17,825,792 events);
+inputs are resident in HBM when timing starts and are larger than L2 (285 MB of events).
+
+`value` = word-level accesses checked per second (whole job, all ranks).  `e2e` = the same
+metric through the C-ABI host entry point (hirace_check_trace_host: pinned host events ->
+H2D -> replay -> collect -> D2H).  `roofline` = the replay kernel against the measured HBM
+copy bandwidth at 32 algorithmic bytes per access.  `cpu_baseline` = the oracle (C, one core).
+`--impl reference` times that oracle as the reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "checked accesses/sec"
+UNIT = "accesses/s"
+BYTES_PER_ACCESS = 32  # 16-B event + 8-B shadow read + 8-B shadow write
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def make_trace(config: int, variant: str):
+    import tracegen as tg
+    if config == 1:
+        return tg.cfg1("post_init" if variant == "racy" else None)
+    if config == 2:
+        return tg.cfg2(variant == "racy")
+    if config == 4:
+        return tg.cfg4("B" if variant == "racy" else None)
+    raise SystemExit(f"config {config} not available in bench yet")
+
+
+def word_accesses(events) -> int:
+    sz = 1 << ((events["meta"] >> 2) & 7).astype(np.int64)
+    return int(np.where(sz <= 4, 1, sz // 4).sum())
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled while the timed region runs."""
+
+    Q = ("timestamp,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+        self.windows = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except (FileNotFoundError, OSError):
+            self.proc = None
+            return
+        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append((time.time(), [x.strip() for x in line.split(",")]))
+
+    def mark(self, t0, t1):
+        self.windows.append((t0, t1))
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        inside = [r for t, r in self.rows if any(a - 0.06 <= t <= b + 0.06 for a, b in self.windows)]
+        rows = inside or [r for _, r in self.rows]
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({n for r in rows for n, v in zip(names, r[5:9]) if v.lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows), "samples_in_timed_region": len(inside)}
+
+
+def load_traffic(config: int, variant: str):
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(f"cfg{config}_{variant}")
+    return None
+
+
+def time_oracle(trace, budget_s: float):
+    """Oracle-D as it stands on a bounded sample: the events of the first m blocks."""
+    import oracle
+    import tracegen as tg
+    ev = trace.events
+    blk = ev["tid"] // trace.block_threads
+    # calibrate on 1/64 of the blocks
+    m0 = max(1, trace.grid_blocks // 64)
+    s0 = ev[blk < m0]
+    t = time.perf_counter()
+    oracle.races(s0, trace.block_threads, trace.warp_size)
+    rate = max(len(s0), 1) / max(time.perf_counter() - t, 1e-6)
+    m = int(min(trace.grid_blocks, max(m0, trace.grid_blocks * min(1.0, budget_s * rate / max(len(ev), 1)))))
+    sample = ev[blk < m]
+    sub = tg.Trace(trace.name, sample, trace.grid_blocks, trace.block_threads, trace.warp_size,
+                   trace.global_words, trace.smem_words)
+    return sub, m
+
+
+def run_reference(args, trace, world):
+    import oracle
+    if int(os.environ.get("RANK", "0")) != 0:
+        return
+    budget = max(0.05, 150.0 / max(args.steps + args.warmup, 1))
+    sub, m = time_oracle(trace, budget)
+    n_acc = word_accesses(sub.events)
+    for _ in range(args.warmup):
+        oracle.races(sub.events, sub.block_threads, sub.warp_size)
+    t = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.races(sub.events, sub.block_threads, sub.warp_size)
+    dt = (time.perf_counter() - t) / max(args.steps, 1)
+    v = n_acc / dt
+    sample = f"events of blocks [0,{m}) of {trace.name} ({n_acc} word accesses) per step"
+    out = {"metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True, "scaling": "weak",
+           "vs_baseline": None, "dtype": "u64", "data": "synthetic", "impl": "reference",
+           "config": config_block(args, trace, world),
+           "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+           "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def config_block(args, trace, world):
+    return {"workload": f"config {args.config} ({trace.name}): {BASELINE_CFG.get(args.config, '')}",
+            "events_per_rank": int(trace.n), "grid_blocks": trace.grid_blocks,
+            "block_threads": trace.block_threads, "batches": trace.batch_count(),
+            "shadow_bytes": 8 * (trace.global_words + trace.grid_blocks * trace.smem_words),
+            "l2": "inputs larger than L2 (events %.0f MB > 126 MB L2)" % (trace.n * 16 / 1e6),
+            "parallelism": f"replicas{world}" if world > 1 else "single"}
+
+
+BASELINE_CFG = {
+    1: "tiny shared-mem reduction, 1 block x 32 threads, missing __syncthreads",
+    2: "tiled shared-memory stencil, 1024 blocks x 256 threads, racy-A (load->compute barrier dropped)",
+    4: "cooperative multi-phase kernel, 592 x 256, 64 grid phases, racy-B",
+}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="hirace", choices=["hirace", "reference"])
+    ap.add_argument("--config", type=int, default=2)
+    ap.add_argument("--variant", default="racy", choices=["racy", "clean"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    trace = make_trace(args.config, args.variant)
+
+    if args.impl == "reference":
+        run_reference(args, trace, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_jacobsonbg24_b200 as hr
+    torch.cuda.set_device(local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+
+    n_acc = word_accesses(trace.events)
+    c = hr.Checker.for_trace(trace, device=local_rank)
+    d_ev = hr.events_to_device(trace.events, f"cuda:{local_rank}")
+    cap = 1 << 20
+    d_out = torch.empty(cap * 16, dtype=torch.uint8, device="cuda")
+    d_total = torch.zeros(1, dtype=torch.int64, device="cuda")
+    stream = torch.cuda.current_stream()
+    K, W = args.steps, args.warmup
+    ks = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
+    ke = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
+    for e in ks + ke:
+        e.record(stream)
+
+    def step(i=None):
+        c.reset(stream)
+        if i is not None:
+            c.set_kernel_timing(ks[i], ke[i])
+        else:
+            c.set_kernel_timing(None, None)
+        c.replay(d_ev, stream=stream)
+        c.collect_device(d_out, cap, d_total, stream=stream)
+
+    clocks = ClockSampler(local_rank)
+    clocks.start()
+    time.sleep(0.3)
+    for _ in range(W):
+        step()
+    torch.cuda.synchronize()
+    flagged = int(d_total.item())
+
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    w0 = time.time()
+    t0.record(stream)
+    for i in range(K):
+        step(i)
+    t1.record(stream)
+    torch.cuda.synchronize()
+    w1 = time.time()
+    if world > 1:
+        dist.barrier()
+    clocks.mark(w0, w1)
+    ms = t0.elapsed_time(t1)
+    kern_ms = sum(a.elapsed_time(b) for a, b in zip(ks, ke)) / K
+    c.set_kernel_timing(None, None)
+    if world > 1:
+        tt = torch.tensor([ms, kern_ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms, kern_ms = float(tt[0]), float(tt[1])
+    ms_per_step = ms / K
+    value = n_acc * world * K / (ms / 1e3)
+    st = c.stats()
+
+    # e2e through the C-ABI host entry point: pinned host events -> H2D -> replay -> D2H
+    e2e = None
+    if not args.no_e2e:
+        pin = torch.empty(trace.n * 16, dtype=torch.uint8, pin_memory=True)
+        pin.numpy()[:] = trace.events.view(np.uint8)
+        hout = torch.empty(cap * 16, dtype=torch.uint8, pin_memory=True)
+        ke2 = max(3, min(K, 10))
+        for _ in range(2):
+            c.reset(stream)
+            c.check_host_ptr(pin.data_ptr(), trace.n, hout.data_ptr(), cap, stream=stream)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        we0 = time.perf_counter()
+        for _ in range(ke2):
+            c.reset(stream)
+            tot = c.check_host_ptr(pin.data_ptr(), trace.n, hout.data_ptr(), cap, stream=stream)
+        torch.cuda.synchronize()
+        e2e_s = (time.perf_counter() - we0) / ke2
+        if world > 1:
+            tt = torch.tensor([e2e_s], dtype=torch.float64, device="cuda")
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            e2e_s = float(tt[0])
+        e2e = {"value": n_acc * world / e2e_s, "unit": UNIT, "h2d_bytes_per_step": int(trace.n * 16),
+               "d2h_bytes_per_step": int(min(tot, cap) * 16 + 8), "ms_per_step": e2e_s * 1e3}
+    clocks.stop()
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+    peak, peak_kind = peaks()
+    achieved = BYTES_PER_ACCESS * n_acc / (kern_ms / 1e3) / 1e9
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        import oracle
+        sub, m = time_oracle(trace, 20.0)
+        t = time.perf_counter()
+        oracle.races(sub.events, sub.block_threads, sub.warp_size)
+        dt = time.perf_counter() - t
+        na = word_accesses(sub.events)
+        cpu = {"value": na / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"events of blocks [0,{m}) of {trace.name} ({na} word accesses), one run, 1 thread"}
+    out = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": W,
+        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "u64", "data": "synthetic", "config": config_block(args, trace, world),
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": load_traffic(args.config, args.variant),
+                     "kernel": "k_replay", "kernel_ms": kern_ms, "kernel_share": kern_ms / ms_per_step,
+                     "bytes_per_access": BYTES_PER_ACCESS, "peak_kind": peak_kind},
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": 6 * K,
+        "clocks": clocks.summary(),
+        "check": {"flagged_words": flagged, "per_step": st},  # stats are per step (reset clears them)
+    }
+    print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,227 @@
+/*
+ * hirace.h — C-ABI of the B200-native HiRace hot path (libhirace.so).
+ *
+ * HiRace (Jacobson, Burtscher, Gopalakrishnan, SC'24; /root/reference/PAPER.md) keeps ONE
+ * constant-size shadow record per tracked memory word — an FSM state plus the last accessor's
+ * id and barrier epochs (Fig. 3) — and advances it on every read, write or
+ * atomic with a lock-free atomicCAS loop (Algorithm 1).  A word whose record
+ * reaches RACE has two accesses that are not ordered by the bulk-synchronous barrier hierarchy
+ * (data-race definition PAPER.md; barriers L120-122, L211-213; atomics/scopes L215-229).
+ *
+ * Plain C: pointers are host or device as stated per argument, sizes are counts, streams are
+ * `cudaStream_t` passed as `void*` (0 = legacy default stream).  No torch types.
+ *
+ * ERRORS.  Every host function returns hirace_status.  Errors are STICKY per context: once a
+ * call returns (or a kernel records) an error, later calls on that context return it too,
+ * except hirace_shadow_free / hirace_get_stats / hirace_status_string.  Races collected before
+ * HIRACE_E_CLOCK_OVERFLOW stay valid ("detection is discontinued with a warning ... after
+ * reporting identified races", PAPER.md L227 fn. 3).  Errors found by kernels (bad trace,
+ * clock overflow) surface at the next synchronising call (collect / get_stats / sync).
+ *
+ * OWNERSHIP.  The context owns the shadow array, the FSM table, the race-report buffer and all
+ * scratch.  The caller owns event buffers and output buffers.
+ *
+ * STREAMS.  Calls taking a stream are asynchronous on it, except where noted.  One context
+ * must not be used from two streams concurrently.
+ */
+#ifndef HIRACE_H
+#define HIRACE_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    HIRACE_OK = 0,
+    HIRACE_E_INVAL = -1,          /* bad argument / config / unsupported combination          */
+    HIRACE_E_NOMEM = -2,          /* device or host allocation failed                          */
+    HIRACE_E_CUDA = -3,           /* a CUDA runtime call failed (no device, launch error, ...) */
+    HIRACE_E_CLOCK_OVERFLOW = -4, /* an epoch counter exceeded its field (g 8 / b 10 / w 9 bits)
+                                     in an inline hook; detection stopped, races so far valid
+                                     (PAPER.md L227 fn. 3, L458)                               */
+    HIRACE_E_REPORT_OVERFLOW = -5,/* reserved: collection never loses races (shadow scan)     */
+    HIRACE_E_BAD_TRACE = -6,      /* replay input not sorted by (g,b,w), tid/address out of
+                                     range, access size > 16 B, or > HIRACE_MAX_BATCHES batches */
+    HIRACE_E_COMM = -7            /* sharded mode exchange failure (set by the Python layer)   */
+} hirace_status;
+
+/* Access kinds: the paper's 4 memory access types. */
+typedef enum {
+    HIRACE_READ = 0,
+    HIRACE_WRITE = 1,
+    HIRACE_ATOMIC_BLOCK = 2, /* block-scope atomic (atomicAdd_block, ...) */
+    HIRACE_ATOMIC_GRID = 3   /* device-scope atomic (atomicMin, ...)       */
+} hirace_kind;
+
+/* Barrier scopes.  GRID = grid-wide sync or kernel boundary. */
+typedef enum { HIRACE_SCOPE_WARP = 1, HIRACE_SCOPE_BLOCK = 2, HIRACE_SCOPE_GRID = 3 } hirace_scope;
+
+/* Race class = the coarsest hierarchy level of the first racing epoch (R6). */
+typedef enum { HIRACE_RACE_WARP = 1, HIRACE_RACE_BLOCK = 2, HIRACE_RACE_GRID = 3 } hirace_race_class;
+
+#define HIRACE_MAX_BATCHES 32767u   /* distinct (g,b,w) batch keys per replay call */
+#define HIRACE_SHARED_BIT (1ull << 63)
+
+/* Tracked geometry.  warp_size may be any value >= 1 (2 reproduces the paper's Fig. 1 toy
+ * hierarchy).  Tracking granularity is the 4-byte word (per array element,
+ * PAPER.md L162): granularity_log2 must be 2.  report_capacity = device race-report records
+ * (16 B each); 0 selects a default of 1<<20. */
+typedef struct {
+    uint32_t grid_blocks;          /* blocks of the checked kernel                        */
+    uint32_t block_threads;        /* threads per block (blockDim.x*y*z)                   */
+    uint32_t warp_size;            /* threads per warp (32 on NVIDIA hardware)             */
+    uint32_t smem_bytes_per_block; /* tracked shared-memory window per block, bytes        */
+    uint64_t global_bytes;         /* tracked global extent, bytes from the tracked base   */
+    uint32_t granularity_log2;     /* must be 2                                            */
+    int32_t device;                /* CUDA device ordinal                                  */
+    uint64_t report_capacity;      /* race-report ring entries (0 = default)               */
+} hirace_config;
+
+/* One traced access, 16 bytes.
+ *   addr: bit 63 = shared space.  Shared: byte offset inside the accessing block's tracked
+ *         shared window.  Global: byte offset from the tracked global base.
+ *   tid:  global thread id = block * block_threads + thread-in-block.
+ *   meta: kind:2 | size_log2:3 | w:9 | b:10 | g:8  (bit 0 upward); size = 1 << size_log2 bytes
+ *         (<= 16); g = grid epochs (kernel boundaries / grid syncs) passed, b = __syncthreads
+ *         passed since the last g, w = full-warp syncs passed since the last b. */
+typedef struct {
+    uint64_t addr;
+    uint32_t tid;
+    uint32_t meta;
+} hirace_event;
+
+/* One flagged word.  key: global -> word index; shared -> 1<<63 | block<<32 | word.
+ * cls_and_epoch = class (1..3) | (g* mod 256) << 8, g* = grid epoch of the first race.
+ * detect_tid = the thread whose access moved the record into RACE (not unique across
+ * interleavings; never compared). */
+typedef struct {
+    uint64_t key;
+    uint32_t cls_and_epoch;
+    uint32_t detect_tid;
+} hirace_race;
+
+typedef struct hirace_ctx hirace_ctx;
+
+/* Device-side context handed by value to instrumented kernels (include/hirace_device.cuh).
+ * All pointers are device pointers owned by the hirace_ctx. */
+typedef struct {
+    unsigned long long *shadow;       /* [global_words | grid_blocks * smem_words] records   */
+    const unsigned char *table;       /* 2048-entry FSM transition table                      */
+    hirace_race *reports;             /* race-report ring                                     */
+    unsigned long long *report_count; /* records appended (may exceed capacity)               */
+    unsigned long long *stats;        /* [checked, cas_retries, cas_ops, no_write]            */
+    unsigned int *error_flags;        /* bit0 bad trace, bit1 clock overflow                  */
+    unsigned long long report_capacity;
+    unsigned long long global_words;
+    const void *global_base;          /* tracked global base for inline hooks (may be NULL)   */
+    unsigned int smem_words;
+    unsigned int grid_blocks, block_threads, warp_size;
+    unsigned int bt_magic, bt_s1, bt_s2; /* fast division by block_threads                    */
+    unsigned int ws_magic, ws_s1, ws_s2; /* fast division by warp_size                        */
+    unsigned int g;                   /* current grid epoch for inline hooks                  */
+} hirace_dev_ctx;
+
+/* ---- lifecycle (a11: shadow alloc/init, "Initially, all State values are set
+ *      to INIT") -------------------------------------------------------------------------- */
+
+/* Allocates shadow = 8 B per tracked word (global_bytes/4 + grid_blocks*smem_bytes/4 words),
+ * all INIT, plus the FSM table and report buffer on cfg->device.  Synchronous.
+ * Errors: INVAL (NULL args, zero geometry, granularity != 2, tid space > 2^32), NOMEM, CUDA. */
+hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out);
+
+/* Frees everything the context owns (synchronises the device first).  NULL is a no-op. */
+hirace_status hirace_shadow_free(hirace_ctx *ctx);
+
+/* Sets every shadow record to INIT, clears reports, stats and sticky errors; g := 0. Async. */
+hirace_status hirace_shadow_reset(hirace_ctx *ctx, void *stream);
+
+/* Host barrier hook.  Only HIRACE_SCOPE_GRID is meaningful on the host: a kernel boundary /
+ * grid sync advances the context's grid epoch g used by inline hooks.  When g
+ * would wrap its 8-bit field the library first runs a rebase sweep (non-RACE records -> INIT,
+ * RACE records retired) so equality-only epoch comparisons stay exact (R7).
+ * WARP/BLOCK scopes are device-side (hirace::barrier) -> INVAL.  Async. */
+hirace_status hirace_barrier(hirace_ctx *ctx, hirace_scope scope, void *stream);
+
+/* ---- replay (a1-a9) ------------------------------------------------------------------- */
+
+/* Replays n DEVICE-resident events through the shadow FSM.  Events must be sorted by batch
+ * key (g,b,w) = meta >> 5; inside a batch any order (all such events are pairwise concurrent
+ * or same-thread, so any order is a linear extension of happens-before).
+ * Batches are found on the device and validated (any unsorted input, out-of-range tid or
+ * address, size > 16 B -> sticky HIRACE_E_BAD_TRACE, reported at the next sync).  At most
+ * HIRACE_MAX_BATCHES batches and n < 2^32 per call; consecutive calls on one stream continue
+ * the same linearisation.  Async on `stream`. */
+hirace_status hirace_replay_trace(hirace_ctx *ctx, const hirace_event *d_events, uint64_t n, void *stream);
+
+/* Same work from HOST events (pinned or pageable): copies through a device staging ring in
+ * chunks, overlapping H2D with replay, then collects like hirace_collect_races.  Synchronous.
+ * This is the end-to-end entry point. */
+hirace_status hirace_check_trace_host(hirace_ctx *ctx, const hirace_event *h_events, uint64_t n,
+                                      hirace_race *h_out, uint64_t cap, uint64_t *n_total, void *stream);
+
+/* ---- results (a7) -------------------------------------------------------------------- */
+
+/* Copies min(cap, n_total) flagged words, sorted by key, unique, to HOST memory h_out and sets
+ * *n_total (call again with a bigger buffer if n_total > cap).  Synchronises `stream`.
+ * Returns the sticky status (e.g. BAD_TRACE) after copying. */
+hirace_status hirace_collect_races(hirace_ctx *ctx, hirace_race *h_out, uint64_t cap, uint64_t *n_total,
+                                   void *stream);
+
+/* Device-side variant: writes min(cap, total) records to DEVICE memory d_out and the total to
+ * DEVICE *d_n_total.  Async (for timed loops / CUDA graphs). */
+hirace_status hirace_collect_races_device(hirace_ctx *ctx, hirace_race *d_out, uint64_t cap,
+                                          unsigned long long *d_n_total, void *stream);
+
+/* Counters since the last reset: word-level accesses checked, CAS retries, CAS issued,
+ * accesses linearised without a store (no-write fast path), reports appended beyond capacity.
+ * Synchronises the device.  Any pointer may be NULL. */
+hirace_status hirace_get_stats(hirace_ctx *ctx, uint64_t *checked, uint64_t *cas_retries, uint64_t *cas_ops,
+                               uint64_t *no_write, uint64_t *dropped_reports);
+
+/* Synchronises and returns the sticky status (HIRACE_OK if none). */
+hirace_status hirace_sync(hirace_ctx *ctx);
+
+/* Copies the device context for inline hooks into *out (host memory).  global_base is the
+ * device address tracked global offsets are measured from (may be NULL for replay-only). */
+hirace_status hirace_get_dev_ctx(hirace_ctx *ctx, const void *global_base, hirace_dev_ctx *out);
+
+/* Measurement hook: when both are non-NULL, every later hirace_replay_trace records `start`
+ * immediately before and `stop` immediately after its replay-kernel launch on the call's
+ * stream (cudaEvent_t handles owned by the caller), so the caller can time the dominant
+ * kernel alone with cudaEventElapsedTime.  NULL, NULL disables it. */
+hirace_status hirace_set_kernel_timing(hirace_ctx *ctx, void *start_event, void *stop_event);
+
+/* ---- sharded mode (a10) ---------------------------------------------------------------- */
+
+/* Buckets n DEVICE events by owner rank for address sharding across nranks GPUs:
+ * owner(global word) = (word >> 14) mod nranks (64 KiB chunks), shared-space events stay on
+ * `my_rank`.  Writes events grouped by owner (stable inside each owner, so batch order is
+ * preserved) to DEVICE d_out (n records) and per-owner counts to HOST h_counts[nranks].
+ * Synchronises `stream` (the counts are needed to size the exchange). */
+hirace_status hirace_bucket_events(hirace_ctx *ctx, const hirace_event *d_in, uint64_t n, int nranks, int my_rank,
+                                   hirace_event *d_out, uint64_t *h_counts, void *stream);
+
+/* ---- verification hooks (host-only, NOT a replay path) --------------------------------- */
+
+/* Writes the 2048-byte FSM transition table: entry[state<<6 | kind<<4 | sync<<2 | rel] =
+ * next_state:5 | keep_record:1 | report:1 (PAPER.md L295 flat-array encoding). */
+hirace_status hirace_fsm_table(unsigned char out[2048]);
+
+/* One FSM step on the host with the same inline function the kernels use, for model checking:
+ * returns the new 64-bit record for old record `old_shadow` and one access. *report is set to
+ * 1 if the step enters or upgrades a RACE state. */
+uint64_t hirace_fsm_step(uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t b, uint32_t w,
+                         uint32_t block_threads, uint32_t warp_size, int *report);
+
+const char *hirace_status_string(hirace_status s);
+
+/* Library version string and the compile target ("sm_100a"). */
+const char *hirace_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HIRACE_H */

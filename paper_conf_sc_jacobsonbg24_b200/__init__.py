@@ -1,0 +1,10 @@
+"""B200-native HiRace hot path: per-access shadow-state update for GPU data-race checking.
+
+The compute path is libhirace.so (sm_100a CUDA kernels behind the C-ABI in include/hirace.h);
+`hirace` is its ctypes binding, `sharded` the address-sharded multi-GPU driver.
+"""
+from .hirace import (ATOMIC_BLOCK, ATOMIC_GRID, EVENT_DTYPE, RACE_DTYPE, READ, WRITE, Checker,  # noqa: F401
+                     HiraceError, events_to_device, fsm_step, fsm_table, load, races_to_dict)
+
+__all__ = ["Checker", "HiraceError", "EVENT_DTYPE", "RACE_DTYPE", "events_to_device", "fsm_step", "fsm_table",
+           "load", "races_to_dict", "READ", "WRITE", "ATOMIC_BLOCK", "ATOMIC_GRID"]

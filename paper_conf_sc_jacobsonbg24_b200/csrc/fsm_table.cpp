@@ -1,0 +1,206 @@
+/*
+ * fsm_table.cpp — builds HiRace's flat transition table (PAPER.md: "The HiRace FSM is
+ * encoded as a flat array indexed by a concatenation of oState and the transition labels").
+ *
+ * The paper's full 25-state table lives in an external artifact; this build
+ * derives its own exact machine from the race definition:
+ * 23 states, labels = 4 kinds x 4 sync statuses (Us, Ws, Bs + Gs for a new grid epoch)
+ * x 4 thread relations (S, W, B, G).  Entry = next_state:5 | keep:1 | report:1.
+ *
+ * Kind classes.  Inside one block atomics of either scope never conflict with each other:
+ *   cls(R)=R, cls(AB)=cls(AG)=A, cls(W)=X.
+ * Across blocks only grid-scope atomics are mutually atomic:
+ *   clsG(R)=R, clsG(AG)=AG, clsG(AB)=clsG(W)=X.
+ * join(x,y) = x if x==y else X.  compat(c,k) <=> c == cls(k) in {R,A};
+ * compatG(c,k) <=> c == clsG(k) in {R,AG}.
+ *
+ * States (per location, within the current grid epoch):
+ *   T(KT,KB,KG)  one thread in the current warp epoch; KT its kinds there, KB its warp's kinds
+ *                in the current block epoch, KG its block's kinds in the grid epoch
+ *   W(c,KB,KG)   >= 2 threads of one warp in the current warp epoch, all of class c
+ *   B(c,KG)      >= 2 warps of one block in the current block epoch, all of class c
+ *   G(c)         >= 2 blocks in the grid epoch, all of class c
+ *   RACE_W/B/G   sticky; class = coarsest level in the first racing epoch (upgrades allowed
+ *                while still in that epoch)
+ * Rules, first match wins (record := the current accessor unless "keep"):
+ *   0 RACE_*: Gs -> keep.  RACE_W & rel B & Us -> RACE_B (report).  RACE_W/B & rel G & !Gs
+ *     -> RACE_G (report).  Otherwise keep.
+ *   1 INIT or Gs -> T(cls k, cls k, clsG k)
+ *   2 G(c): compatG(c,k) -> G(c) keep, else RACE_G
+ *   3 rel G: compatG(KG,k) -> G(KG), else RACE_G
+ *   4 Bs -> T(cls k, cls k, KG')
+ *   5 B(c,KG): compat(c,k) -> B(c,KG') keep, else RACE_B
+ *   6 rel B: compat(KB,k) -> B(KB,KG'), else RACE_B
+ *   7 Ws -> T(cls k, KB', KG')
+ *   8 W(c,KB,KG): compat(c,k) -> W(c,KB',KG') keep, else RACE_W
+ *   9 rel W (state T): compat(KT,k) -> W(KT,KB',KG'), else RACE_W
+ *  10 rel S (state T): T(join(KT,cls k), KB', KG') keep
+ * with KB' = join(KB, cls k), KG' = join(KG, clsG k).
+ */
+#include <stdint.h>
+#include <string.h>
+
+#include "hirace.h"
+#include "hirace_device.cuh"
+
+namespace {
+
+enum Cl { C_R = 0, C_A = 1, C_AG = 2, C_X = 3 };
+
+enum Group { G_INIT, G_T, G_W, G_B, G_G, G_RACE, G_NONE };
+
+struct Desc {
+    Group grp;
+    int a, b, c; /* T: KT,KB,KG  W: c,KB,KG  B: c,KG  G: c */
+};
+
+const Desc kStates[hirace::ST_COUNT] = {
+    {G_INIT, 0, 0, 0},
+    {G_T, C_R, C_R, C_R},   {G_T, C_R, C_R, C_X},  {G_T, C_R, C_X, C_X}, {G_T, C_X, C_X, C_X},
+    {G_T, C_A, C_A, C_AG},  {G_T, C_A, C_A, C_X},  {G_T, C_A, C_X, C_X},
+    {G_W, C_R, C_R, C_R},   {G_W, C_R, C_R, C_X},  {G_W, C_R, C_X, C_X},
+    {G_W, C_A, C_A, C_AG},  {G_W, C_A, C_A, C_X},  {G_W, C_A, C_X, C_X},
+    {G_B, C_R, C_R, 0},     {G_B, C_R, C_X, 0},    {G_B, C_A, C_AG, 0},  {G_B, C_A, C_X, 0},
+    {G_G, C_R, 0, 0},       {G_G, C_AG, 0, 0},
+    {G_RACE, 1, 0, 0},      {G_RACE, 2, 0, 0},     {G_RACE, 3, 0, 0},
+};
+
+int cls_low(uint32_t k) { return k == HIRACE_READ ? C_R : (k == HIRACE_WRITE ? C_X : C_A); }
+int cls_grid(uint32_t k) { return k == HIRACE_READ ? C_R : (k == HIRACE_ATOMIC_GRID ? C_AG : C_X); }
+int join(int x, int y) { return x == y ? x : C_X; }
+bool compat(int c, uint32_t k) { return (c == C_R || c == C_A) && c == cls_low(k); }
+bool compatG(int c, uint32_t k) { return (c == C_R || c == C_AG) && c == cls_grid(k); }
+
+int find(Group grp, int a, int b, int c)
+{
+    for (int s = 0; s < (int)hirace::ST_COUNT; s++) {
+        const Desc &d = kStates[s];
+        if (d.grp != grp || d.a != a)
+            continue;
+        if (grp == G_G || grp == G_RACE)
+            return s;
+        if (grp == G_B && d.b == b)
+            return s;
+        if ((grp == G_T || grp == G_W) && d.b == b && d.c == c)
+            return s;
+    }
+    return -1; /* unreachable for consistent tuples; checked by the caller */
+}
+
+struct Out {
+    int next;
+    bool keep, report;
+};
+
+Out rules(int s, uint32_t k, uint32_t sync, uint32_t rel)
+{
+    using namespace hirace;
+    const Desc d = kStates[s];
+    const int ck = cls_low(k), gk = cls_grid(k);
+    const int RW = ST_RACE_W, RB = ST_RACE_B, RG = ST_RACE_G;
+    /* rule 0 */
+    if (d.grp == G_RACE) {
+        if (sync == SYNC_GS)
+            return {s, true, false};
+        if (s == RW && rel == REL_B && sync == SYNC_US)
+            return {RB, true, true};
+        if ((s == RW || s == RB) && rel == REL_G)
+            return {RG, true, true};
+        return {s, true, false};
+    }
+    /* rule 1 */
+    if (d.grp == G_INIT || sync == SYNC_GS)
+        return {find(G_T, ck, ck, gk), false, false};
+    /* rule 2 */
+    if (d.grp == G_G)
+        return compatG(d.a, k) ? Out{s, true, false} : Out{RG, false, true};
+    int KT = 0, KB = 0, KG = 0;
+    if (d.grp == G_T) {
+        KT = d.a;
+        KB = d.b;
+        KG = d.c;
+    } else if (d.grp == G_W) {
+        KT = d.a;
+        KB = d.b;
+        KG = d.c;
+    } else { /* G_B */
+        KB = d.a;
+        KG = d.b;
+    }
+    const int KBp = join(KB, ck), KGp = join(KG, gk);
+    /* rule 3 */
+    if (rel == REL_G)
+        return compatG(KG, k) ? Out{find(G_G, KG, 0, 0), false, false} : Out{RG, false, true};
+    /* rule 4 */
+    if (sync == SYNC_BS)
+        return {find(G_T, ck, ck, KGp), false, false};
+    /* rule 5 */
+    if (d.grp == G_B)
+        return compat(d.a, k) ? Out{find(G_B, d.a, KGp, 0), true, false} : Out{RB, false, true};
+    /* rule 6 */
+    if (rel == REL_B)
+        return compat(KB, k) ? Out{find(G_B, KB, KGp, 0), false, false} : Out{RB, false, true};
+    /* rule 7 */
+    if (sync == SYNC_WS)
+        return {find(G_T, ck, KBp, KGp), false, false};
+    /* rule 8 */
+    if (d.grp == G_W)
+        return compat(d.a, k) ? Out{find(G_W, d.a, KBp, KGp), true, false} : Out{RW, false, true};
+    /* rule 9 */
+    if (rel == REL_W)
+        return compat(KT, k) ? Out{find(G_W, KT, KBp, KGp), false, false} : Out{RW, false, true};
+    /* rule 10 */
+    return {find(G_T, join(KT, ck), KBp, KGp), true, false};
+}
+
+} // namespace
+
+extern "C" hirace_status hirace_fsm_table(unsigned char out[2048])
+{
+    if (!out)
+        return HIRACE_E_INVAL;
+    for (int s = 0; s < 32; s++) {
+        for (uint32_t k = 0; k < 4; k++)
+            for (uint32_t y = 0; y < 4; y++)
+                for (uint32_t r = 0; r < 4; r++) {
+                    uint32_t idx = ((uint32_t)s << 6) | (k << 4) | (y << 2) | r;
+                    if (s >= (int)hirace::ST_COUNT) {
+                        out[idx] = (unsigned char)(s | hirace::E_KEEP); /* unused codes */
+                        continue;
+                    }
+                    Out o = rules(s, k, y, r);
+                    if (o.next < 0)
+                        return HIRACE_E_INVAL; /* inconsistent tuple: a rule-table bug */
+                    out[idx] = (unsigned char)(o.next | (o.keep ? hirace::E_KEEP : 0) |
+                                               (o.report ? hirace::E_REPORT : 0));
+                }
+    }
+    return HIRACE_OK;
+}
+
+extern "C" uint64_t hirace_fsm_step(uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t b,
+                                    uint32_t w, uint32_t block_threads, uint32_t warp_size, int *report)
+{
+    static unsigned char table[2048];
+    static bool built = false;
+    if (!built) {
+        hirace_fsm_table(table);
+        built = true;
+    }
+    hirace::geom G;
+    G.bt = block_threads ? block_threads : 1;
+    hirace::fastdiv_init(G.bt, &G.bt_m, &G.bt_s1, &G.bt_s2);
+    hirace::fastdiv_init(warp_size ? warp_size : 1, &G.ws_m, &G.ws_s1, &G.ws_s2);
+    hirace::access a;
+    a.tid = tid;
+    hirace::coords(tid, G, &a.block, &a.warp);
+    a.kind = kind & 3;
+    a.g = g;
+    a.b = b;
+    a.w = w;
+    uint32_t rep = 0;
+    uint64_t n = hirace::step(old_shadow, a, table, G, &rep);
+    if (report)
+        *report = (int)rep;
+    return n;
+}

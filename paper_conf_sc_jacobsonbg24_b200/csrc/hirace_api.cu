@@ -1,0 +1,454 @@
+/*
+ * hirace_api.cu — host implementation of the C-ABI declared in include/hirace.h.
+ * Every step of the hot path runs in the kernels of hirace_kernels.cu; this file only
+ * validates arguments, owns device memory and sequences launches on the caller's stream.
+ * There is no CPU fallback: without a CUDA device every entry point that needs one fails
+ * with HIRACE_E_CUDA.
+ */
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <mutex>
+
+#include "hirace.h"
+#include "hirace_device.cuh"
+#include "internal.h"
+
+using namespace hirace_impl;
+
+struct hirace_ctx {
+    hirace_config cfg;
+    int device = 0;
+    int sm_count = 0;
+    int replay_grid = 0;
+    uint64_t global_words = 0, shadow_words = 0;
+    unsigned long long *d_shadow = nullptr;
+    unsigned char *d_table = nullptr;
+    hirace_race *d_reports = nullptr;
+    unsigned long long *d_report_count = nullptr;
+    unsigned long long *d_stats = nullptr;
+    unsigned int *d_err = nullptr;
+    Scratch scr{};
+    /* collect staging (host API) */
+    hirace_race *d_collect = nullptr;
+    uint64_t collect_cap = 0;
+    unsigned long long *d_total = nullptr;
+    /* bucket scratch */
+    uint32_t *d_bucket_hist = nullptr;
+    uint64_t bucket_hist_cap = 0;
+    unsigned long long *d_bucket_counts = nullptr;
+    /* host-trace staging ring */
+    hirace_event *d_stage[2] = {nullptr, nullptr};
+    uint64_t stage_cap = 0;
+    cudaStream_t copy_stream = nullptr;
+    cudaEvent_t ev_copied[2] = {nullptr, nullptr}, ev_used[2] = {nullptr, nullptr};
+    hirace_dev_ctx dev{};
+    uint32_t g = 0;
+    cudaEvent_t t_start = nullptr, t_stop = nullptr;
+    hirace_status sticky = HIRACE_OK;
+};
+
+namespace {
+
+hirace_status set_sticky(hirace_ctx *c, hirace_status s)
+{
+    if (c && s != HIRACE_OK && c->sticky == HIRACE_OK)
+        c->sticky = s;
+    return s;
+}
+
+hirace_status from_cuda(hirace_ctx *c, cudaError_t e)
+{
+    if (e == cudaSuccess)
+        return HIRACE_OK;
+    return set_sticky(c, e == cudaErrorMemoryAllocation ? HIRACE_E_NOMEM : HIRACE_E_CUDA);
+}
+
+#define HR_CUDA(c, x)                                  \
+    do {                                               \
+        cudaError_t _e = (x);                          \
+        if (_e != cudaSuccess)                         \
+            return from_cuda((c), _e);                 \
+    } while (0)
+
+hirace_status device_errors(hirace_ctx *c)
+{
+    unsigned int flags = 0;
+    cudaError_t e = cudaMemcpy(&flags, c->d_err, sizeof(flags), cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess)
+        return from_cuda(c, e);
+    if (flags & hirace::ERR_BAD_TRACE)
+        set_sticky(c, HIRACE_E_BAD_TRACE);
+    if (flags & hirace::ERR_CLOCK)
+        set_sticky(c, HIRACE_E_CLOCK_OVERFLOW);
+    return c->sticky;
+}
+
+} // namespace
+
+extern "C" {
+
+const char *hirace_version(void) { return "hirace-b200 0.1 (sm_100a)"; }
+
+const char *hirace_status_string(hirace_status s)
+{
+    switch (s) {
+    case HIRACE_OK: return "ok";
+    case HIRACE_E_INVAL: return "invalid argument";
+    case HIRACE_E_NOMEM: return "out of memory";
+    case HIRACE_E_CUDA: return "CUDA error";
+    case HIRACE_E_CLOCK_OVERFLOW: return "epoch clock overflow: detection stopped";
+    case HIRACE_E_REPORT_OVERFLOW: return "report overflow";
+    case HIRACE_E_BAD_TRACE: return "bad trace";
+    case HIRACE_E_COMM: return "communication error";
+    }
+    return "unknown";
+}
+
+hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
+{
+    if (!cfg || !out)
+        return HIRACE_E_INVAL;
+    *out = nullptr;
+    if (cfg->grid_blocks == 0 || cfg->block_threads == 0 || cfg->warp_size == 0 || cfg->granularity_log2 != 2)
+        return HIRACE_E_INVAL;
+    if ((uint64_t)cfg->grid_blocks * cfg->block_threads > 0xffffffffull)
+        return HIRACE_E_INVAL;
+    if ((cfg->smem_bytes_per_block & 3) || (cfg->global_bytes & 3))
+        return HIRACE_E_INVAL;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0 || cfg->device < 0 || cfg->device >= ndev)
+        return HIRACE_E_CUDA;
+    hirace_ctx *c = new (std::nothrow) hirace_ctx();
+    if (!c)
+        return HIRACE_E_NOMEM;
+    c->cfg = *cfg;
+    if (c->cfg.report_capacity == 0)
+        c->cfg.report_capacity = 1ull << 20;
+    c->device = cfg->device;
+    c->global_words = cfg->global_bytes >> 2;
+    const uint64_t smem_words = cfg->smem_bytes_per_block >> 2;
+    c->shadow_words = c->global_words + (uint64_t)cfg->grid_blocks * smem_words;
+    if (c->shadow_words == 0)
+        c->shadow_words = 1;
+    hirace_status st = HIRACE_OK;
+    auto fail = [&](cudaError_t e) {
+        st = e == cudaErrorMemoryAllocation ? HIRACE_E_NOMEM : HIRACE_E_CUDA;
+        hirace_shadow_free(c);
+        return st;
+    };
+    cudaError_t e;
+    if ((e = cudaSetDevice(c->device)) != cudaSuccess)
+        return fail(e);
+    static std::once_flag once[64];
+    static cudaError_t init_err[64];
+    std::call_once(once[c->device & 63], [&] { init_err[c->device & 63] = kernels_init(c->device); });
+    if ((e = init_err[c->device & 63]) != cudaSuccess)
+        return fail(e);
+    cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, c->device);
+    c->replay_grid = replay_max_grid(c->device);
+    unsigned char table[2048];
+    if (hirace_fsm_table(table) != HIRACE_OK) {
+        hirace_shadow_free(c);
+        return HIRACE_E_INVAL;
+    }
+    c->scr.ntiles = (c->shadow_words + kCollectTile - 1) / kCollectTile;
+    if ((e = cudaMalloc(&c->d_shadow, c->shadow_words * 8)) != cudaSuccess ||
+        (e = cudaMalloc(&c->d_table, 2048)) != cudaSuccess ||
+        (e = cudaMalloc(&c->d_reports, c->cfg.report_capacity * sizeof(hirace_race))) != cudaSuccess ||
+        (e = cudaMalloc(&c->d_report_count, sizeof(unsigned long long))) != cudaSuccess ||
+        (e = cudaMalloc(&c->d_stats, 4 * sizeof(unsigned long long))) != cudaSuccess ||
+        (e = cudaMalloc(&c->d_err, sizeof(unsigned int))) != cudaSuccess ||
+        (e = cudaMalloc(&c->scr.raw_pos, HIRACE_MAX_BATCHES * sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&c->scr.raw_count, sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&c->scr.batch_off, (HIRACE_MAX_BATCHES + 1) * sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&c->scr.nbatches, sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&c->scr.grid_bar, sizeof(unsigned int))) != cudaSuccess ||
+        (e = cudaMalloc(&c->scr.tile_counts, c->scr.ntiles * sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&c->d_total, sizeof(unsigned long long))) != cudaSuccess)
+        return fail(e);
+    if ((e = cudaMemcpy(c->d_table, table, 2048, cudaMemcpyHostToDevice)) != cudaSuccess)
+        return fail(e);
+    hirace_dev_ctx &d = c->dev;
+    d.shadow = c->d_shadow;
+    d.table = c->d_table;
+    d.reports = c->d_reports;
+    d.report_count = c->d_report_count;
+    d.stats = c->d_stats;
+    d.error_flags = c->d_err;
+    d.report_capacity = c->cfg.report_capacity;
+    d.global_words = c->global_words;
+    d.global_base = nullptr;
+    d.smem_words = (unsigned int)smem_words;
+    d.grid_blocks = cfg->grid_blocks;
+    d.block_threads = cfg->block_threads;
+    d.warp_size = cfg->warp_size;
+    hirace::fastdiv_init(cfg->block_threads, &d.bt_magic, &d.bt_s1, &d.bt_s2);
+    hirace::fastdiv_init(cfg->warp_size, &d.ws_magic, &d.ws_s1, &d.ws_s2);
+    d.g = 0;
+    if (hirace_shadow_reset(c, nullptr) != HIRACE_OK || cudaDeviceSynchronize() != cudaSuccess) {
+        hirace_shadow_free(c);
+        return HIRACE_E_CUDA;
+    }
+    *out = c;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_shadow_free(hirace_ctx *c)
+{
+    if (!c)
+        return HIRACE_OK;
+    cudaSetDevice(c->device);
+    cudaDeviceSynchronize();
+    void *ptrs[] = {c->d_shadow, c->d_table, c->d_reports, c->d_report_count, c->d_stats, c->d_err,
+                    c->scr.raw_pos, c->scr.raw_count, c->scr.batch_off, c->scr.nbatches, c->scr.grid_bar,
+                    c->scr.tile_counts, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
+                    c->d_stage[0], c->d_stage[1]};
+    for (void *p : ptrs)
+        if (p)
+            cudaFree(p);
+    for (int i = 0; i < 2; i++) {
+        if (c->ev_copied[i])
+            cudaEventDestroy(c->ev_copied[i]);
+        if (c->ev_used[i])
+            cudaEventDestroy(c->ev_used[i]);
+    }
+    if (c->copy_stream)
+        cudaStreamDestroy(c->copy_stream);
+    delete c;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_shadow_reset(hirace_ctx *c, void *stream)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    HR_CUDA(c, cudaMemsetAsync(c->d_shadow, 0, c->shadow_words * 8, st));
+    HR_CUDA(c, cudaMemsetAsync(c->d_report_count, 0, sizeof(unsigned long long), st));
+    HR_CUDA(c, cudaMemsetAsync(c->d_stats, 0, 4 * sizeof(unsigned long long), st));
+    HR_CUDA(c, cudaMemsetAsync(c->d_err, 0, sizeof(unsigned int), st));
+    c->g = 0;
+    c->dev.g = 0;
+    c->sticky = HIRACE_OK;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_barrier(hirace_ctx *c, hirace_scope scope, void *stream)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    if (scope != HIRACE_SCOPE_GRID)
+        return set_sticky(c, HIRACE_E_INVAL);
+    HR_CUDA(c, cudaSetDevice(c->device));
+    if (c->g + 1 >= 255u) {
+        HR_CUDA(c, launch_rebase(c->dev, c->shadow_words, (cudaStream_t)stream));
+        c->g = 0;
+    } else {
+        c->g++;
+    }
+    c->dev.g = c->g;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_replay_trace(hirace_ctx *c, const hirace_event *d_events, uint64_t n, void *stream)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    if (n == 0)
+        return HIRACE_OK;
+    if (!d_events || n >= 0xffffffffull)
+        return set_sticky(c, HIRACE_E_INVAL);
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    HR_CUDA(c, launch_find_batches(d_events, (uint32_t)n, c->scr, c->d_err, c->sm_count, st));
+    if (c->t_start)
+        HR_CUDA(c, cudaEventRecord(c->t_start, st));
+    HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st));
+    if (c->t_stop)
+        HR_CUDA(c, cudaEventRecord(c->t_stop, st));
+    return HIRACE_OK;
+}
+
+hirace_status hirace_set_kernel_timing(hirace_ctx *c, void *start_event, void *stop_event)
+{
+    if (!c || (!start_event) != (!stop_event))
+        return HIRACE_E_INVAL;
+    c->t_start = (cudaEvent_t)start_event;
+    c->t_stop = (cudaEvent_t)stop_event;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_collect_races_device(hirace_ctx *c, hirace_race *d_out, uint64_t cap,
+                                          unsigned long long *d_n_total, void *stream)
+{
+    if (!c || !d_n_total || (cap && !d_out))
+        return HIRACE_E_INVAL;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    HR_CUDA(c, launch_collect(c->dev, c->shadow_words, c->scr, d_out, cap, d_n_total, (cudaStream_t)stream));
+    return c->sticky;
+}
+
+hirace_status hirace_collect_races(hirace_ctx *c, hirace_race *h_out, uint64_t cap, uint64_t *n_total, void *stream)
+{
+    if (!c || !n_total || (cap && !h_out))
+        return HIRACE_E_INVAL;
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    if (cap > c->collect_cap) {
+        if (c->d_collect)
+            cudaFree(c->d_collect);
+        c->d_collect = nullptr;
+        c->collect_cap = 0;
+        HR_CUDA(c, cudaMalloc(&c->d_collect, cap * sizeof(hirace_race)));
+        c->collect_cap = cap;
+    }
+    HR_CUDA(c, launch_collect(c->dev, c->shadow_words, c->scr, c->d_collect, cap, c->d_total, st));
+    unsigned long long total = 0;
+    HR_CUDA(c, cudaMemcpyAsync(&total, c->d_total, sizeof(total), cudaMemcpyDeviceToHost, st));
+    HR_CUDA(c, cudaStreamSynchronize(st));
+    *n_total = total;
+    uint64_t m = total < cap ? total : cap;
+    if (m)
+        HR_CUDA(c, cudaMemcpy(h_out, c->d_collect, m * sizeof(hirace_race), cudaMemcpyDeviceToHost));
+    return device_errors(c);
+}
+
+hirace_status hirace_check_trace_host(hirace_ctx *c, const hirace_event *h_events, uint64_t n, hirace_race *h_out,
+                                      uint64_t cap, uint64_t *n_total, void *stream)
+{
+    if (!c || !n_total || (n && !h_events))
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    const uint64_t chunk = 1ull << 22; /* 4 Mi events = 64 MiB per staging buffer */
+    if (!c->copy_stream) {
+        HR_CUDA(c, cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
+        for (int i = 0; i < 2; i++) {
+            HR_CUDA(c, cudaEventCreateWithFlags(&c->ev_copied[i], cudaEventDisableTiming));
+            HR_CUDA(c, cudaEventCreateWithFlags(&c->ev_used[i], cudaEventDisableTiming));
+        }
+    }
+    const uint64_t need = n < chunk ? (n ? n : 1) : chunk;
+    if (need > c->stage_cap) {
+        for (int i = 0; i < 2; i++) {
+            if (c->d_stage[i])
+                cudaFree(c->d_stage[i]);
+            c->d_stage[i] = nullptr;
+        }
+        c->stage_cap = 0;
+        HR_CUDA(c, cudaMalloc(&c->d_stage[0], need * sizeof(hirace_event)));
+        HR_CUDA(c, cudaMalloc(&c->d_stage[1], need * sizeof(hirace_event)));
+        c->stage_cap = need;
+    }
+    /* the copy stream must not run ahead of work already queued on `st` */
+    HR_CUDA(c, cudaEventRecord(c->ev_used[0], st));
+    HR_CUDA(c, cudaStreamWaitEvent(c->copy_stream, c->ev_used[0], 0));
+    HR_CUDA(c, cudaEventRecord(c->ev_used[1], st));
+    for (uint64_t off = 0, k = 0; off < n; off += chunk, k++) {
+        const int b = (int)(k & 1);
+        const uint64_t m = n - off < chunk ? n - off : chunk;
+        HR_CUDA(c, cudaStreamWaitEvent(c->copy_stream, c->ev_used[b], 0));
+        HR_CUDA(c, cudaMemcpyAsync(c->d_stage[b], h_events + off, m * sizeof(hirace_event), cudaMemcpyHostToDevice,
+                                   c->copy_stream));
+        HR_CUDA(c, cudaEventRecord(c->ev_copied[b], c->copy_stream));
+        HR_CUDA(c, cudaStreamWaitEvent(st, c->ev_copied[b], 0));
+        hirace_status s = hirace_replay_trace(c, c->d_stage[b], m, stream);
+        if (s != HIRACE_OK)
+            return s;
+        HR_CUDA(c, cudaEventRecord(c->ev_used[b], st));
+    }
+    return hirace_collect_races(c, h_out, cap, n_total, stream);
+}
+
+hirace_status hirace_get_stats(hirace_ctx *c, uint64_t *checked, uint64_t *cas_retries, uint64_t *cas_ops,
+                               uint64_t *no_write, uint64_t *dropped_reports)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    HR_CUDA(c, cudaDeviceSynchronize());
+    unsigned long long s[4] = {0, 0, 0, 0}, rc = 0;
+    HR_CUDA(c, cudaMemcpy(s, c->d_stats, sizeof(s), cudaMemcpyDeviceToHost));
+    HR_CUDA(c, cudaMemcpy(&rc, c->d_report_count, sizeof(rc), cudaMemcpyDeviceToHost));
+    if (checked)
+        *checked = s[0];
+    if (cas_retries)
+        *cas_retries = s[1];
+    if (cas_ops)
+        *cas_ops = s[2];
+    if (no_write)
+        *no_write = s[3];
+    if (dropped_reports)
+        *dropped_reports = rc > c->cfg.report_capacity ? rc - c->cfg.report_capacity : 0;
+    device_errors(c);
+    return HIRACE_OK;
+}
+
+hirace_status hirace_sync(hirace_ctx *c)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    HR_CUDA(c, cudaDeviceSynchronize());
+    return device_errors(c);
+}
+
+hirace_status hirace_get_dev_ctx(hirace_ctx *c, const void *global_base, hirace_dev_ctx *out)
+{
+    if (!c || !out)
+        return HIRACE_E_INVAL;
+    *out = c->dev;
+    out->global_base = global_base;
+    out->g = c->g;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_bucket_events(hirace_ctx *c, const hirace_event *d_in, uint64_t n, int nranks, int my_rank,
+                                   hirace_event *d_out, uint64_t *h_counts, void *stream)
+{
+    if (!c || !h_counts || nranks < 1 || nranks > 32 || my_rank < 0 || my_rank >= nranks || n >= 0xffffffffull ||
+        (n && (!d_in || !d_out)))
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    if (n == 0) {
+        for (int r = 0; r < nranks; r++)
+            h_counts[r] = 0;
+        return HIRACE_OK;
+    }
+    const uint32_t ntiles = (uint32_t)((n + 4095) / 4096);
+    const uint64_t need = (uint64_t)ntiles * nranks;
+    if (need > c->bucket_hist_cap) {
+        if (c->d_bucket_hist)
+            cudaFree(c->d_bucket_hist);
+        c->d_bucket_hist = nullptr;
+        c->bucket_hist_cap = 0;
+        HR_CUDA(c, cudaMalloc(&c->d_bucket_hist, need * sizeof(uint32_t)));
+        c->bucket_hist_cap = need;
+    }
+    if (!c->d_bucket_counts)
+        HR_CUDA(c, cudaMalloc(&c->d_bucket_counts, 32 * sizeof(unsigned long long)));
+    HR_CUDA(c, launch_bucket(c->dev, d_in, (uint32_t)n, nranks, my_rank, d_out, c->d_bucket_counts, c->d_bucket_hist,
+                             ntiles, st));
+    unsigned long long tmp[32];
+    HR_CUDA(c, cudaMemcpyAsync(tmp, c->d_bucket_counts, nranks * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+    HR_CUDA(c, cudaStreamSynchronize(st));
+    for (int r = 0; r < nranks; r++)
+        h_counts[r] = tmp[r];
+    return HIRACE_OK;
+}
+
+} /* extern "C" */

@@ -1,0 +1,259 @@
+"""Thin ctypes binding over libhirace.so (include/hirace.h).  Argument marshalling only:
+every step of the hot path runs in the library's sm_100a kernels.  PyTorch provides device
+memory and streams.  There is no CPU fallback: if the library or a CUDA device is missing,
+every call raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+SO_PATH = os.path.join(_PKG, "lib", "libhirace.so")
+
+EVENT_DTYPE = np.dtype([("addr", "<u8"), ("tid", "<u4"), ("meta", "<u4")])
+RACE_DTYPE = np.dtype([("key", "<u8"), ("cls_and_epoch", "<u4"), ("detect_tid", "<u4")])
+
+READ, WRITE, ATOMIC_BLOCK, ATOMIC_GRID = 0, 1, 2, 3
+SCOPE_WARP, SCOPE_BLOCK, SCOPE_GRID = 1, 2, 3
+RACE_WARP, RACE_BLOCK, RACE_GRID = 1, 2, 3
+MAX_BATCHES = 32767
+
+STATUS = {0: "HIRACE_OK", -1: "HIRACE_E_INVAL", -2: "HIRACE_E_NOMEM", -3: "HIRACE_E_CUDA",
+          -4: "HIRACE_E_CLOCK_OVERFLOW", -5: "HIRACE_E_REPORT_OVERFLOW", -6: "HIRACE_E_BAD_TRACE",
+          -7: "HIRACE_E_COMM"}
+
+# every symbol include/hirace.h declares (checked by tests/test_abi.py against the header)
+EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_free", "hirace_shadow_reset", "hirace_barrier",
+           "hirace_replay_trace", "hirace_check_trace_host", "hirace_collect_races",
+           "hirace_collect_races_device", "hirace_get_stats", "hirace_sync", "hirace_get_dev_ctx",
+           "hirace_bucket_events", "hirace_set_kernel_timing", "hirace_fsm_table", "hirace_fsm_step", "hirace_status_string",
+           "hirace_version")
+
+
+class HiraceError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        super().__init__(f"{where}: {STATUS.get(status, status)}")
+
+
+class Config(ctypes.Structure):
+    _fields_ = [("grid_blocks", ctypes.c_uint32), ("block_threads", ctypes.c_uint32),
+                ("warp_size", ctypes.c_uint32), ("smem_bytes_per_block", ctypes.c_uint32),
+                ("global_bytes", ctypes.c_uint64), ("granularity_log2", ctypes.c_uint32),
+                ("device", ctypes.c_int32), ("report_capacity", ctypes.c_uint64)]
+
+
+class DevCtx(ctypes.Structure):
+    _fields_ = [("shadow", ctypes.c_void_p), ("table", ctypes.c_void_p), ("reports", ctypes.c_void_p),
+                ("report_count", ctypes.c_void_p), ("stats", ctypes.c_void_p),
+                ("error_flags", ctypes.c_void_p), ("report_capacity", ctypes.c_uint64),
+                ("global_words", ctypes.c_uint64), ("global_base", ctypes.c_void_p),
+                ("smem_words", ctypes.c_uint32), ("grid_blocks", ctypes.c_uint32),
+                ("block_threads", ctypes.c_uint32), ("warp_size", ctypes.c_uint32),
+                ("bt_magic", ctypes.c_uint32), ("bt_s1", ctypes.c_uint32), ("bt_s2", ctypes.c_uint32),
+                ("ws_magic", ctypes.c_uint32), ("ws_s1", ctypes.c_uint32), ("ws_s2", ctypes.c_uint32),
+                ("g", ctypes.c_uint32)]
+
+
+_lib = None
+
+
+def load():
+    """Loads the in-tree library; raises if it was not built (no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(SO_PATH):
+        raise RuntimeError(f"{SO_PATH} missing: build it with `python -m paper_conf_sc_jacobsonbg24_b200.build` "
+                           "(the CUDA path has no fallback)")
+    lib = ctypes.CDLL(SO_PATH)
+    P, U64, U32, I32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int
+    sig = {
+        "hirace_shadow_alloc": (I32, [ctypes.POINTER(Config), ctypes.POINTER(P)]),
+        "hirace_shadow_free": (I32, [P]),
+        "hirace_shadow_reset": (I32, [P, P]),
+        "hirace_barrier": (I32, [P, I32, P]),
+        "hirace_replay_trace": (I32, [P, P, U64, P]),
+        "hirace_check_trace_host": (I32, [P, P, U64, P, U64, ctypes.POINTER(U64), P]),
+        "hirace_collect_races": (I32, [P, P, U64, ctypes.POINTER(U64), P]),
+        "hirace_collect_races_device": (I32, [P, P, U64, P, P]),
+        "hirace_get_stats": (I32, [P] + [ctypes.POINTER(U64)] * 5),
+        "hirace_sync": (I32, [P]),
+        "hirace_get_dev_ctx": (I32, [P, P, ctypes.POINTER(DevCtx)]),
+        "hirace_bucket_events": (I32, [P, P, U64, I32, I32, P, ctypes.POINTER(U64), P]),
+        "hirace_set_kernel_timing": (I32, [P, P, P]),
+        "hirace_fsm_table": (I32, [P]),
+        "hirace_fsm_step": (U64, [U64, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
+        "hirace_status_string": (ctypes.c_char_p, [I32]),
+        "hirace_version": (ctypes.c_char_p, []),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(lib, name)
+        f.restype, f.argtypes = res, args
+    _lib = lib
+    return lib
+
+
+def _check(st: int, where: str):
+    if st != 0:
+        raise HiraceError(st, where)
+
+
+def fsm_table() -> np.ndarray:
+    t = np.zeros(2048, np.uint8)
+    _check(load().hirace_fsm_table(t.ctypes.data), "hirace_fsm_table")
+    return t
+
+
+def fsm_step(old: int, tid: int, kind: int, g: int, b: int, w: int, block_threads: int, warp_size: int):
+    rep = ctypes.c_int(0)
+    n = load().hirace_fsm_step(old, tid, kind, g, b, w, block_threads, warp_size, ctypes.byref(rep))
+    return int(n), int(rep.value)
+
+
+def _stream_handle(stream):
+    if stream is None:
+        import torch
+        return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, int):
+        return ctypes.c_void_p(stream)
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def events_to_device(events: np.ndarray, device="cuda"):
+    """Copies an EVENT_DTYPE array into a CUDA uint8 tensor (16 bytes per event)."""
+    import torch
+    ev = np.ascontiguousarray(events)
+    assert ev.dtype == EVENT_DTYPE
+    return torch.from_numpy(ev.view(np.uint8).reshape(-1)).to(device)
+
+
+class Checker:
+    """One hirace_ctx: shadow (8 B per tracked 4-byte word), FSM table, report buffer."""
+
+    def __init__(self, grid_blocks: int, block_threads: int, warp_size: int = 32, global_words: int = 0,
+                 smem_words: int = 0, report_capacity: int = 0, device: int = 0):
+        self.lib = load()
+        cfg = Config(grid_blocks, block_threads, warp_size, 4 * smem_words, 4 * global_words, 2, device,
+                     report_capacity)
+        h = ctypes.c_void_p()
+        _check(self.lib.hirace_shadow_alloc(ctypes.byref(cfg), ctypes.byref(h)), "hirace_shadow_alloc")
+        self.h = h
+        self.geometry = dict(grid_blocks=grid_blocks, block_threads=block_threads, warp_size=warp_size,
+                             global_words=global_words, smem_words=smem_words)
+        self.device = device
+
+    @classmethod
+    def for_trace(cls, trace, report_capacity: int = 0, device: int = 0):
+        return cls(trace.grid_blocks, trace.block_threads, trace.warp_size, trace.global_words, trace.smem_words,
+                   report_capacity, device)
+
+    @property
+    def shadow_bytes(self) -> int:
+        g = self.geometry
+        return 8 * (g["global_words"] + g["grid_blocks"] * g["smem_words"])
+
+    def close(self):
+        if getattr(self, "h", None):
+            self.lib.hirace_shadow_free(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def reset(self, stream=None):
+        _check(self.lib.hirace_shadow_reset(self.h, _stream_handle(stream)), "hirace_shadow_reset")
+
+    def barrier(self, scope=SCOPE_GRID, stream=None):
+        _check(self.lib.hirace_barrier(self.h, scope, _stream_handle(stream)), "hirace_barrier")
+
+    def replay(self, events_dev, n: int | None = None, stream=None):
+        """events_dev: CUDA tensor holding 16-byte events (uint8 [16n] or int64 [n,2])."""
+        nbytes = events_dev.numel() * events_dev.element_size()
+        if n is None:
+            n = nbytes // 16
+        _check(self.lib.hirace_replay_trace(self.h, ctypes.c_void_p(events_dev.data_ptr()), n,
+                                            _stream_handle(stream)), "hirace_replay_trace")
+
+    def replay_ptr(self, ptr: int, n: int, stream=None):
+        _check(self.lib.hirace_replay_trace(self.h, ctypes.c_void_p(ptr), n, _stream_handle(stream)),
+               "hirace_replay_trace")
+
+    def collect(self, cap: int | None = None, stream=None) -> np.ndarray:
+        """Flagged words sorted by key (RACE_DTYPE).  Raises on a sticky error."""
+        total = ctypes.c_uint64(0)
+        cap = 1 << 16 if cap is None else cap
+        while True:
+            out = np.empty(max(cap, 1), RACE_DTYPE)
+            st = self.lib.hirace_collect_races(self.h, out.ctypes.data, cap, ctypes.byref(total),
+                                               _stream_handle(stream))
+            _check(st, "hirace_collect_races")
+            if total.value <= cap:
+                return out[: total.value]
+            cap = int(total.value)
+
+    def collect_device(self, out_dev, cap: int, total_dev, stream=None):
+        _check(self.lib.hirace_collect_races_device(self.h, ctypes.c_void_p(out_dev.data_ptr()), cap,
+                                                    ctypes.c_void_p(total_dev.data_ptr()),
+                                                    _stream_handle(stream)), "hirace_collect_races_device")
+
+    def check_host(self, events: np.ndarray, cap: int | None = None, stream=None) -> np.ndarray:
+        """End-to-end from HOST events: H2D (chunked, overlapped) + replay + collect + D2H."""
+        ev = np.ascontiguousarray(events)
+        cap = max(1 << 16, 0) if cap is None else cap
+        total = ctypes.c_uint64(0)
+        while True:
+            out = np.empty(max(cap, 1), RACE_DTYPE)
+            st = self.lib.hirace_check_trace_host(self.h, ev.ctypes.data, ev.shape[0], out.ctypes.data, cap,
+                                                  ctypes.byref(total), _stream_handle(stream))
+            _check(st, "hirace_check_trace_host")
+            if total.value <= cap:
+                return out[: total.value]
+            cap = int(total.value)
+            self.reset(stream)
+
+    def check_host_ptr(self, ptr: int, n: int, out_ptr: int, cap: int, stream=None) -> int:
+        total = ctypes.c_uint64(0)
+        _check(self.lib.hirace_check_trace_host(self.h, ctypes.c_void_p(ptr), n, ctypes.c_void_p(out_ptr), cap,
+                                                ctypes.byref(total), _stream_handle(stream)),
+               "hirace_check_trace_host")
+        return int(total.value)
+
+    def set_kernel_timing(self, start=None, stop=None):
+        """torch.cuda.Event pair (already recorded once) or None: times the replay kernel."""
+        a = ctypes.c_void_p(start.cuda_event if start is not None else 0)
+        b = ctypes.c_void_p(stop.cuda_event if stop is not None else 0)
+        _check(self.lib.hirace_set_kernel_timing(self.h, a, b), "hirace_set_kernel_timing")
+
+    def stats(self) -> dict:
+        v = [ctypes.c_uint64(0) for _ in range(5)]
+        _check(self.lib.hirace_get_stats(self.h, *[ctypes.byref(x) for x in v]), "hirace_get_stats")
+        return dict(checked=v[0].value, cas_retries=v[1].value, cas_ops=v[2].value, no_write=v[3].value,
+                    dropped_reports=v[4].value)
+
+    def sync(self) -> int:
+        return int(self.lib.hirace_sync(self.h))
+
+    def dev_ctx(self, global_base: int = 0) -> DevCtx:
+        d = DevCtx()
+        _check(self.lib.hirace_get_dev_ctx(self.h, ctypes.c_void_p(global_base), ctypes.byref(d)),
+               "hirace_get_dev_ctx")
+        return d
+
+    def bucket(self, events_dev, n: int, nranks: int, my_rank: int, out_dev, stream=None) -> list[int]:
+        counts = (ctypes.c_uint64 * nranks)()
+        _check(self.lib.hirace_bucket_events(self.h, ctypes.c_void_p(events_dev.data_ptr()), n, nranks, my_rank,
+                                             ctypes.c_void_p(out_dev.data_ptr()), counts, _stream_handle(stream)),
+               "hirace_bucket_events")
+        return [int(x) for x in counts]
+
+
+def races_to_dict(races: np.ndarray) -> dict:
+    """{key: class} from collected records."""
+    return {int(k): int(c) & 0xFF for k, c in zip(races["key"], races["cls_and_epoch"])}
