@@ -187,13 +187,14 @@ extern "C" uint64_t hirace_fsm_step(uint64_t old_shadow, uint32_t tid, uint32_t 
         hirace_fsm_table(table);
         built = true;
     }
-    hirace::geom G;
-    G.bt = block_threads ? block_threads : 1;
-    hirace::fastdiv_init(G.bt, &G.bt_m, &G.bt_s1, &G.bt_s2);
-    hirace::fastdiv_init(warp_size ? warp_size : 1, &G.ws_m, &G.ws_s1, &G.ws_s2);
+    hirace_dev_ctx c{};
+    c.block_threads = block_threads ? block_threads : 1;
+    c.warp_size = warp_size ? warp_size : 1;
+    hirace::fastdiv_init(c.block_threads, &c.bt_magic, &c.bt_s1, &c.bt_s2);
+    hirace::fastdiv_init(c.warp_size, &c.ws_magic, &c.ws_s1, &c.ws_s2);
+    const hirace::geom G = hirace::make_geom(c);
     hirace::access a;
     a.tid = tid;
-    hirace::coords(tid, G, &a.block, &a.warp);
     a.kind = kind & 3;
     a.g = g;
     a.b = b;

@@ -166,6 +166,7 @@ hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
         (e = cudaMalloc(&c->scr.raw_count, sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&c->scr.batch_off, (HIRACE_MAX_BATCHES + 1) * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&c->scr.nbatches, sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&c->scr.batch_ctr, HIRACE_MAX_BATCHES * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&c->scr.grid_bar, sizeof(unsigned int))) != cudaSuccess ||
         (e = cudaMalloc(&c->scr.tile_counts, c->scr.ntiles * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&c->d_total, sizeof(unsigned long long))) != cudaSuccess)
@@ -204,7 +205,7 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
     cudaSetDevice(c->device);
     cudaDeviceSynchronize();
     void *ptrs[] = {c->d_shadow, c->d_table, c->d_reports, c->d_report_count, c->d_stats, c->d_err,
-                    c->scr.raw_pos, c->scr.raw_count, c->scr.batch_off, c->scr.nbatches, c->scr.grid_bar,
+                    c->scr.raw_pos, c->scr.raw_count, c->scr.batch_off, c->scr.nbatches, c->scr.batch_ctr, c->scr.grid_bar,
                     c->scr.tile_counts, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
                     c->d_stage[0], c->d_stage[1]};
     for (void *p : ptrs)

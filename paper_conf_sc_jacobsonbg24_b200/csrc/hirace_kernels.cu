@@ -3,12 +3,7 @@
  *
  *   k_find_batches / k_sort_batches  a9  batch discovery + validation (replay input sorted by
  *                                         (g,b,w))
- *   k_replay                          a1-a9 persistent cooperative trace replay: streams events,
- *                                         warp-aggregates same-word accesses (__match_any_sync),
- *                                         folds them through the FSM and commits one CAS per
- *                                         word (Algorithm 1), appends race
- *                                         reports with warp-level compaction, grid barrier
- *                                         between batches
+ *   (k_replay, the a1-a9 hot kernel, lives in replay.cu)
  *   k_collect_*                       a7  order-preserving compaction of RACE records
  *   k_rebase                          a8  grid-epoch wrap sweep
  *   k_bucket_*                        a10 owner bucketing for the address-sharded mode
@@ -18,51 +13,11 @@
 
 #include "hirace_device.cuh"
 #include "internal.h"
+#include "kernel_common.cuh"
 
 namespace hirace_impl {
 
 using namespace hirace;
-
-/* ---------------------------------------------------------------------------------------- */
-/* small helpers                                                                             */
-/* ---------------------------------------------------------------------------------------- */
-
-__device__ __forceinline__ uint32_t batch_key_at(const hirace_event *ev, uint32_t p)
-{
-    return __ldg(&ev[p].meta) >> 5;
-}
-
-__device__ __forceinline__ void ld_event_stream(const hirace_event *p, uint64_t &addr, uint32_t &tid, uint32_t &meta)
-{
-    /* events are read exactly once: streaming, no L1 allocation */
-    uint32_t a0, a1, t, m;
-    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
-                 : "=r"(a0), "=r"(a1), "=r"(t), "=r"(m)
-                 : "l"(p));
-    addr = ((uint64_t)a1 << 32) | a0;
-    tid = t;
-    meta = m;
-}
-
-__device__ __forceinline__ void grid_sync(unsigned int *bar, unsigned int nctas, unsigned int &epoch)
-{
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        epoch++;
-        const unsigned int target = epoch * nctas;
-        __threadfence();
-        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(bar) : "memory");
-        unsigned int v;
-        for (;;) {
-            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
-            if (v >= target)
-                break;
-            __nanosleep(20);
-        }
-        __threadfence();
-    }
-    __syncthreads();
-}
 
 /* ---------------------------------------------------------------------------------------- */
 /* a9: batch discovery.  Boundaries = {p : key(p) != key(p-1)}.  A chunk [lo,hi) can hold a  */
@@ -137,7 +92,8 @@ __global__ void __launch_bounds__(kFindWarps * 32) k_find_batches(const hirace_e
 /* check that batch keys strictly increase                                                   */
 __global__ void __launch_bounds__(1024) k_sort_batches(const hirace_event *__restrict__ ev, uint32_t n,
                                                        const uint32_t *raw, const uint32_t *raw_count,
-                                                       uint32_t *off, uint32_t *nbatches, unsigned int *err)
+                                                       uint32_t *off, uint32_t *nbatches, uint32_t *batch_ctr,
+                                                       unsigned int *err)
 {
     extern __shared__ uint32_t s[];
     const uint32_t found = *raw_count;
@@ -180,6 +136,7 @@ __global__ void __launch_bounds__(1024) k_sort_batches(const hirace_event *__res
     }
     for (uint32_t i = threadIdx.x; i < nb; i += blockDim.x) {
         off[i] = s[i];
+        batch_ctr[i] = 0; /* tile-claim counters of the replay kernel */
         if (i > 0 && !(batch_key_at(ev, s[i]) > batch_key_at(ev, s[i - 1])))
             atomicOr(err, ERR_BAD_TRACE);
     }
@@ -203,196 +160,8 @@ cudaError_t launch_find_batches(const hirace_event *ev, uint32_t n, const Scratc
     }
     /* dynamic smem sized for the worst case; the kernel uses next_pow2(nb) of it */
     k_sort_batches<<<1, 1024, 32768 * sizeof(uint32_t), st>>>(ev, n, s.raw_pos, s.raw_count, s.batch_off,
-                                                              s.nbatches, err);
+                                                              s.nbatches, s.batch_ctr, err);
     return cudaGetLastError();
-}
-
-/* ---------------------------------------------------------------------------------------- */
-/* a1-a9: the replay kernel                                                                  */
-/* ---------------------------------------------------------------------------------------- */
-
-struct lane_acc {
-    uint32_t tid, block, warp, kind;
-};
-
-constexpr int kReplayWarps = kReplayThreads / 32;
-
-__global__ void __launch_bounds__(kReplayThreads) k_replay(hirace_dev_ctx c, const hirace_event *__restrict__ ev,
-                                                           const uint32_t *__restrict__ off,
-                                                           const uint32_t *__restrict__ nbp, unsigned int *bar)
-{
-    __shared__ __align__(16) unsigned char s_table[2048];
-    __shared__ lane_acc s_acc[kReplayWarps][32];
-    __shared__ unsigned long long s_stats[4];
-
-    const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    for (int i = threadIdx.x; i < 2048 / 16; i += blockDim.x)
-        reinterpret_cast<uint4 *>(s_table)[i] = __ldg(reinterpret_cast<const uint4 *>(c.table) + i);
-    if (threadIdx.x < 4)
-        s_stats[threadIdx.x] = 0;
-    __syncthreads();
-
-    const geom G = make_geom(c);
-    const uint32_t nb = *nbp;
-    const uint64_t total_threads = (uint64_t)c.grid_blocks * c.block_threads;
-    const uint32_t warp_global = blockIdx.x * kReplayWarps + wid;
-    const uint32_t nwarps = gridDim.x * kReplayWarps;
-    unsigned int bar_epoch = 0;
-    unsigned long long n_checked = 0, n_retry = 0, n_cas = 0, n_nowrite = 0;
-    unsigned int bad = 0;
-
-    for (uint32_t bi = 0; bi < nb; bi++) {
-        const uint32_t start = __ldg(&off[bi]), end = __ldg(&off[bi + 1]);
-        const uint32_t bkey = batch_key_at(ev, start);
-        const uint32_t bg = bkey >> 19, bb = (bkey >> 9) & 1023u, bw = bkey & 511u;
-        if (bg == 255u)
-            bad = 1; /* g = 255 is reserved for retired RACE records (R7) */
-
-        for (uint64_t base = (uint64_t)start + (uint64_t)warp_global * 32; base < end; base += (uint64_t)nwarps * 32) {
-            const uint64_t i = base + lane;
-            bool valid = i < end;
-            uint64_t idx = 0, keyhi = 0, word = 0;
-            uint32_t nw = 0;
-            lane_acc a{0, 0, 0, 0};
-            if (valid) {
-                uint64_t addr;
-                uint32_t tid, meta;
-                ld_event_stream(ev + i, addr, tid, meta);
-                const uint32_t szl = (meta >> 2) & 7u;
-                nw = szl <= 2 ? 1u : (1u << (szl - 2));
-                word = (addr & ~HIRACE_SHARED_BIT) >> 2;
-                bool ok = (meta >> 5) == bkey && tid < total_threads && szl <= 4;
-                if (ok) {
-                    coords(tid, G, &a.block, &a.warp);
-                    a.tid = tid;
-                    a.kind = meta & 3u;
-                    if (addr & HIRACE_SHARED_BIT) {
-                        ok = word + nw <= c.smem_words;
-                        idx = c.global_words + (uint64_t)a.block * c.smem_words + word;
-                        keyhi = HIRACE_SHARED_BIT | ((uint64_t)a.block << 32);
-                    } else {
-                        ok = word + nw <= c.global_words;
-                        idx = word;
-                    }
-                }
-                if (!ok) {
-                    bad = 1;
-                    valid = false;
-                    nw = 0;
-                }
-            }
-            s_acc[wid][lane] = a;
-            __syncwarp();
-            const uint32_t maxnw = __reduce_max_sync(0xffffffffu, nw);
-            for (uint32_t k = 0; k < maxnw; k++) {
-                const bool act = k < nw;
-                const uint64_t myidx = act ? idx + k : ~0ull;
-                const uint32_t peers = __match_any_sync(0xffffffffu, myidx);
-                const bool leader = act && (__ffs(peers) - 1) == (int)lane;
-                uint32_t rep_cls = 0, rep_tid = 0;
-                n_checked += act ? 1 : 0;
-                if (leader) {
-                    unsigned long long *p = c.shadow + myidx;
-                    uint64_t o = ld_coherent(p);
-                    for (;;) {
-                        uint64_t nsh = o;
-                        uint32_t rep = 0, rtid = 0;
-                        for (uint32_t m = peers; m; m &= m - 1) {
-                            const lane_acc &q = s_acc[wid][__ffs(m) - 1];
-                            access x{q.tid, q.block, q.warp, q.kind, bg, bb, bw};
-                            uint32_t r1 = 0;
-                            nsh = step(nsh, x, s_table, G, &r1);
-                            if (r1) {
-                                rep = 1;
-                                rtid = q.tid;
-                            }
-                        }
-                        if (nsh == o) {
-                            n_nowrite++;
-                            break;
-                        }
-                        n_cas++;
-                        const uint64_t prev = cas64(p, o, nsh);
-                        if (prev == o) {
-                            const uint32_t cn = race_class(st_of(nsh)), co = race_class(st_of(o));
-                            if (rep && cn > co) {
-                                rep_cls = cn;
-                                rep_tid = rtid;
-                            }
-                            break;
-                        }
-                        o = prev;
-                        n_retry++;
-                    }
-                }
-                /* a7: warp-compacted report append */
-                const uint32_t rmask = __ballot_sync(0xffffffffu, rep_cls != 0);
-                if (rmask) {
-                    unsigned long long basepos = 0;
-                    const int first = __ffs(rmask) - 1;
-                    if ((int)lane == first)
-                        basepos = atomicAdd(c.report_count, (unsigned long long)__popc(rmask));
-                    basepos = __shfl_sync(0xffffffffu, basepos, first);
-                    if (rep_cls) {
-                        const unsigned long long posn = basepos + __popc(rmask & ((1u << lane) - 1));
-                        if (posn < c.report_capacity) {
-                            hirace_race r;
-                            r.key = keyhi | (word + k);
-                            r.cls_and_epoch = rep_cls | (bg << 8);
-                            r.detect_tid = rep_tid;
-                            c.reports[posn] = r;
-                        }
-                    }
-                }
-            }
-            __syncwarp();
-        }
-        if (bi + 1 < nb)
-            grid_sync(bar, gridDim.x, bar_epoch);
-    }
-    if (__any_sync(0xffffffffu, bad) && lane == 0)
-        atomicOr(c.error_flags, ERR_BAD_TRACE);
-    /* stats: warp reduce -> shared -> one global atomic per CTA */
-    for (int o = 16; o > 0; o >>= 1) {
-        n_checked += __shfl_xor_sync(0xffffffffu, n_checked, o);
-        n_retry += __shfl_xor_sync(0xffffffffu, n_retry, o);
-        n_cas += __shfl_xor_sync(0xffffffffu, n_cas, o);
-        n_nowrite += __shfl_xor_sync(0xffffffffu, n_nowrite, o);
-    }
-    if (lane == 0) {
-        atomicAdd(&s_stats[0], n_checked);
-        atomicAdd(&s_stats[1], n_retry);
-        atomicAdd(&s_stats[2], n_cas);
-        atomicAdd(&s_stats[3], n_nowrite);
-    }
-    __syncthreads();
-    if (threadIdx.x < 4 && s_stats[threadIdx.x])
-        atomicAdd(&c.stats[threadIdx.x], s_stats[threadIdx.x]);
-}
-
-int replay_max_grid(int device)
-{
-    int sms = 0, occ = 0;
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_replay, kReplayThreads, 0);
-    if (occ < 1)
-        occ = 1;
-    return sms * occ;
-}
-
-cudaError_t launch_replay(const hirace_dev_ctx &c, const hirace_event *ev, const Scratch &s, int grid,
-                          cudaStream_t st)
-{
-    cudaError_t e = cudaMemsetAsync(s.grid_bar, 0, sizeof(unsigned int), st);
-    if (e != cudaSuccess)
-        return e;
-    hirace_dev_ctx cc = c;
-    const hirace_event *evp = ev;
-    const uint32_t *offp = s.batch_off;
-    const uint32_t *nbp = s.nbatches;
-    unsigned int *barp = s.grid_bar;
-    void *args[] = {&cc, &evp, &offp, &nbp, &barp};
-    return cudaLaunchCooperativeKernel((const void *)k_replay, dim3(grid), dim3(kReplayThreads), args, 0, st);
 }
 
 /* ---------------------------------------------------------------------------------------- */

@@ -9,7 +9,7 @@
 
 namespace hirace_impl {
 
-constexpr int kReplayThreads = 256;
+constexpr int kReplayThreads = 256;  /* 8 warps */
 constexpr int kCollectTile = 4096;     /* shadow words per collect CTA                 */
 constexpr int kCollectThreads = 256;
 constexpr uint32_t kFindChunk = 32768; /* top-level batch-boundary probe chunk (32^3)   */
@@ -19,6 +19,7 @@ struct Scratch {
     uint32_t *raw_count;     /* number found (excluding position 0)                          */
     uint32_t *batch_off;     /* sorted batch offsets [0..nb], HIRACE_MAX_BATCHES + 1         */
     uint32_t *nbatches;      /* nb                                                            */
+    uint32_t *batch_ctr;     /* per-batch tile-claim counters, HIRACE_MAX_BATCHES             */
     unsigned int *grid_bar;  /* grid barrier counter                                          */
     uint32_t *tile_counts;   /* collect: per-tile counts / offsets                           */
     uint64_t ntiles;

@@ -1,0 +1,382 @@
+/*
+ * replay.cu — the hot kernel: persistent, cooperative trace replay through the HiRace FSM
+ * (§8(a) rows a1-a9; Algorithm 1).
+ *
+ * Work layout.  Batches (g,b,w) are processed in order with a grid barrier between them;
+ * inside a batch any order is a linear extension of happens-before.  Each warp
+ * walks the batch in 32-event chunks (grid-stride, one event per lane) and keeps the next
+ * chunk's 16-byte events in flight while it works on the current one (a1).
+ *
+ * Per chunk, the common path is short and branch-free (optimistic concurrency):
+ *   a2  decode: one compare checks batch key + access size, shadow index from the address;
+ *   a4  each lane's coherent 8-byte shadow load (ld.relaxed.gpu: never a stale L1 line);
+ *   a5  relation/sync label by XOR+shift, one lookup in the 2 KB shared-memory table, pack;
+ *   a6  one atom.cas.b64 per changed word; an unchanged record issues no CAS (the access is
+ *       linearised at the load: no-write fast path, e.g. every read of a G_R word).
+ * a3 warp aggregation happens only where it pays: lanes whose CAS lost (typically lanes of
+ * the same warp on the same word) are grouped with __match_any_sync and the group leader folds
+ * all members' accesses in lane order from the record its CAS returned, then commits them with
+ * one CAS (Algorithm 1's retry loop).  Other rare cases also leave the
+ * common path behind warp-uniform votes: 8/16-byte accesses, race reports (a7: warp-compacted
+ * append, one atomicAdd per warp), invalid events.
+ */
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "hirace_device.cuh"
+#include "internal.h"
+#include "kernel_common.cuh"
+
+namespace hirace_impl {
+
+using namespace hirace;
+
+namespace {
+
+constexpr uint32_t FULL = 0xffffffffu;
+constexpr uint64_t NONE = ~0ull;
+constexpr int kMinBlocks = 4; /* 32 warps per SM at <= 64 registers */
+
+struct Batch {
+    uint32_t key, g, b, w, ep; /* ep = epochs in record layout */
+};
+
+struct Counters {
+    uint32_t checked, retry, cas, nowrite; /* per thread; widened at the end */
+};
+
+__device__ __forceinline__ uint32_t lds_u8(uint32_t saddr)
+{
+    uint32_t v;
+    asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(saddr));
+    return v;
+}
+
+__device__ __forceinline__ uint4 ld_event(const uint4 *p)
+{
+    uint4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                 : "l"(p));
+    return v;
+}
+
+/* race key (include/hirace.h) of word k of event e */
+__device__ __forceinline__ uint64_t key_of(const geom &G, const uint4 &e, uint32_t k)
+{
+    const uint64_t addr = ((uint64_t)e.y << 32) | e.x;
+    const uint64_t word = ((addr & ~HIRACE_SHARED_BIT) >> 2) + k;
+    if (addr & HIRACE_SHARED_BIT)
+        return HIRACE_SHARED_BIT | ((uint64_t)block_of(e.z, G) << 32) | word;
+    return word;
+}
+
+/* Fold, for every lane with a non-zero `peers` (a group leader), its group's accesses into
+ * record o in lane order: the same sequence of Algorithm-1 transitions as if their CASes had
+ * won one after another.  Accessors are broadcast by shuffle, so all lanes must call it. */
+__device__ __forceinline__ uint64_t fold_shfl(uint64_t o, uint32_t peers, uint32_t my_tid, uint32_t my_kind,
+                                              const geom &G, const unsigned char *tab, const Batch &B,
+                                              uint32_t &rep, uint32_t &rtid)
+{
+    uint64_t n = o;
+    for (uint32_t uni = __reduce_or_sync(FULL, peers); uni; uni &= uni - 1) {
+        const int m = __ffs(uni) - 1;
+        const uint32_t t = __shfl_sync(FULL, my_tid, m);
+        const uint32_t k = __shfl_sync(FULL, my_kind, m);
+        if ((peers >> m) & 1u) {
+            access a{t, k, B.g, B.b, B.w};
+            uint32_t r = 0;
+            n = step(n, a, tab, G, &r);
+            if (r) {
+                rep = 1;
+                rtid = t;
+            }
+        }
+    }
+    return n;
+}
+
+/* Commit for group leaders (peers != 0 only in leaders) starting from observed records o:
+ * fold, CAS, re-fold on failure until every leader's CAS sticks or the record is unchanged.
+ * Returns the report class for this lane; counts into cnt. */
+__device__ __forceinline__ uint32_t commit_groups(unsigned long long *p, uint64_t o, uint32_t peers, uint32_t tid,
+                                                  uint32_t kind, const geom &G, const unsigned char *tab,
+                                                  const Batch &B, Counters &cnt, uint32_t &rtid, bool first)
+{
+    bool pending = peers != 0;
+    uint32_t cls = 0;
+    while (__any_sync(FULL, pending)) {
+        uint32_t rep = 0, rt = 0;
+        const uint64_t n = fold_shfl(o, pending ? peers : 0u, tid, kind, G, tab, B, rep, rt);
+        if (pending) {
+            if (n == o) {
+                pending = false;
+                cnt.nowrite++;
+            } else {
+                cnt.cas++;
+                cnt.retry += first ? 0u : 1u;
+                const uint64_t prev = cas64(p, o, n);
+                if (prev == o) {
+                    pending = false;
+                    const uint32_t cn = race_class(st_of(n)), co = race_class(st_of(o));
+                    cls = (rep && cn > co) ? cn : 0u;
+                    rtid = rt;
+                } else {
+                    o = prev;
+                }
+            }
+        }
+        first = false;
+    }
+    return cls;
+}
+
+/* a7: warp-compacted report append (one atomicAdd per warp) */
+__device__ __forceinline__ void append_reports(const hirace_dev_ctx &c, uint32_t cls, uint64_t key, uint32_t g,
+                                               uint32_t rtid, uint32_t lane)
+{
+    const uint32_t m = __ballot_sync(FULL, cls != 0);
+    if (!m)
+        return;
+    unsigned long long base = 0;
+    const int first = __ffs(m) - 1;
+    if ((int)lane == first)
+        base = atomicAdd(c.report_count, (unsigned long long)__popc(m));
+    base = __shfl_sync(FULL, base, first);
+    if (cls) {
+        const unsigned long long pos = base + __popc(m & ((1u << lane) - 1));
+        if (pos < c.report_capacity) {
+            hirace_race r;
+            r.key = key;
+            r.cls_and_epoch = cls | (g << 8);
+            r.detect_tid = rtid;
+            c.reports[pos] = r;
+        }
+    }
+}
+
+/* chunks holding 8/16-byte accesses: word by word through the group commit (rare; the configs
+ * emit 4-byte accesses).  `take` marks this lane's event as one to process here. */
+__device__ __noinline__ uint4 chunk_multiword(const hirace_dev_ctx c, const geom G, const unsigned char *tab,
+                                              const Batch B, uint4 e, bool take, uint32_t lane)
+{
+    Counters cnt{0, 0, 0, 0};
+    const uint64_t addr = ((uint64_t)e.y << 32) | e.x;
+    const uint32_t szl = (e.w >> 2) & 7u;
+    const uint32_t nw = szl <= 2 ? 1u : (1u << (szl - 2));
+    const uint64_t word = (addr & ~HIRACE_SHARED_BIT) >> 2;
+    const bool sh = (addr & HIRACE_SHARED_BIT) != 0;
+    const uint64_t base = sh ? c.global_words + (uint64_t)block_of(e.z, G) * c.smem_words + word : word;
+    const uint32_t maxnw = __reduce_max_sync(FULL, take ? nw : 0u);
+    for (uint32_t k = 0; k < maxnw; k++) {
+        const bool act = take && k < nw;
+        const uint64_t my = act ? base + k : NONE;
+        const uint32_t peers = __match_any_sync(FULL, my);
+        cnt.checked += act;
+        const bool lead = act && (peers & ((1u << lane) - 1)) == 0;
+        const uint64_t o = lead ? ld_coherent(c.shadow + my) : 0;
+        uint32_t rtid = 0;
+        const uint32_t cls =
+            commit_groups(c.shadow + my, o, lead ? peers : 0u, e.z, e.w & 3u, G, tab, B, cnt, rtid, true);
+        if (__any_sync(FULL, cls != 0))
+            append_reports(c, cls, key_of(G, e, k), B.g, rtid, lane);
+    }
+    return make_uint4(cnt.checked, cnt.retry, cnt.cas, cnt.nowrite);
+}
+
+/* one lane's decoded access for the pipeline */
+struct Lane {
+    uint64_t idx;
+    uint32_t tid, kind;
+    bool ok;
+};
+
+/* a2: decode + validate one lane's event (sub-word accesses map to their word); 8/16-byte
+ * accesses of the chunk are committed right here, word by word */
+__device__ __forceinline__ Lane decode(const uint4 &e, bool valid, uint32_t keysz, const Batch &B,
+                                       uint64_t total_threads, const hirace_dev_ctx &c, const geom &G,
+                                       const unsigned char *tab, Counters &cnt, uint32_t &bad, uint32_t lane)
+{
+    Lane L;
+    L.tid = e.z;
+    L.kind = e.w & 3u;
+    const uint32_t meta = e.w;
+    const bool sh = (int)e.y < 0;
+    const bool key_ok = (meta >> 2) - keysz <= 2u; /* same batch, size <= 4 bytes */
+    const bool tid_ok = L.tid < total_threads;
+    const uint64_t word = ((uint64_t)(e.y & 0x7fffffffu) << 30) | (e.x >> 2);
+    const bool in_range = sh ? word < c.smem_words : word < c.global_words;
+    L.ok = valid && key_ok && tid_ok && in_range;
+    if (__any_sync(FULL, valid && !L.ok)) {
+        const uint32_t szl = (meta >> 2) & 7u;
+        const bool multi = valid && (meta >> 5) == B.key && (szl == 3 || szl == 4) && tid_ok &&
+                           (sh ? word + (1u << (szl - 2)) <= c.smem_words : word + (1u << (szl - 2)) <= c.global_words);
+        if (valid && !L.ok && !multi)
+            bad = 1;
+        if (__any_sync(FULL, multi)) {
+            const uint4 d = chunk_multiword(c, G, tab, B, e, multi, lane);
+            cnt.checked += d.x;
+            cnt.retry += d.y;
+            cnt.cas += d.z;
+            cnt.nowrite += d.w;
+        }
+    }
+    L.idx = !L.ok ? NONE : (sh ? c.global_words + (uint64_t)block_of(L.tid, G) * c.smem_words + word : word);
+    return L;
+}
+
+/* race key of a decoded lane (include/hirace.h) */
+__device__ __forceinline__ uint64_t key_of_idx(const Lane &L, const hirace_dev_ctx &c, const geom &G)
+{
+    if (L.idx < c.global_words)
+        return L.idx;
+    const uint32_t blk = block_of(L.tid, G);
+    return HIRACE_SHARED_BIT | ((uint64_t)blk << 32) | (L.idx - c.global_words - (uint64_t)blk * c.smem_words);
+}
+
+template <bool P2>
+__global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
+    k_replay(hirace_dev_ctx c, const uint4 *__restrict__ ev, const uint32_t *__restrict__ off,
+             const uint32_t *__restrict__ nbp, unsigned int *bar)
+{
+    __shared__ __align__(16) unsigned char s_table[2048];
+    __shared__ unsigned long long s_stats[4];
+    const uint32_t lane = threadIdx.x & 31;
+    for (int i = threadIdx.x; i < 2048 / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(s_table)[i] = __ldg(reinterpret_cast<const uint4 *>(c.table) + i);
+    if (threadIdx.x < 4)
+        s_stats[threadIdx.x] = 0;
+    __syncthreads();
+
+    geom G = make_geom(c);
+    G.pow2 = P2; /* compile-time geometry mode: shifts (P2) or fast division */
+    const uint32_t nb = *nbp;
+    const uint64_t total_threads = (uint64_t)c.grid_blocks * c.block_threads;
+    const uint32_t below = (1u << lane) - 1;
+    const uint32_t tab_s = smem_u32(s_table);
+    const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t stride = (gridDim.x * blockDim.x) >> 5 << 5; /* events per grid-wide sweep */
+    unsigned int bar_epoch = 0;
+    Counters cnt{0, 0, 0, 0};
+    uint32_t bad = 0;
+
+    /* a1: events of the first chunk of every batch are requested before the barrier that
+     * precedes the batch, so the HBM latency overlaps the barrier */
+    uint32_t bstart = nb ? __ldg(&off[0]) : 0, bend = nb ? __ldg(&off[1]) : 0;
+    uint32_t i = bstart + warp_global * 32 + lane;
+    uint4 e0 = i < bend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
+    uint4 e1 = i + stride < bend ? ld_event(ev + i + stride) : make_uint4(0, 0, 0, 0);
+    for (uint32_t bi = 0; bi < nb; bi++) {
+        const uint32_t end = bend;
+        Batch B;
+        B.key = __ldg(&ev[bstart].w) >> 5;
+        B.g = B.key >> 19;
+        B.b = (B.key >> 9) & 1023u;
+        B.w = B.key & 511u;
+        B.ep = (B.g << SH_G) | (B.b << SH_B) | (B.w << SH_W);
+        const uint32_t keysz = B.key << 3; /* (meta >> 2) - keysz = size_log2 for this batch */
+        if (B.g == 255u)
+            bad = 1; /* reserved for retired RACE records (R7) */
+
+        for (uint32_t base = bstart + warp_global * 32; base < end; base += stride) {
+            const Lane cur = decode(e0, i < end, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+            e0 = e1; /* a1: keep the next chunks' events in flight */
+            e1 = i + 2 * stride < end ? ld_event(ev + i + 2 * stride) : make_uint4(0, 0, 0, 0);
+            i += stride;
+
+            /* a4: optimistic: every lane reads its own word (coherent load); lanes that share
+             * a word are grouped only if their CAS collides (below) */
+            unsigned long long *const p = c.shadow + cur.idx;
+            const uint64_t o = cur.ok ? ld_coherent(p) : 0;
+            cnt.checked += cur.ok;
+
+            /* a5: transition */
+            const access a{cur.tid, cur.kind, B.g, B.b, B.w};
+            const uint32_t ent = lds_u8(tab_s + ((st_of(o) << 6) | label(o, a, G)));
+            const uint64_t n = (ent & E_KEEP) ? ((o & ~(uint64_t)31) | (ent & E_STATE))
+                                              : (((uint64_t)cur.tid << SH_TID) | B.ep | (ent & E_STATE));
+            /* a6: one CAS per changed word; unchanged = linearised at the load */
+            const bool do_cas = cur.ok && n != o;
+            cnt.nowrite += cur.ok && !do_cas;
+            cnt.cas += do_cas;
+            const uint64_t prev = do_cas ? cas64(p, o, n) : o;
+            uint32_t cls = 0, rtid = cur.tid;
+            if (do_cas && prev == o) {
+                const uint32_t cn = race_class(st_of(n)), co = race_class(st_of(o));
+                cls = ((ent & E_REPORT) && cn > co) ? cn : 0u;
+            }
+            const bool failed = do_cas && prev != o;
+            if (__any_sync(FULL, failed)) {
+                /* Algorithm 1's retry for the lanes whose CAS lost: group them by word, the
+                 * group leader folds its members' accesses from the record it observed */
+                const uint32_t peers = __match_any_sync(FULL, failed ? cur.idx : NONE);
+                const bool lead = failed && (peers & below) == 0;
+                cnt.retry += lead;
+                cls |= commit_groups(p, prev, lead ? peers : 0u, cur.tid, cur.kind, G, s_table, B, cnt, rtid, true);
+            }
+            /* a7 */
+            if (__any_sync(FULL, cls != 0))
+                append_reports(c, cls, key_of_idx(cur, c, G), B.g, rtid, lane);
+        }
+        if (bi + 1 < nb) {
+            bstart = __ldg(&off[bi + 1]);
+            bend = __ldg(&off[bi + 2]);
+            i = bstart + warp_global * 32 + lane;
+            e0 = i < bend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
+            e1 = i + stride < bend ? ld_event(ev + i + stride) : make_uint4(0, 0, 0, 0);
+            grid_sync(bar, gridDim.x, bar_epoch);
+        }
+    }
+
+    if (__any_sync(FULL, bad) && lane == 0)
+        atomicOr(c.error_flags, ERR_BAD_TRACE);
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) {
+        cnt.checked += __shfl_xor_sync(FULL, cnt.checked, d);
+        cnt.retry += __shfl_xor_sync(FULL, cnt.retry, d);
+        cnt.cas += __shfl_xor_sync(FULL, cnt.cas, d);
+        cnt.nowrite += __shfl_xor_sync(FULL, cnt.nowrite, d);
+    }
+    if (lane == 0) {
+        atomicAdd(&s_stats[0], (unsigned long long)cnt.checked);
+        atomicAdd(&s_stats[1], (unsigned long long)cnt.retry);
+        atomicAdd(&s_stats[2], (unsigned long long)cnt.cas);
+        atomicAdd(&s_stats[3], (unsigned long long)cnt.nowrite);
+    }
+    __syncthreads();
+    if (threadIdx.x < 4 && s_stats[threadIdx.x])
+        atomicAdd(&c.stats[threadIdx.x], s_stats[threadIdx.x]);
+}
+
+} // namespace
+
+int replay_max_grid(int device)
+{
+    int sms = 0, occ = 0, occ2 = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_replay<true>, kReplayThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_replay<false>, kReplayThreads, 0);
+    occ = occ < occ2 ? occ : occ2;
+    if (occ < 1)
+        occ = 1;
+    return sms * occ;
+}
+
+cudaError_t launch_replay(const hirace_dev_ctx &c, const hirace_event *ev, const Scratch &s, int grid,
+                          cudaStream_t st)
+{
+    cudaError_t e = cudaMemsetAsync(s.grid_bar, 0, sizeof(unsigned int), st);
+    if (e != cudaSuccess)
+        return e;
+    hirace_dev_ctx cc = c;
+    const uint4 *evp = reinterpret_cast<const uint4 *>(ev);
+    const uint32_t *offp = s.batch_off;
+    const uint32_t *nbp = s.nbatches;
+    unsigned int *barp = s.grid_bar;
+    void *args[] = {&cc, &evp, &offp, &nbp, &barp};
+    const bool p2 = (c.block_threads & (c.block_threads - 1)) == 0 && (c.warp_size & (c.warp_size - 1)) == 0;
+    const void *fn = p2 ? (const void *)k_replay<true> : (const void *)k_replay<false>;
+    return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kReplayThreads), args, 0, st);
+}
+
+} // namespace hirace_impl
