@@ -4,8 +4,8 @@
  *
  * Work layout.  Batches (g,b,w) are processed in order with a grid barrier between them;
  * inside a batch any order is a linear extension of happens-before.  Each warp
- * walks the batch in 32-event chunks (grid-stride, one event per lane) and keeps the next
- * chunk's 16-byte events in flight while it works on the current one (a1).
+ * owns a contiguous, balanced share of the batch and walks it in 32-event chunks (one event
+ * per lane), keeping the next two chunks' 16-byte events in flight (a1).
  *
  * Per chunk, the common path is short and branch-free (optimistic concurrency):
  *   a2  decode: one compare checks batch key + access size, shadow index from the address;
@@ -184,7 +184,21 @@ __device__ __noinline__ uint4 chunk_multiword(const hirace_dev_ctx c, const geom
     return make_uint4(cnt.checked, cnt.retry, cnt.cas, cnt.nowrite);
 }
 
-/* one lane's decoded access for the pipeline */
+/* Contiguous, balanced share of a batch [bstart, bend) for warp w of nw: whole 32-event
+ * chunks [c0, c1).  Consecutive chunks of a batch are usually consecutive instructions of the
+ * same traced warp and touch the same words; giving them to one replay warp processes them in
+ * sequence instead of racing their CASes (grid-stride would run them concurrently). */
+__device__ __forceinline__ void warp_share(uint32_t bstart, uint32_t bend, uint32_t w, uint32_t nw, uint32_t lane,
+                                           uint32_t &i, uint32_t &iend)
+{
+    const uint32_t nchunks = (bend - bstart + 31) / 32;
+    const uint32_t c0 = (uint32_t)(((uint64_t)nchunks * w) / nw);
+    const uint32_t c1 = (uint32_t)(((uint64_t)nchunks * (w + 1)) / nw);
+    i = bstart + c0 * 32 + lane;
+    iend = min(bend, bstart + c1 * 32);
+}
+
+/* one lane's decoded access */
 struct Lane {
     uint64_t idx;
     uint32_t tid, kind;
@@ -255,7 +269,7 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     const uint32_t below = (1u << lane) - 1;
     const uint32_t tab_s = smem_u32(s_table);
     const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint32_t stride = (gridDim.x * blockDim.x) >> 5 << 5; /* events per grid-wide sweep */
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
     unsigned int bar_epoch = 0;
     Counters cnt{0, 0, 0, 0};
     uint32_t bad = 0;
@@ -263,11 +277,11 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     /* a1: events of the first chunk of every batch are requested before the barrier that
      * precedes the batch, so the HBM latency overlaps the barrier */
     uint32_t bstart = nb ? __ldg(&off[0]) : 0, bend = nb ? __ldg(&off[1]) : 0;
-    uint32_t i = bstart + warp_global * 32 + lane;
-    uint4 e0 = i < bend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
-    uint4 e1 = i + stride < bend ? ld_event(ev + i + stride) : make_uint4(0, 0, 0, 0);
+    uint32_t i, iend; /* this warp's contiguous share of the batch: events [i - lane, iend) */
+    warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
+    uint4 e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
+    uint4 e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
     for (uint32_t bi = 0; bi < nb; bi++) {
-        const uint32_t end = bend;
         Batch B;
         B.key = __ldg(&ev[bstart].w) >> 5;
         B.g = B.key >> 19;
@@ -278,11 +292,10 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
         if (B.g == 255u)
             bad = 1; /* reserved for retired RACE records (R7) */
 
-        for (uint32_t base = bstart + warp_global * 32; base < end; base += stride) {
-            const Lane cur = decode(e0, i < end, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+        for (; i - lane < iend; i += 32) {
+            const Lane cur = decode(e0, i < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
             e0 = e1; /* a1: keep the next chunks' events in flight */
-            e1 = i + 2 * stride < end ? ld_event(ev + i + 2 * stride) : make_uint4(0, 0, 0, 0);
-            i += stride;
+            e1 = i + 64 < iend ? ld_event(ev + i + 64) : make_uint4(0, 0, 0, 0);
 
             /* a4: optimistic: every lane reads its own word (coherent load); lanes that share
              * a word are grouped only if their CAS collides (below) */
@@ -321,9 +334,9 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
         if (bi + 1 < nb) {
             bstart = __ldg(&off[bi + 1]);
             bend = __ldg(&off[bi + 2]);
-            i = bstart + warp_global * 32 + lane;
-            e0 = i < bend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
-            e1 = i + stride < bend ? ld_event(ev + i + stride) : make_uint4(0, 0, 0, 0);
+            warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
+            e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
+            e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
             grid_sync(bar, gridDim.x, bar_epoch);
         }
     }

@@ -11,7 +11,7 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(_PKG, "lib", "libhirace.so")
+SO_PATH = os.environ.get("HIRACE_LIB") or os.path.join(_PKG, "lib", "libhirace.so")  # override: A/B builds
 
 EVENT_DTYPE = np.dtype([("addr", "<u8"), ("tid", "<u4"), ("meta", "<u4")])
 RACE_DTYPE = np.dtype([("key", "<u8"), ("cls_and_epoch", "<u4"), ("detect_tid", "<u4")])
