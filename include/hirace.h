@@ -156,6 +156,14 @@ hirace_status hirace_barrier(hirace_ctx *ctx, hirace_scope scope, void *stream);
  * the same linearisation.  Async on `stream`. */
 hirace_status hirace_replay_trace(hirace_ctx *ctx, const hirace_event *d_events, uint64_t n, void *stream);
 
+/* hirace_replay_trace + hirace_collect_races_device fused into one persistent kernel: the
+ * collection runs as a final grid-wide phase of the replay kernel (no extra launches).  Writes
+ * min(cap, total) unique key-sorted records to DEVICE d_out and the total to DEVICE
+ * *d_n_total.  Async on `stream`.  Kernel-detected errors surface at the next sync. */
+hirace_status hirace_check_trace_device(hirace_ctx *ctx, const hirace_event *d_events, uint64_t n,
+                                        hirace_race *d_out, uint64_t cap, unsigned long long *d_n_total,
+                                        void *stream);
+
 /* Same work from HOST events (pinned or pageable): copies through a device staging ring in
  * chunks, overlapping H2D with replay, then collects like hirace_collect_races.  Synchronous.
  * This is the end-to-end entry point. */
@@ -203,6 +211,18 @@ hirace_status hirace_set_kernel_timing(hirace_ctx *ctx, void *start_event, void 
  * Synchronises `stream` (the counts are needed to size the exchange). */
 hirace_status hirace_bucket_events(hirace_ctx *ctx, const hirace_event *d_in, uint64_t n, int nranks, int my_rank,
                                    hirace_event *d_out, uint64_t *h_counts, void *stream);
+
+/* ---- microbenchmarks for the roofline (diagnostics; not part of the checking path) -------- */
+
+/* Rate of 64-bit operations on `nwords` distinct words of a fresh device array (nwords*8 bytes;
+ * <= ~64 MiB stays L2-resident), coalesced (random = 0) or uniformly random (random = 1).
+ * op: 0 atomicCAS, 1 atomicAdd, 2 coherent load (ld.relaxed.gpu), 3 load + CAS pair.
+ * Writes operations per second to *ops_per_s.  Synchronous. */
+hirace_status hirace_microbench_atomics(int device, uint64_t nwords, int random, int op, uint64_t nops,
+                                        double *ops_per_s, void *stream);
+
+/* Cost of one grid barrier of the persistent replay kernel (its grid size), microseconds. */
+hirace_status hirace_microbench_grid_sync(int device, int iters, double *us_per_barrier, void *stream);
 
 /* ---- verification hooks (host-only, NOT a replay path) --------------------------------- */
 

@@ -155,20 +155,19 @@ hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
         hirace_shadow_free(c);
         return HIRACE_E_INVAL;
     }
-    c->scr.ntiles = (c->shadow_words + kCollectTile - 1) / kCollectTile;
+    c->scr.collect_grid = collect_max_grid(c->device);
     if ((e = cudaMalloc(&c->d_shadow, c->shadow_words * 8)) != cudaSuccess ||
         (e = cudaMalloc(&c->d_table, 2048)) != cudaSuccess ||
         (e = cudaMalloc(&c->d_reports, c->cfg.report_capacity * sizeof(hirace_race))) != cudaSuccess ||
         (e = cudaMalloc(&c->d_report_count, sizeof(unsigned long long))) != cudaSuccess ||
         (e = cudaMalloc(&c->d_stats, 4 * sizeof(unsigned long long))) != cudaSuccess ||
         (e = cudaMalloc(&c->d_err, sizeof(unsigned int))) != cudaSuccess ||
-        (e = cudaMalloc(&c->scr.raw_pos, HIRACE_MAX_BATCHES * sizeof(uint32_t))) != cudaSuccess ||
-        (e = cudaMalloc(&c->scr.raw_count, sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&c->scr.batch_off, (HIRACE_MAX_BATCHES + 1) * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&c->scr.nbatches, sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&c->scr.batch_ctr, HIRACE_MAX_BATCHES * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&c->scr.grid_bar, sizeof(unsigned int))) != cudaSuccess ||
-        (e = cudaMalloc(&c->scr.tile_counts, c->scr.ntiles * sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&c->scr.grid_bar2, sizeof(unsigned int))) != cudaSuccess ||
+        (e = cudaMalloc(&c->scr.cta_cnt, kMaxCtas * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&c->d_total, sizeof(unsigned long long))) != cudaSuccess)
         return fail(e);
     if ((e = cudaMemcpy(c->d_table, table, 2048, cudaMemcpyHostToDevice)) != cudaSuccess)
@@ -205,8 +204,8 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
     cudaSetDevice(c->device);
     cudaDeviceSynchronize();
     void *ptrs[] = {c->d_shadow, c->d_table, c->d_reports, c->d_report_count, c->d_stats, c->d_err,
-                    c->scr.raw_pos, c->scr.raw_count, c->scr.batch_off, c->scr.nbatches, c->scr.batch_ctr, c->scr.grid_bar,
-                    c->scr.tile_counts, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
+                    c->scr.batch_off, c->scr.nbatches, c->scr.batch_ctr, c->scr.grid_bar,
+                    c->scr.grid_bar2, c->scr.cta_cnt, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
                     c->d_stage[0], c->d_stage[1]};
     for (void *p : ptrs)
         if (p)
@@ -285,6 +284,28 @@ hirace_status hirace_set_kernel_timing(hirace_ctx *c, void *start_event, void *s
         return HIRACE_E_INVAL;
     c->t_start = (cudaEvent_t)start_event;
     c->t_stop = (cudaEvent_t)stop_event;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_events, uint64_t n, hirace_race *d_out,
+                                        uint64_t cap, unsigned long long *d_n_total, void *stream)
+{
+    if (!c || !d_n_total || (cap && !d_out))
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    if (n >= 0xffffffffull || (n && !d_events))
+        return set_sticky(c, HIRACE_E_INVAL);
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    if (n == 0)
+        return hirace_collect_races_device(c, d_out, cap, d_n_total, stream);
+    HR_CUDA(c, launch_find_batches(d_events, (uint32_t)n, c->scr, c->d_err, c->sm_count, st));
+    if (c->t_start)
+        HR_CUDA(c, cudaEventRecord(c->t_start, st));
+    HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st, c->shadow_words, d_out, cap, d_n_total));
+    if (c->t_stop)
+        HR_CUDA(c, cudaEventRecord(c->t_stop, st));
     return HIRACE_OK;
 }
 

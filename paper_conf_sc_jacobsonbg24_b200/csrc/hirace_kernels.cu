@@ -1,10 +1,10 @@
 /*
  * hirace_kernels.cu — sm_100a kernels of the HiRace hot path.
  *
- *   k_find_batches / k_sort_batches  a9  batch discovery + validation (replay input sorted by
- *                                         (g,b,w))
+ *   k_batches                         a9  batch discovery + validation (replay input sorted by
+ *                                         (g,b,w)), one CTA
  *   (k_replay, the a1-a9 hot kernel, lives in replay.cu)
- *   k_collect_*                       a7  order-preserving compaction of RACE records
+ *   k_collect                         a7  order-preserving compaction of RACE records (collect.cuh)
  *   k_rebase                          a8  grid-epoch wrap sweep
  *   k_bucket_*                        a10 owner bucketing for the address-sharded mode
  */
@@ -13,6 +13,7 @@
 
 #include "hirace_device.cuh"
 #include "internal.h"
+#include "collect.cuh"
 #include "kernel_common.cuh"
 
 namespace hirace_impl {
@@ -27,7 +28,8 @@ using namespace hirace;
 /* flags HIRACE_E_BAD_TRACE, so validation is complete without a second full read.          */
 /* ---------------------------------------------------------------------------------------- */
 
-constexpr int kFindWarps = 8;
+constexpr int kFindThreads = 1024;
+constexpr int kFindWarps = kFindThreads / 32;
 constexpr int kFindStack = 160;
 
 __device__ __forceinline__ bool chunk_dirty(const hirace_event *ev, uint32_t lo, uint32_t hi)
@@ -38,65 +40,28 @@ __device__ __forceinline__ bool chunk_dirty(const hirace_event *ev, uint32_t lo,
     return batch_key_at(ev, q - 1) != batch_key_at(ev, hi - 1);
 }
 
-__global__ void __launch_bounds__(kFindWarps * 32) k_find_batches(const hirace_event *__restrict__ ev, uint32_t n,
-                                                                  uint32_t *pos, uint32_t *count, uint32_t cap)
-{
-    __shared__ uint32_t s_lo[kFindWarps][kFindStack];
-    __shared__ uint32_t s_len[kFindWarps][kFindStack];
-    const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const uint32_t wg = blockIdx.x * kFindWarps + wid, nwarps = gridDim.x * kFindWarps;
-    for (uint64_t t = wg; t * kFindChunk < n; t += nwarps) {
-        uint32_t lo = (uint32_t)(t * kFindChunk);
-        uint32_t len = min(kFindChunk, n - lo);
-        int sp = 0;
-        bool d = lane == 0 && chunk_dirty(ev, lo, lo + len);
-        if (__shfl_sync(0xffffffffu, d ? 1 : 0, 0)) {
-            if (lane == 0) {
-                s_lo[wid][0] = lo;
-                s_len[wid][0] = len;
-            }
-            sp = 1;
-        }
-        __syncwarp();
-        while (sp > 0) {
-            sp--;
-            uint32_t clo = s_lo[wid][sp], clen = s_len[wid][sp];
-            __syncwarp();
-            if (clen <= 32) {
-                uint32_t p = clo + lane;
-                bool b = lane < clen && p >= 1 && batch_key_at(ev, p) != batch_key_at(ev, p - 1);
-                if (b) {
-                    uint32_t i = atomicAdd(count, 1u);
-                    if (i < cap)
-                        pos[i] = p;
-                }
-            } else {
-                uint32_t sub = (clen + 31) / 32;
-                uint32_t slo = clo + lane * sub;
-                uint32_t shi = min(slo + sub, clo + clen);
-                bool dd = slo < clo + clen && chunk_dirty(ev, slo, shi);
-                uint32_t mask = __ballot_sync(0xffffffffu, dd);
-                uint32_t rank = __popc(mask & ((1u << lane) - 1));
-                if (dd && sp + rank < kFindStack) {
-                    s_lo[wid][sp + rank] = slo;
-                    s_len[wid][sp + rank] = shi - slo;
-                }
-                sp = min(sp + __popc(mask), kFindStack);
-                __syncwarp();
-            }
-        }
-    }
-}
+struct FindSmem {
+    uint32_t list[32768];                 /* boundary positions; list[0] = 0 */
+    uint32_t lo[kFindWarps][kFindStack];  /* per-warp refinement stacks */
+    uint32_t len[kFindWarps][kFindStack];
+    uint32_t count;
+};
 
-/* single CTA: sort boundary positions (bitonic in shared memory), emit batch_off[0..nb] and  */
-/* check that batch keys strictly increase                                                   */
-__global__ void __launch_bounds__(1024) k_sort_batches(const hirace_event *__restrict__ ev, uint32_t n,
-                                                       const uint32_t *raw, const uint32_t *raw_count,
-                                                       uint32_t *off, uint32_t *nbatches, uint32_t *batch_ctr,
-                                                       unsigned int *err)
+/* One CTA: (1) each lane probes one 32768-event chunk (2 loads), (2) the warp refines each
+ * dirty chunk 32-way down to single positions, (3) bitonic sort of the boundaries, emit
+ * batch_off[0..nb], zero the per-batch claim counters, check keys strictly increase. */
+__global__ void __launch_bounds__(kFindThreads) k_batches(const hirace_event *__restrict__ ev, uint32_t n,
+                                                          uint32_t *off, uint32_t *nbatches, uint32_t *batch_ctr,
+                                                          unsigned int *err)
 {
-    extern __shared__ uint32_t s[];
-    const uint32_t found = *raw_count;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    FindSmem &S = *reinterpret_cast<FindSmem *>(smem_raw);
+    const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    if (threadIdx.x == 0) {
+        S.count = 1;
+        S.list[0] = 0;
+    }
+    __syncthreads();
     if (n == 0) {
         if (threadIdx.x == 0) {
             *nbatches = 0;
@@ -104,30 +69,71 @@ __global__ void __launch_bounds__(1024) k_sort_batches(const hirace_event *__res
         }
         return;
     }
-    if (found + 1 > HIRACE_MAX_BATCHES) {
+    const uint64_t nchunks = (n + kFindChunk - 1) / kFindChunk;
+    for (uint64_t t0 = (uint64_t)wid * 32; t0 < nchunks; t0 += (uint64_t)kFindWarps * 32) {
+        const uint64_t t = t0 + lane;
+        const uint32_t lo = (uint32_t)(t * kFindChunk);
+        const bool d = t < nchunks && chunk_dirty(ev, lo, (uint32_t)min((uint64_t)lo + kFindChunk, (uint64_t)n));
+        for (uint32_t dm = __ballot_sync(0xffffffffu, d); dm; dm &= dm - 1) {
+            const uint32_t clo0 = (uint32_t)((t0 + __ffs(dm) - 1) * kFindChunk);
+            int sp = 1;
+            if (lane == 0) {
+                S.lo[wid][0] = clo0;
+                S.len[wid][0] = (uint32_t)min((uint64_t)kFindChunk, (uint64_t)n - clo0);
+            }
+            __syncwarp();
+            while (sp > 0) {
+                sp--;
+                const uint32_t clo = S.lo[wid][sp], clen = S.len[wid][sp];
+                __syncwarp();
+                if (clen <= 32) {
+                    const uint32_t p = clo + lane;
+                    if (lane < clen && p >= 1 && batch_key_at(ev, p) != batch_key_at(ev, p - 1)) {
+                        const uint32_t k = atomicAdd(&S.count, 1u);
+                        if (k < 32768u)
+                            S.list[k] = p;
+                    }
+                } else {
+                    const uint32_t sub = (clen + 31) / 32;
+                    const uint32_t slo = clo + lane * sub;
+                    const uint32_t shi = min(slo + sub, clo + clen);
+                    const bool dd = slo < clo + clen && chunk_dirty(ev, slo, shi);
+                    const uint32_t mask = __ballot_sync(0xffffffffu, dd);
+                    const uint32_t rank = __popc(mask & ((1u << lane) - 1));
+                    if (dd && sp + rank < kFindStack) {
+                        S.lo[wid][sp + rank] = slo;
+                        S.len[wid][sp + rank] = shi - slo;
+                    }
+                    sp = min(sp + __popc(mask), kFindStack);
+                    __syncwarp();
+                }
+            }
+        }
+    }
+    __syncthreads();
+    const uint32_t nb = S.count;
+    if (nb > HIRACE_MAX_BATCHES) {
         if (threadIdx.x == 0) {
             *nbatches = 0;
             atomicOr(err, ERR_BATCHES | ERR_BAD_TRACE);
         }
         return;
     }
-    const uint32_t nb = found + 1;
     uint32_t P = 1;
     while (P < nb)
         P <<= 1;
-    for (uint32_t i = threadIdx.x; i < P; i += blockDim.x)
-        s[i] = i == 0 ? 0u : (i < nb ? raw[i - 1] : 0xffffffffu);
+    for (uint32_t i = nb + threadIdx.x; i < P; i += blockDim.x)
+        S.list[i] = 0xffffffffu;
     __syncthreads();
     for (uint32_t k = 2; k <= P; k <<= 1) {
         for (uint32_t j = k >> 1; j > 0; j >>= 1) {
             for (uint32_t i = threadIdx.x; i < P; i += blockDim.x) {
-                uint32_t ixj = i ^ j;
+                const uint32_t ixj = i ^ j;
                 if (ixj > i) {
-                    uint32_t a = s[i], b = s[ixj];
-                    bool up = (i & k) == 0;
-                    if ((a > b) == up) {
-                        s[i] = b;
-                        s[ixj] = a;
+                    const uint32_t x = S.list[i], y = S.list[ixj];
+                    if ((x > y) == ((i & k) == 0)) {
+                        S.list[i] = y;
+                        S.list[ixj] = x;
                     }
                 }
             }
@@ -135,9 +141,9 @@ __global__ void __launch_bounds__(1024) k_sort_batches(const hirace_event *__res
         }
     }
     for (uint32_t i = threadIdx.x; i < nb; i += blockDim.x) {
-        off[i] = s[i];
-        batch_ctr[i] = 0; /* tile-claim counters of the replay kernel */
-        if (i > 0 && !(batch_key_at(ev, s[i]) > batch_key_at(ev, s[i - 1])))
+        off[i] = S.list[i];
+        batch_ctr[i] = 0;
+        if (i > 0 && !(batch_key_at(ev, S.list[i]) > batch_key_at(ev, S.list[i - 1])))
             atomicOr(err, ERR_BAD_TRACE);
     }
     if (threadIdx.x == 0) {
@@ -149,18 +155,8 @@ __global__ void __launch_bounds__(1024) k_sort_batches(const hirace_event *__res
 cudaError_t launch_find_batches(const hirace_event *ev, uint32_t n, const Scratch &s, unsigned int *err,
                                 int sm_count, cudaStream_t st)
 {
-    cudaError_t e = cudaMemsetAsync(s.raw_count, 0, sizeof(uint32_t), st);
-    if (e != cudaSuccess)
-        return e;
-    if (n > 1) {
-        uint64_t chunks = (n + kFindChunk - 1) / kFindChunk;
-        uint64_t ctas = (chunks + kFindWarps - 1) / kFindWarps;
-        int grid = (int)(ctas < (uint64_t)sm_count * 4 ? ctas : (uint64_t)sm_count * 4);
-        k_find_batches<<<grid, kFindWarps * 32, 0, st>>>(ev, n, s.raw_pos, s.raw_count, HIRACE_MAX_BATCHES - 1);
-    }
-    /* dynamic smem sized for the worst case; the kernel uses next_pow2(nb) of it */
-    k_sort_batches<<<1, 1024, 32768 * sizeof(uint32_t), st>>>(ev, n, s.raw_pos, s.raw_count, s.batch_off,
-                                                              s.nbatches, s.batch_ctr, err);
+    (void)sm_count;
+    k_batches<<<1, kFindThreads, sizeof(FindSmem), st>>>(ev, n, s.batch_off, s.nbatches, s.batch_ctr, err);
     return cudaGetLastError();
 }
 
@@ -169,139 +165,31 @@ cudaError_t launch_find_batches(const hirace_event *ev, uint32_t n, const Scratc
 /* words first, then shared words block-major)                                               */
 /* ---------------------------------------------------------------------------------------- */
 
-__global__ void __launch_bounds__(kCollectThreads) k_collect_count(const unsigned long long *__restrict__ shadow,
-                                                                   uint64_t nwords, uint32_t *tile_counts)
+/* standalone collect: one cooperative kernel running collect_phase (collect.cuh) */
+__global__ void __launch_bounds__(256) k_collect(hirace_dev_ctx c, uint64_t nwords, hirace_race *out, uint64_t cap,
+                                                 unsigned long long *d_total, uint32_t *cta_cnt, unsigned int *bar)
 {
-    __shared__ uint32_t s_w[kCollectThreads / 32];
-    const uint64_t base = (uint64_t)blockIdx.x * kCollectTile;
-    uint32_t cnt = 0;
-    for (int it = 0; it < kCollectTile / kCollectThreads / 2; it++) {
-        uint64_t wi = base + ((uint64_t)it * kCollectThreads + threadIdx.x) * 2;
-        if (wi + 1 < nwords) {
-            ulonglong2 v = __ldcs(reinterpret_cast<const ulonglong2 *>(shadow + wi));
-            cnt += (st_of(v.x) >= ST_RACE_W) + (st_of(v.y) >= ST_RACE_W);
-        } else if (wi < nwords) {
-            cnt += st_of(shadow[wi]) >= ST_RACE_W;
-        }
-    }
-    cnt = __reduce_add_sync(0xffffffffu, cnt);
-    if ((threadIdx.x & 31) == 0)
-        s_w[threadIdx.x >> 5] = cnt;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        uint32_t t = 0;
-        for (int i = 0; i < kCollectThreads / 32; i++)
-            t += s_w[i];
-        tile_counts[blockIdx.x] = t;
-    }
-}
-
-/* single CTA exclusive scan of tile counts; total -> *d_total */
-__global__ void __launch_bounds__(1024) k_collect_scan(uint32_t *tile_counts, uint64_t ntiles,
-                                                       unsigned long long *d_total)
-{
-    __shared__ unsigned long long s_w[32];
-    __shared__ unsigned long long s_carry;
-    if (threadIdx.x == 0)
-        s_carry = 0;
-    __syncthreads();
-    const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    for (uint64_t b0 = 0; b0 < ntiles; b0 += 1024) {
-        uint64_t i = b0 + threadIdx.x;
-        unsigned long long v = i < ntiles ? tile_counts[i] : 0;
-        unsigned long long x = v;
-        for (int o = 1; o < 32; o <<= 1) {
-            unsigned long long y = __shfl_up_sync(0xffffffffu, x, o);
-            if ((int)lane >= o)
-                x += y;
-        }
-        if (lane == 31)
-            s_w[wid] = x;
-        __syncthreads();
-        if (wid == 0) {
-            unsigned long long t = s_w[lane];
-            for (int o = 1; o < 32; o <<= 1) {
-                unsigned long long y = __shfl_up_sync(0xffffffffu, t, o);
-                if ((int)lane >= o)
-                    t += y;
-            }
-            s_w[lane] = t;
-        }
-        __syncthreads();
-        unsigned long long excl = s_carry + (wid ? s_w[wid - 1] : 0) + x - v;
-        if (i < ntiles)
-            tile_counts[i] = (uint32_t)excl; /* offsets fit: at most shadow words < 2^37; see cap */
-        __syncthreads();
-        if (threadIdx.x == 0)
-            s_carry += s_w[31];
-        __syncthreads();
-    }
-    if (threadIdx.x == 0)
-        *d_total = s_carry;
-}
-
-__global__ void __launch_bounds__(kCollectThreads) k_collect_write(const unsigned long long *__restrict__ shadow,
-                                                                   uint64_t nwords, uint64_t global_words,
-                                                                   uint32_t smem_words,
-                                                                   const uint32_t *__restrict__ tile_off,
-                                                                   hirace_race *out, uint64_t cap)
-{
-    __shared__ uint32_t s_w[kCollectThreads / 32];
-    __shared__ uint32_t s_run;
-    const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const uint64_t base = (uint64_t)blockIdx.x * kCollectTile;
-    if (threadIdx.x == 0)
-        s_run = 0;
-    __syncthreads();
-    const uint64_t toff = tile_off[blockIdx.x];
-    for (int it = 0; it < kCollectTile / kCollectThreads; it++) {
-        const uint64_t wi = base + (uint64_t)it * kCollectThreads + threadIdx.x;
-        uint64_t o = wi < nwords ? shadow[wi] : 0;
-        const bool f = st_of(o) >= ST_RACE_W;
-        const uint32_t m = __ballot_sync(0xffffffffu, f);
-        if (lane == 0)
-            s_w[wid] = __popc(m);
-        __syncthreads();
-        uint32_t before = s_run;
-        for (uint32_t w = 0; w < wid; w++)
-            before += s_w[w];
-        if (f) {
-            const uint64_t posn = toff + before + __popc(m & ((1u << lane) - 1));
-            if (posn < cap) {
-                hirace_race r;
-                if (wi < global_words) {
-                    r.key = wi;
-                } else {
-                    const uint64_t sidx = wi - global_words;
-                    const uint64_t blk = sidx / smem_words;
-                    r.key = HIRACE_SHARED_BIT | (blk << 32) | (sidx - blk * smem_words);
-                }
-                r.cls_and_epoch = race_class(st_of(o)) | (g_of(o) << 8);
-                r.detect_tid = tid_of(o);
-                out[posn] = r;
-            }
-        }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            uint32_t t = 0;
-            for (int w = 0; w < kCollectThreads / 32; w++)
-                t += s_w[w];
-            s_run += t;
-        }
-        __syncthreads();
-    }
+    unsigned int epoch = 0;
+    collect_phase(c, nwords, out, cap, d_total, cta_cnt, bar, epoch);
 }
 
 cudaError_t launch_collect(const hirace_dev_ctx &c, uint64_t shadow_words, const Scratch &s, hirace_race *out,
                            uint64_t cap, unsigned long long *d_total, cudaStream_t st)
 {
-    const uint64_t ntiles = s.ntiles;
-    k_collect_count<<<(unsigned)ntiles, kCollectThreads, 0, st>>>(c.shadow, shadow_words, s.tile_counts);
-    k_collect_scan<<<1, 1024, 0, st>>>(s.tile_counts, ntiles, d_total);
-    k_collect_write<<<(unsigned)ntiles, kCollectThreads, 0, st>>>(c.shadow, shadow_words, c.global_words,
-                                                                  c.smem_words ? c.smem_words : 1, s.tile_counts,
-                                                                  out, cap);
-    return cudaGetLastError();
+    cudaError_t e = cudaMemsetAsync(s.grid_bar2, 0, sizeof(unsigned int), st);
+    if (e != cudaSuccess)
+        return e;
+    hirace_dev_ctx cc = c;
+    uint64_t nw = shadow_words;
+    hirace_race *o = out;
+    uint64_t cp = cap;
+    unsigned long long *dt = d_total;
+    uint32_t *cnt = s.cta_cnt;
+    unsigned int *bar = s.grid_bar2;
+    void *args[] = {&cc, &nw, &o, &cp, &dt, &cnt, &bar};
+    const uint64_t ntiles = (shadow_words + kCollectTile - 1) / kCollectTile;
+    const int grid = (int)(ntiles < (uint64_t)s.collect_grid ? ntiles : (uint64_t)s.collect_grid);
+    return cudaLaunchCooperativeKernel((const void *)k_collect, dim3(grid), dim3(256), args, 0, st);
 }
 
 /* ---------------------------------------------------------------------------------------- */
@@ -467,8 +355,7 @@ cudaError_t launch_bucket(const hirace_dev_ctx &c, const hirace_event *in, uint3
 cudaError_t kernels_init(int device)
 {
     (void)device;
-    return cudaFuncSetAttribute(k_sort_batches, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                32768 * (int)sizeof(uint32_t));
+    return cudaFuncSetAttribute(k_batches, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(FindSmem));
 }
 
 } // namespace hirace_impl

@@ -9,28 +9,33 @@
 
 namespace hirace_impl {
 
-constexpr int kReplayThreads = 256;  /* 8 warps */
+constexpr int kReplayThreads = 512;  /* 16 warps */
 constexpr int kCollectTile = 4096;     /* shadow words per collect CTA                 */
 constexpr int kCollectThreads = 256;
 constexpr uint32_t kFindChunk = 32768; /* top-level batch-boundary probe chunk (32^3)   */
+constexpr int kMaxCtas = 4096;         /* upper bound on co-resident CTAs of our kernels */
 
 struct Scratch {
-    uint32_t *raw_pos;       /* boundary positions found (unsorted), HIRACE_MAX_BATCHES      */
-    uint32_t *raw_count;     /* number found (excluding position 0)                          */
     uint32_t *batch_off;     /* sorted batch offsets [0..nb], HIRACE_MAX_BATCHES + 1         */
     uint32_t *nbatches;      /* nb                                                            */
     uint32_t *batch_ctr;     /* per-batch tile-claim counters, HIRACE_MAX_BATCHES             */
-    unsigned int *grid_bar;  /* grid barrier counter                                          */
-    uint32_t *tile_counts;   /* collect: per-tile counts / offsets                           */
-    uint64_t ntiles;
+    unsigned int *grid_bar;  /* grid barrier counter (replay)                                 */
+    unsigned int *grid_bar2; /* grid barrier counter (standalone collect)                     */
+    uint32_t *cta_cnt;       /* collect: per-CTA flagged-word counts, kMaxCtas                */
+    int collect_grid;        /* co-resident CTAs of k_collect                                  */
 };
 
-/* batch discovery: find_batches + sort_batches */
+/* batch discovery (one CTA): boundaries, sort, validation */
 cudaError_t launch_find_batches(const hirace_event *ev, uint32_t n, const Scratch &s, unsigned int *err,
                                 int sm_count, cudaStream_t st);
 /* persistent cooperative replay over the discovered batches */
+/* optional fused collect at the end of the replay (out == nullptr: none) */
 cudaError_t launch_replay(const hirace_dev_ctx &c, const hirace_event *ev, const Scratch &s, int grid,
-                          cudaStream_t st);
+                          cudaStream_t st, uint64_t shadow_words = 0, hirace_race *out = nullptr, uint64_t cap = 0,
+                          unsigned long long *d_total = nullptr);
+int collect_max_grid(int device);
+__global__ void k_collect(hirace_dev_ctx c, uint64_t nwords, hirace_race *out, uint64_t cap,
+                          unsigned long long *d_total, uint32_t *cta_cnt, unsigned int *bar);
 int replay_max_grid(int device);
 /* order-preserving compaction of RACE records from the shadow */
 cudaError_t launch_collect(const hirace_dev_ctx &c, uint64_t shadow_words, const Scratch &s, hirace_race *out,

@@ -24,6 +24,7 @@
 #include <stdint.h>
 
 #include "hirace_device.cuh"
+#include "collect.cuh"
 #include "internal.h"
 #include "kernel_common.cuh"
 
@@ -35,7 +36,7 @@ namespace {
 
 constexpr uint32_t FULL = 0xffffffffu;
 constexpr uint64_t NONE = ~0ull;
-constexpr int kMinBlocks = 4; /* 32 warps per SM at <= 64 registers */
+constexpr int kMinBlocks = 2; /* 2 x 16 warps per SM at <= 64 registers */
 
 struct Batch {
     uint32_t key, g, b, w, ep; /* ep = epochs in record layout */
@@ -248,10 +249,20 @@ __device__ __forceinline__ uint64_t key_of_idx(const Lane &L, const hirace_dev_c
     return HIRACE_SHARED_BIT | ((uint64_t)blk << 32) | (L.idx - c.global_words - (uint64_t)blk * c.smem_words);
 }
 
+/* out of line so the collect's registers do not raise the replay loop's allocation */
+__device__ __noinline__ unsigned int collect_call(const hirace_dev_ctx c, uint64_t nwords, hirace_race *out, uint64_t cap,
+                                                  unsigned long long *d_total, uint32_t *cta_cnt, unsigned int *bar,
+                                                  unsigned int epoch)
+{
+    collect_phase(c, nwords, out, cap, d_total, cta_cnt, bar, epoch);
+    return epoch;
+}
+
 template <bool P2>
 __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     k_replay(hirace_dev_ctx c, const uint4 *__restrict__ ev, const uint32_t *__restrict__ off,
-             const uint32_t *__restrict__ nbp, unsigned int *bar)
+             const uint32_t *__restrict__ nbp, unsigned int *bar, uint64_t shadow_words, hirace_race *out,
+             uint64_t cap, unsigned long long *d_total, uint32_t *cta_cnt)
 {
     __shared__ __align__(16) unsigned char s_table[2048];
     __shared__ unsigned long long s_stats[4];
@@ -341,6 +352,12 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
         }
     }
 
+    /* fused a7 collection (hirace_check_trace_device): one more barrier, then the shadow scan */
+    if (d_total) {
+        grid_sync(bar, gridDim.x, bar_epoch);
+        bar_epoch = collect_call(c, shadow_words, out, cap, d_total, cta_cnt, bar, bar_epoch);
+    }
+
     if (__any_sync(FULL, bad) && lane == 0)
         atomicOr(c.error_flags, ERR_BAD_TRACE);
 #pragma unroll
@@ -375,8 +392,19 @@ int replay_max_grid(int device)
     return sms * occ;
 }
 
+int collect_max_grid(int device)
+{
+    int sms = 0, occ = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_collect, 256, 0);
+    if (occ < 1)
+        occ = 1;
+    return sms * occ < kMaxCtas ? sms * occ : kMaxCtas;
+}
+
 cudaError_t launch_replay(const hirace_dev_ctx &c, const hirace_event *ev, const Scratch &s, int grid,
-                          cudaStream_t st)
+                          cudaStream_t st, uint64_t shadow_words, hirace_race *out, uint64_t cap,
+                          unsigned long long *d_total)
 {
     cudaError_t e = cudaMemsetAsync(s.grid_bar, 0, sizeof(unsigned int), st);
     if (e != cudaSuccess)
@@ -386,7 +414,11 @@ cudaError_t launch_replay(const hirace_dev_ctx &c, const hirace_event *ev, const
     const uint32_t *offp = s.batch_off;
     const uint32_t *nbp = s.nbatches;
     unsigned int *barp = s.grid_bar;
-    void *args[] = {&cc, &evp, &offp, &nbp, &barp};
+    uint64_t nw = shadow_words, cp = cap;
+    hirace_race *o = out;
+    unsigned long long *dt = d_total;
+    uint32_t *cnt = s.cta_cnt;
+    void *args[] = {&cc, &evp, &offp, &nbp, &barp, &nw, &o, &cp, &dt, &cnt};
     const bool p2 = (c.block_threads & (c.block_threads - 1)) == 0 && (c.warp_size & (c.warp_size - 1)) == 0;
     const void *fn = p2 ? (const void *)k_replay<true> : (const void *)k_replay<false>;
     return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kReplayThreads), args, 0, st);

@@ -27,9 +27,9 @@ STATUS = {0: "HIRACE_OK", -1: "HIRACE_E_INVAL", -2: "HIRACE_E_NOMEM", -3: "HIRAC
 
 # every symbol include/hirace.h declares (checked by tests/test_abi.py against the header)
 EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_free", "hirace_shadow_reset", "hirace_barrier",
-           "hirace_replay_trace", "hirace_check_trace_host", "hirace_collect_races",
+           "hirace_replay_trace", "hirace_check_trace_device", "hirace_check_trace_host", "hirace_collect_races",
            "hirace_collect_races_device", "hirace_get_stats", "hirace_sync", "hirace_get_dev_ctx",
-           "hirace_bucket_events", "hirace_set_kernel_timing", "hirace_fsm_table", "hirace_fsm_step", "hirace_status_string",
+           "hirace_bucket_events", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_fsm_table", "hirace_fsm_step", "hirace_status_string",
            "hirace_version")
 
 
@@ -78,6 +78,7 @@ def load():
         "hirace_barrier": (I32, [P, I32, P]),
         "hirace_replay_trace": (I32, [P, P, U64, P]),
         "hirace_check_trace_host": (I32, [P, P, U64, P, U64, ctypes.POINTER(U64), P]),
+        "hirace_check_trace_device": (I32, [P, P, U64, P, U64, P, P]),
         "hirace_collect_races": (I32, [P, P, U64, ctypes.POINTER(U64), P]),
         "hirace_collect_races_device": (I32, [P, P, U64, P, P]),
         "hirace_get_stats": (I32, [P] + [ctypes.POINTER(U64)] * 5),
@@ -85,6 +86,8 @@ def load():
         "hirace_get_dev_ctx": (I32, [P, P, ctypes.POINTER(DevCtx)]),
         "hirace_bucket_events": (I32, [P, P, U64, I32, I32, P, ctypes.POINTER(U64), P]),
         "hirace_set_kernel_timing": (I32, [P, P, P]),
+        "hirace_microbench_atomics": (I32, [I32, U64, I32, I32, U64, ctypes.POINTER(ctypes.c_double), P]),
+        "hirace_microbench_grid_sync": (I32, [I32, I32, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_fsm_table": (I32, [P]),
         "hirace_fsm_step": (U64, [U64, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
         "hirace_status_string": (ctypes.c_char_p, [I32]),
@@ -112,6 +115,22 @@ def fsm_step(old: int, tid: int, kind: int, g: int, b: int, w: int, block_thread
     rep = ctypes.c_int(0)
     n = load().hirace_fsm_step(old, tid, kind, g, b, w, block_threads, warp_size, ctypes.byref(rep))
     return int(n), int(rep.value)
+
+
+def microbench_atomics(nwords: int, random: bool, op: int, nops: int, device: int = 0, stream=None) -> float:
+    """64-bit op rate on distinct words (op 0 CAS, 1 add, 2 coherent load, 3 load+CAS)."""
+    r = ctypes.c_double(0)
+    _check(load().hirace_microbench_atomics(device, nwords, int(random), op, nops, ctypes.byref(r),
+                                            _stream_handle(stream)), "hirace_microbench_atomics")
+    return r.value
+
+
+def microbench_grid_sync(iters: int = 200, device: int = 0, stream=None) -> float:
+    """Microseconds per grid barrier of the persistent replay kernel."""
+    r = ctypes.c_double(0)
+    _check(load().hirace_microbench_grid_sync(device, iters, ctypes.byref(r), _stream_handle(stream)),
+           "hirace_microbench_grid_sync")
+    return r.value
 
 
 def _stream_handle(stream):
@@ -202,6 +221,15 @@ class Checker:
         _check(self.lib.hirace_collect_races_device(self.h, ctypes.c_void_p(out_dev.data_ptr()), cap,
                                                     ctypes.c_void_p(total_dev.data_ptr()),
                                                     _stream_handle(stream)), "hirace_collect_races_device")
+
+    def check_device(self, events_dev, out_dev, cap: int, total_dev, n: int | None = None, stream=None):
+        """Fused replay + collect on device-resident events (one persistent kernel)."""
+        if n is None:
+            n = events_dev.numel() * events_dev.element_size() // 16
+        _check(self.lib.hirace_check_trace_device(self.h, ctypes.c_void_p(events_dev.data_ptr()), n,
+                                                  ctypes.c_void_p(out_dev.data_ptr()), cap,
+                                                  ctypes.c_void_p(total_dev.data_ptr()), _stream_handle(stream)),
+               "hirace_check_trace_device")
 
     def check_host(self, events: np.ndarray, cap: int | None = None, stream=None) -> np.ndarray:
         """End-to-end from HOST events: H2D (chunked, overlapped) + replay + collect + D2H."""

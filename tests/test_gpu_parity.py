@@ -265,3 +265,44 @@ def test_report_buffer_counts_every_class_transition():
     st = c.stats()
     assert st["dropped_reports"] >= len(r) - 16
     c.close()
+
+
+def _fused(trace, cap=1 << 20):
+    c = hr.Checker.for_trace(trace)
+    c.reset()
+    d = hr.events_to_device(trace.events)
+    out = torch.zeros(max(cap, 1) * 16, dtype=torch.uint8, device="cuda")
+    tot = torch.zeros(1, dtype=torch.int64, device="cuda")
+    c.check_device(d, out, cap, tot)
+    torch.cuda.synchronize()
+    assert c.sync() == 0
+    n = int(tot.item())
+    recs = out.cpu().numpy().view(hr.RACE_DTYPE)[: min(n, cap)]
+    c.close()
+    return n, recs
+
+
+@pytest.mark.parametrize("make", [lambda: tg.cfg1("post_init"), lambda: tg.cfg2(True, n=128, steps=3),
+                                  lambda: tg.cfg4("B", 6, 128, 34), lambda: tg.listing5(40, 1, 64),
+                                  lambda: tg.cfg2(False, n=64, steps=2)])
+def test_fused_check_device_matches_oracle(make):
+    t = make()
+    n, recs = _fused(t)
+    want = oracle_dict(t)
+    assert n == len(want)
+    assert as_dict(recs) == want
+    assert bool(np.all(recs["key"][1:] > recs["key"][:-1]))
+
+
+def test_collect_with_small_capacity_reports_total():
+    t = tg.cfg2(True, n=128, steps=2)
+    want = oracle_dict(t)
+    n, recs = _fused(t, cap=100)
+    assert n == len(want) and len(recs) == 100
+    keys = sorted(want)[:100]
+    assert recs["key"].tolist() == keys
+    c = hr.Checker.for_trace(t)
+    c.replay(hr.events_to_device(t.events))
+    r = c.collect(cap=10)           # grows the buffer and retries
+    assert as_dict(r) == want
+    c.close()
