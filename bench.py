@@ -50,6 +50,8 @@ def make_trace(config: int, variant: str):
         return tg.cfg1("post_init" if variant == "racy" else None)
     if config == 2:
         return tg.cfg2(variant == "racy")
+    if config == 3:
+        return tg.cfg3("bfs", variant == "racy")
     if config == 4:
         return tg.cfg4("B" if variant == "racy" else None)
     raise SystemExit(f"config {config} not available in bench yet")
@@ -176,6 +178,7 @@ def config_block(args, trace, world):
 BASELINE_CFG = {
     1: "tiny shared-mem reduction, 1 block x 32 threads, missing __syncthreads",
     2: "tiled shared-memory stencil, 1024 blocks x 256 threads, racy-A (load->compute barrier dropped)",
+    3: "Indigo-style BFS on RMAT-20 (1M vertices, edge factor 16), atomicBug racy variant",
     4: "cooperative multi-phase kernel, 592 x 256, 64 grid phases, racy-B",
 }
 

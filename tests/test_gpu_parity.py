@@ -306,3 +306,30 @@ def test_collect_with_small_capacity_reports_total():
     r = c.collect(cap=10)           # grows the buffer and retries
     assert as_dict(r) == want
     c.close()
+
+
+@pytest.mark.parametrize("kind", ["bfs", "cc"])
+@pytest.mark.parametrize("racy", [False, True])
+def test_cfg3_graph_kernels_vs_oracle(kind, racy):
+    # RMAT scale 14 (16K vertices, hubs of degree ~1e3): hot words, atomics, plain R/W races
+    t = tg.cfg3(kind, racy, scale=14, edge_factor=16)
+    want = oracle_dict(t)
+    assert bool(want) == racy
+    for seed in (None, 0, 1):
+        ts = t if seed is None else tg.Trace(t.name, tg._shuffle_within_batches(t.events, seed), t.grid_blocks,
+                                              t.block_threads, t.warp_size, t.global_words, t.smem_words)
+        r, st = gpu_races(ts)
+        assert as_dict(r) == want
+        assert st["checked"] == t.n
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("racy", [False, True])
+def test_cfg3_full_rmat20_bfs_vs_oracle(racy):
+    # BASELINE configs[2]: RMAT-20 (1,048,576 vertices, ~3.1e7 CSR entries), BFS, ~7e7-1e8 events
+    t = tg.cfg3("bfs", racy)
+    assert t.n > 6e7
+    want = oracle_dict(t)
+    n, recs = _fused(t, cap=max(1, len(want)) + 16)
+    assert n == len(want)
+    assert as_dict(recs) == want

@@ -164,3 +164,20 @@ def test_multiword_accesses_expand_to_words():
     t = tg.Trace("mw", ev, 1, 32, 32, 4, 0)
     assert as_dict(*oracle.races_of(t)[:2]) == {2: 1, 3: 1}
     assert as_dict(*oracle.races_of(t)[:2]) == {k: c for k, (c, _) in brute.races(ev, 32, 32).items()}
+
+
+def test_cfg3_clean_graph_kernels_never_race():
+    # the atomic (clean) BFS/CC variants must give the empty set
+    for kind in ("bfs", "cc"):
+        t = tg.cfg3(kind, racy=False, scale=12, edge_factor=8)
+        assert t.n > 10_000
+        assert as_dict(*oracle.races_of(t)[:2]) == {}
+
+
+@pytest.mark.parametrize("kind", ["bfs", "cc"])
+def test_cfg3_racy_small_graph_oracle_matches_bruteforce(kind):
+    t = tg.cfg3(kind, racy=True, scale=4, edge_factor=2, bs=8, ws=4)
+    assert 20 < t.n < 700
+    want = {k: c for k, (c, _) in brute.races(t.events, t.block_threads, t.warp_size).items()}
+    assert want, "the racy graph kernels must race"
+    assert as_dict(*oracle.races_of(t)[:2]) == want
