@@ -164,6 +164,13 @@ hirace_status hirace_check_trace_device(hirace_ctx *ctx, const hirace_event *d_e
                                         hirace_race *d_out, uint64_t cap, unsigned long long *d_n_total,
                                         void *stream);
 
+/* Batch discovery only (a9, as run by hirace_replay_trace): writes the batch start offsets
+ * (nb + 1 entries, last = n) and batch keys (g<<19 | b<<9 | w) of DEVICE events to HOST arrays
+ * of capacity cap and *nbatches = nb.  Synchronises `stream`.  Used by the sharded driver to
+ * exchange events batch by batch.  BAD_TRACE if the keys do not strictly increase. */
+hirace_status hirace_find_batches(hirace_ctx *ctx, const hirace_event *d_events, uint64_t n, uint32_t *h_offsets,
+                                  uint32_t *h_keys, uint64_t cap, uint64_t *nbatches, void *stream);
+
 /* Same work from HOST events (pinned or pageable): copies through a device staging ring in
  * chunks, overlapping H2D with replay, then collects like hirace_collect_races.  Synchronous.
  * This is the end-to-end entry point. */
@@ -204,11 +211,14 @@ hirace_status hirace_set_kernel_timing(hirace_ctx *ctx, void *start_event, void 
 
 /* ---- sharded mode (a10) ---------------------------------------------------------------- */
 
-/* Buckets n DEVICE events by owner rank for address sharding across nranks GPUs:
- * owner(global word) = (word >> 14) mod nranks (64 KiB chunks), shared-space events stay on
- * `my_rank`.  Writes events grouped by owner (stable inside each owner, so batch order is
- * preserved) to DEVICE d_out (n records) and per-owner counts to HOST h_counts[nranks].
- * Synchronises `stream` (the counts are needed to size the exchange). */
+/* Buckets n DEVICE events by owner rank for address sharding across nranks GPUs
+ * (SURVEY §8(e)): owner(global word) = (word >> 14) mod nranks (64 KiB chunks, so coalesced
+ * runs stay on one owner); shared-space events stay on `my_rank` (shared memory is per block,
+ * PAPER.md L118).  Writes the events grouped by owner — stable inside each owner, so batch
+ * order is preserved — to DEVICE d_out (n records), with every global address rewritten to
+ * the owner's shard-local word ((word >> 14) / nranks) << 14 | (word mod 2^14), so the owner's
+ * context tracks ceil(global_words / (2^14 nranks)) * 2^14 words.  Per-owner counts go to HOST
+ * h_counts[nranks].  Synchronises `stream` (the counts size the exchange).  nranks <= 32. */
 hirace_status hirace_bucket_events(hirace_ctx *ctx, const hirace_event *d_in, uint64_t n, int nranks, int my_rank,
                                    hirace_event *d_out, uint64_t *h_counts, void *stream);
 

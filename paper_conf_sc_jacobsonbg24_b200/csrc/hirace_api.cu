@@ -287,6 +287,37 @@ hirace_status hirace_set_kernel_timing(hirace_ctx *c, void *start_event, void *s
     return HIRACE_OK;
 }
 
+hirace_status hirace_find_batches(hirace_ctx *c, const hirace_event *d_events, uint64_t n, uint32_t *h_offsets,
+                                  uint32_t *h_keys, uint64_t cap, uint64_t *nbatches, void *stream)
+{
+    if (!c || !nbatches || (cap && (!h_offsets || !h_keys)) || (n && !d_events) || n >= 0xffffffffull)
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    *nbatches = 0;
+    if (n == 0)
+        return HIRACE_OK;
+    HR_CUDA(c, launch_find_batches(d_events, (uint32_t)n, c->scr, c->d_err, c->sm_count, st));
+    uint32_t nb = 0;
+    HR_CUDA(c, cudaMemcpyAsync(&nb, c->scr.nbatches, sizeof(nb), cudaMemcpyDeviceToHost, st));
+    HR_CUDA(c, cudaStreamSynchronize(st));
+    hirace_status s = device_errors(c);
+    if (s != HIRACE_OK)
+        return s;
+    *nbatches = nb;
+    if (nb + 1 > cap)
+        return HIRACE_OK; /* caller retries with a bigger buffer */
+    HR_CUDA(c, cudaMemcpy(h_offsets, c->scr.batch_off, (nb + 1) * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+    for (uint32_t i = 0; i < nb; i++) {
+        uint32_t meta = 0;
+        HR_CUDA(c, cudaMemcpy(&meta, &d_events[h_offsets[i]].meta, sizeof(meta), cudaMemcpyDeviceToHost));
+        h_keys[i] = meta >> 5;
+    }
+    return HIRACE_OK;
+}
+
 hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_events, uint64_t n, hirace_race *d_out,
                                         uint64_t cap, unsigned long long *d_n_total, void *stream)
 {

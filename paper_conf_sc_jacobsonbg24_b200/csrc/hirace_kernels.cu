@@ -223,11 +223,25 @@ constexpr int kBucketThreads = 256;
 constexpr int kBucketTile = 4096;
 constexpr int kMaxRanks = 32;
 
+constexpr uint32_t kShardChunkLog2 = 14; /* owner granularity: 2^14 words = 64 KiB */
+
 __device__ __forceinline__ uint32_t owner_of(const hirace_event &e, int nranks, int my_rank)
 {
     if (e.addr & HIRACE_SHARED_BIT)
         return (uint32_t)my_rank;
-    return (uint32_t)((((e.addr & ~HIRACE_SHARED_BIT) >> 2) >> 14) % (uint64_t)nranks);
+    return (uint32_t)((((e.addr & ~HIRACE_SHARED_BIT) >> 2) >> kShardChunkLog2) % (uint64_t)nranks);
+}
+
+/* global byte address -> the owner's shard-local byte address (chunk c of the owner becomes
+ * local chunk c / nranks); shared addresses are unchanged */
+__device__ __forceinline__ uint64_t shard_local_addr(uint64_t addr, int nranks)
+{
+    if (addr & HIRACE_SHARED_BIT)
+        return addr;
+    const uint64_t word = addr >> 2;
+    const uint64_t chunk = word >> kShardChunkLog2;
+    const uint64_t local = ((chunk / (uint64_t)nranks) << kShardChunkLog2) | (word & ((1u << kShardChunkLog2) - 1));
+    return (local << 2) | (addr & 3u);
 }
 
 __global__ void __launch_bounds__(kBucketThreads) k_bucket_hist(const hirace_event *__restrict__ in, uint32_t n,
@@ -328,6 +342,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_scatter(const hirace_
             uint32_t before = s_run[own];
             for (uint32_t w = 0; w < wid; w++)
                 before += s_wc[w][own];
+            e.addr = shard_local_addr(e.addr, nranks);
             out[before + rank_in_warp] = e;
         }
         __syncthreads();

@@ -27,7 +27,7 @@ STATUS = {0: "HIRACE_OK", -1: "HIRACE_E_INVAL", -2: "HIRACE_E_NOMEM", -3: "HIRAC
 
 # every symbol include/hirace.h declares (checked by tests/test_abi.py against the header)
 EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_free", "hirace_shadow_reset", "hirace_barrier",
-           "hirace_replay_trace", "hirace_check_trace_device", "hirace_check_trace_host", "hirace_collect_races",
+           "hirace_replay_trace", "hirace_find_batches", "hirace_check_trace_device", "hirace_check_trace_host", "hirace_collect_races",
            "hirace_collect_races_device", "hirace_get_stats", "hirace_sync", "hirace_get_dev_ctx",
            "hirace_bucket_events", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_fsm_table", "hirace_fsm_step", "hirace_status_string",
            "hirace_version")
@@ -79,6 +79,7 @@ def load():
         "hirace_replay_trace": (I32, [P, P, U64, P]),
         "hirace_check_trace_host": (I32, [P, P, U64, P, U64, ctypes.POINTER(U64), P]),
         "hirace_check_trace_device": (I32, [P, P, U64, P, U64, P, P]),
+        "hirace_find_batches": (I32, [P, P, U64, P, P, U64, ctypes.POINTER(U64), P]),
         "hirace_collect_races": (I32, [P, P, U64, ctypes.POINTER(U64), P]),
         "hirace_collect_races_device": (I32, [P, P, U64, P, P]),
         "hirace_get_stats": (I32, [P] + [ctypes.POINTER(U64)] * 5),
@@ -203,6 +204,22 @@ class Checker:
     def replay_ptr(self, ptr: int, n: int, stream=None):
         _check(self.lib.hirace_replay_trace(self.h, ctypes.c_void_p(ptr), n, _stream_handle(stream)),
                "hirace_replay_trace")
+
+    def find_batches(self, events_dev, n: int | None = None, stream=None):
+        """(offsets[nb+1], keys[nb]) of device events (batch discovery as the replay does it)."""
+        if n is None:
+            n = events_dev.numel() * events_dev.element_size() // 16
+        cap = 64
+        while True:
+            offs = np.zeros(cap, np.uint32)
+            keys = np.zeros(cap, np.uint32)
+            nb = ctypes.c_uint64(0)
+            _check(self.lib.hirace_find_batches(self.h, ctypes.c_void_p(events_dev.data_ptr()), n, offs.ctypes.data,
+                                                keys.ctypes.data, cap, ctypes.byref(nb), _stream_handle(stream)),
+                   "hirace_find_batches")
+            if nb.value + 1 <= cap:
+                return offs[: nb.value + 1].copy(), keys[: nb.value].copy()
+            cap = int(nb.value) + 1
 
     def collect(self, cap: int | None = None, stream=None) -> np.ndarray:
         """Flagged words sorted by key (RACE_DTYPE).  Raises on a sticky error."""

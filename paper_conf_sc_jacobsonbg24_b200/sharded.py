@@ -1,0 +1,172 @@
+"""Address-sharded multi-GPU mode.
+
+One process per GPU.  Each rank holds the trace events of its own blocks (any partition of the
+trace's events works).  Global words are owned by rank (word >> 14) mod P (64 KiB chunks, so
+coalesced runs stay together); shared-memory words stay with the rank that holds the block.
+Batch by batch — in the global (g,b,w) order every rank agrees on — each rank
+
+  1. buckets its events of the batch by owner on the GPU (`hirace_bucket_events`: a stable
+     partition that also rewrites global addresses to the owner's shard-local word index),
+  2. exchanges them with `all_to_all_single` (counts, then payload; NCCL over NVLink/NVSwitch
+     with device tensors, or gloo through host staging for CPU tests / single-GPU runs),
+  3. replays what it received on its own shard of the shadow (`hirace_replay_trace`).
+
+Every word's events therefore reach exactly one rank, in batch order, so each rank's race set
+is exact for the words it owns; the union (keys mapped back to global words) is the answer.
+Inside a batch any order is a linear extension of happens-before, so the
+received segments need no merge.
+
+The orchestration is written against three small interfaces (`ops`: find_batches / bucket /
+replay / collect, and an exchange) so the host logic can be tested on CPU with gloo and
+world_size > 1; the GPU ops are the library's kernels, there is no CPU fallback for them.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+CHUNK_LOG2 = 14
+SHARED_BIT = np.uint64(1) << np.uint64(63)
+
+
+def shard_words(global_words: int, nranks: int) -> int:
+    """Shadow words a rank must track for its shard of `global_words` tracked global words."""
+    chunk = 1 << CHUNK_LOG2
+    nchunks = -(-global_words // chunk)
+    return max(1, -(-nchunks // nranks)) * chunk
+
+
+def owner_of_words(words: np.ndarray, nranks: int) -> np.ndarray:
+    return (np.asarray(words, np.uint64) >> np.uint64(CHUNK_LOG2)) % np.uint64(nranks)
+
+
+def local_to_global_keys(keys: np.ndarray, rank: int, nranks: int) -> np.ndarray:
+    """Shard-local race keys -> global keys (shared keys are unchanged)."""
+    keys = np.asarray(keys, dtype=np.uint64)
+    sh = (keys & SHARED_BIT) != 0
+    c = np.uint64(CHUNK_LOG2)
+    mask = np.uint64((1 << CHUNK_LOG2) - 1)
+    glob = (((keys >> c) * np.uint64(nranks) + np.uint64(rank)) << c) | (keys & mask)
+    return np.where(sh, keys, glob)
+
+
+# ---------------------------------------------------------------------------------------------
+# exchanges
+# ---------------------------------------------------------------------------------------------
+
+class NcclExchange:
+    """all_to_all_single on device tensors (NCCL over NVLink 5 / NVSwitch)."""
+
+    def __init__(self, group, device):
+        import torch
+        import torch.distributed as dist
+        self.dist, self.torch, self.group, self.device = dist, torch, group, device
+
+    def counts(self, send_counts: list[int]) -> list[int]:
+        t = self.torch.tensor(send_counts, dtype=self.torch.int64, device=self.device)
+        r = self.torch.empty_like(t)
+        self.dist.all_to_all_single(r, t, group=self.group)
+        return [int(x) for x in r.cpu()]
+
+    def payload(self, send, send_counts: list[int], recv_counts: list[int]):
+        """send: int64 tensor [n, 2] (16-byte events) grouped by destination rank."""
+        out = self.torch.empty((sum(recv_counts), 2), dtype=self.torch.int64, device=self.device)
+        self.dist.all_to_all_single(out, send, output_split_sizes=recv_counts, input_split_sizes=send_counts,
+                                    group=self.group)
+        return out
+
+
+class HostExchange(NcclExchange):
+    """The same exchange through host memory (gloo): CPU tests and several ranks on one GPU."""
+
+    def __init__(self, group, device=None):
+        super().__init__(group, "cpu")
+        self.out_device = device
+
+    def payload(self, send, send_counts, recv_counts):
+        cpu = send.cpu() if hasattr(send, "cpu") else send
+        out = super().payload(cpu, send_counts, recv_counts)
+        return out.to(self.out_device) if self.out_device is not None else out
+
+
+# ---------------------------------------------------------------------------------------------
+# GPU ops (the library's kernels)
+# ---------------------------------------------------------------------------------------------
+
+class GpuOps:
+    """Per-rank shard context on one GPU; every step is a libhirace kernel."""
+
+    def __init__(self, grid_blocks, block_threads, warp_size, global_words, smem_words, nranks, rank,
+                 device=0, report_capacity=0):
+        import torch
+
+        from .hirace import Checker
+        self.torch = torch
+        self.nranks, self.rank, self.device = nranks, rank, device
+        self.ctx = Checker(grid_blocks, block_threads, warp_size, shard_words(global_words, nranks), smem_words,
+                           report_capacity, device)
+        self.ctx.reset()
+
+    def find_batches(self, events):
+        """events: CUDA int64 tensor [n, 2] -> (offsets[nb+1], keys[nb]) numpy."""
+        if events.shape[0] == 0:
+            return np.zeros(1, np.uint32), np.zeros(0, np.uint32)
+        return self.ctx.find_batches(events, events.shape[0])
+
+    def bucket(self, events):
+        out = self.torch.empty_like(events)
+        counts = self.ctx.bucket(events, events.shape[0], self.nranks, self.rank, out) if events.shape[0] else \
+            [0] * self.nranks
+        return out, counts
+
+    def replay(self, events):
+        if events.shape[0]:
+            self.ctx.replay(events, events.shape[0])
+
+    def collect(self):
+        r = self.ctx.collect()
+        keys = local_to_global_keys(r["key"], self.rank, self.nranks)
+        out = r.copy()
+        out["key"] = keys
+        return out
+
+
+# ---------------------------------------------------------------------------------------------
+# orchestration
+# ---------------------------------------------------------------------------------------------
+
+def all_batch_keys(local_keys: np.ndarray, group, dist) -> np.ndarray:
+    """Union of every rank's batch keys, sorted: the global batch order all ranks follow."""
+    objs = [None] * dist.get_world_size(group)
+    dist.all_gather_object(objs, [int(k) for k in local_keys], group=group)
+    return np.array(sorted(set().union(*[set(o) for o in objs])), dtype=np.uint32)
+
+
+def run_sharded(local_events, ops, exchange, group, dist, on_batch=None):
+    """Replays this rank's events (int64 tensor [n, 2], sorted by batch key) across all ranks.
+    Returns the number of events this rank replayed (received).  `on_batch(key, n_recv)` is an
+    optional hook for tests/telemetry."""
+    offs, keys = ops.find_batches(local_events)
+    order = all_batch_keys(keys, group, dist)
+    where = {int(k): i for i, k in enumerate(keys)}
+    received = 0
+    for key in order:
+        i = where.get(int(key))
+        part = local_events[int(offs[i]):int(offs[i + 1])] if i is not None else local_events[0:0]
+        send, send_counts = ops.bucket(part)
+        recv_counts = exchange.counts(send_counts)
+        recv = exchange.payload(send, send_counts, recv_counts)
+        ops.replay(recv)
+        received += int(recv.shape[0])
+        if on_batch is not None:
+            on_batch(int(key), int(recv.shape[0]))
+    return received
+
+
+def gather_races(races: np.ndarray, group, dist, dst: int = 0):
+    """Union of the per-rank race sets (disjoint by owner), sorted by key, on rank `dst`."""
+    objs = [None] * dist.get_world_size(group)
+    dist.all_gather_object(objs, races.tobytes(), group=group)
+    if dist.get_rank(group) != dst:
+        return None
+    allr = np.concatenate([np.frombuffer(b, dtype=races.dtype) for b in objs]) if objs else races[:0]
+    return allr[np.argsort(allr["key"], kind="stable")]
