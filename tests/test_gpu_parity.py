@@ -333,3 +333,37 @@ def test_cfg3_full_rmat20_bfs_vs_oracle(racy):
     n, recs = _fused(t, cap=max(1, len(want)) + 16)
     assert n == len(want)
     assert as_dict(recs) == want
+
+
+def _cfg5_check(t, sample=4000):
+    from tests.helpers import oracle_on_words
+    want = {w: CLS[c] for w, c in t.info["expected"].items()}
+    n, recs = _fused(t, cap=len(want) + 1024)
+    got = as_dict(recs)
+    assert n == len(want) and got == want          # by construction
+    rng = np.random.default_rng(1)
+    reg = t.info["regions"]
+    sample_words = np.concatenate([
+        np.array(list(want)[:200], np.uint64),
+        rng.integers(0, reg["gather"], sample // 4).astype(np.uint64),          # private
+        rng.integers(reg["gather"], reg["hot"], sample // 4).astype(np.uint64),  # gather
+        rng.integers(reg["hot"], reg["hot"] + 64, sample // 4).astype(np.uint64),  # hottest atomics
+        rng.integers(reg["inj"], reg["pat"] + 2048, sample // 4).astype(np.uint64)])
+    sampled = oracle_on_words(t, sample_words)
+    assert {w: got[w] for w in sampled if w in got} == sampled
+    assert all(int(w) not in got or int(w) in sampled for w in sample_words)
+
+
+def test_cfg5_medium_vs_construction_and_sampled_oracle():
+    # 2^28 tracked words, 8192 blocks x 256 threads, 32 batches: ~1.3e8 events
+    t = tg.cfg5(grid_blocks=8192, words_log2=28)
+    assert t.n > 1e8
+    _cfg5_check(t)
+
+
+@pytest.mark.slow
+def test_cfg5_full_1e9_vs_construction_and_sampled_oracle():
+    # BASELINE configs[4] on one GPU: 2^32 tracked words (32 GiB shadow), 1.07e9 events (17 GB)
+    t = tg.cfg5()
+    assert t.n > 1.07e9
+    _cfg5_check(t)

@@ -181,3 +181,19 @@ def test_cfg3_racy_small_graph_oracle_matches_bruteforce(kind):
     want = {k: c for k, (c, _) in brute.races(t.events, t.block_threads, t.warp_size).items()}
     assert want, "the racy graph kernels must race"
     assert as_dict(*oracle.races_of(t)[:2]) == want
+
+
+def test_cfg5_construction_and_rank_partition():
+    # config 5 (App. C): the injected pairs race with their class, decoys (separated by the
+    # matching barrier) do not, and the filler regions never race; rank slices partition it
+    kw = dict(grid_blocks=64, block_threads=256, words_log2=24, npatterns=300)
+    t = tg.cfg5(**kw)
+    want = {w: CLS[c] for w, c in t.info["expected"].items()}
+    assert len(want) == 150 and set(want.values()) == {1, 2, 3}
+    assert as_dict(*oracle.races_of(t)[:2]) == want
+    parts = [tg.cfg5(nranks=3, rank=r, **kw) for r in range(3)]
+    allev = np.concatenate([p.events for p in parts])
+    assert allev.shape[0] == t.n
+    key = lambda e: np.sort(e.view(np.dtype((np.void, 16))))  # noqa: E731
+    assert np.array_equal(key(allev), key(t.events))
+    assert all(p.batch_count() == 32 for p in parts)
