@@ -44,7 +44,7 @@ def peaks():
     return 6650.0, "fallback"
 
 
-def make_trace(config: int, variant: str):
+def make_trace(config: int, variant: str, nranks: int = 1, rank: int = 0):
     import tracegen as tg
     if config == 1:
         return tg.cfg1("post_init" if variant == "racy" else None)
@@ -54,7 +54,9 @@ def make_trace(config: int, variant: str):
         return tg.cfg3("bfs", variant == "racy")
     if config == 4:
         return tg.cfg4("B" if variant == "racy" else None)
-    raise SystemExit(f"config {config} not available in bench yet")
+    if config == 5:
+        return tg.cfg5(nranks=nranks, rank=rank)
+    raise SystemExit(f"unknown config {config}")
 
 
 def word_accesses(events) -> int:
@@ -180,7 +182,86 @@ BASELINE_CFG = {
     2: "tiled shared-memory stencil, 1024 blocks x 256 threads, racy-A (load->compute barrier dropped)",
     3: "Indigo-style BFS on RMAT-20 (1M vertices, edge factor 16), atomicBug racy variant",
     4: "cooperative multi-phase kernel, 592 x 256, 64 grid phases, racy-B",
+    5: "1.07e9 accesses over 2^32 tracked words (16 GiB tracked, 32 GiB shadow), 65536 x 256 threads, 32 batches",
 }
+
+
+def run_sharded_bench(args, world, rank, local_rank):
+    """Config 5 across `world` GPUs: each rank generates its blocks' events; per batch the events
+    are bucketed by owner (64 KiB chunks of the 2^32-word space) on the GPU and exchanged with
+    NCCL all_to_all_single, then replayed on the owner's shard (strong scaling: fixed trace)."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_jacobsonbg24_b200 import sharded
+    dev = local_rank % torch.cuda.device_count()
+    torch.cuda.set_device(dev)
+    if args.transport == "nccl":
+        dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        ex = sharded.NcclExchange(None, f"cuda:{dev}")
+    else:
+        dist.init_process_group("gloo")
+        ex = sharded.HostExchange(None, device=f"cuda:{dev}")
+    t = make_trace(5, args.variant, world, rank)
+    n_local = word_accesses(t.events)
+    tot = torch.tensor([n_local], dtype=torch.int64, device=f"cuda:{dev}" if args.transport == "nccl" else "cpu")
+    dist.all_reduce(tot)
+    n_total = int(tot.item())
+    ops = sharded.GpuOps(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words, world, rank,
+                         device=dev)
+    ev = torch.from_numpy(t.events.view(np.int64).reshape(-1, 2)).to(f"cuda:{dev}")
+    cap = 1 << 20
+    d_out = torch.empty(cap * 16, dtype=torch.uint8, device=f"cuda:{dev}")
+    d_total = torch.zeros(1, dtype=torch.int64, device=f"cuda:{dev}")
+
+    def step():
+        ops.ctx.reset()
+        sharded.run_sharded(ev, ops, ex, None, dist)
+        ops.ctx.collect_device(d_out, cap, d_total)
+
+    clocks = ClockSampler(dev)
+    clocks.start()
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    flagged = int(d_total.item())
+    dist.barrier()
+    torch.cuda.synchronize()
+    w0 = time.time()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(args.steps):
+        step()
+    e1.record()
+    torch.cuda.synchronize()
+    w1 = time.time()
+    dist.barrier()
+    clocks.mark(w0, w1)
+    clocks.stop()
+    ms = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64)
+    fl = torch.tensor([flagged], dtype=torch.int64)
+    if args.transport == "nccl":
+        ms, fl = ms.cuda(), fl.cuda()
+    dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+    dist.all_reduce(fl)
+    ms, flagged = float(ms.item()), int(fl.item())
+    if rank == 0:
+        peak, peak_kind = peaks()
+        per_step = ms / args.steps
+        out = {"metric": METRIC, "value": n_total * args.steps / (ms / 1e3), "unit": UNIT, "n_gpus": world,
+               "steps": args.steps, "warmup": args.warmup, "ms_per_step": per_step, "higher_is_better": True,
+               "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+               "config": {"workload": f"config 5: {BASELINE_CFG[5]}", "events_total": n_total,
+                          "parallelism": f"address-sharded x{world} ({args.transport} all_to_all per batch)",
+                          "l2": "inputs larger than L2"},
+               "roofline": {"bound": "hbm", "achieved": BYTES_PER_ACCESS * n_total / world / (per_step / 1e3) / 1e9,
+                            "peak": peak, "unit": "GB/s",
+                            "frac": BYTES_PER_ACCESS * n_total / world / (per_step / 1e3) / 1e9 / peak,
+                            "traffic": None, "kernel": "whole sharded step per GPU", "peak_kind": peak_kind},
+               "cpu_baseline": None, "e2e": None, "gpu_launches": None, "clocks": clocks.summary(),
+               "check": {"flagged_words": flagged, "expected": len(t.info["expected"])}}
+        print(json.dumps(out), flush=True)
+    dist.destroy_process_group()
 
 
 def main():
@@ -193,12 +274,17 @@ def main():
     ap.add_argument("--variant", default="racy", choices=["racy", "clean"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "host"],
+                    help="config-5 shard exchange: NCCL device all_to_all, or gloo host staging")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.config == 5 and world > 1 and args.impl != "reference":
+        run_sharded_bench(args, world, rank, local_rank)
+        return
     trace = make_trace(args.config, args.variant)
 
     if args.impl == "reference":
@@ -271,7 +357,8 @@ def main():
     # e2e through the C-ABI host entry point: pinned host events -> H2D -> replay -> D2H
     e2e = None
     if not args.no_e2e:
-        pin = torch.empty(trace.n * 16, dtype=torch.uint8, pin_memory=True)
+        small = trace.n * 16 <= (4 << 30)
+        pin = torch.empty(trace.n * 16, dtype=torch.uint8, pin_memory=small)
         pin.numpy()[:] = trace.events.view(np.uint8)
         hout = torch.empty(cap * 16, dtype=torch.uint8, pin_memory=True)
         ke2 = max(3, min(K, 10))
@@ -292,6 +379,7 @@ def main():
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             e2e_s = float(tt[0])
         e2e = {"value": n_acc * world / e2e_s, "unit": UNIT, "h2d_bytes_per_step": int(trace.n * 16),
+               "host_memory": "pinned" if small else "pageable",
                "d2h_bytes_per_step": int(min(tot, cap) * 16 + 8), "ms_per_step": e2e_s * 1e3}
     clocks.stop()
 
