@@ -15,6 +15,8 @@ CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIBDIR = os.path.join(PKG, "lib")
 SO = os.path.join(LIBDIR, "libhirace.so")
+EXDIR = os.path.join(PKG, "examples")
+EXSO = os.path.join(LIBDIR, "libhirace_examples.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -27,23 +29,33 @@ def headers():
     return sorted(glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(INCLUDE, "*")))
 
 
-def stale() -> bool:
-    if not os.path.exists(SO):
+def ex_sources():
+    return sorted(glob.glob(os.path.join(EXDIR, "*.cu")))
+
+
+def stale(so, srcs) -> bool:
+    if not os.path.exists(so):
         return True
-    t = os.path.getmtime(SO)
-    return any(os.path.getmtime(p) > t for p in sources() + headers())
+    t = os.path.getmtime(so)
+    return any(os.path.getmtime(p) > t for p in srcs + headers())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not stale():
-        return SO
-    os.makedirs(LIBDIR, exist_ok=True)
+def _nvcc(so, srcs, verbose):
     cmd = [NVCC, *ARCH, "-lineinfo", "-O3", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "-shared",
-           "-I", INCLUDE, "-I", CSRC, "-o", SO + ".tmp", *sources()]
+           "-I", INCLUDE, "-I", CSRC, "-o", so + ".tmp", *srcs]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     subprocess.check_call(cmd)
-    os.replace(SO + ".tmp", SO)
+    os.replace(so + ".tmp", so)
+
+
+def build(force: bool = False, verbose: bool = False) -> str:
+    """libhirace.so (the checker) and libhirace_examples.so (native programs checked inline)."""
+    os.makedirs(LIBDIR, exist_ok=True)
+    if force or stale(SO, sources()):
+        _nvcc(SO, sources(), verbose)
+    if force or stale(EXSO, ex_sources()):
+        _nvcc(EXSO, ex_sources(), verbose)
     return SO
 
 

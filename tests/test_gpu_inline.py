@@ -1,0 +1,103 @@
+"""Inline mode: native CUDA programs checked by the device hooks while they run
+(hirace::on_access / hirace::barrier).  The race set of a data race is a
+property of the program, not of the schedule, so the inline result must equal the oracle on
+the trace generator's model of the same program (configs 1-4) and the closed forms."""
+import numpy as np
+import pytest
+
+import oracle
+import tracegen as tg
+from tests.helpers import CLS, skey
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import paper_conf_sc_jacobsonbg24_b200 as hr  # noqa: E402
+from paper_conf_sc_jacobsonbg24_b200 import examples as ex  # noqa: E402
+
+
+def odict(t):
+    k, c, _ = oracle.races_of(t)
+    return {int(a): int(b) for a, b in zip(k, c)}
+
+
+def rdict(r):
+    return {int(k): int(c) & 0xFF for k, c in zip(r["key"], r["cls_and_epoch"])}
+
+
+@pytest.mark.parametrize("racy", [False, True])
+@pytest.mark.parametrize("n,steps", [(128, 3), (512, 8)])
+def test_inline_stencil(racy, n, steps):
+    t = tg.cfg2(racy, n=n, steps=steps)
+    c = hr.Checker.for_trace(t)
+    buf = torch.rand(2 * n * n, device="cuda")
+    ex.stencil(c, buf, n, steps, racy)
+    got = rdict(c.collect())
+    want = odict(t)
+    assert got == want
+    if n == 512 and racy:
+        assert sorted(np.bincount(list(got.values()), minlength=4).tolist()) == [0, 0, 32768, 229376]
+    st = c.stats()
+    c.close()
+    assert st["dropped_reports"] == 0
+
+
+@pytest.mark.parametrize("bs", [32, 64])
+@pytest.mark.parametrize("racy", [0, 1, 2])
+def test_inline_reduction(bs, racy):
+    t = tg.cfg1([None, "post_init", "level"][racy], block_threads=bs)
+    c = hr.Checker.for_trace(t)
+    out = torch.zeros(8, device="cuda")
+    ex.reduce(c, out, bs, 8, racy)
+    assert rdict(c.collect()) == odict(t)
+    c.close()
+
+
+@pytest.mark.parametrize("racy", [0, 1, 2])
+def test_inline_multiphase_small(racy):
+    nb, phases = 6, 34
+    t = tg.cfg4([None, "G", "B"][racy], nb, 256, phases)
+    c = hr.Checker.for_trace(t)
+    AB = torch.rand(4 * nb * 256, device="cuda")
+    bar = torch.zeros(1, dtype=torch.int32, device="cuda")
+    ex.multiphase(c, AB, nb, phases, racy, bar)
+    assert rdict(c.collect()) == odict(t)
+    c.close()
+
+
+@pytest.mark.parametrize("racy", [1, 2])
+def test_inline_multiphase_full_closed_form(racy):
+    nb, phases = 592, 64
+    t_geom = dict(grid_blocks=nb, block_threads=256, warp_size=32, global_words=4 * nb * 256, smem_words=514)
+    c = hr.Checker(**t_geom)
+    AB = torch.rand(4 * nb * 256, device="cuda")
+    bar = torch.zeros(1, dtype=torch.int32, device="cuda")
+    ex.multiphase(c, AB, nb, phases, racy, bar)
+    d = rdict(c.collect())
+    c.close()
+    if racy == 1:
+        assert len(d) == 2 * 1182 and set(d.values()) == {CLS["GRID"]}
+    else:
+        assert len(d) == 301_920 and sum(v == CLS["BLOCK"] for v in d.values()) == 8_288
+        assert d[skey(0, 64)] == CLS["BLOCK"] and d[skey(3, 5)] == CLS["WARP"]
+
+
+@pytest.mark.parametrize("racy", [False, True])
+def test_inline_bfs(racy):
+    nindex, nlist = tg.rmat_graph(12, 8)
+    t = tg.cfg3("bfs", racy, graph=(nindex, nlist))
+    V, E = nindex.shape[0] - 1, nlist.shape[0]
+    buf = torch.empty(V + 1 + E + V, dtype=torch.int32, device="cuda")
+    buf[:V + 1] = torch.from_numpy(nindex.astype(np.int32))
+    buf[V + 1:V + 1 + E] = torch.from_numpy(nlist.astype(np.int32))
+    dist = buf[V + 1 + E:]
+    dist.fill_(2**31 - 1)
+    dist[int(np.argmax(nindex[1:] - nindex[:-1]))] = 0
+    c = hr.Checker.for_trace(t)
+    levels = ex.bfs(c, buf.data_ptr(), buf[:V + 1], buf[V + 1:V + 1 + E], dist, V, racy)
+    assert levels == t.batch_count()
+    assert rdict(c.collect()) == odict(t)
+    c.close()
