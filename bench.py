@@ -186,6 +186,74 @@ BASELINE_CFG = {
 }
 
 
+def measure_slowdown(dev: int, reps: int = 5) -> dict:
+    """Instrumented slowdown (BASELINE.json metric): native CUDA programs timed uninstrumented
+    and with every tracked access / barrier checked inline by the HiRace device hooks
+    (examples.cu).  Shadow resets are outside the timed regions."""
+    import torch
+
+    import paper_conf_sc_jacobsonbg24_b200 as hr
+    import tracegen as tg
+    from paper_conf_sc_jacobsonbg24_b200 import examples as ex
+
+    def timed(fn, prep=None):
+        fn()
+        torch.cuda.synchronize()
+        tot = 0.0
+        for _ in range(reps):
+            if prep:
+                prep()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fn()
+            b.record()
+            torch.cuda.synchronize()
+            tot += a.elapsed_time(b)
+        return tot / reps
+
+    out = {}
+    n, steps = 512, 8
+    c = hr.Checker(1024, 256, 32, 2 * n * n, 324, device=dev)
+    buf = torch.rand(2 * n * n, device=f"cuda:{dev}")
+    nat = timed(lambda: ex.stencil(None, buf, n, steps, True))
+    ins = timed(lambda: ex.stencil(c, buf, n, steps, True), c.reset)
+    out["cfg2_stencil_racy"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat}
+    c.close()
+    nb, phases = 592, 64
+    c = hr.Checker(nb, 256, 32, 4 * nb * 256, 514, device=dev)
+    AB = torch.rand(4 * nb * 256, device=f"cuda:{dev}")
+    bar = torch.zeros(1, dtype=torch.int32, device=f"cuda:{dev}")
+    nat = timed(lambda: ex.multiphase(None, AB, nb, phases, 0, bar))
+    ins = timed(lambda: ex.multiphase(c, AB, nb, phases, 0, bar), c.reset)
+    out["cfg4_multiphase_clean"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat}
+    c.close()
+    c = hr.Checker(1, 32, 32, 8, 32, device=dev)
+    o = torch.zeros(8, device=f"cuda:{dev}")
+    nat = timed(lambda: ex.reduce(None, o, 32, 8, 1))
+    ins = timed(lambda: ex.reduce(c, o, 32, 8, 1), c.reset)
+    out["cfg1_reduction_racy"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat}
+    c.close()
+    nindex, nlist = tg.rmat_graph(18, 16)
+    V, E = nindex.shape[0] - 1, nlist.shape[0]
+    gb = torch.empty(V + 1 + E + V, dtype=torch.int32, device=f"cuda:{dev}")
+    gb[:V + 1] = torch.from_numpy(nindex.astype(np.int32))
+    gb[V + 1:V + 1 + E] = torch.from_numpy(nlist.astype(np.int32))
+    dist = gb[V + 1 + E:]
+    src = int(np.argmax(nindex[1:] - nindex[:-1]))
+
+    def reset_dist():
+        dist.fill_(2**31 - 1)
+        dist[src] = 0
+
+    c = hr.Checker(-(-V // 256), 256, 32, V + 1 + E + V + V + 1, 0, device=dev)
+    nat = timed(lambda: ex.bfs(None, gb.data_ptr(), gb[:V + 1], gb[V + 1:V + 1 + E], dist, V, False), reset_dist)
+    ins = timed(lambda: ex.bfs(c, gb.data_ptr(), gb[:V + 1], gb[V + 1:V + 1 + E], dist, V, False),
+                lambda: (reset_dist(), c.reset()))
+    out["cfg3_bfs_rmat18_clean"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat}
+    c.close()
+    return out
+
+
 def run_sharded_bench(args, world, rank, local_rank):
     """Config 5 across `world` GPUs: each rank generates its blocks' events; per batch the events
     are bucketed by owner (64 KiB chunks of the 2^32-word space) on the GPU and exchanged with
@@ -274,6 +342,7 @@ def main():
     ap.add_argument("--variant", default="racy", choices=["racy", "clean"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-slowdown", action="store_true")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "host"],
                     help="config-5 shard exchange: NCCL device all_to_all, or gloo host staging")
     args = ap.parse_args()
@@ -389,6 +458,7 @@ def main():
         return
     peak, peak_kind = peaks()
     achieved = BYTES_PER_ACCESS * n_acc / (kern_ms / 1e3) / 1e9
+    slow = None if args.no_slowdown else measure_slowdown(local_rank)
     cpu = None
     if not args.no_cpu_baseline and world == 1:
         import oracle
@@ -412,6 +482,9 @@ def main():
         "gpu_launches": 2 * K,  # k_batches + k_replay (fused collect) per step
         "clocks": clocks.summary(),
         "check": {"flagged_words": flagged, "per_step": st},  # stats are per step (reset clears them)
+        "instrumented_slowdown": slow,
+        "shadow_overhead": {"bytes_per_tracked_word": 8, "ratio_to_tracked_bytes": 2.0,
+                            "iguard_ratio_context": 4.0},
     }
     print(json.dumps(out), flush=True)
     if world > 1:
