@@ -343,7 +343,6 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-slowdown", action="store_true")
-    ap.add_argument("--no-hint", action="store_true", help="do not promise block-grouped batches")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "host"],
                     help="config-5 shard exchange: NCCL device all_to_all, or gloo host staging")
     args = ap.parse_args()
@@ -371,8 +370,6 @@ def main():
 
     n_acc = word_accesses(trace.events)
     c = hr.Checker.for_trace(trace, device=local_rank)
-    # the generators emit natural per-block order: promise it (checked by the kernel)
-    c.set_hints(block_grouped=not args.no_hint)
     d_ev = hr.events_to_device(trace.events, f"cuda:{local_rank}")
     cap = 1 << 20
     d_out = torch.empty(cap * 16, dtype=torch.uint8, device="cuda")

@@ -63,15 +63,6 @@ typedef enum { HIRACE_SCOPE_WARP = 1, HIRACE_SCOPE_BLOCK = 2, HIRACE_SCOPE_GRID 
 typedef enum { HIRACE_RACE_WARP = 1, HIRACE_RACE_BLOCK = 2, HIRACE_RACE_GRID = 3 } hirace_race_class;
 
 #define HIRACE_MAX_BATCHES 32767u   /* distinct (g,b,w) batch keys per replay call */
-
-/* Trace-order hints (hirace_set_hints).  HIRACE_HINT_BLOCK_GROUPED: inside every batch the
- * events are ordered by block (non-decreasing tid / block_threads), as a per-block recorder
- * emits them.  The replay then keeps the shared-space records of the blocks that lie entirely
- * inside one CTA's share in that CTA's shared memory (the paper keeps shared variables' shadows
- * in shared memory).  The kernel checks the order of every adjacent event pair;
- * a trace that breaks the promise is reported as HIRACE_E_BAD_TRACE (its result is not
- * trustworthy), never silently accepted. */
-#define HIRACE_HINT_BLOCK_GROUPED 1u
 #define HIRACE_SHARED_BIT (1ull << 63)
 
 /* Tracked geometry.  warp_size may be any value >= 1 (2 reproduces the paper's Fig. 1 toy
@@ -211,9 +202,6 @@ hirace_status hirace_sync(hirace_ctx *ctx);
 /* Copies the device context for inline hooks into *out (host memory).  global_base is the
  * device address tracked global offsets are measured from (may be NULL for replay-only). */
 hirace_status hirace_get_dev_ctx(hirace_ctx *ctx, const void *global_base, hirace_dev_ctx *out);
-
-/* Sets the trace-order hints (HIRACE_HINT_*) used by later replays; 0 = no promise. */
-hirace_status hirace_set_hints(hirace_ctx *ctx, uint32_t hints);
 
 /* Measurement hook: when both are non-NULL, every later hirace_replay_trace records `start`
  * immediately before and `stop` immediately after its replay-kernel launch on the call's

@@ -278,14 +278,6 @@ hirace_status hirace_replay_trace(hirace_ctx *c, const hirace_event *d_events, u
     return HIRACE_OK;
 }
 
-hirace_status hirace_set_hints(hirace_ctx *c, uint32_t hints)
-{
-    if (!c || (hints & ~HIRACE_HINT_BLOCK_GROUPED))
-        return HIRACE_E_INVAL;
-    c->scr.hints = hints;
-    return HIRACE_OK;
-}
-
 hirace_status hirace_set_kernel_timing(hirace_ctx *c, void *start_event, void *stop_event)
 {
     if (!c || (!start_event) != (!stop_event))

@@ -23,7 +23,6 @@ struct Scratch {
     unsigned int *grid_bar2; /* grid barrier counter (standalone collect)                     */
     uint32_t *cta_cnt;       /* collect: per-CTA flagged-word counts, kMaxCtas                */
     int collect_grid;        /* co-resident CTAs of k_collect                                  */
-    uint32_t hints;          /* HIRACE_HINT_* of the context                                   */
 };
 
 /* batch discovery (one CTA): boundaries, sort, validation */

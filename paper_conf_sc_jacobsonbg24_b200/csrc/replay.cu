@@ -37,7 +37,6 @@ namespace {
 constexpr uint32_t FULL = 0xffffffffu;
 constexpr uint64_t NONE = ~0ull;
 constexpr int kMinBlocks = 2; /* 2 x 16 warps per SM at <= 64 registers */
-constexpr uint32_t kCacheWords = 12288; /* 96 KiB of shared memory per CTA for owned shared-space records */
 
 struct Batch {
     uint32_t key, g, b, w, ep; /* ep = epochs in record layout */
@@ -60,29 +59,6 @@ __device__ __forceinline__ uint4 ld_event(const uint4 *p)
     asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
                  : "l"(p));
-    return v;
-}
-
-/* Where a shadow record lives: the global array, or — for the shared-space words of blocks a
- * CTA owns in the current batch (block-grouped traces, HIRACE_HINT_BLOCK_GROUPED) — a copy in
- * the CTA's shared memory covering global shadow indices [base, base + len).  Generic
- * pointers let the same load / CAS code serve both. */
-struct ShadowMap {
-    unsigned long long *shadow;
-    unsigned long long *cache;
-    uint64_t base, len;
-    __device__ __forceinline__ unsigned long long *ptr(uint64_t idx) const
-    {
-        return idx - base < len ? cache + (idx - base) : shadow + idx;
-    }
-};
-
-/* coherent 8-byte load through a generic address (global: L2, never a stale L1 line; shared:
- * the CTA's copy) */
-__device__ __forceinline__ uint64_t ld_gen(const unsigned long long *p)
-{
-    uint64_t v;
-    asm volatile("ld.relaxed.gpu.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
 
@@ -183,7 +159,7 @@ __device__ __forceinline__ void append_reports(const hirace_dev_ctx &c, uint32_t
 /* chunks holding 8/16-byte accesses: word by word through the group commit (rare; the configs
  * emit 4-byte accesses).  `take` marks this lane's event as one to process here. */
 __device__ __noinline__ uint4 chunk_multiword(const hirace_dev_ctx c, const geom G, const unsigned char *tab,
-                                              const Batch B, uint4 e, bool take, uint32_t lane, const ShadowMap M)
+                                              const Batch B, uint4 e, bool take, uint32_t lane)
 {
     Counters cnt{0, 0, 0, 0};
     const uint64_t addr = ((uint64_t)e.y << 32) | e.x;
@@ -199,10 +175,10 @@ __device__ __noinline__ uint4 chunk_multiword(const hirace_dev_ctx c, const geom
         const uint32_t peers = __match_any_sync(FULL, my);
         cnt.checked += act;
         const bool lead = act && (peers & ((1u << lane) - 1)) == 0;
-        unsigned long long *const p = M.ptr(act ? my : 0);
-        const uint64_t o = lead ? ld_gen(p) : 0;
+        const uint64_t o = lead ? ld_coherent(c.shadow + my) : 0;
         uint32_t rtid = 0;
-        const uint32_t cls = commit_groups(p, o, lead ? peers : 0u, e.z, e.w & 3u, G, tab, B, cnt, rtid, true);
+        const uint32_t cls =
+            commit_groups(c.shadow + my, o, lead ? peers : 0u, e.z, e.w & 3u, G, tab, B, cnt, rtid, true);
         if (__any_sync(FULL, cls != 0))
             append_reports(c, cls, key_of(G, e, k), B.g, rtid, lane);
     }
@@ -234,19 +210,8 @@ struct Lane {
  * accesses of the chunk are committed right here, word by word */
 __device__ __forceinline__ Lane decode(const uint4 &e, bool valid, uint32_t keysz, const Batch &B,
                                        uint64_t total_threads, const hirace_dev_ctx &c, const geom &G,
-                                       const unsigned char *tab, Counters &cnt, uint32_t &bad, uint32_t lane,
-                                       const ShadowMap &M, bool grouped, uint32_t &last_blk)
+                                       const unsigned char *tab, Counters &cnt, uint32_t &bad, uint32_t lane)
 {
-    if (grouped) { /* HIRACE_HINT_BLOCK_GROUPED: blocks must not decrease along the batch */
-        const uint32_t blk = block_of(e.z, G);
-        const uint32_t prev = __shfl_up_sync(FULL, blk, 1);
-        const uint32_t pv = __shfl_up_sync(FULL, valid ? 1u : 0u, 1);
-        if (valid && ((lane > 0 && pv && blk < prev) || (lane == 0 && blk < last_blk)))
-            bad = 1;
-        const uint32_t nv = __popc(__ballot_sync(FULL, valid));
-        if (nv)
-            last_blk = __shfl_sync(FULL, blk, nv - 1);
-    }
     Lane L;
     L.tid = e.z;
     L.kind = e.w & 3u;
@@ -264,7 +229,7 @@ __device__ __forceinline__ Lane decode(const uint4 &e, bool valid, uint32_t keys
         if (valid && !L.ok && !multi)
             bad = 1;
         if (__any_sync(FULL, multi)) {
-            const uint4 d = chunk_multiword(c, G, tab, B, e, multi, lane, M);
+            const uint4 d = chunk_multiword(c, G, tab, B, e, multi, lane);
             cnt.checked += d.x;
             cnt.retry += d.y;
             cnt.cas += d.z;
@@ -297,9 +262,8 @@ template <bool P2>
 __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     k_replay(hirace_dev_ctx c, const uint4 *__restrict__ ev, const uint32_t *__restrict__ off,
              const uint32_t *__restrict__ nbp, unsigned int *bar, uint64_t shadow_words, hirace_race *out,
-             uint64_t cap, unsigned long long *d_total, uint32_t *cta_cnt, uint32_t hints, uint32_t cache_words)
+             uint64_t cap, unsigned long long *d_total, uint32_t *cta_cnt)
 {
-    extern __shared__ __align__(16) unsigned long long s_cache[]; /* cache_words records */
     __shared__ __align__(16) unsigned char s_table[2048];
     __shared__ unsigned long long s_stats[4];
     const uint32_t lane = threadIdx.x & 31;
@@ -328,32 +292,7 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
     uint4 e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
     uint4 e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
-    const bool grouped = (hints & HIRACE_HINT_BLOCK_GROUPED) != 0;
-    const uint32_t wpc = blockDim.x >> 5;
     for (uint32_t bi = 0; bi < nb; bi++) {
-        /* shared-space words of the blocks lying entirely inside this CTA's share of a
-         * block-grouped batch are owned by this CTA: copy them to shared memory */
-        ShadowMap M{c.shadow, s_cache, 0, 0};
-        uint32_t last_blk = 0;
-        if (grouped) {
-            uint32_t lo, hi, d0, d1;
-            warp_share(bstart, bend, blockIdx.x * wpc, nwarps, 0, lo, d0);
-            warp_share(bstart, bend, blockIdx.x * wpc + wpc - 1, nwarps, 0, d1, hi);
-            (void)d0;
-            (void)d1;
-            if (i - lane > bstart && i - lane < iend)
-                last_blk = block_of(__ldg(&ev[i - lane - 1].z), G);
-            if (hi > lo && c.smem_words && cache_words >= c.smem_words) {
-                const uint32_t bf = block_of(__ldg(&ev[lo].z), G), bl = block_of(__ldg(&ev[hi - 1].z), G);
-                const uint32_t nint = bl > bf + 1 ? bl - bf - 1 : 0;
-                const uint32_t ncache = min(nint, cache_words / c.smem_words);
-                M.base = c.global_words + (uint64_t)(bf + 1) * c.smem_words;
-                M.len = (uint64_t)ncache * c.smem_words;
-                for (uint32_t k = threadIdx.x; k < M.len; k += blockDim.x)
-                    s_cache[k] = __ldcg(c.shadow + M.base + k);
-            }
-            __syncthreads();
-        }
         Batch B;
         B.key = __ldg(&ev[bstart].w) >> 5;
         B.g = B.key >> 19;
@@ -365,15 +304,14 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
             bad = 1; /* reserved for retired RACE records (R7) */
 
         for (; i - lane < iend; i += 32) {
-            const Lane cur =
-                decode(e0, i < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane, M, grouped, last_blk);
+            const Lane cur = decode(e0, i < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
             e0 = e1; /* a1: keep the next chunks' events in flight */
             e1 = i + 64 < iend ? ld_event(ev + i + 64) : make_uint4(0, 0, 0, 0);
 
             /* a4: optimistic: every lane reads its own word (coherent load); lanes that share
              * a word are grouped only if their CAS collides (below) */
-            unsigned long long *const p = M.ptr(cur.ok ? cur.idx : 0);
-            const uint64_t o = cur.ok ? ld_gen(p) : 0;
+            unsigned long long *const p = c.shadow + cur.idx;
+            const uint64_t o = cur.ok ? ld_coherent(p) : 0;
             cnt.checked += cur.ok;
 
             /* a5: transition */
@@ -403,11 +341,6 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
             /* a7 */
             if (__any_sync(FULL, cls != 0))
                 append_reports(c, cls, key_of_idx(cur, c, G), B.g, rtid, lane);
-        }
-        if (M.len) { /* write the owned words back before anyone else may touch them */
-            __syncthreads();
-            for (uint32_t k = threadIdx.x; k < M.len; k += blockDim.x)
-                __stcg(c.shadow + M.base + k, s_cache[k]);
         }
         if (bi + 1 < nb) {
             bstart = __ldg(&off[bi + 1]);
@@ -451,10 +384,8 @@ int replay_max_grid(int device)
 {
     int sms = 0, occ = 0, occ2 = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    cudaFuncSetAttribute(k_replay<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCacheWords * 8);
-    cudaFuncSetAttribute(k_replay<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kCacheWords * 8);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_replay<true>, kReplayThreads, kCacheWords * 8);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_replay<false>, kReplayThreads, kCacheWords * 8);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_replay<true>, kReplayThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_replay<false>, kReplayThreads, 0);
     occ = occ < occ2 ? occ : occ2;
     if (occ < 1)
         occ = 1;
@@ -487,11 +418,10 @@ cudaError_t launch_replay(const hirace_dev_ctx &c, const hirace_event *ev, const
     hirace_race *o = out;
     unsigned long long *dt = d_total;
     uint32_t *cnt = s.cta_cnt;
-    uint32_t hints = s.hints, cw = kCacheWords;
-    void *args[] = {&cc, &evp, &offp, &nbp, &barp, &nw, &o, &cp, &dt, &cnt, &hints, &cw};
+    void *args[] = {&cc, &evp, &offp, &nbp, &barp, &nw, &o, &cp, &dt, &cnt};
     const bool p2 = (c.block_threads & (c.block_threads - 1)) == 0 && (c.warp_size & (c.warp_size - 1)) == 0;
     const void *fn = p2 ? (const void *)k_replay<true> : (const void *)k_replay<false>;
-    return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kReplayThreads), args, kCacheWords * 8, st);
+    return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kReplayThreads), args, 0, st);
 }
 
 } // namespace hirace_impl

@@ -20,7 +20,6 @@ READ, WRITE, ATOMIC_BLOCK, ATOMIC_GRID = 0, 1, 2, 3
 SCOPE_WARP, SCOPE_BLOCK, SCOPE_GRID = 1, 2, 3
 RACE_WARP, RACE_BLOCK, RACE_GRID = 1, 2, 3
 MAX_BATCHES = 32767
-HINT_BLOCK_GROUPED = 1
 
 STATUS = {0: "HIRACE_OK", -1: "HIRACE_E_INVAL", -2: "HIRACE_E_NOMEM", -3: "HIRACE_E_CUDA",
           -4: "HIRACE_E_CLOCK_OVERFLOW", -5: "HIRACE_E_REPORT_OVERFLOW", -6: "HIRACE_E_BAD_TRACE",
@@ -30,7 +29,7 @@ STATUS = {0: "HIRACE_OK", -1: "HIRACE_E_INVAL", -2: "HIRACE_E_NOMEM", -3: "HIRAC
 EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_free", "hirace_shadow_reset", "hirace_barrier",
            "hirace_replay_trace", "hirace_find_batches", "hirace_check_trace_device", "hirace_check_trace_host", "hirace_collect_races",
            "hirace_collect_races_device", "hirace_get_stats", "hirace_sync", "hirace_get_dev_ctx",
-           "hirace_bucket_events", "hirace_set_hints", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_fsm_table", "hirace_fsm_step", "hirace_status_string",
+           "hirace_bucket_events", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_fsm_table", "hirace_fsm_step", "hirace_status_string",
            "hirace_version")
 
 
@@ -88,7 +87,6 @@ def load():
         "hirace_get_dev_ctx": (I32, [P, P, ctypes.POINTER(DevCtx)]),
         "hirace_bucket_events": (I32, [P, P, U64, I32, I32, P, ctypes.POINTER(U64), P]),
         "hirace_set_kernel_timing": (I32, [P, P, P]),
-        "hirace_set_hints": (I32, [P, U32]),
         "hirace_microbench_atomics": (I32, [I32, U64, I32, I32, U64, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_microbench_grid_sync": (I32, [I32, I32, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_fsm_table": (I32, [P]),
@@ -271,11 +269,6 @@ class Checker:
                                                 ctypes.byref(total), _stream_handle(stream)),
                "hirace_check_trace_host")
         return int(total.value)
-
-    def set_hints(self, block_grouped: bool = False):
-        """Promise block-grouped batches (natural per-block order): shared-space records of owned
-        blocks are checked in shared memory.  A broken promise is reported as BAD_TRACE."""
-        _check(self.lib.hirace_set_hints(self.h, HINT_BLOCK_GROUPED if block_grouped else 0), "hirace_set_hints")
 
     def set_kernel_timing(self, start=None, stop=None):
         """torch.cuda.Event pair (already recorded once) or None: times the replay kernel."""

@@ -367,60 +367,3 @@ def test_cfg5_full_1e9_vs_construction_and_sampled_oracle():
     t = tg.cfg5()
     assert t.n > 1.07e9
     _cfg5_check(t)
-
-
-def _grouped_races(t):
-    c = hr.Checker.for_trace(t)
-    c.set_hints(block_grouped=True)
-    c.reset()
-    c.replay(hr.events_to_device(t.events))
-    r = c.collect()
-    st = c.stats()
-    c.close()
-    return r, st
-
-
-@pytest.mark.parametrize("make", [lambda: tg.cfg1("post_init"), lambda: tg.cfg1(None, block_threads=64),
-                                  lambda: tg.cfg2(True, n=128, steps=3), lambda: tg.cfg2(False, n=128, steps=3),
-                                  lambda: tg.cfg2(True), lambda: tg.cfg4("B", 6, 128, 34),
-                                  lambda: tg.cfg4("G", 40, 256, 34), lambda: tg.listing4(64, 3),
-                                  lambda: tg.listing3(4, 64)])
-def test_block_grouped_hint_shared_memory_shadow(make):
-    # natural (per-block) order satisfies HIRACE_HINT_BLOCK_GROUPED: owned blocks' shared-space
-    # records are checked in shared memory; the result must not change
-    t = make()
-    r, st = _grouped_races(t)
-    assert as_dict(r) == oracle_dict(t)
-    assert st["checked"] == word_accesses(t)
-    n, recs = _fused_hint(t)
-    assert as_dict(recs) == oracle_dict(t)
-
-
-def _fused_hint(t):
-    c = hr.Checker.for_trace(t)
-    c.set_hints(block_grouped=True)
-    c.reset()
-    out = torch.zeros((1 << 20) * 16, dtype=torch.uint8, device="cuda")
-    tot = torch.zeros(1, dtype=torch.int64, device="cuda")
-    c.check_device(hr.events_to_device(t.events), out, 1 << 20, tot)
-    torch.cuda.synchronize()
-    assert c.sync() == 0
-    n = int(tot.item())
-    recs = out.cpu().numpy().view(hr.RACE_DTYPE)[:n]
-    c.close()
-    return n, recs
-
-
-def test_block_grouped_hint_violation_is_reported():
-    t = tg.cfg2(True, n=128, steps=2, shuffle_seed=3)   # legal trace, but not block-grouped
-    c = hr.Checker.for_trace(t)
-    c.set_hints(block_grouped=True)
-    c.replay(hr.events_to_device(t.events))
-    with pytest.raises(hr.HiraceError) as e:
-        c.collect()
-    assert e.value.status == -6
-    c.reset()
-    c.set_hints(block_grouped=False)
-    c.replay(hr.events_to_device(t.events))
-    assert as_dict(c.collect()) == oracle_dict(t)
-    c.close()
