@@ -231,8 +231,9 @@ hirace_status hirace_bucket_events(hirace_ctx *ctx, const hirace_event *d_in, ui
 hirace_status hirace_microbench_atomics(int device, uint64_t nwords, int random, int op, uint64_t nops,
                                         double *ops_per_s, void *stream);
 
-/* Cost of one grid barrier of the persistent replay kernel (its grid size), microseconds. */
-hirace_status hirace_microbench_grid_sync(int device, int iters, double *us_per_barrier, void *stream);
+/* Cost of one grid barrier at the persistent replay kernel's grid size, microseconds.
+ * mode 0 = the library's barrier; 1 = busy polling; 2 = generation flag set by the last CTA. */
+hirace_status hirace_microbench_grid_sync(int device, int iters, int mode, double *us_per_barrier, void *stream);
 
 /* ---- verification hooks (host-only, NOT a replay path) --------------------------------- */
 

@@ -27,11 +27,11 @@ __device__ __forceinline__ void grid_sync(unsigned int *bar, unsigned int nctas,
         /* bar.sync above orders the CTA's accesses before this release (cumulativity) */
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(bar) : "memory");
         unsigned int v;
-        for (;;) { /* relaxed spin (no L1 invalidation per poll), one acquire fence after */
+        for (;;) { /* relaxed busy poll (no sleep: 1.5 vs 2.9 us per barrier on B200, no L1
+                      * invalidation per poll), one acquire fence after */
             asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
             if (v >= target)
                 break;
-            __nanosleep(20);
         }
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
     }

@@ -52,11 +52,48 @@ __global__ void __launch_bounds__(256) k_mb_atomics(unsigned long long *a, uint6
         *sink = acc;
 }
 
-__global__ void __launch_bounds__(kReplayThreads) k_mb_grid_sync(unsigned int *bar, int iters)
+/* barrier variants: 0 = grid_sync (library), 1 = no sleep while polling, 2 = last arriver
+ * flips a separate generation flag that the others poll */
+__device__ __forceinline__ void grid_sync_variant(unsigned int *bar, unsigned int nctas, unsigned int &epoch,
+                                                  int mode)
+{
+    if (mode == 0) {
+        grid_sync(bar, nctas, epoch);
+        return;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        epoch++;
+        if (mode == 1) {
+            const unsigned int target = epoch * nctas;
+            asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(bar) : "memory");
+            unsigned int v;
+            do {
+                asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
+            } while (v < target);
+        } else {
+            unsigned int *flag = bar + 32; /* another 128-byte line */
+            unsigned int old;
+            asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(bar) : "memory");
+            if (old == epoch * nctas - 1) {
+                asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(flag), "r"(epoch) : "memory");
+            } else {
+                unsigned int v;
+                do {
+                    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
+                } while (v < epoch);
+            }
+        }
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+    }
+    __syncthreads();
+}
+
+__global__ void __launch_bounds__(kReplayThreads) k_mb_grid_sync(unsigned int *bar, int iters, int mode)
 {
     unsigned int epoch = 0;
     for (int i = 0; i < iters; i++)
-        grid_sync(bar, gridDim.x, epoch);
+        grid_sync_variant(bar, gridDim.x, epoch, mode);
 }
 
 } // namespace
@@ -102,7 +139,8 @@ extern "C" hirace_status hirace_microbench_atomics(int device, uint64_t nwords, 
     return s;
 }
 
-extern "C" hirace_status hirace_microbench_grid_sync(int device, int iters, double *us_per_barrier, void *stream)
+extern "C" hirace_status hirace_microbench_grid_sync(int device, int iters, int mode, double *us_per_barrier,
+                                                     void *stream)
 {
     if (!us_per_barrier || iters < 1)
         return HIRACE_E_INVAL;
@@ -110,7 +148,7 @@ extern "C" hirace_status hirace_microbench_grid_sync(int device, int iters, doub
     if (cudaSetDevice(device) != cudaSuccess)
         return HIRACE_E_CUDA;
     unsigned int *bar = nullptr;
-    if (cudaMalloc(&bar, sizeof(unsigned int)) != cudaSuccess)
+    if (cudaMalloc(&bar, 64 * sizeof(unsigned int)) != cudaSuccess)
         return HIRACE_E_NOMEM;
     const int grid = replay_max_grid(device);
     cudaEvent_t e0, e1;
@@ -120,8 +158,8 @@ extern "C" hirace_status hirace_microbench_grid_sync(int device, int iters, doub
     hirace_status s = HIRACE_OK;
     for (int rep = 0; rep < 2; rep++) { /* iters and 1 barrier: the difference is the barrier cost */
         int it = rep == 0 ? iters : 1;
-        void *args[] = {&bar, &it};
-        cudaMemsetAsync(bar, 0, sizeof(unsigned int), st);
+        void *args[] = {&bar, &it, &mode};
+        cudaMemsetAsync(bar, 0, 64 * sizeof(unsigned int), st);
         cudaEventRecord(e0, st);
         if (cudaLaunchCooperativeKernel((const void *)k_mb_grid_sync, dim3(grid), dim3(kReplayThreads), args, 0, st) !=
             cudaSuccess)

@@ -32,6 +32,17 @@ namespace hirace_impl {
 
 using namespace hirace;
 
+#ifdef HIRACE_BARRIER_TRACE
+/* diagnostics build only: per (batch, CTA) globaltimer at arrival and after release */
+__device__ unsigned long long g_bar_trace[128 * 2048 * 2];
+__device__ __forceinline__ unsigned long long gtimer()
+{
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#endif
+
 namespace {
 
 constexpr uint32_t FULL = 0xffffffffu;
@@ -348,7 +359,16 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
             warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
             e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
             e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
+#ifdef HIRACE_BARRIER_TRACE
+            __syncthreads();
+            if (threadIdx.x == 0 && bi < 128 && blockIdx.x < 2048)
+                g_bar_trace[(bi * 2048 + blockIdx.x) * 2] = gtimer();
+#endif
             grid_sync(bar, gridDim.x, bar_epoch);
+#ifdef HIRACE_BARRIER_TRACE
+            if (threadIdx.x == 0 && bi < 128 && blockIdx.x < 2048)
+                g_bar_trace[(bi * 2048 + blockIdx.x) * 2 + 1] = gtimer();
+#endif
         }
     }
 
@@ -379,6 +399,13 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
 }
 
 } // namespace
+
+#ifdef HIRACE_BARRIER_TRACE
+extern "C" int hirace_debug_barrier_trace(unsigned long long *host, uint64_t n)
+{
+    return (int)cudaMemcpyFromSymbol(host, g_bar_trace, n * sizeof(unsigned long long));
+}
+#endif
 
 int replay_max_grid(int device)
 {

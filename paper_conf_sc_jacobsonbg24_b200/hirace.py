@@ -88,7 +88,7 @@ def load():
         "hirace_bucket_events": (I32, [P, P, U64, I32, I32, P, ctypes.POINTER(U64), P]),
         "hirace_set_kernel_timing": (I32, [P, P, P]),
         "hirace_microbench_atomics": (I32, [I32, U64, I32, I32, U64, ctypes.POINTER(ctypes.c_double), P]),
-        "hirace_microbench_grid_sync": (I32, [I32, I32, ctypes.POINTER(ctypes.c_double), P]),
+        "hirace_microbench_grid_sync": (I32, [I32, I32, I32, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_fsm_table": (I32, [P]),
         "hirace_fsm_step": (U64, [U64, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
         "hirace_status_string": (ctypes.c_char_p, [I32]),
@@ -126,10 +126,10 @@ def microbench_atomics(nwords: int, random: bool, op: int, nops: int, device: in
     return r.value
 
 
-def microbench_grid_sync(iters: int = 200, device: int = 0, stream=None) -> float:
-    """Microseconds per grid barrier of the persistent replay kernel."""
+def microbench_grid_sync(iters: int = 200, mode: int = 0, device: int = 0, stream=None) -> float:
+    """Microseconds per grid barrier of the persistent replay kernel (mode: see hirace.h)."""
     r = ctypes.c_double(0)
-    _check(load().hirace_microbench_grid_sync(device, iters, ctypes.byref(r), _stream_handle(stream)),
+    _check(load().hirace_microbench_grid_sync(device, iters, mode, ctypes.byref(r), _stream_handle(stream)),
            "hirace_microbench_grid_sync")
     return r.value
 

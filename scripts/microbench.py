@@ -9,7 +9,7 @@ import torch  # noqa: E402
 from paper_conf_sc_jacobsonbg24_b200 import hirace as h  # noqa: E402
 
 torch.cuda.set_device(0)
-out = {"grid_sync_us": h.microbench_grid_sync(400)}
+out = {f"grid_sync_mode{m}_us": h.microbench_grid_sync(400, m) for m in (0, 1, 2)}
 ops = {0: "cas", 1: "add", 2: "load", 3: "load+cas"}
 for label, nwords in (("l2_4MiB", 1 << 19), ("l2_32MiB", 1 << 22), ("hbm_4GiB", 1 << 29)):
     for rnd in (0, 1):
