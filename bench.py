@@ -217,7 +217,9 @@ def measure_slowdown(dev: int, reps: int = 5) -> dict:
     buf = torch.rand(2 * n * n, device=f"cuda:{dev}")
     nat = timed(lambda: ex.stencil(None, buf, n, steps, True))
     ins = timed(lambda: ex.stencil(c, buf, n, steps, True), c.reset)
-    out["cfg2_stencil_racy"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat}
+    ins_g = timed(lambda: ex.stencil(c, buf, n, steps, True, smem_shadow=False), c.reset)
+    out["cfg2_stencil_racy"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat,
+                                "slowdown_global_shadow": ins_g / nat}
     c.close()
     nb, phases = 592, 64
     c = hr.Checker(nb, 256, 32, 4 * nb * 256, 514, device=dev)
@@ -225,7 +227,9 @@ def measure_slowdown(dev: int, reps: int = 5) -> dict:
     bar = torch.zeros(1, dtype=torch.int32, device=f"cuda:{dev}")
     nat = timed(lambda: ex.multiphase(None, AB, nb, phases, 0, bar))
     ins = timed(lambda: ex.multiphase(c, AB, nb, phases, 0, bar), c.reset)
-    out["cfg4_multiphase_clean"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat}
+    ins_g = timed(lambda: ex.multiphase(c, AB, nb, phases, 0, bar, smem_shadow=False), c.reset)
+    out["cfg4_multiphase_clean"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat,
+                                    "slowdown_global_shadow": ins_g / nat}
     c.close()
     c = hr.Checker(1, 32, 32, 8, 32, device=dev)
     o = torch.zeros(8, device=f"cuda:{dev}")

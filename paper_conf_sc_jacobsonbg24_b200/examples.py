@@ -20,9 +20,9 @@ def load():
             raise RuntimeError(f"{_LIB} missing: python -m paper_conf_sc_jacobsonbg24_b200.build")
         lib = ctypes.CDLL(_LIB)
         P, I, U = ctypes.c_void_p, ctypes.c_int, ctypes.c_uint
-        lib.hx_stencil.argtypes = [P, P, I, I, I, U, P]
-        lib.hx_reduce.argtypes = [P, P, I, I, I, U, P]
-        lib.hx_multiphase.argtypes = [P, P, I, I, I, I, I, P, U, P]
+        lib.hx_stencil.argtypes = [P, P, I, I, I, U, I, P]
+        lib.hx_reduce.argtypes = [P, P, I, I, I, U, I, P]
+        lib.hx_multiphase.argtypes = [P, P, I, I, I, I, I, P, U, I, P]
         lib.hx_bfs.argtypes = [P, P, P, P, I, I, U, ctypes.POINTER(I), P]
         for f in (lib.hx_stencil, lib.hx_reduce, lib.hx_multiphase, lib.hx_bfs):
             f.restype = I
@@ -42,27 +42,30 @@ def _ok(rc, name):
         raise RuntimeError(f"{name}: CUDA error {rc}")
 
 
-def stencil(checker, buf, n: int, steps: int, racy: bool, g0: int = 0, stream=None):
-    """buf: CUDA float32 tensor of 2 n^2 (A then B; the tracked global base)."""
+def stencil(checker, buf, n: int, steps: int, racy: bool, g0: int = 0, smem_shadow: bool = True, stream=None):
+    """buf: CUDA float32 tensor of 2 n^2 (A then B; the tracked global base).  smem_shadow: keep the
+    tile's shadow records in shared memory (else in the context's global shadow)."""
     d, p = _ctx(checker, buf.data_ptr())
-    _ok(load().hx_stencil(p, ctypes.c_void_p(buf.data_ptr()), n, steps, int(racy), g0, _stream_handle(stream)),
-        "hx_stencil")
+    _ok(load().hx_stencil(p, ctypes.c_void_p(buf.data_ptr()), n, steps, int(racy), g0, int(smem_shadow),
+                          _stream_handle(stream)), "hx_stencil")
 
 
-def reduce(checker, out, block_threads: int, passes: int, racy: int, g0: int = 0, stream=None):
+def reduce(checker, out, block_threads: int, passes: int, racy: int, g0: int = 0, smem_shadow: bool = True,
+           stream=None):
     """racy: 0 clean, 1 post-init barrier dropped, 2 first level barrier dropped."""
     d, p = _ctx(checker, out.data_ptr())
-    _ok(load().hx_reduce(p, ctypes.c_void_p(out.data_ptr()), block_threads, passes, racy, g0,
+    _ok(load().hx_reduce(p, ctypes.c_void_p(out.data_ptr()), block_threads, passes, racy, g0, int(smem_shadow),
                          _stream_handle(stream)), "hx_reduce")
 
 
 def multiphase(checker, AB, grid: int, phases: int, racy: int, bar, racy_phase_g: int = 31, racy_phase_b: int = 7,
-               g0: int = 0, stream=None):
+               g0: int = 0, smem_shadow: bool = True, stream=None):
     """racy: 0 clean, 1 grid barrier after racy_phase_g demoted, 2 tile barrier of racy_phase_b dropped."""
     d, p = _ctx(checker, AB.data_ptr())
     bar.zero_()
     _ok(load().hx_multiphase(p, ctypes.c_void_p(AB.data_ptr()), grid, phases, racy, racy_phase_g, racy_phase_b,
-                             ctypes.c_void_p(bar.data_ptr()), g0, _stream_handle(stream)), "hx_multiphase")
+                             ctypes.c_void_p(bar.data_ptr()), g0, int(smem_shadow), _stream_handle(stream)),
+        "hx_multiphase")
 
 
 def bfs(checker, base, nindex, nlist, dist, V: int, racy: bool, g0: int = 0, stream=None) -> int:

@@ -28,13 +28,14 @@ def rdict(r):
     return {int(k): int(c) & 0xFF for k, c in zip(r["key"], r["cls_and_epoch"])}
 
 
+@pytest.mark.parametrize("smem", [True, False])
 @pytest.mark.parametrize("racy", [False, True])
 @pytest.mark.parametrize("n,steps", [(128, 3), (512, 8)])
-def test_inline_stencil(racy, n, steps):
+def test_inline_stencil(racy, n, steps, smem):
     t = tg.cfg2(racy, n=n, steps=steps)
     c = hr.Checker.for_trace(t)
     buf = torch.rand(2 * n * n, device="cuda")
-    ex.stencil(c, buf, n, steps, racy)
+    ex.stencil(c, buf, n, steps, racy, smem_shadow=smem)
     got = rdict(c.collect())
     want = odict(t)
     assert got == want
@@ -45,31 +46,33 @@ def test_inline_stencil(racy, n, steps):
     assert st["dropped_reports"] == 0
 
 
+@pytest.mark.parametrize("smem", [True, False])
 @pytest.mark.parametrize("bs", [32, 64])
 @pytest.mark.parametrize("racy", [0, 1, 2])
-def test_inline_reduction(bs, racy):
+def test_inline_reduction(bs, racy, smem):
     t = tg.cfg1([None, "post_init", "level"][racy], block_threads=bs)
     c = hr.Checker.for_trace(t)
     out = torch.zeros(8, device="cuda")
-    ex.reduce(c, out, bs, 8, racy)
+    ex.reduce(c, out, bs, 8, racy, smem_shadow=smem)
     assert rdict(c.collect()) == odict(t)
     c.close()
 
 
+@pytest.mark.parametrize("smem", [True, False])
 @pytest.mark.parametrize("racy", [0, 1, 2])
-def test_inline_multiphase_small(racy):
+def test_inline_multiphase_small(racy, smem):
     nb, phases = 6, 34
     t = tg.cfg4([None, "G", "B"][racy], nb, 256, phases)
     c = hr.Checker.for_trace(t)
     AB = torch.rand(4 * nb * 256, device="cuda")
     bar = torch.zeros(1, dtype=torch.int32, device="cuda")
-    ex.multiphase(c, AB, nb, phases, racy, bar)
+    ex.multiphase(c, AB, nb, phases, racy, bar, smem_shadow=smem)
     assert rdict(c.collect()) == odict(t)
     c.close()
 
 
 @pytest.mark.parametrize("racy", [1, 2])
-def test_inline_multiphase_full_closed_form(racy):
+def test_inline_multiphase_full_closed_form(racy):  # shared-variable shadows in shared memory
     nb, phases = 592, 64
     t_geom = dict(grid_blocks=nb, block_threads=256, warp_size=32, global_words=4 * nb * 256, smem_words=514)
     c = hr.Checker(**t_geom)
@@ -100,4 +103,17 @@ def test_inline_bfs(racy):
     levels = ex.bfs(c, buf.data_ptr(), buf[:V + 1], buf[V + 1:V + 1 + E], dist, V, racy)
     assert levels == t.batch_count()
     assert rdict(c.collect()) == odict(t)
+    c.close()
+
+
+def test_inline_sticky_race_across_launches_with_smem_shadow():
+    # a shared word that raced in launch g=0 stays RACE (class from g*) after clean launches:
+    # the shared-memory shadow is loaded from and written back to the context every launch
+    t = tg.cfg1("post_init")
+    c = hr.Checker.for_trace(t)
+    out = torch.zeros(8, device="cuda")
+    ex.reduce(c, out, 32, 1, 1, g0=0)            # racy pass
+    ex.reduce(c, out, 32, 3, 0, g0=1)            # clean passes
+    got = rdict(c.collect())
+    assert got == {skey(0, w): CLS["WARP"] for w in range(16, 32)}
     c.close()
