@@ -62,6 +62,13 @@ typedef enum { HIRACE_SCOPE_WARP = 1, HIRACE_SCOPE_BLOCK = 2, HIRACE_SCOPE_GRID 
 /* Race class = the coarsest hierarchy level of the first racing epoch (R6). */
 typedef enum { HIRACE_RACE_WARP = 1, HIRACE_RACE_BLOCK = 2, HIRACE_RACE_GRID = 3 } hirace_race_class;
 
+/* Conflict policy (R2 / SURVEY §8(f) f2).  STRICT (default, the paper's Table 1
+ * reading): a plain read conflicts with an atomic; atomics of different blocks conflict unless
+ * both are grid-scope.  RELAXED_READ_ATOMIC: a plain read never conflicts with an atomic and
+ * atomics of one block never conflict; across blocks AB-AB and AB-AG still do.  Writes conflict
+ * with everything under both. */
+typedef enum { HIRACE_POLICY_STRICT = 0, HIRACE_POLICY_RELAXED_READ_ATOMIC = 1 } hirace_policy;
+
 #define HIRACE_MAX_BATCHES 32767u   /* distinct (g,b,w) batch keys per replay call */
 #define HIRACE_SHARED_BIT (1ull << 63)
 
@@ -235,17 +242,30 @@ hirace_status hirace_microbench_atomics(int device, uint64_t nwords, int random,
  * mode 0 = the library's barrier; 1 = busy polling; 2 = generation flag set by the last CTA. */
 hirace_status hirace_microbench_grid_sync(int device, int iters, int mode, double *us_per_barrier, void *stream);
 
+/* Selects the conflict policy of a context by uploading that policy's FSM table (stream-ordered
+ * on `stream`).  Takes effect for later replays and inline launches; call it on a reset shadow
+ * (records written under one policy are states of that policy's automaton).
+ * Errors: INVAL (NULL ctx, unknown policy), CUDA. */
+hirace_status hirace_set_policy(hirace_ctx *ctx, int policy, void *stream);
+
 /* ---- verification hooks (host-only, NOT a replay path) --------------------------------- */
 
 /* Writes the 2048-byte FSM transition table: entry[state<<6 | kind<<4 | sync<<2 | rel] =
  * next_state:5 | keep_record:1 | report:1 (PAPER.md L295 flat-array encoding). */
 hirace_status hirace_fsm_table(unsigned char out[2048]);
 
+/* hirace_fsm_table for a given hirace_policy.  Errors: INVAL (NULL out, unknown policy). */
+hirace_status hirace_fsm_table_policy(int policy, unsigned char out[2048]);
+
 /* One FSM step on the host with the same inline function the kernels use, for model checking:
  * returns the new 64-bit record for old record `old_shadow` and one access. *report is set to
  * 1 if the step enters or upgrades a RACE state. */
 uint64_t hirace_fsm_step(uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t b, uint32_t w,
                          uint32_t block_threads, uint32_t warp_size, int *report);
+
+/* hirace_fsm_step under a given hirace_policy (unknown values select STRICT). */
+uint64_t hirace_fsm_step_policy(int policy, uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t b,
+                                uint32_t w, uint32_t block_threads, uint32_t warp_size, int *report);
 
 const char *hirace_status_string(hirace_status s);
 

@@ -39,15 +39,17 @@ def _load():
     if _lib is None:
         build()
         lib = ctypes.CDLL(_SO)
-        lib.oracle_races.restype = ctypes.c_int64
-        lib.oracle_races.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
-                                     ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64]
+        lib.oracle_races_policy.restype = ctypes.c_int64
+        lib.oracle_races_policy.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                                            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                                            ctypes.c_int]
         _lib = lib
     return _lib
 
 
-def races(events: np.ndarray, block_threads: int, warp_size: int):
-    """Oracle-D.  Returns (keys u64[], cls u8[], gstar u8[]) sorted by key."""
+def races(events: np.ndarray, block_threads: int, warp_size: int, policy: int = 0):
+    """Oracle-D.  Returns (keys u64[], cls u8[], gstar u8[]) sorted by key.  policy 0 = strict
+    conflict rule (C1.3), 1 = relaxed read-vs-atomic (R2b)."""
     lib = _load()
     ev = np.ascontiguousarray(events)
     n = int(ev.shape[0])
@@ -56,8 +58,8 @@ def races(events: np.ndarray, block_threads: int, warp_size: int):
         keys = np.empty(cap, np.uint64)
         cls = np.empty(cap, np.uint8)
         gs = np.empty(cap, np.uint8)
-        r = lib.oracle_races(ev.ctypes.data if n else None, n, block_threads, warp_size,
-                             keys.ctypes.data, cls.ctypes.data, gs.ctypes.data, cap)
+        r = lib.oracle_races_policy(ev.ctypes.data if n else None, n, block_threads, warp_size,
+                                    keys.ctypes.data, cls.ctypes.data, gs.ctypes.data, cap, policy)
         if r < 0:
             raise RuntimeError(f"oracle_races failed ({r})")
         if r <= cap:
@@ -65,10 +67,10 @@ def races(events: np.ndarray, block_threads: int, warp_size: int):
         cap = int(r)
 
 
-def races_of(trace):
-    return races(trace.events, trace.block_threads, trace.warp_size)
+def races_of(trace, policy: int = 0):
+    return races(trace.events, trace.block_threads, trace.warp_size, policy)
 
 
-def races_dict(trace) -> dict:
-    k, c, _ = races_of(trace)
+def races_dict(trace, policy: int = 0) -> dict:
+    k, c, _ = races_of(trace, policy)
     return {int(a): int(b) for a, b in zip(k, c)}

@@ -40,10 +40,13 @@ def concurrent(a, c):
     return wp1 != wp2 or w1 == w2
 
 
-def conflict(a, c):
-    """C1.3."""
+def conflict(a, c, policy=0):
+    """C1.3.  policy 1 = relaxed: a plain read never conflicts with an
+    atomic (reading R2b)."""
     k1, k2 = a[2], c[2]
     if k1 == R and k2 == R:
+        return False
+    if policy == 1 and W not in (k1, k2) and R in (k1, k2):
         return False
     if k1 in (AB, AG) and k2 in (AB, AG):
         if k1 == AG and k2 == AG:
@@ -60,14 +63,14 @@ def level(a, c):
     return WARP
 
 
-def races(events, block_threads, warp_size):
+def races(events, block_threads, warp_size, policy=0):
     """Returns {key: (class, g*)} by literal enumeration of all pairs (C1.4-C1.6)."""
     acc = accesses(events, block_threads, warp_size)
     pairs = {}
     for i in range(len(acc)):
         for j in range(i + 1, len(acc)):
             a, c = acc[i], acc[j]
-            if a[0] == c[0] and concurrent(a, c) and conflict(a, c):
+            if a[0] == c[0] and concurrent(a, c) and conflict(a, c, policy):
                 # racing pair: record (g, b, level); b is shared by intra-block pairs
                 pairs.setdefault(a[0], []).append((a[3], a[4], level(a, c)))
     out = {}

@@ -19,6 +19,9 @@
  *   C1.3  Conflict: R-R never; atomic-atomic only if not both grid-scope and the two threads
  *         are in different blocks; every other pair (incl. plain read vs atomic) conflicts
  *         ("at least one of the accesses is a write", L223-229; readings R2, R3)
+ *         policy 1 (RELAXED_READ_ATOMIC, reading R2b): a pair
+ *         conflicts iff one is a write, or both are atomics of different blocks and not both
+ *         grid-scope (a plain read never conflicts with an atomic)
  *   C1.4  racing pair = Concurrent and Conflict; level GRID / BLOCK / WARP
  *   C1.5  a key is flagged iff it has a racing pair
  *   C1.6  class: g* = smallest g with a racing pair; GRID if a racing pair of g* is GRID-level;
@@ -55,8 +58,10 @@ static const uint64_t SHARED = 1ull << 63;
 static int is_atomic(uint32_t k) { return k == K_ATOMIC_BLOCK || k == K_ATOMIC_GRID; }
 
 /* C1.3 */
-static int conflict(uint32_t k1, uint32_t k2, int same_block)
+static int conflict(uint32_t k1, uint32_t k2, int same_block, int policy)
 {
+    if (policy == 1 && (k1 == K_READ || k2 == K_READ) && k1 != K_WRITE && k2 != K_WRITE)
+        return 0; /* read vs read or read vs atomic */
     if (k1 == K_READ && k2 == K_READ)
         return 0;
     if (is_atomic(k1) && is_atomic(k2)) {
@@ -70,11 +75,11 @@ static int conflict(uint32_t k1, uint32_t k2, int same_block)
 }
 
 /* exists i != j with kind k1 in masks[i], kind k2 in masks[j], conflict(k1,k2) */
-static int distinct_conflict(const uint8_t *masks, size_t n, int same_block)
+static int distinct_conflict(const uint8_t *masks, size_t n, int same_block, int policy)
 {
     for (uint32_t k1 = 0; k1 < 4; k1++) {
         for (uint32_t k2 = 0; k2 < 4; k2++) {
-            if (!conflict(k1, k2, same_block))
+            if (!conflict(k1, k2, same_block, policy))
                 continue;
             size_t c1 = 0, c2 = 0, f1 = 0, f2 = 0;
             for (size_t i = 0; i < n; i++) {
@@ -134,9 +139,11 @@ static int masks_push(masks_t *s, uint8_t v)
  * by C1.2/C1.3 and is reported so a test can pin it).
  * out_g receives g* (the grid epoch of the first racing pair).
  */
-int64_t oracle_races(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
-                     uint64_t *out_key, uint8_t *out_cls, uint8_t *out_g, uint64_t cap)
+int64_t oracle_races_policy(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
+                            uint64_t *out_key, uint8_t *out_cls, uint8_t *out_g, uint64_t cap, int policy)
 {
+    if (policy != 0 && policy != 1)
+        return -1;
     if (block_threads == 0 || warp_size == 0 || (n && !ev))
         return -1;
     /* C1.1: expand to word-level accesses */
@@ -235,13 +242,13 @@ int64_t oracle_races(const oracle_event *ev, uint64_t n, uint32_t block_threads,
                                 if (masks_push(&threads, tmask))
                                     err = -1;
                             }
-                            if (distinct_conflict(threads.m, threads.n, 1))
+                            if (distinct_conflict(threads.m, threads.n, 1, policy))
                                 warp_race = 1;
                             xs = xe;
                         }
                         ws = we;
                     }
-                    int block_race = distinct_conflict(warps.m, warps.n, 1);
+                    int block_race = distinct_conflict(warps.m, warps.n, 1, policy);
                     if ((block_race || warp_race) && (!have_min_b || b < min_b)) {
                         have_min_b = 1;
                         min_b = b;
@@ -253,7 +260,7 @@ int64_t oracle_races(const oracle_event *ev, uint64_t n, uint32_t block_threads,
                 }
                 bs = be;
             }
-            int grid_race = distinct_conflict(blocks.m, blocks.n, 0);
+            int grid_race = distinct_conflict(blocks.m, blocks.n, 0, policy);
             if (grid_race) {
                 cls = CLS_GRID;
             } else if (have_min_b) {
@@ -282,4 +289,10 @@ int64_t oracle_races(const oracle_event *ev, uint64_t n, uint32_t block_threads,
     free(threads.m);
     free(acc);
     return err ? err : nflag;
+}
+
+int64_t oracle_races(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
+                     uint64_t *out_key, uint8_t *out_cls, uint8_t *out_g, uint64_t cap)
+{
+    return oracle_races_policy(ev, n, block_threads, warp_size, out_key, out_cls, out_g, cap, 0);
 }

@@ -153,11 +153,155 @@ Out rules(int s, uint32_t k, uint32_t sync, uint32_t rel)
     return {find(G_T, join(KT, ck), KBp, KGp), true, false};
 }
 
+/* ---- relaxed read-vs-atomic policy (reading R2 alternative) ----
+ * Conflicts: W with anything; across blocks AB-AB and AB-AG.  A plain read never conflicts with
+ * an atomic, and atomics of one block never conflict.  Inside a block only W matters (classes
+ * N = non-write, X = write).  Across blocks a block's kinds summarise into the chain
+ * R < RAG (some AG) < RAB (some AB) < X (some W): a new R is compatible unless X, an AG only
+ * with R/RAG, an AB only with R.  With >= 2 blocks and no race the configurations are:
+ *   G_R   only reads;                       G_AG1 AG in exactly one block (the record's), R elsewhere;
+ *   G_AGn AG in >= 2 blocks, R elsewhere;   G_AB1 AB (+ maybe AG) in exactly one block (the record's).
+ * State codes keep INIT = 0 and RACE_W/B/G = 20/21/22. */
+namespace relaxed {
+
+enum { N = 0, X = 1 };
+enum { GR = 0, GRAG = 1, GRAB = 2, GX = 3 };
+enum { S_INIT = 0, T0 = 1, W0 = 7, B0 = 12, G_R = 16, G_AG1 = 17, G_AGn = 18, G_AB1 = 19 };
+
+struct RDesc {
+    Group grp;
+    int a, b, c; /* T: KT, KB, KG   W: KB, KG   B: KG */
+};
+
+const RDesc kR[hirace::ST_COUNT] = {
+    {G_INIT, 0, 0, 0},
+    {G_T, N, N, GR},  {G_T, N, N, GRAG}, {G_T, N, N, GRAB}, {G_T, N, N, GX}, {G_T, N, X, GX}, {G_T, X, X, GX},
+    {G_W, N, GR, 0},  {G_W, N, GRAG, 0}, {G_W, N, GRAB, 0}, {G_W, N, GX, 0}, {G_W, X, GX, 0},
+    {G_B, GR, 0, 0},  {G_B, GRAG, 0, 0}, {G_B, GRAB, 0, 0}, {G_B, GX, 0, 0},
+    {G_G, 0, 0, 0},   {G_G, 1, 0, 0},    {G_G, 2, 0, 0},    {G_G, 3, 0, 0},
+    {G_RACE, 1, 0, 0}, {G_RACE, 2, 0, 0}, {G_RACE, 3, 0, 0},
+};
+
+int clsL(uint32_t k) { return k == HIRACE_WRITE ? X : N; }
+int clsG(uint32_t k)
+{
+    return k == HIRACE_READ ? GR : (k == HIRACE_ATOMIC_GRID ? GRAG : (k == HIRACE_ATOMIC_BLOCK ? GRAB : GX));
+}
+int jmax(int x, int y) { return x > y ? x : y; }
+
+int findT(int kt, int kb, int kg)
+{
+    for (int s = T0; s < W0; s++)
+        if (kR[s].a == kt && kR[s].b == kb && kR[s].c == kg)
+            return s;
+    return -1;
+}
+int findW(int kb, int kg)
+{
+    for (int s = W0; s < B0; s++)
+        if (kR[s].a == kb && kR[s].b == kg)
+            return s;
+    return -1;
+}
+int findB(int kg) { return B0 + kg; }
+
+Out rules(int s, uint32_t k, uint32_t sync, uint32_t rel)
+{
+    using namespace hirace;
+    const RDesc d = kR[s];
+    const int RW = ST_RACE_W, RB = ST_RACE_B, RG = ST_RACE_G;
+    /* rule 0: RACE records are frozen; class upgrades inside the first racing epoch */
+    if (d.grp == G_RACE) {
+        if (sync == SYNC_GS)
+            return {s, true, false};
+        if (s == RW && rel == REL_B && sync == SYNC_US)
+            return {RB, true, true};
+        if ((s == RW || s == RB) && rel == REL_G)
+            return {RG, true, true};
+        return {s, true, false};
+    }
+    /* rule 1 */
+    if (d.grp == G_INIT || sync == SYNC_GS)
+        return {findT(clsL(k), clsL(k), clsG(k)), false, false};
+    const bool same = rel != REL_G;
+    /* rule 2: >= 2 blocks in the grid epoch */
+    if (d.grp == G_G) {
+        if (k == HIRACE_WRITE)
+            return {RG, false, true};
+        switch (s) {
+        case G_R:
+            if (k == HIRACE_READ)
+                return {G_R, true, false};
+            return {k == HIRACE_ATOMIC_GRID ? G_AG1 : G_AB1, false, false}; /* record := the atomic's block */
+        case G_AG1:
+            if (k == HIRACE_READ)
+                return {G_AG1, true, false};
+            if (k == HIRACE_ATOMIC_GRID)
+                return {same ? G_AG1 : G_AGn, true, false};
+            return same ? Out{G_AB1, true, false} : Out{RG, false, true}; /* AB */
+        case G_AGn:
+            if (k == HIRACE_ATOMIC_BLOCK)
+                return {RG, false, true};
+            return {G_AGn, true, false};
+        default: /* G_AB1 */
+            if (k == HIRACE_READ || same)
+                return {G_AB1, true, false};
+            return {RG, false, true};
+        }
+    }
+    int KT = N, KB, KG;
+    if (d.grp == G_T) {
+        KT = d.a;
+        KB = d.b;
+        KG = d.c;
+    } else if (d.grp == G_W) {
+        KB = d.a;
+        KG = d.b;
+    } else { /* B */
+        KB = N;
+        KG = d.a;
+    }
+    const int cl = clsL(k), cg = clsG(k);
+    const int KBp = jmax(KB, cl), KGp = jmax(KG, cg);
+    /* rule 3: first access of another block in this grid epoch */
+    if (rel == REL_G) {
+        if (k == HIRACE_WRITE || KG == GX)
+            return {RG, false, true};
+        if (k == HIRACE_READ)
+            return KG == GR ? Out{G_R, false, false} : Out{KG == GRAG ? G_AG1 : G_AB1, true, false};
+        if (k == HIRACE_ATOMIC_GRID)
+            return KG == GR ? Out{G_AG1, false, false} : (KG == GRAG ? Out{G_AGn, true, false} : Out{RG, false, true});
+        return KG == GR ? Out{G_AB1, false, false} : Out{RG, false, true}; /* AB */
+    }
+    /* rule 4 */
+    if (sync == SYNC_BS)
+        return {findT(cl, cl, KGp), false, false};
+    /* rule 5 */
+    if (d.grp == G_B)
+        return k != HIRACE_WRITE ? Out{findB(KGp), true, false} : Out{RB, false, true};
+    /* rule 6 */
+    if (rel == REL_B)
+        return (KB == N && k != HIRACE_WRITE) ? Out{findB(KGp), false, false} : Out{RB, false, true};
+    /* rule 7 */
+    if (sync == SYNC_WS)
+        return {findT(cl, KBp, KGp), false, false};
+    /* rule 8 */
+    if (d.grp == G_W)
+        return k != HIRACE_WRITE ? Out{findW(KBp, KGp), true, false} : Out{RW, false, true};
+    /* rule 9 */
+    if (rel == REL_W)
+        return (KT == N && k != HIRACE_WRITE) ? Out{findW(KBp, KGp), false, false} : Out{RW, false, true};
+    /* rule 10 */
+    return {findT(jmax(KT, cl), KBp, KGp), true, false};
+}
+
+} // namespace relaxed
+
 } // namespace
 
-extern "C" hirace_status hirace_fsm_table(unsigned char out[2048])
+extern "C" hirace_status hirace_fsm_table_policy(int policy, unsigned char out[2048])
 {
-    if (!out)
+    if (!out || policy < 0 || policy > 1)
         return HIRACE_E_INVAL;
     for (int s = 0; s < 32; s++) {
         for (uint32_t k = 0; k < 4; k++)
@@ -168,7 +312,7 @@ extern "C" hirace_status hirace_fsm_table(unsigned char out[2048])
                         out[idx] = (unsigned char)(s | hirace::E_KEEP); /* unused codes */
                         continue;
                     }
-                    Out o = rules(s, k, y, r);
+                    Out o = policy == 0 ? rules(s, k, y, r) : relaxed::rules(s, k, y, r);
                     if (o.next < 0)
                         return HIRACE_E_INVAL; /* inconsistent tuple: a rule-table bug */
                     out[idx] = (unsigned char)(o.next | (o.keep ? hirace::E_KEEP : 0) |
@@ -178,15 +322,20 @@ extern "C" hirace_status hirace_fsm_table(unsigned char out[2048])
     return HIRACE_OK;
 }
 
-extern "C" uint64_t hirace_fsm_step(uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t b,
-                                    uint32_t w, uint32_t block_threads, uint32_t warp_size, int *report)
+extern "C" hirace_status hirace_fsm_table(unsigned char out[2048]) { return hirace_fsm_table_policy(0, out); }
+
+extern "C" uint64_t hirace_fsm_step_policy(int policy, uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g,
+                                           uint32_t b, uint32_t w, uint32_t block_threads, uint32_t warp_size,
+                                           int *report)
 {
-    static unsigned char table[2048];
-    static bool built = false;
-    if (!built) {
-        hirace_fsm_table(table);
-        built = true;
+    static unsigned char tables[2][2048];
+    static bool built[2] = {false, false};
+    policy = policy == 1 ? 1 : 0;
+    if (!built[policy]) {
+        hirace_fsm_table_policy(policy, tables[policy]);
+        built[policy] = true;
     }
+    const unsigned char *table = tables[policy];
     hirace_dev_ctx c{};
     c.block_threads = block_threads ? block_threads : 1;
     c.warp_size = warp_size ? warp_size : 1;
@@ -204,4 +353,10 @@ extern "C" uint64_t hirace_fsm_step(uint64_t old_shadow, uint32_t tid, uint32_t 
     if (report)
         *report = (int)rep;
     return n;
+}
+
+extern "C" uint64_t hirace_fsm_step(uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t b,
+                                    uint32_t w, uint32_t block_threads, uint32_t warp_size, int *report)
+{
+    return hirace_fsm_step_policy(0, old_shadow, tid, kind, g, b, w, block_threads, warp_size, report);
 }

@@ -27,6 +27,8 @@ struct hirace_ctx {
     uint64_t global_words = 0, shadow_words = 0;
     unsigned long long *d_shadow = nullptr;
     unsigned char *d_table = nullptr;
+    unsigned char h_table[2048];
+    int policy = HIRACE_POLICY_STRICT;
     hirace_race *d_reports = nullptr;
     unsigned long long *d_report_count = nullptr;
     unsigned long long *d_stats = nullptr;
@@ -219,6 +221,23 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
     if (c->copy_stream)
         cudaStreamDestroy(c->copy_stream);
     delete c;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_set_policy(hirace_ctx *c, int policy, void *stream)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    if (policy == c->policy)
+        return HIRACE_OK;
+    if (hirace_fsm_table_policy(policy, c->h_table) != HIRACE_OK)
+        return HIRACE_E_INVAL;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    /* h_table is context-owned and only rewritten by a later policy change, which first waits */
+    HR_CUDA(c, cudaStreamSynchronize((cudaStream_t)stream));
+    HR_CUDA(c, cudaMemcpyAsync(c->d_table, c->h_table, 2048, cudaMemcpyHostToDevice, (cudaStream_t)stream));
+    HR_CUDA(c, cudaStreamSynchronize((cudaStream_t)stream));
+    c->policy = policy;
     return HIRACE_OK;
 }
 

@@ -25,11 +25,14 @@ STATUS = {0: "HIRACE_OK", -1: "HIRACE_E_INVAL", -2: "HIRACE_E_NOMEM", -3: "HIRAC
           -4: "HIRACE_E_CLOCK_OVERFLOW", -5: "HIRACE_E_REPORT_OVERFLOW", -6: "HIRACE_E_BAD_TRACE",
           -7: "HIRACE_E_COMM"}
 
+POLICY_STRICT, POLICY_RELAXED_READ_ATOMIC = 0, 1
+
 # every symbol include/hirace.h declares (checked by tests/test_abi.py against the header)
 EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_free", "hirace_shadow_reset", "hirace_barrier",
            "hirace_replay_trace", "hirace_find_batches", "hirace_check_trace_device", "hirace_check_trace_host", "hirace_collect_races",
            "hirace_collect_races_device", "hirace_get_stats", "hirace_sync", "hirace_get_dev_ctx",
-           "hirace_bucket_events", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_fsm_table", "hirace_fsm_step", "hirace_status_string",
+           "hirace_bucket_events", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_set_policy",
+           "hirace_fsm_table", "hirace_fsm_table_policy", "hirace_fsm_step", "hirace_fsm_step_policy", "hirace_status_string",
            "hirace_version")
 
 
@@ -89,8 +92,11 @@ def load():
         "hirace_set_kernel_timing": (I32, [P, P, P]),
         "hirace_microbench_atomics": (I32, [I32, U64, I32, I32, U64, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_microbench_grid_sync": (I32, [I32, I32, I32, ctypes.POINTER(ctypes.c_double), P]),
+        "hirace_set_policy": (I32, [P, I32, P]),
         "hirace_fsm_table": (I32, [P]),
+        "hirace_fsm_table_policy": (I32, [I32, P]),
         "hirace_fsm_step": (U64, [U64, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
+        "hirace_fsm_step_policy": (U64, [I32, U64, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
         "hirace_status_string": (ctypes.c_char_p, [I32]),
         "hirace_version": (ctypes.c_char_p, []),
     }
@@ -106,15 +112,23 @@ def _check(st: int, where: str):
         raise HiraceError(st, where)
 
 
-def fsm_table() -> np.ndarray:
+def fsm_table(policy: int = 0) -> np.ndarray:
     t = np.zeros(2048, np.uint8)
-    _check(load().hirace_fsm_table(t.ctypes.data), "hirace_fsm_table")
+    if policy == POLICY_STRICT:
+        _check(load().hirace_fsm_table(t.ctypes.data), "hirace_fsm_table")
+    else:
+        _check(load().hirace_fsm_table_policy(policy, t.ctypes.data), "hirace_fsm_table_policy")
     return t
 
 
-def fsm_step(old: int, tid: int, kind: int, g: int, b: int, w: int, block_threads: int, warp_size: int):
+def fsm_step(old: int, tid: int, kind: int, g: int, b: int, w: int, block_threads: int, warp_size: int,
+             policy: int = 0):
     rep = ctypes.c_int(0)
-    n = load().hirace_fsm_step(old, tid, kind, g, b, w, block_threads, warp_size, ctypes.byref(rep))
+    if policy == POLICY_STRICT:
+        n = load().hirace_fsm_step(old, tid, kind, g, b, w, block_threads, warp_size, ctypes.byref(rep))
+    else:
+        n = load().hirace_fsm_step_policy(policy, old, tid, kind, g, b, w, block_threads, warp_size,
+                                          ctypes.byref(rep))
     return int(n), int(rep.value)
 
 
@@ -155,7 +169,7 @@ class Checker:
     """One hirace_ctx: shadow (8 B per tracked 4-byte word), FSM table, report buffer."""
 
     def __init__(self, grid_blocks: int, block_threads: int, warp_size: int = 32, global_words: int = 0,
-                 smem_words: int = 0, report_capacity: int = 0, device: int = 0):
+                 smem_words: int = 0, report_capacity: int = 0, device: int = 0, policy: int = 0):
         self.lib = load()
         cfg = Config(grid_blocks, block_threads, warp_size, 4 * smem_words, 4 * global_words, 2, device,
                      report_capacity)
@@ -165,11 +179,19 @@ class Checker:
         self.geometry = dict(grid_blocks=grid_blocks, block_threads=block_threads, warp_size=warp_size,
                              global_words=global_words, smem_words=smem_words)
         self.device = device
+        self.policy = POLICY_STRICT
+        if policy != POLICY_STRICT:
+            self.set_policy(policy)
 
     @classmethod
-    def for_trace(cls, trace, report_capacity: int = 0, device: int = 0):
+    def for_trace(cls, trace, report_capacity: int = 0, device: int = 0, policy: int = 0):
         return cls(trace.grid_blocks, trace.block_threads, trace.warp_size, trace.global_words, trace.smem_words,
-                   report_capacity, device)
+                   report_capacity, device, policy)
+
+    def set_policy(self, policy: int, stream=None):
+        """POLICY_STRICT or POLICY_RELAXED_READ_ATOMIC (include/hirace.h hirace_policy)."""
+        _check(self.lib.hirace_set_policy(self.h, policy, _stream_handle(stream)), "hirace_set_policy")
+        self.policy = policy
 
     @property
     def shadow_bytes(self) -> int:

@@ -367,3 +367,63 @@ def test_cfg5_full_1e9_vs_construction_and_sampled_oracle():
     t = tg.cfg5()
     assert t.n > 1.07e9
     _cfg5_check(t)
+
+
+# ---- relaxed read-vs-atomic policy (reading R2b) ----------------
+
+def _relaxed(t, seeds=(None, 0, 1)):
+    want = {int(a): int(b) for a, b in zip(*oracle.races_of(t, hr.POLICY_RELAXED_READ_ATOMIC)[:2])}
+    c = hr.Checker.for_trace(t, policy=hr.POLICY_RELAXED_READ_ATOMIC)
+    for seed in seeds:
+        ts = t if seed is None else tg.Trace(t.name, tg._shuffle_within_batches(t.events, seed), t.grid_blocks,
+                                              t.block_threads, t.warp_size, t.global_words, t.smem_words)
+        r, _ = gpu_races(ts, checker=c)
+        assert as_dict(r) == want, seed
+    c.close()
+    return want
+
+
+@pytest.mark.parametrize("chunk", range(2))
+def test_relaxed_policy_random_tiny_vs_oracle(chunk):
+    for seed in range(chunk * 250, (chunk + 1) * 250):
+        _relaxed(tg.random_tiny(seed, max_events=40, probs=(.35, .15, .25, .25)), seeds=(None, seed))
+
+
+def test_relaxed_policy_dense_atomics_vs_oracle():
+    rng = np.random.default_rng(12)
+    differ = 0
+    for it in range(20):
+        nb, bs, ws = int(rng.integers(1, 6)), 64, 32
+        n = int(rng.integers(500, 20000))
+        ev = np.empty(n, dtype=tg.EVENT_DTYPE)
+        nkeys = int(rng.integers(1, 50))
+        ev["tid"] = rng.integers(0, nb * bs, n)
+        ev["addr"] = rng.integers(0, nkeys, n).astype(np.uint64) << np.uint64(2)
+        kinds = rng.choice(4, n, p=[0.6, 0.002, 0.15, 0.248])
+        ev["meta"] = tg.pack_meta(kinds, 2, rng.integers(0, 3, n), rng.integers(0, 3, n), rng.integers(0, 3, n))
+        t = tg.Trace("dense", tg.sort_by_batch(ev), nb, bs, ws, nkeys, nkeys)
+        differ += _relaxed(t, seeds=(None,)) != oracle_dict(t)
+    assert differ > 0
+
+
+@pytest.mark.parametrize("kind", ["bfs", "cc"])
+def test_relaxed_policy_cfg3_graph_kernels(kind):
+    # graph kernels mix plain reads of dist/labels with atomicMin: the policy changes the verdict
+    t = tg.cfg3(kind, True, scale=14, edge_factor=16)
+    _relaxed(t)
+
+
+def test_relaxed_policy_cfg5_small_and_switch_on_one_context():
+    # config-5 mix (App. C): its injected GRID patterns are half AB/AB, half R vs AG; under the
+    # relaxed policy the R-vs-AG half is not a race (oracle: 129 flagged strict, 107 relaxed)
+    t = tg.cfg5(grid_blocks=64, words_log2=20, npatterns=256)
+    c = hr.Checker.for_trace(t)
+    got = []
+    for pol in (0, 1, 0, 1):
+        c.set_policy(pol)
+        r, _ = gpu_races(t, checker=c)
+        want = {int(a): int(b) for a, b in zip(*oracle.races_of(t, pol)[:2])}
+        assert as_dict(r) == want, pol
+        got.append(len(want))
+    c.close()
+    assert got[0] > got[1]
