@@ -9,7 +9,10 @@
 
 namespace hirace_impl {
 
-constexpr int kReplayThreads = 512;  /* 16 warps */
+#ifndef HIRACE_REPLAY_THREADS
+#define HIRACE_REPLAY_THREADS 512 /* 16 warps */
+#endif
+constexpr int kReplayThreads = HIRACE_REPLAY_THREADS;
 constexpr int kCollectTile = 4096;     /* shadow words per collect CTA                 */
 constexpr int kCollectThreads = 256;
 constexpr uint32_t kFindChunk = 32768; /* top-level batch-boundary probe chunk (32^3)   */

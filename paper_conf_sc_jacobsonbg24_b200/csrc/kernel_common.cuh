@@ -32,6 +32,9 @@ __device__ __forceinline__ void grid_sync(unsigned int *bar, unsigned int nctas,
             asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
             if (v >= target)
                 break;
+#ifdef HIRACE_BAR_SLEEP
+            __nanosleep(HIRACE_BAR_SLEEP);
+#endif
         }
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
     }

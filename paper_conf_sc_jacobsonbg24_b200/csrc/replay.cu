@@ -32,6 +32,12 @@ namespace hirace_impl {
 
 using namespace hirace;
 
+#ifdef HIRACE_WARP_TRACE
+/* diagnostics build only: per (batch, replay warp) globaltimer when its share is done, and smid */
+__device__ unsigned long long g_warp_trace[16 * 8192 * 4];
+/* per replay warp: max (over all chunks of all batches) of load wait, CAS wait, fold time (ns) */
+__device__ unsigned long long g_chunk_detail[8192 * 4];
+#endif
 #ifdef HIRACE_BARRIER_TRACE
 /* diagnostics build only: per (batch, CTA) globaltimer at arrival and after release */
 __device__ unsigned long long g_bar_trace[128 * 2048 * 2];
@@ -47,7 +53,10 @@ namespace {
 
 constexpr uint32_t FULL = 0xffffffffu;
 constexpr uint64_t NONE = ~0ull;
-constexpr int kMinBlocks = 2; /* 2 x 16 warps per SM at <= 64 registers */
+#ifndef HIRACE_REPLAY_MINB
+#define HIRACE_REPLAY_MINB 2 /* 2 x 16 warps per SM at <= 64 registers */
+#endif
+constexpr int kMinBlocks = HIRACE_REPLAY_MINB;
 
 struct Batch {
     uint32_t key, g, b, w, ep; /* ep = epochs in record layout */
@@ -67,7 +76,12 @@ __device__ __forceinline__ uint32_t lds_u8(uint32_t saddr)
 __device__ __forceinline__ uint4 ld_event(const uint4 *p)
 {
     uint4 v;
+#ifdef HIRACE_EV_EVICT_FIRST
+    asm volatile("{\n\t.reg .b64 pol;\n\tcreatepolicy.fractional.L2::evict_first.b64 pol, 1.0;\n\t"
+                 "ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], pol;\n\t}"
+#else
     asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+#endif
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
                  : "l"(p));
     return v;
@@ -196,6 +210,7 @@ __device__ __noinline__ uint4 chunk_multiword(const hirace_dev_ctx c, const geom
     return make_uint4(cnt.checked, cnt.retry, cnt.cas, cnt.nowrite);
 }
 
+#ifndef HIRACE_STEAL
 /* Contiguous, balanced share of a batch [bstart, bend) for warp w of nw: whole 32-event
  * chunks [c0, c1).  Consecutive chunks of a batch are usually consecutive instructions of the
  * same traced warp and touch the same words; giving them to one replay warp processes them in
@@ -209,6 +224,7 @@ __device__ __forceinline__ void warp_share(uint32_t bstart, uint32_t bend, uint3
     i = bstart + c0 * 32 + lane;
     iend = min(bend, bstart + c1 * 32);
 }
+#endif
 
 /* one lane's decoded access */
 struct Lane {
@@ -269,6 +285,247 @@ __device__ __noinline__ unsigned int collect_call(const hirace_dev_ctx c, uint64
     return epoch;
 }
 
+/* One 32-event chunk (one event per lane): a2 decode, a4 load, a5 transition, a6 CAS, a3
+ * collision fold, a7 report.  All lanes of the warp call it (warp-collective). */
+__device__ __forceinline__ void process_decoded(const Lane &cur, const Batch &B, const hirace_dev_ctx &c,
+                                                const geom &G, const unsigned char *s_table, uint32_t tab_s,
+                                                Counters &cnt, uint32_t lane, uint32_t below);
+
+__device__ __forceinline__ void process_chunk(const uint4 &e, bool valid, uint32_t keysz, const Batch &B,
+                                              uint64_t total_threads, const hirace_dev_ctx &c, const geom &G,
+                                              const unsigned char *s_table, uint32_t tab_s, Counters &cnt,
+                                              uint32_t &bad, uint32_t lane, uint32_t below)
+{
+    const Lane cur = decode(e, valid, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+    process_decoded(cur, B, c, G, s_table, tab_s, cnt, lane, below);
+}
+
+__device__ __forceinline__ void process_decoded(const Lane &cur, const Batch &B, const hirace_dev_ctx &c,
+                                                const geom &G, const unsigned char *s_table, uint32_t tab_s,
+                                                Counters &cnt, uint32_t lane, uint32_t below)
+{
+
+    /* a4: optimistic: every lane reads its own word (coherent load); lanes that share a word
+     * are grouped only if their CAS collides (below) */
+    unsigned long long *const p = c.shadow + cur.idx;
+#ifdef HIRACE_WARP_TRACE
+    const unsigned long long tt0 = gtimer();
+#endif
+    const uint64_t o = cur.ok ? ld_coherent(p) : 0;
+    cnt.checked += cur.ok;
+#ifdef HIRACE_WARP_TRACE
+    uint32_t dmy;
+    asm volatile("add.u32 %0, %1, 0;" : "=r"(dmy) : "r"((uint32_t)o));
+    const unsigned long long tt1 = gtimer();
+#endif
+
+    /* a5: transition */
+    const access a{cur.tid, cur.kind, B.g, B.b, B.w};
+    const uint32_t ent = lds_u8(tab_s + ((st_of(o) << 6) | label(o, a, G)));
+    const uint64_t n = (ent & E_KEEP) ? ((o & ~(uint64_t)31) | (ent & E_STATE))
+                                      : (((uint64_t)cur.tid << SH_TID) | B.ep | (ent & E_STATE));
+    /* a6: one CAS per changed word; unchanged = linearised at the load */
+    const bool do_cas = cur.ok && n != o;
+    cnt.nowrite += cur.ok && !do_cas;
+    cnt.cas += do_cas;
+    const uint64_t prev = do_cas ? cas64(p, o, n) : o;
+    const bool failed = do_cas && prev != o;
+    /* common case: no lane lost its CAS and no lane's transition reports -> one vote */
+    const bool rep = (ent & E_REPORT) && do_cas && !failed;
+#ifndef HIRACE_WARP_TRACE
+    if (!__any_sync(FULL, failed || rep))
+        return;
+#endif
+    uint32_t cls = 0, rtid = cur.tid;
+    if (rep) {
+        const uint32_t cn = race_class(st_of(n)), co = race_class(st_of(o));
+        cls = cn > co ? cn : 0u;
+    }
+#ifdef HIRACE_WARP_TRACE
+    const unsigned long long tt2 = gtimer();
+    const bool failed_any = __any_sync(FULL, failed);
+#endif
+    if (__any_sync(FULL, failed)) {
+        /* Algorithm 1's retry for the lanes whose CAS lost: group them by word, the group
+         * leader folds its members' accesses from the record it observed */
+        const uint32_t peers = __match_any_sync(FULL, failed ? cur.idx : NONE);
+        const bool lead = failed && (peers & below) == 0;
+        cnt.retry += lead;
+        cls |= commit_groups(p, prev, lead ? peers : 0u, cur.tid, cur.kind, G, s_table, B, cnt, rtid, true);
+    }
+    /* a7 */
+    if (__any_sync(FULL, cls != 0))
+        append_reports(c, cls, key_of_idx(cur, c, G), B.g, rtid, lane);
+#ifdef HIRACE_WARP_TRACE
+    const unsigned long long tt3 = gtimer();
+    if (lane == 0) {
+        const uint32_t wg = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+        if (wg < 8192) {
+            unsigned long long *d = &g_chunk_detail[wg * 4];
+            const bool anyf = __any_sync(1u, failed_any);
+            if (!anyf && tt3 - tt0 > d[0]) d[0] = tt3 - tt0;
+            if (anyf && tt3 - tt0 > d[1]) d[1] = tt3 - tt0;
+            d[2] += anyf;
+            if (tt1 - tt0 > d[3]) d[3] = tt1 - tt0;
+        }
+    }
+#endif
+}
+
+#ifdef HIRACE_PIPE
+/* Pipelined chunk processing (opt-in, -DHIRACE_PIPE; measured slower).  The shadow loads of chunk i+1 are issued right after
+ * chunk i's CASes, before their results are awaited, so each chunk costs about one L2 round
+ * trip instead of two (load, then CAS).  Issued after the CASes in program order, the loads
+ * normally observe them; a load that does not (another lane's word, reordered in the memory
+ * system) is only stale for a same-batch access, which is either linearised before the CAS
+ * (no store) or fails its own CAS and retries: the same argument as for concurrent warps
+ * (Algorithm 1; any in-batch order is a linear extension, L177). */
+struct Staged {
+    Lane L;
+    uint64_t o; /* observed record */
+};
+
+__device__ __forceinline__ Staged stage_chunk(const uint4 &e, bool valid, uint32_t keysz, const Batch &B,
+                                              uint64_t total_threads, const hirace_dev_ctx &c, const geom &G,
+                                              const unsigned char *s_table, Counters &cnt, uint32_t &bad,
+                                              uint32_t lane)
+{
+    Staged S;
+    S.L = decode(e, valid, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+    S.o = ld_coherent_if(c.shadow + S.L.idx, S.L.ok, 0); /* a4 */
+    return S;
+}
+
+/* a5 + a6 issue: transition of the staged record and its CAS (result not awaited here) */
+struct Issued {
+    uint64_t n, prev;
+    uint32_t ent;
+    bool do_cas;
+};
+
+__device__ __forceinline__ Issued issue_chunk(const Staged &S, const Batch &B, const geom &G, uint32_t tab_s,
+                                              const hirace_dev_ctx &c, Counters &cnt)
+{
+    Issued I;
+    const access a{S.L.tid, S.L.kind, B.g, B.b, B.w};
+    I.ent = lds_u8(tab_s + ((st_of(S.o) << 6) | label(S.o, a, G)));
+    I.n = (I.ent & E_KEEP) ? ((S.o & ~(uint64_t)31) | (I.ent & E_STATE))
+                           : (((uint64_t)S.L.tid << SH_TID) | B.ep | (I.ent & E_STATE));
+    I.do_cas = S.L.ok && I.n != S.o;
+    cnt.checked += S.L.ok;
+    cnt.nowrite += S.L.ok && !I.do_cas;
+    cnt.cas += I.do_cas;
+    I.prev = cas64_if(c.shadow + S.L.idx, S.o, I.n, I.do_cas);
+    return I;
+}
+
+/* a6 result, a3 fold of lost CASes, a7 report (warp-collective) */
+__device__ __forceinline__ void finish_chunk(const Staged &S, const Issued &I, const Batch &B, const geom &G,
+                                             const unsigned char *s_table, const hirace_dev_ctx &c, Counters &cnt,
+                                             uint32_t lane, uint32_t below)
+{
+    uint32_t cls = 0, rtid = S.L.tid;
+    if (I.do_cas && I.prev == S.o) {
+        const uint32_t cn = race_class(st_of(I.n)), co = race_class(st_of(S.o));
+        cls = ((I.ent & E_REPORT) && cn > co) ? cn : 0u;
+    }
+    const bool failed = I.do_cas && I.prev != S.o;
+    if (__any_sync(FULL, failed)) {
+        const uint32_t peers = __match_any_sync(FULL, failed ? S.L.idx : NONE);
+        const bool lead = failed && (peers & below) == 0;
+        cnt.retry += lead;
+        cls |= commit_groups(c.shadow + S.L.idx, I.prev, lead ? peers : 0u, S.L.tid, S.L.kind, G, s_table, B, cnt,
+                             rtid, true);
+    }
+    if (__any_sync(FULL, cls != 0))
+        append_reports(c, cls, key_of_idx(S.L, c, G), B.g, rtid, lane);
+}
+#endif
+
+#ifdef HIRACE_STEAL
+/* Work stealing inside a CTA (cuts the batch tail before each grid barrier).  Each warp's
+ * contiguous share [c0, c1) of the batch's chunks sits in one shared 32-bit word
+ * back:16 | front:16 (relative to c0; native 32-bit shared atomics).  The owner claims from
+ * the front with an atomic add of 1, issued one hand-out ahead so its latency is hidden (the
+ * result is consumed a chunk later); a warp whose share is exhausted takes single chunks from
+ * the back of the CTA's fullest share with an atomic add of -2^16.  Claims linearise on the
+ * word, so every chunk is replayed exactly once; owner and thieves work at opposite ends of a
+ * share, far apart until it is nearly drained (adjacent chunks touch the same words).  Any
+ * order of a batch's events is a linear extension of happens-before.
+ * Double-buffered by batch parity, so the next batch's shares are published (and the owners'
+ * first claims issued) before the grid barrier.  Shares must stay below 2^15 chunks. */
+__device__ __forceinline__ uint32_t atom_add_shared_if(uint32_t *p, uint32_t v, bool pred)
+{
+    uint32_t r = 0;
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q atom.shared.add.u32 %0, [%1], %2;\n\t}"
+                 : "+r"(r)
+                 : "r"(smem_u32(p)), "r"(v), "r"((uint32_t)pred)
+                 : "memory");
+    return r;
+}
+
+__device__ __forceinline__ int share_begin(uint32_t nchunks, uint32_t w, uint32_t nw)
+{
+    return (int)(((uint64_t)nchunks * w) / nw);
+}
+
+__device__ __forceinline__ void share_init(uint32_t *s_rng, uint32_t bstart, uint32_t bend, uint32_t w, uint32_t nw,
+                                           uint32_t wib, uint32_t lane, int &ca, int &cb, int &c0,
+                                           uint32_t &pend)
+{
+    const uint32_t nchunks = (bend - bstart + 31) / 32;
+    c0 = share_begin(nchunks, w, nw);
+    const int len = share_begin(nchunks, w + 1, nw) - c0;
+    ca = len > 0 ? c0 : -1;
+    cb = len > 1 ? c0 + 1 : -1;
+    if (lane == 0)
+        s_rng[wib] = ((uint32_t)len << 16) | 2u;
+    pend = atom_add_shared_if(&s_rng[wib], 1u, lane == 0); /* same thread: ordered after the store */
+}
+
+__device__ __forceinline__ uint4 chunk_event(const uint4 *ev, int ch, uint32_t bstart, uint32_t bend, uint32_t lane)
+{
+    const uint32_t i = bstart + (uint32_t)ch * 32u + lane;
+    return (ch >= 0 && i < bend) ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
+}
+
+/* consume the pending front claim (lane 0's atomic result) and issue the next one */
+__device__ __forceinline__ int claim_front(uint32_t *r, uint32_t &pend, int c0, uint32_t lane)
+{
+    const int f = (int)(int16_t)(pend & 0xffffu), bk = (int)(int16_t)(pend >> 16);
+    const int ch = __shfl_sync(FULL, f < bk ? c0 + f : -1, 0);
+    if (ch >= 0)
+        pend = atom_add_shared_if(r, 1u, lane == 0);
+    return ch;
+}
+
+/* a chunk from the back of the fullest share of this CTA, or -1 when all are drained */
+__device__ __forceinline__ int steal_back(uint32_t *s_rng, uint32_t nwib, uint32_t lane, uint32_t nchunks,
+                                          uint32_t warp0, uint32_t nw)
+{
+    for (;;) {
+        int rem = -1;
+        if (lane < nwib) {
+            const uint32_t r = *(volatile uint32_t *)&s_rng[lane];
+            rem = (int)(int16_t)(r >> 16) - (int)(int16_t)(r & 0xffffu);
+        }
+        const int best = __reduce_max_sync(FULL, rem);
+        if (best <= 0)
+            return -1;
+        const uint32_t v = __ffs(__ballot_sync(FULL, rem == best)) - 1;
+        int ch = -1;
+        if (lane == 0) {
+            const uint32_t old = atomicAdd(&s_rng[v], 0xffff0000u);
+            const int f = (int)(int16_t)(old & 0xffffu), bk = (int)(int16_t)(old >> 16);
+            ch = f < bk ? share_begin(nchunks, warp0 + v, nw) + bk - 1 : -1;
+        }
+        ch = __shfl_sync(FULL, ch, 0);
+        if (ch >= 0)
+            return ch;
+    }
+}
+#endif
+
 template <bool P2>
 __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     k_replay(hirace_dev_ctx c, const uint4 *__restrict__ ev, const uint32_t *__restrict__ off,
@@ -282,7 +539,6 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
         reinterpret_cast<uint4 *>(s_table)[i] = __ldg(reinterpret_cast<const uint4 *>(c.table) + i);
     if (threadIdx.x < 4)
         s_stats[threadIdx.x] = 0;
-    __syncthreads();
 
     geom G = make_geom(c);
     G.pow2 = P2; /* compile-time geometry mode: shifts (P2) or fast division */
@@ -296,13 +552,26 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     Counters cnt{0, 0, 0, 0};
     uint32_t bad = 0;
 
-    /* a1: events of the first chunk of every batch are requested before the barrier that
+    /* a1: events of the first chunks of every batch are requested before the barrier that
      * precedes the batch, so the HBM latency overlaps the barrier */
     uint32_t bstart = nb ? __ldg(&off[0]) : 0, bend = nb ? __ldg(&off[1]) : 0;
+#ifdef HIRACE_STEAL
+    __shared__ uint32_t s_rng[2][kReplayThreads / 32];
+    const uint32_t wib = threadIdx.x >> 5, nwib = blockDim.x >> 5;
+    int ca, cb, c0; /* this warp's next two chunks (batch-relative, -1 = none); share start */
+    uint32_t pend;  /* lane 0: result of the in-flight front claim */
+    const uint32_t warp0 = blockIdx.x * nwib;
+    share_init(s_rng[0], bstart, bend, warp_global, nwarps, wib, lane, ca, cb, c0, pend);
+    uint4 e0 = chunk_event(ev, ca, bstart, bend, lane);
+    uint4 e1 = chunk_event(ev, cb, bstart, bend, lane);
+    __syncthreads();
+#else
+    __syncthreads();
     uint32_t i, iend; /* this warp's contiguous share of the batch: events [i - lane, iend) */
     warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
     uint4 e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
     uint4 e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
+#endif
     for (uint32_t bi = 0; bi < nb; bi++) {
         Batch B;
         B.key = __ldg(&ev[bstart].w) >> 5;
@@ -314,51 +583,125 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
         if (B.g == 255u)
             bad = 1; /* reserved for retired RACE records (R7) */
 
+#ifdef HIRACE_STEAL
+        uint32_t *const rng = s_rng[bi & 1];
+        const uint32_t nchunks = (bend - bstart + 31) / 32;
+        bool own = true; /* still claiming from this warp's own share */
+        while (ca >= 0) {
+            const uint4 e = e0;
+            const bool valid = bstart + (uint32_t)ca * 32u + lane < bend;
+            e0 = e1; /* a1: keep the next chunks' events in flight */
+            ca = cb;
+            if (own) { /* own share front to back, then the back ends of the CTA's other shares */
+                cb = claim_front(&rng[wib], pend, c0, lane);
+                own = cb >= 0;
+            }
+#ifndef HIRACE_STEAL_OFF
+            if (!own)
+                cb = steal_back(rng, nwib, lane, nchunks, warp0, nwarps);
+#endif
+            e1 = chunk_event(ev, cb, bstart, bend, lane);
+            process_chunk(e, valid, keysz, B, total_threads, c, G, s_table, tab_s, cnt, bad, lane, below);
+        }
+#ifdef HIRACE_WARP_TRACE
+        if (lane == 0 && bi < 16 && warp_global < 8192) {
+            uint32_t smid;
+            asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+            g_warp_trace[(bi * 8192 + warp_global) * 4] = gtimer();
+            g_warp_trace[(bi * 8192 + warp_global) * 4 + 1] = smid;
+        }
+#endif
+        if (bi + 1 < nb) {
+            bstart = __ldg(&off[bi + 1]);
+            bend = __ldg(&off[bi + 2]);
+            share_init(s_rng[(bi + 1) & 1], bstart, bend, warp_global, nwarps, wib, lane, ca, cb, c0, pend);
+            e0 = chunk_event(ev, ca, bstart, bend, lane);
+            e1 = chunk_event(ev, cb, bstart, bend, lane);
+#else
+#if defined(HIRACE_UNROLL2) && !defined(HIRACE_PIPE)
+        /* two chunks per trip: e0/e1 are refilled in place right after their decode, so the
+         * prefetch pipeline costs no register moves */
+        for (;;) {
+            if (i - lane >= iend)
+                break;
+            Lane cur = decode(e0, i < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+            e0 = i + 64 < iend ? ld_event(ev + i + 64) : make_uint4(0, 0, 0, 0);
+            process_decoded(cur, B, c, G, s_table, tab_s, cnt, lane, below);
+            i += 32;
+            if (i - lane >= iend)
+                break;
+            cur = decode(e1, i < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+            e1 = i + 64 < iend ? ld_event(ev + i + 64) : make_uint4(0, 0, 0, 0);
+            process_decoded(cur, B, c, G, s_table, tab_s, cnt, lane, below);
+            i += 32;
+        }
+#elif !defined(HIRACE_PIPE)
+#ifdef HIRACE_WARP_TRACE
+        unsigned long long t_prev = gtimer(), t_max = 0, t_at = 0, t_evmax = 0;
+#endif
         for (; i - lane < iend; i += 32) {
-            const Lane cur = decode(e0, i < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+            const uint4 e = e0;
+            const bool valid = i < iend;
             e0 = e1; /* a1: keep the next chunks' events in flight */
             e1 = i + 64 < iend ? ld_event(ev + i + 64) : make_uint4(0, 0, 0, 0);
-
-            /* a4: optimistic: every lane reads its own word (coherent load); lanes that share
-             * a word are grouped only if their CAS collides (below) */
-            unsigned long long *const p = c.shadow + cur.idx;
-            const uint64_t o = cur.ok ? ld_coherent(p) : 0;
-            cnt.checked += cur.ok;
-
-            /* a5: transition */
-            const access a{cur.tid, cur.kind, B.g, B.b, B.w};
-            const uint32_t ent = lds_u8(tab_s + ((st_of(o) << 6) | label(o, a, G)));
-            const uint64_t n = (ent & E_KEEP) ? ((o & ~(uint64_t)31) | (ent & E_STATE))
-                                              : (((uint64_t)cur.tid << SH_TID) | B.ep | (ent & E_STATE));
-            /* a6: one CAS per changed word; unchanged = linearised at the load */
-            const bool do_cas = cur.ok && n != o;
-            cnt.nowrite += cur.ok && !do_cas;
-            cnt.cas += do_cas;
-            const uint64_t prev = do_cas ? cas64(p, o, n) : o;
-            uint32_t cls = 0, rtid = cur.tid;
-            if (do_cas && prev == o) {
-                const uint32_t cn = race_class(st_of(n)), co = race_class(st_of(o));
-                cls = ((ent & E_REPORT) && cn > co) ? cn : 0u;
+#ifdef HIRACE_WARP_TRACE
+            {
+                uint32_t dmy;
+                asm volatile("add.u32 %0, %1, %2;" : "=r"(dmy) : "r"(e.x), "r"(e.w));
+                const unsigned long long t_ev = gtimer();
+                if (t_ev - t_prev > t_evmax)
+                    t_evmax = t_ev - t_prev;
             }
-            const bool failed = do_cas && prev != o;
-            if (__any_sync(FULL, failed)) {
-                /* Algorithm 1's retry for the lanes whose CAS lost: group them by word, the
-                 * group leader folds its members' accesses from the record it observed */
-                const uint32_t peers = __match_any_sync(FULL, failed ? cur.idx : NONE);
-                const bool lead = failed && (peers & below) == 0;
-                cnt.retry += lead;
-                cls |= commit_groups(p, prev, lead ? peers : 0u, cur.tid, cur.kind, G, s_table, B, cnt, rtid, true);
+#endif
+            process_chunk(e, valid, keysz, B, total_threads, c, G, s_table, tab_s, cnt, bad, lane, below);
+#ifdef HIRACE_WARP_TRACE
+            const unsigned long long t_now = gtimer();
+            if (t_now - t_prev > t_max) {
+                t_max = t_now - t_prev;
+                t_at = i - lane;
             }
-            /* a7 */
-            if (__any_sync(FULL, cls != 0))
-                append_reports(c, cls, key_of_idx(cur, c, G), B.g, rtid, lane);
+            t_prev = t_now;
+#endif
         }
+#else
+        if (i - lane < iend) {
+            Staged cur = stage_chunk(e0, i < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+            e0 = e1; /* a1: keep the next chunks' events in flight */
+            e1 = i + 64 < iend ? ld_event(ev + i + 64) : make_uint4(0, 0, 0, 0);
+            for (;; i += 32) {
+                const Issued I = issue_chunk(cur, B, G, tab_s, c, cnt);
+                const bool more = i + 32 - lane < iend; /* warp-uniform */
+                Staged nxt;
+                if (more) { /* next chunk's shadow loads go out behind this chunk's CASes */
+                    nxt = stage_chunk(e0, i + 32 < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+                    e0 = e1;
+                    e1 = i + 96 < iend ? ld_event(ev + i + 96) : make_uint4(0, 0, 0, 0);
+                }
+                finish_chunk(cur, I, B, G, s_table, c, cnt, lane, below);
+                if (!more)
+                    break;
+                cur = nxt;
+            }
+            i += 32;
+        }
+#endif
+#ifdef HIRACE_WARP_TRACE
+        if (lane == 0 && bi < 16 && warp_global < 8192) {
+            uint32_t smid;
+            asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+            g_warp_trace[(bi * 8192 + warp_global) * 4] = gtimer();
+            g_warp_trace[(bi * 8192 + warp_global) * 4 + 1] = smid;
+            g_warp_trace[(bi * 8192 + warp_global) * 4 + 2] = t_max;
+            g_warp_trace[(bi * 8192 + warp_global) * 4 + 3] = t_at | (t_evmax << 32);
+        }
+#endif
         if (bi + 1 < nb) {
             bstart = __ldg(&off[bi + 1]);
             bend = __ldg(&off[bi + 2]);
             warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
             e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
             e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
+#endif
 #ifdef HIRACE_BARRIER_TRACE
             __syncthreads();
             if (threadIdx.x == 0 && bi < 128 && blockIdx.x < 2048)
@@ -400,6 +743,16 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
 
 } // namespace
 
+#ifdef HIRACE_WARP_TRACE
+extern "C" int hirace_debug_chunk_detail(unsigned long long *host, uint64_t n)
+{
+    return (int)cudaMemcpyFromSymbol(host, g_chunk_detail, n * sizeof(unsigned long long));
+}
+extern "C" int hirace_debug_warp_trace(unsigned long long *host, uint64_t n)
+{
+    return (int)cudaMemcpyFromSymbol(host, g_warp_trace, n * sizeof(unsigned long long));
+}
+#endif
 #ifdef HIRACE_BARRIER_TRACE
 extern "C" int hirace_debug_barrier_trace(unsigned long long *host, uint64_t n)
 {
