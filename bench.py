@@ -259,9 +259,10 @@ def measure_slowdown(dev: int, reps: int = 5) -> dict:
 
 
 def run_sharded_bench(args, world, rank, local_rank):
-    """Config 5 across `world` GPUs: each rank generates its blocks' events; per batch the events
-    are bucketed by owner (64 KiB chunks of the 2^32-word space) on the GPU and exchanged with
-    NCCL all_to_all_single, then replayed on the owner's shard (strong scaling: fixed trace)."""
+    """Config 5 across `world` GPUs: each rank generates its blocks' events; they are bucketed by
+    owner (64 KiB chunks of the 2^32-word space) into 8-byte wire records on the GPU, exchanged
+    per batch with NCCL all_to_all_single (all batches in flight, overlapped with the replays),
+    and replayed on the owner's shard (strong scaling: fixed trace)."""
     import torch
     import torch.distributed as dist
 
@@ -286,9 +287,12 @@ def run_sharded_bench(args, world, rank, local_rank):
     d_out = torch.empty(cap * 16, dtype=torch.uint8, device=f"cuda:{dev}")
     d_total = torch.zeros(1, dtype=torch.int64, device=f"cuda:{dev}")
 
+    wire = sharded.wire_fits(t.grid_blocks * t.block_threads, t.global_words, t.smem_words, world)
+    run = sharded.run_sharded_wire if wire else sharded.run_sharded
+
     def step():
         ops.ctx.reset()
-        sharded.run_sharded(ev, ops, ex, None, dist)
+        run(ev, ops, ex, None, dist)
         ops.ctx.collect_device(d_out, cap, d_total)
 
     clocks = ClockSampler(dev)
@@ -324,7 +328,9 @@ def run_sharded_bench(args, world, rank, local_rank):
                "steps": args.steps, "warmup": args.warmup, "ms_per_step": per_step, "higher_is_better": True,
                "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
                "config": {"workload": f"config 5: {BASELINE_CFG[5]}", "events_total": n_total,
-                          "parallelism": f"address-sharded x{world} ({args.transport} all_to_all per batch)",
+                          "parallelism": (f"address-sharded x{world} ({args.transport} all_to_all per batch, "
+                                          + ("8-byte wire records, async exchange overlapped with replay)" if wire
+                                             else "16-byte events)")),
                           "l2": "inputs larger than L2"},
                "roofline": {"bound": "hbm", "achieved": BYTES_PER_ACCESS * n_total / world / (per_step / 1e3) / 1e9,
                             "peak": peak, "unit": "GB/s",

@@ -229,6 +229,40 @@ hirace_status hirace_set_kernel_timing(hirace_ctx *ctx, void *start_event, void 
 hirace_status hirace_bucket_events(hirace_ctx *ctx, const hirace_event *d_in, uint64_t n, int nranks, int my_rank,
                                    hirace_event *d_out, uint64_t *h_counts, void *stream);
 
+/* ---- sharded mode, 8-byte wire format (a10) -------------------------------- */
+
+/* Wire record, 8 bytes (half the 16-byte event on the NVLink exchange):
+ *   bits  0..30  word: the owner's shard-local global word, or (bit 31 set) the word inside the
+ *                accessing block's shared window (shared events stay on my_rank)
+ *   bit  31      shared
+ *   bits 32..61  tid (global thread id, < 2^30)
+ *   bits 62..63  kind
+ * The batch (g,b,w) is implied: records travel and replay one batch at a time.  Global words
+ * are owned as in hirace_bucket_events (64 KiB chunks, owner = (word >> 14) mod nranks, local
+ * word = ((word >> 14) / nranks) << 14 | word mod 2^14).  8/16-byte accesses are expanded into
+ * one record per word, each routed to its own word's owner (an access may straddle chunks). */
+#define HIRACE_WIRE_MAX_TIDS (1ull << 30)
+#define HIRACE_WIRE_MAX_WORDS (1ull << 31)
+
+/* Buckets the nb batches of DEVICE events d_in (batch b = [h_offsets[b], h_offsets[b+1]),
+ * HOST offsets as returned by hirace_find_batches) into wire records at DEVICE d_out
+ * (capacity cap records): batch-major, owner-grouped inside a batch (order inside a
+ * (batch, owner) segment is unspecified).  Writes HOST h_counts[nb * nranks]
+ * (row b = batch b's records per owner) and *n_words = total records.  If *n_words > cap the
+ * counts are still written and HIRACE_E_INVAL is returned (not sticky): call again with a
+ * buffer of *n_words records.  Synchronises `stream`.
+ * Errors: INVAL (NULL args, nranks not in 1..32, my_rank out of range, grid threads > 2^30 or
+ * shared-window words > 2^31 — such configurations use hirace_bucket_events), BAD_TRACE
+ * (sticky: access size > 16 B, or a shard-local word >= 2^31 — those records are dropped), CUDA. */
+hirace_status hirace_bucket_wire(hirace_ctx *ctx, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
+                                 int nranks, int my_rank, uint64_t *d_out, uint64_t cap, uint64_t *h_counts,
+                                 uint64_t *n_words, void *stream);
+
+/* Replays n DEVICE wire records of ONE batch, key = g<<19 | b<<9 | w, on ctx (the owner's shard
+ * context: its global extent is the shard's).  Successive calls must follow the global batch
+ * order.  Records with tid or word out of range -> sticky BAD_TRACE at the next sync.  Async. */
+hirace_status hirace_replay_wire(hirace_ctx *ctx, const uint64_t *d_wire, uint64_t n, uint32_t batch_key, void *stream);
+
 /* ---- microbenchmarks for the roofline (diagnostics; not part of the checking path) -------- */
 
 /* Rate of 64-bit operations on `nwords` distinct words of a fresh device array (nwords*8 bytes;

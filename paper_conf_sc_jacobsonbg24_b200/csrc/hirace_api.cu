@@ -42,6 +42,12 @@ struct hirace_ctx {
     uint32_t *d_bucket_hist = nullptr;
     uint64_t bucket_hist_cap = 0;
     unsigned long long *d_bucket_counts = nullptr;
+    /* wire bucket scratch */
+    unsigned long long *d_wire_off = nullptr;   /* per-tile offsets of one batch       */
+    uint64_t wire_off_cap = 0;
+    unsigned long long *d_wire_counts = nullptr; /* nb x nranks (+1: running total)    */
+    uint64_t wire_counts_cap = 0;
+    unsigned int *d_wire_flag = nullptr;
     /* host-trace staging ring */
     hirace_event *d_stage[2] = {nullptr, nullptr};
     uint64_t stage_cap = 0;
@@ -208,7 +214,7 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
     void *ptrs[] = {c->d_shadow, c->d_table, c->d_reports, c->d_report_count, c->d_stats, c->d_err,
                     c->scr.batch_off, c->scr.nbatches, c->scr.batch_ctr, c->scr.grid_bar,
                     c->scr.grid_bar2, c->scr.cta_cnt, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
-                    c->d_stage[0], c->d_stage[1]};
+                    c->d_stage[0], c->d_stage[1], c->d_wire_off, c->d_wire_counts, c->d_wire_flag};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
@@ -520,6 +526,99 @@ hirace_status hirace_bucket_events(hirace_ctx *c, const hirace_event *d_in, uint
     HR_CUDA(c, cudaStreamSynchronize(st));
     for (int r = 0; r < nranks; r++)
         h_counts[r] = tmp[r];
+    return HIRACE_OK;
+}
+
+hirace_status hirace_bucket_wire(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
+                                 int nranks, int my_rank, uint64_t *d_out, uint64_t cap, uint64_t *h_counts,
+                                 uint64_t *n_words, void *stream)
+{
+    if (!c || !h_offsets || !h_counts || !n_words || nranks < 1 || nranks > 32 || my_rank < 0 || my_rank >= nranks ||
+        nb > HIRACE_MAX_BATCHES || (nb && !d_in) || (cap && !d_out))
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    const uint64_t threads = (uint64_t)c->cfg.grid_blocks * c->cfg.block_threads;
+    if (threads > HIRACE_WIRE_MAX_TIDS || (uint64_t)c->dev.smem_words > HIRACE_WIRE_MAX_WORDS)
+        return HIRACE_E_INVAL;
+    for (uint64_t b = 0; b < nb; b++)
+        if (h_offsets[b + 1] < h_offsets[b] || h_offsets[b + 1] >= 0xffffffffu)
+            return HIRACE_E_INVAL;
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    uint32_t maxlen = 0;
+    for (uint64_t b = 0; b < nb; b++)
+        maxlen = h_offsets[b + 1] - h_offsets[b] > maxlen ? h_offsets[b + 1] - h_offsets[b] : maxlen;
+    const uint64_t ntiles = (maxlen + kWireTile - 1) / kWireTile;
+    const uint64_t need_hist = ntiles * (uint64_t)nranks;
+    if (need_hist > c->bucket_hist_cap) {
+        if (c->d_bucket_hist)
+            cudaFree(c->d_bucket_hist);
+        c->d_bucket_hist = nullptr;
+        c->bucket_hist_cap = 0;
+        HR_CUDA(c, cudaMalloc(&c->d_bucket_hist, need_hist * sizeof(uint32_t)));
+        c->bucket_hist_cap = need_hist;
+    }
+    if (need_hist > c->wire_off_cap) {
+        if (c->d_wire_off)
+            cudaFree(c->d_wire_off);
+        c->d_wire_off = nullptr;
+        c->wire_off_cap = 0;
+        HR_CUDA(c, cudaMalloc(&c->d_wire_off, need_hist * sizeof(unsigned long long)));
+        c->wire_off_cap = need_hist;
+    }
+    const uint64_t need_counts = nb * (uint64_t)nranks + 1;
+    if (need_counts > c->wire_counts_cap) {
+        if (c->d_wire_counts)
+            cudaFree(c->d_wire_counts);
+        c->d_wire_counts = nullptr;
+        c->wire_counts_cap = 0;
+        HR_CUDA(c, cudaMalloc(&c->d_wire_counts, need_counts * sizeof(unsigned long long)));
+        c->wire_counts_cap = need_counts;
+    }
+    if (!c->d_wire_flag)
+        HR_CUDA(c, cudaMalloc(&c->d_wire_flag, sizeof(unsigned int)));
+    unsigned long long *running = c->d_wire_counts + nb * (uint64_t)nranks;
+    HR_CUDA(c, cudaMemsetAsync(running, 0, sizeof(unsigned long long), st));
+    HR_CUDA(c, cudaMemsetAsync(c->d_wire_flag, 0, sizeof(unsigned int), st));
+    for (uint64_t b = 0; b < nb; b++)
+        HR_CUDA(c, launch_bucket_wire(d_in, h_offsets[b], h_offsets[b + 1], nranks, my_rank,
+                                      reinterpret_cast<unsigned long long *>(d_out), cap, c->d_bucket_hist,
+                                      c->d_wire_off, running, c->d_wire_counts + b * (uint64_t)nranks, c->d_wire_flag,
+                                      st));
+    HR_CUDA(c, cudaMemcpyAsync(h_counts, c->d_wire_counts, nb * (uint64_t)nranks * sizeof(uint64_t),
+                               cudaMemcpyDeviceToHost, st));
+    unsigned long long total = 0;
+    unsigned int flag = 0;
+    HR_CUDA(c, cudaMemcpyAsync(&total, running, sizeof(total), cudaMemcpyDeviceToHost, st));
+    HR_CUDA(c, cudaMemcpyAsync(&flag, c->d_wire_flag, sizeof(flag), cudaMemcpyDeviceToHost, st));
+    HR_CUDA(c, cudaStreamSynchronize(st));
+    *n_words = total;
+    if (flag & hirace::ERR_BAD_TRACE)
+        return set_sticky(c, HIRACE_E_BAD_TRACE);
+    if (total > cap)
+        return HIRACE_E_INVAL;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_replay_wire(hirace_ctx *c, const uint64_t *d_wire, uint64_t n, uint32_t batch_key, void *stream)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    if (n == 0)
+        return HIRACE_OK;
+    if (!d_wire || n >= 0xffffffffull || batch_key >= (1u << 27))
+        return set_sticky(c, HIRACE_E_INVAL);
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    if (c->t_start)
+        HR_CUDA(c, cudaEventRecord(c->t_start, st));
+    HR_CUDA(c, launch_replay_wire(c->dev, reinterpret_cast<const unsigned long long *>(d_wire), (uint32_t)n, batch_key,
+                                  c->replay_grid, st));
+    if (c->t_stop)
+        HR_CUDA(c, cudaEventRecord(c->t_stop, st));
     return HIRACE_OK;
 }
 

@@ -367,6 +367,178 @@ cudaError_t launch_bucket(const hirace_dev_ctx &c, const hirace_event *in, uint3
     return cudaGetLastError();
 }
 
+/* ---------------------------------------------------------------------------------------- */
+/* a10: wire bucketing — one batch at a time, owner-grouped 8-byte wire records               */
+/* ---------------------------------------------------------------------------------------- */
+
+/* words covered by an event of size 1 << szl (sub-word accesses map to their word) */
+__device__ __forceinline__ uint32_t words_of(uint32_t szl) { return szl <= 2 ? 1u : (szl <= 4 ? 1u << (szl - 2) : 0u); }
+
+/* wire record of word k of event e, and its owner (include/hirace.h) */
+__device__ __forceinline__ uint64_t wire_of(const hirace_event &e, uint32_t k, int nranks, int my_rank,
+                                            uint32_t &owner)
+{
+    const bool sh = (e.addr & HIRACE_SHARED_BIT) != 0;
+    const uint64_t word = ((e.addr & ~HIRACE_SHARED_BIT) >> 2) + k;
+    uint64_t w;
+    if (sh) {
+        owner = (uint32_t)my_rank;
+        w = word;
+    } else {
+        const uint64_t chunk = word >> kShardChunkLog2;
+        owner = (uint32_t)(chunk % (uint64_t)nranks);
+        w = ((chunk / (uint64_t)nranks) << kShardChunkLog2) | (word & ((1u << kShardChunkLog2) - 1));
+    }
+    if (w >= (1ull << 31) || e.tid >= (1u << 30)) { /* beyond the wire format: bad input */
+        owner = 0xffffffffu;
+        return 0;
+    }
+    return w | (sh ? 0x80000000ull : 0ull) | ((uint64_t)e.tid << 32) | ((uint64_t)(e.meta & 3u) << 62);
+}
+
+__global__ void __launch_bounds__(kBucketThreads) k_wire_hist(const hirace_event *__restrict__ in, uint32_t lo,
+                                                              uint32_t hi, int nranks, int my_rank,
+                                                              uint32_t *tile_hist, unsigned int *err)
+{
+    __shared__ uint32_t s_h[kMaxRanks];
+    if (threadIdx.x < kMaxRanks)
+        s_h[threadIdx.x] = 0;
+    __syncthreads();
+    const uint32_t base = lo + blockIdx.x * kBucketTile;
+    for (uint32_t it = 0; it < kBucketTile / kBucketThreads; it++) {
+        const uint32_t i = base + it * kBucketThreads + threadIdx.x;
+        if (i < hi) {
+            const hirace_event e = in[i];
+            const uint32_t nw = words_of((e.meta >> 2) & 7u);
+            if (nw == 0)
+                atomicOr(err, hirace::ERR_BAD_TRACE);
+            for (uint32_t k = 0; k < nw; k++) {
+                uint32_t own;
+                (void)wire_of(e, k, nranks, my_rank, own);
+                if (own < (uint32_t)nranks)
+                    atomicAdd(&s_h[own], 1u);
+                else
+                    atomicOr(err, hirace::ERR_BAD_TRACE);
+            }
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x < (unsigned)nranks)
+        tile_hist[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x] = s_h[threadIdx.x];
+}
+
+/* exclusive scan of this batch's [owner][tile] histogram, offset by the records of earlier
+ * batches (*running, updated); the batch's per-owner counts go to counts_row[nranks] */
+__global__ void __launch_bounds__(1024) k_wire_scan(uint32_t *tile_hist, uint32_t ntiles, int nranks,
+                                                    unsigned long long *running, unsigned long long *counts_row,
+                                                    unsigned long long *tile_off)
+{
+    __shared__ unsigned long long s_w[32];
+    __shared__ unsigned long long s_carry;
+    const uint64_t total = (uint64_t)ntiles * nranks;
+    const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const unsigned long long base = *running;
+    if (threadIdx.x == 0)
+        s_carry = 0;
+    __syncthreads();
+    for (uint64_t b0 = 0; b0 < total; b0 += 1024) {
+        const uint64_t i = b0 + threadIdx.x;
+        const unsigned long long v = i < total ? tile_hist[i] : 0;
+        unsigned long long x = v;
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned long long y = __shfl_up_sync(0xffffffffu, x, o);
+            if ((int)lane >= o)
+                x += y;
+        }
+        if (lane == 31)
+            s_w[wid] = x;
+        __syncthreads();
+        if (wid == 0) {
+            unsigned long long t = s_w[lane];
+            for (int o = 1; o < 32; o <<= 1) {
+                const unsigned long long y = __shfl_up_sync(0xffffffffu, t, o);
+                if ((int)lane >= o)
+                    t += y;
+            }
+            s_w[lane] = t;
+        }
+        __syncthreads();
+        if (i < total)
+            tile_off[i] = base + s_carry + (wid ? s_w[wid - 1] : 0) + x - v;
+        __syncthreads();
+        if (threadIdx.x == 0)
+            s_carry += s_w[31];
+        __syncthreads();
+    }
+    if (threadIdx.x < (unsigned)nranks) {
+        const unsigned long long start = tile_off[(uint64_t)threadIdx.x * ntiles];
+        const unsigned long long next =
+            threadIdx.x + 1 < (unsigned)nranks ? tile_off[(uint64_t)(threadIdx.x + 1) * ntiles] : base + s_carry;
+        counts_row[threadIdx.x] = next - start;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0)
+        *running = base + s_carry;
+}
+
+/* scatter: each word gets a slot in its (owner) segment; order inside a batch is free
+ * (PAPER.md L177), so slots are taken with warp-aggregated shared-memory counters */
+__global__ void __launch_bounds__(kBucketThreads) k_wire_scatter(const hirace_event *__restrict__ in, uint32_t lo,
+                                                                 uint32_t hi, int nranks, int my_rank,
+                                                                 const unsigned long long *__restrict__ tile_off,
+                                                                 unsigned long long *out, uint64_t cap,
+                                                                 unsigned int *err)
+{
+    __shared__ unsigned long long s_run[kMaxRanks];
+    const uint32_t lane = threadIdx.x & 31;
+    if (threadIdx.x < (unsigned)nranks)
+        s_run[threadIdx.x] = tile_off[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x];
+    __syncthreads();
+    const uint32_t base = lo + blockIdx.x * kBucketTile;
+    for (uint32_t it = 0; it < kBucketTile / kBucketThreads; it++) {
+        const uint32_t i = base + it * kBucketThreads + threadIdx.x;
+        hirace_event e{0, 0, 0};
+        uint32_t nw = 0;
+        if (i < hi) {
+            e = in[i];
+            nw = words_of((e.meta >> 2) & 7u);
+        }
+        const uint32_t maxw = __reduce_max_sync(0xffffffffu, nw);
+        for (uint32_t k = 0; k < maxw; k++) {
+            uint32_t own = 0xffffffffu;
+            uint64_t w = 0;
+            if (k < nw)
+                w = wire_of(e, k, nranks, my_rank, own); /* own = ~0: invalid, skipped (hist flagged it) */
+            const uint32_t peers = __match_any_sync(0xffffffffu, own);
+            const int leader = __ffs(peers) - 1;
+            unsigned long long slot = 0;
+            if (own != 0xffffffffu && (int)lane == leader)
+                slot = atomicAdd(&s_run[own], (unsigned long long)__popc(peers));
+            slot = __shfl_sync(0xffffffffu, slot, leader) + __popc(peers & ((1u << lane) - 1));
+            if (own != 0xffffffffu) {
+                if (slot < cap)
+                    out[slot] = w;
+                else
+                    atomicOr(err, 8u); /* capacity exceeded: reported by the host call */
+            }
+        }
+    }
+}
+
+cudaError_t launch_bucket_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, int my_rank,
+                               unsigned long long *out, uint64_t cap, uint32_t *d_tile_hist,
+                               unsigned long long *d_tile_off, unsigned long long *d_running,
+                               unsigned long long *d_counts_row, unsigned int *err, cudaStream_t st)
+{
+    const uint32_t ntiles = (hi - lo + kBucketTile - 1) / kBucketTile;
+    if (ntiles == 0)
+        return cudaMemsetAsync(d_counts_row, 0, nranks * sizeof(unsigned long long), st);
+    k_wire_hist<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_hist, err);
+    k_wire_scan<<<1, 1024, 0, st>>>(d_tile_hist, ntiles, nranks, d_running, d_counts_row, d_tile_off);
+    k_wire_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_off, out, cap, err);
+    return cudaGetLastError();
+}
+
 cudaError_t kernels_init(int device)
 {
     (void)device;

@@ -47,6 +47,15 @@ cudaError_t launch_rebase(const hirace_dev_ctx &c, uint64_t shadow_words, cudaSt
 cudaError_t launch_bucket(const hirace_dev_ctx &c, const hirace_event *in, uint32_t n, int nranks, int my_rank,
                           hirace_event *out, unsigned long long *d_counts, uint32_t *d_tile_hist, uint32_t ntiles,
                           cudaStream_t st);
+/* one batch [lo, hi) of events -> owner-grouped 8-byte wire records at out[*running ...] */
+cudaError_t launch_bucket_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, int my_rank,
+                               unsigned long long *out, uint64_t cap, uint32_t *d_tile_hist,
+                               unsigned long long *d_tile_off, unsigned long long *d_running,
+                               unsigned long long *d_counts_row, unsigned int *err, cudaStream_t st);
+/* single-batch replay of 8-byte wire records (batch key given) */
+cudaError_t launch_replay_wire(const hirace_dev_ctx &c, const unsigned long long *wire, uint32_t n, uint32_t batch_key,
+                               int grid, cudaStream_t st);
+constexpr int kWireTile = 4096;
 cudaError_t kernels_init(int device);
 
 } // namespace hirace_impl

@@ -741,6 +741,80 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
         atomicAdd(&c.stats[threadIdx.x], s_stats[threadIdx.x]);
 }
 
+/* Single-batch replay of 8-byte wire records (sharded mode): word:31 |
+ * shared:1 | tid:30 | kind:2; the batch's (g,b,w) is given, so no batch discovery and no grid
+ * barrier — a plain launch.  Each warp walks a contiguous balanced share of 32-record chunks
+ * with the same per-chunk path (a4-a7) as k_replay. */
+template <bool P2>
+__global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
+    k_replay_wire(hirace_dev_ctx c, const unsigned long long *__restrict__ wire, uint32_t n, uint32_t key)
+{
+    __shared__ __align__(16) unsigned char s_table[2048];
+    __shared__ unsigned long long s_stats[4];
+    const uint32_t lane = threadIdx.x & 31;
+    for (int i = threadIdx.x; i < 2048 / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(s_table)[i] = __ldg(reinterpret_cast<const uint4 *>(c.table) + i);
+    if (threadIdx.x < 4)
+        s_stats[threadIdx.x] = 0;
+    __syncthreads();
+    geom G = make_geom(c);
+    G.pow2 = P2;
+    const uint64_t total_threads = (uint64_t)c.grid_blocks * c.block_threads;
+    const uint32_t below = (1u << lane) - 1;
+    const uint32_t tab_s = smem_u32(s_table);
+    Counters cnt{0, 0, 0, 0};
+    Batch B;
+    B.key = key;
+    B.g = key >> 19;
+    B.b = (key >> 9) & 1023u;
+    B.w = key & 511u;
+    B.ep = (B.g << SH_G) | (B.b << SH_B) | (B.w << SH_W);
+    const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    const uint32_t nchunks = (n + 31) / 32;
+    const uint32_t c0 = (uint32_t)(((uint64_t)nchunks * warp_global) / nwarps);
+    const uint32_t c1 = (uint32_t)(((uint64_t)nchunks * (warp_global + 1)) / nwarps);
+    const uint32_t iend = min(n, c1 * 32);
+    uint32_t bad = 0;
+    uint32_t i = c0 * 32 + lane;
+    unsigned long long w0 = i < iend ? __ldcs(wire + i) : 0ull;
+    unsigned long long w1 = i + 32 < iend ? __ldcs(wire + i + 32) : 0ull;
+    for (; i - lane < iend; i += 32) {
+        const unsigned long long w = w0;
+        const bool valid = i < iend;
+        w0 = w1;
+        w1 = i + 64 < iend ? __ldcs(wire + i + 64) : 0ull;
+        Lane L;
+        const uint32_t lo = (uint32_t)w, hi = (uint32_t)(w >> 32);
+        const uint32_t word = lo & 0x7fffffffu;
+        const bool sh = (lo >> 31) != 0;
+        L.tid = hi & 0x3fffffffu;
+        L.kind = hi >> 30;
+        L.ok = valid && L.tid < total_threads && (sh ? word < c.smem_words : word < c.global_words);
+        bad |= (valid && !L.ok) ? 1u : 0u;
+        L.idx = !L.ok ? NONE : (sh ? c.global_words + (uint64_t)block_of(L.tid, G) * c.smem_words + word : (uint64_t)word);
+        process_decoded(L, B, c, G, s_table, tab_s, cnt, lane, below);
+    }
+    if ((__any_sync(FULL, bad) || B.g == 255u) && lane == 0)
+        atomicOr(c.error_flags, ERR_BAD_TRACE);
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) {
+        cnt.checked += __shfl_xor_sync(FULL, cnt.checked, d);
+        cnt.retry += __shfl_xor_sync(FULL, cnt.retry, d);
+        cnt.cas += __shfl_xor_sync(FULL, cnt.cas, d);
+        cnt.nowrite += __shfl_xor_sync(FULL, cnt.nowrite, d);
+    }
+    if (lane == 0) {
+        atomicAdd(&s_stats[0], (unsigned long long)cnt.checked);
+        atomicAdd(&s_stats[1], (unsigned long long)cnt.retry);
+        atomicAdd(&s_stats[2], (unsigned long long)cnt.cas);
+        atomicAdd(&s_stats[3], (unsigned long long)cnt.nowrite);
+    }
+    __syncthreads();
+    if (threadIdx.x < 4 && s_stats[threadIdx.x])
+        atomicAdd(&c.stats[threadIdx.x], s_stats[threadIdx.x]);
+}
+
 } // namespace
 
 #ifdef HIRACE_WARP_TRACE
@@ -780,6 +854,20 @@ int collect_max_grid(int device)
     if (occ < 1)
         occ = 1;
     return sms * occ < kMaxCtas ? sms * occ : kMaxCtas;
+}
+
+cudaError_t launch_replay_wire(const hirace_dev_ctx &c, const unsigned long long *wire, uint32_t n, uint32_t batch_key,
+                               int grid, cudaStream_t st)
+{
+    const bool p2 = (c.block_threads & (c.block_threads - 1)) == 0 && (c.warp_size & (c.warp_size - 1)) == 0;
+    const uint32_t need = (n + 31) / 32; /* no more warps than chunks */
+    const uint64_t want = ((uint64_t)need * 32 + kReplayThreads - 1) / kReplayThreads;
+    const int g2 = (int)(want < (uint64_t)grid ? want : (uint64_t)grid);
+    if (p2)
+        k_replay_wire<true><<<g2, kReplayThreads, 0, st>>>(c, wire, n, batch_key);
+    else
+        k_replay_wire<false><<<g2, kReplayThreads, 0, st>>>(c, wire, n, batch_key);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_replay(const hirace_dev_ctx &c, const hirace_event *ev, const Scratch &s, int grid,

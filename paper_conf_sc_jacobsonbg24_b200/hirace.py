@@ -31,7 +31,7 @@ POLICY_STRICT, POLICY_RELAXED_READ_ATOMIC = 0, 1
 EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_free", "hirace_shadow_reset", "hirace_barrier",
            "hirace_replay_trace", "hirace_find_batches", "hirace_check_trace_device", "hirace_check_trace_host", "hirace_collect_races",
            "hirace_collect_races_device", "hirace_get_stats", "hirace_sync", "hirace_get_dev_ctx",
-           "hirace_bucket_events", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_set_policy",
+           "hirace_bucket_events", "hirace_bucket_wire", "hirace_replay_wire", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_set_policy",
            "hirace_fsm_table", "hirace_fsm_table_policy", "hirace_fsm_step", "hirace_fsm_step_policy", "hirace_status_string",
            "hirace_version")
 
@@ -89,6 +89,8 @@ def load():
         "hirace_sync": (I32, [P]),
         "hirace_get_dev_ctx": (I32, [P, P, ctypes.POINTER(DevCtx)]),
         "hirace_bucket_events": (I32, [P, P, U64, I32, I32, P, ctypes.POINTER(U64), P]),
+        "hirace_bucket_wire": (I32, [P, P, P, U64, I32, I32, P, U64, P, ctypes.POINTER(U64), P]),
+        "hirace_replay_wire": (I32, [P, P, U64, U32, P]),
         "hirace_set_kernel_timing": (I32, [P, P, P]),
         "hirace_microbench_atomics": (I32, [I32, U64, I32, I32, U64, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_microbench_grid_sync": (I32, [I32, I32, I32, ctypes.POINTER(ctypes.c_double), P]),
@@ -319,6 +321,34 @@ class Checker:
                                              ctypes.c_void_p(out_dev.data_ptr()), counts, _stream_handle(stream)),
                "hirace_bucket_events")
         return [int(x) for x in counts]
+
+    def bucket_wire(self, events_dev, offsets: np.ndarray, nranks: int, my_rank: int, stream=None):
+        """8-byte wire records of all batches (include/hirace.h hirace_bucket_wire).
+        offsets: batch start offsets (nb + 1, as from find_batches).  Returns (wire int64 CUDA
+        tensor [m], counts uint64 [nb, nranks]); batch-major, owner-grouped."""
+        import torch
+        offs = np.ascontiguousarray(offsets, dtype=np.uint32)
+        nb = max(len(offs) - 1, 0)
+        counts = np.zeros((max(nb, 1), nranks), np.uint64)
+        total = ctypes.c_uint64(0)
+        n_ev = int(offs[-1]) if nb else 0
+        cap = n_ev + n_ev // 8 + 64
+        dev = events_dev.device
+        while True:
+            out = torch.empty(cap, dtype=torch.int64, device=dev)
+            st = self.lib.hirace_bucket_wire(self.h, ctypes.c_void_p(events_dev.data_ptr() if nb else 0),
+                                             offs.ctypes.data, nb, nranks, my_rank, ctypes.c_void_p(out.data_ptr()),
+                                             cap, counts.ctypes.data, ctypes.byref(total), _stream_handle(stream))
+            if st == -1 and total.value > cap:
+                cap = int(total.value)
+                continue
+            _check(st, "hirace_bucket_wire")
+            return out[: total.value], counts[:nb]
+
+    def replay_wire(self, wire_dev, n: int, batch_key: int, stream=None):
+        """Replays n wire records of one batch (key g<<19 | b<<9 | w)."""
+        _check(self.lib.hirace_replay_wire(self.h, ctypes.c_void_p(wire_dev.data_ptr() if n else 0), n, batch_key,
+                                           _stream_handle(stream)), "hirace_replay_wire")
 
 
 def races_to_dict(races: np.ndarray) -> dict:

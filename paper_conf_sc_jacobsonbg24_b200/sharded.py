@@ -16,6 +16,15 @@ is exact for the words it owns; the union (keys mapped back to global words) is 
 Inside a batch any order is a linear extension of happens-before, so the
 received segments need no merge.
 
+`run_sharded_wire` is the default pipeline: ONE bucketing launch sequence over
+all local batches into 8-byte wire records (hirace_bucket_wire; g,b,w implied by the batch),
+ONE all_to_all of the [ranks x batches] count matrix, then every batch's payload
+all_to_all posted asynchronously up front while the replays (hirace_replay_wire) consume
+them in batch order — the exchange of batch k+1 overlaps the replay of batch k, and the host
+never waits on the exchange with NCCL (work.wait() orders the streams).  `run_sharded` (16-byte
+events, per-batch synchronous exchange) remains for geometries beyond the wire format's
+limits (> 2^30 threads or > 2^31 words per shard).
+
 The orchestration is written against three small interfaces (`ops`: find_batches / bucket /
 replay / collect, and an exchange) so the host logic can be tested on CPU with gloo and
 world_size > 1; the GPU ops are the library's kernels, there is no CPU fallback for them.
@@ -74,6 +83,28 @@ class NcclExchange:
                                     group=self.group)
         return out
 
+    def counts_matrix(self, send):
+        """send: int64 numpy [P, nb] (row = destination) -> recv [P, nb] (row = source)."""
+        P, nb = send.shape
+        t = self.torch.from_numpy(np.ascontiguousarray(send, dtype=np.int64).reshape(-1)).to(self.device)
+        r = self.torch.empty_like(t)
+        if nb:
+            self.dist.all_to_all_single(r, t, group=self.group)
+        return r.cpu().numpy().reshape(P, nb)
+
+    def payload_async(self, send, send_counts: list[int], recv_counts: list[int]):
+        """Posts one batch's exchange of 8-byte wire records (int64 [n]); returns a handle for
+        finish().  NCCL: device tensors, the collective runs on NCCL's stream."""
+        out = self.torch.empty(sum(recv_counts), dtype=self.torch.int64, device=self.device)
+        work = self.dist.all_to_all_single(out, send, output_split_sizes=recv_counts, input_split_sizes=send_counts,
+                                           group=self.group, async_op=True)
+        return out, work
+
+    def finish(self, handle):
+        out, work = handle
+        work.wait()  # NCCL: the current stream waits on the collective; the host does not block
+        return out
+
 
 class HostExchange(NcclExchange):
     """The same exchange through host memory (gloo): CPU tests and several ranks on one GPU."""
@@ -85,6 +116,14 @@ class HostExchange(NcclExchange):
     def payload(self, send, send_counts, recv_counts):
         cpu = send.cpu() if hasattr(send, "cpu") else send
         out = super().payload(cpu, send_counts, recv_counts)
+        return out.to(self.out_device) if self.out_device is not None else out
+
+    def payload_async(self, send, send_counts, recv_counts):
+        cpu = send.cpu() if hasattr(send, "cpu") else send
+        return super().payload_async(cpu, send_counts, recv_counts)
+
+    def finish(self, handle):
+        out = super().finish(handle)
         return out.to(self.out_device) if self.out_device is not None else out
 
 
@@ -121,6 +160,17 @@ class GpuOps:
     def replay(self, events):
         if events.shape[0]:
             self.ctx.replay(events, events.shape[0])
+
+    def bucket_wire(self, events, offsets):
+        """All local batches -> (wire int64 [m], counts [nb, P]) (hirace_bucket_wire)."""
+        if len(offsets) <= 1:
+            return self.torch.empty(0, dtype=self.torch.int64, device=events.device), np.zeros((0, self.nranks),
+                                                                                                np.uint64)
+        return self.ctx.bucket_wire(events, offsets, self.nranks, self.rank)
+
+    def replay_wire(self, wire, key: int):
+        if wire.shape[0]:
+            self.ctx.replay_wire(wire, int(wire.shape[0]), key)
 
     def collect(self):
         r = self.ctx.collect()
@@ -160,6 +210,48 @@ def run_sharded(local_events, ops, exchange, group, dist, on_batch=None):
         if on_batch is not None:
             on_batch(int(key), int(recv.shape[0]))
     return received
+
+
+def run_sharded_wire(local_events, ops, exchange, group, dist, on_batch=None):
+    """The default sharded pipeline (module docstring): bucket all batches once, exchange the
+    count matrix once, post every batch's payload exchange asynchronously, replay in the global
+    batch order as each arrives.  Returns the number of wire records (word accesses) replayed
+    on this rank."""
+    offs, keys = ops.find_batches(local_events)
+    order = all_batch_keys(keys, group, dist)
+    P = dist.get_world_size(group)
+    wire, counts = ops.bucket_wire(local_events, offs)
+    counts = np.asarray(counts, dtype=np.int64).reshape(-1, P)
+    row_start = np.concatenate(([0], np.cumsum(counts.sum(axis=1)))).astype(np.int64)
+    where = {int(k): i for i, k in enumerate(keys)}
+    nbg = len(order)
+    send = np.zeros((P, nbg), np.int64)
+    seg = np.zeros(nbg, np.int64)
+    for j, k in enumerate(order):
+        i = where.get(int(k))
+        if i is not None:
+            send[:, j] = counts[i]
+            seg[j] = row_start[i]
+    recv = exchange.counts_matrix(send)
+    handles = []
+    for j in range(nbg):  # all payload exchanges in flight; the replays below consume them in order
+        n = int(send[:, j].sum())
+        handles.append(exchange.payload_async(wire[int(seg[j]):int(seg[j]) + n], send[:, j].tolist(),
+                                              recv[:, j].tolist()))
+    received = 0
+    for j, k in enumerate(order):
+        got = exchange.finish(handles[j])
+        handles[j] = None
+        ops.replay_wire(got, int(k))
+        received += int(got.shape[0])
+        if on_batch is not None:
+            on_batch(int(k), int(got.shape[0]))
+    return received
+
+
+def wire_fits(grid_threads: int, global_words: int, smem_words: int, nranks: int) -> bool:
+    """Whether the 8-byte wire format covers this geometry (include/hirace.h limits)."""
+    return grid_threads <= (1 << 30) and shard_words(global_words, nranks) <= (1 << 31) and smem_words <= (1 << 31)
 
 
 def gather_races(races: np.ndarray, group, dist, dst: int = 0):

@@ -20,7 +20,7 @@ import torch.multiprocessing as mp  # noqa: E402
 
 import paper_conf_sc_jacobsonbg24_b200 as hr  # noqa: E402
 from paper_conf_sc_jacobsonbg24_b200 import sharded  # noqa: E402
-from tests.test_sharded import CpuTestOps, _make, _to_events, _to_tensor  # noqa: E402
+from tests.test_sharded import CpuTestOps, _make, _to_events, _to_tensor, _words, wire_bucket_np  # noqa: E402
 
 
 @pytest.mark.parametrize("nranks,rank", [(1, 0), (2, 1), (3, 2), (8, 5), (32, 17)])
@@ -44,7 +44,72 @@ def test_bucket_kernel_matches_contract(nranks, rank):
     c.close()
 
 
-def _gpu_worker(rank, world, port, name, q):
+@pytest.mark.parametrize("nranks,rank", [(1, 0), (2, 1), (3, 0), (8, 5), (32, 31)])
+def test_bucket_wire_kernel_matches_contract(nranks, rank):
+    t = _make("multi")
+    c = hr.Checker(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words)
+    d = _to_tensor(t.events).cuda()
+    offs, keys = c.find_batches(d)
+    wire, counts = c.bucket_wire(d, offs, nranks, rank)
+    want, want_counts = wire_bucket_np(t.events, offs, nranks, rank)
+    assert np.array_equal(counts, want_counts)
+    got = wire.cpu().numpy()
+    ref = want.numpy()
+    assert got.shape == ref.shape == (_words(t),)
+    flat = want_counts.reshape(-1)
+    pos = np.concatenate(([0], np.cumsum(flat.astype(np.int64))))
+    for i in range(len(flat)):  # every (batch, owner) segment holds the same records
+        a, b = int(pos[i]), int(pos[i + 1])
+        assert np.array_equal(np.sort(got[a:b]), np.sort(ref[a:b]))
+    c.close()
+
+
+def test_bucket_wire_capacity_and_bad_sizes():
+    t = _make("multi")
+    c = hr.Checker(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words)
+    d = _to_tensor(t.events).cuda()
+    offs, _ = c.find_batches(d)
+    wire, counts = c.bucket_wire(d, offs, 2, 0)   # the binding grows its buffer on INVAL
+    assert wire.shape[0] == _words(t) > t.n
+    ev = t.events.copy()
+    ev["meta"][5] = (ev["meta"][5] & ~np.uint32(7 << 2)) | np.uint32(5 << 2)  # 32-byte access
+    with pytest.raises(hr.HiraceError):
+        c.bucket_wire(_to_tensor(ev).cuda(), offs, 2, 0)
+    c.close()
+
+
+def test_replay_wire_matches_replay_trace():
+    """Single rank: wire replay of every batch == the 16-byte replay (same race set)."""
+    for name in ("cfg2", "multi", "cfg4"):
+        t = _make(name)
+        d = _to_tensor(t.events).cuda()
+        a = hr.Checker.for_trace(t)
+        a.replay(d, t.n)
+        want = a.collect()
+        b = hr.Checker.for_trace(t)
+        offs, keys = b.find_batches(d)
+        wire, counts = b.bucket_wire(d, offs, 1, 0)
+        start = 0
+        for k, n in zip(keys, counts.sum(axis=1)):
+            b.replay_wire(wire[start:start + int(n)], int(n), int(k))
+            start += int(n)
+        got = b.collect()
+        assert got["key"].tolist() == want["key"].tolist()
+        assert ((got["cls_and_epoch"] & 0xFF) == (want["cls_and_epoch"] & 0xFF)).all()
+        assert b.stats()["checked"] == _words(t)
+        a.close()
+        b.close()
+
+
+def test_replay_wire_rejects_out_of_range():
+    c = hr.Checker(4, 64, 32, 1 << 14, 16)
+    bad = torch.tensor([np.int64(1 << 20)], dtype=torch.int64, device="cuda")  # word 2^20 > 2^14 tracked
+    c.replay_wire(bad, 1, 0)
+    assert c.sync() == -6
+    c.close()
+
+
+def _gpu_worker(rank, world, port, name, q, wire=False):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     torch.cuda.set_device(0)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -55,7 +120,8 @@ def _gpu_worker(rank, world, port, name, q):
         ops = sharded.GpuOps(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words, world,
                              rank, device=0)
         ex = sharded.HostExchange(None, device="cuda:0")
-        n = sharded.run_sharded(_to_tensor(mine).cuda(), ops, ex, None, dist)
+        run = sharded.run_sharded_wire if wire else sharded.run_sharded
+        n = run(_to_tensor(mine).cuda(), ops, ex, None, dist)
         races = sharded.gather_races(ops.collect(), None, dist)
         tot = torch.tensor([n])
         dist.all_reduce(tot)
@@ -88,6 +154,43 @@ def test_sharded_gpu_ranks_reproduce_the_oracle(world, name):
     assert total == t.n
     assert keys == [int(x) for x in k]
     assert cls == [int(x) for x in c]
+
+
+@pytest.mark.parametrize("world,name", [(2, "cfg2"), (3, "multi"), (4, "cfg4"), (2, "cfg3")])
+def test_sharded_wire_gpu_ranks_reproduce_the_oracle(world, name):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_gpu_worker, args=(r, world, port, name, q, True)) for r in range(world)]
+    for p in procs:
+        p.start()
+    total, keys, cls = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    t = _make(name)
+    k, c, _ = oracle.races_of(t)
+    assert total == _words(t)
+    assert keys == [int(x) for x in k]
+    assert cls == [int(x) for x in c]
+
+
+def test_sharded_wire_single_rank_nccl():
+    port = _free_port()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        t = _make("multi")
+        ops = sharded.GpuOps(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words, 1, 0)
+        ex = sharded.NcclExchange(None, "cuda:0")
+        n = sharded.run_sharded_wire(_to_tensor(t.events).cuda(), ops, ex, None, dist)
+        races = sharded.gather_races(ops.collect(), None, dist)
+    finally:
+        dist.destroy_process_group()
+    k, c, _ = oracle.races_of(t)
+    assert n == _words(t)
+    assert races["key"].tolist() == [int(x) for x in k]
+    assert (races["cls_and_epoch"] & 0xFF).tolist() == [int(x) for x in c]
 
 
 def test_sharded_single_rank_nccl():

@@ -62,6 +62,12 @@ class CpuTestOps:
     def replay(self, events):
         self.got.append(_to_events(events).copy())
 
+    def bucket_wire(self, events, offsets):
+        return wire_bucket_np(_to_events(events), offsets, self.P, self.r)
+
+    def replay_wire(self, wire, key):
+        self.got.append(wire_to_events(np.asarray(wire), key))
+
     def collect(self):
         ev = np.concatenate(self.got) if self.got else np.empty(0, tg.EVENT_DTYPE)
         k, c, g = oracle.races(ev, self.t.block_threads, self.t.warp_size)
@@ -70,6 +76,46 @@ class CpuTestOps:
         out["cls_and_epoch"] = c.astype(np.uint32) | (g.astype(np.uint32) << 8)
         out["detect_tid"] = 0
         return out
+
+
+def wire_bucket_np(ev, offsets, P, r):
+    """Reference of the hirace_bucket_wire contract (include/hirace.h): per batch, one record per
+    covered word, routed to its word's owner, shard-local words, owner-grouped (stable here;
+    the kernel's order inside a (batch, owner) segment is unspecified)."""
+    nb = len(offsets) - 1
+    counts = np.zeros((max(nb, 0), P), np.uint64)
+    parts = []
+    for b in range(nb):
+        e = ev[int(offsets[b]):int(offsets[b + 1])]
+        szl = (e["meta"] >> 2) & 7
+        nw = np.where(szl <= 2, 1, 1 << np.maximum(szl.astype(np.int64) - 2, 0)).astype(np.int64)
+        rep = np.repeat(e, nw)
+        k = np.arange(rep.shape[0]) - np.repeat(np.cumsum(nw) - nw, nw)
+        sh = (rep["addr"] & tg.SHARED_BIT) != 0
+        word = ((rep["addr"] & ~tg.SHARED_BIT) >> np.uint64(2)) + k.astype(np.uint64)
+        c = np.uint64(sharded.CHUNK_LOG2)
+        owner = np.where(sh, r, (word >> c) % np.uint64(P)).astype(np.int64)
+        local = np.where(sh, word, (((word >> c) // np.uint64(P)) << c) | (word & np.uint64((1 << 14) - 1)))
+        w = (local | (sh.astype(np.uint64) << np.uint64(31)) | (rep["tid"].astype(np.uint64) << np.uint64(32)) |
+             ((rep["meta"] & 3).astype(np.uint64) << np.uint64(62)))
+        order = np.argsort(owner, kind="stable")
+        parts.append(w[order])
+        counts[b] = np.bincount(owner, minlength=P)
+    wire = np.concatenate(parts) if parts else np.zeros(0, np.uint64)
+    return torch.from_numpy(wire.view(np.int64).copy()), counts
+
+
+def wire_to_events(wire, key):
+    """Wire records of batch `key` back to 4-byte events (for the oracle)."""
+    w = np.asarray(wire).view(np.uint64)
+    ev = np.empty(w.shape[0], tg.EVENT_DTYPE)
+    word = w & np.uint64(0x7FFFFFFF)
+    sh = (w >> np.uint64(31)) & np.uint64(1)
+    ev["addr"] = (word << np.uint64(2)) | (sh << np.uint64(63))
+    ev["tid"] = (w >> np.uint64(32)) & np.uint64(0x3FFFFFFF)
+    g, b, ww = key >> 19, (key >> 9) & 1023, key & 511
+    ev["meta"] = tg.pack_meta((w >> np.uint64(62)).astype(np.uint32), 2, ww, b, g)
+    return ev
 
 
 def _make(name):
@@ -89,10 +135,31 @@ def _make(name):
         ev["meta"] = tg.pack_meta(rng.choice(4, n, p=[.5, .3, .1, .1]), 2, 0, rng.integers(0, 3, n),
                                   rng.integers(0, 3, n))
         return tg.Trace("wide", tg.sort_by_batch(ev), 8, 64, 32, 1 << 20, 0)
+    if name == "multi":
+        # 8- and 16-byte accesses, many straddling a 64 KiB owner chunk, plus shared words
+        rng = np.random.default_rng(11)
+        n = 20000
+        ev = np.empty(n, dtype=tg.EVENT_DTYPE)
+        ev["tid"] = rng.integers(0, 8 * 64, n)
+        chunk_edge = (rng.integers(1, 16, n).astype(np.uint64) << np.uint64(14)) - rng.integers(0, 3, n).astype(
+            np.uint64)
+        words = np.where(rng.random(n) < 0.5, chunk_edge, rng.integers(0, 1 << 18, n).astype(np.uint64))
+        sh = rng.random(n) < 0.15
+        szl = rng.choice([2, 3, 4], n, p=[.4, .3, .3])
+        words = np.where(sh, rng.integers(0, 60, n).astype(np.uint64), words)
+        ev["addr"] = (words << np.uint64(2)) | (sh.astype(np.uint64) << np.uint64(63))
+        ev["meta"] = tg.pack_meta(rng.choice(4, n, p=[.5, .3, .1, .1]), szl, 0, rng.integers(0, 2, n),
+                                  rng.integers(0, 3, n))
+        return tg.Trace("multi", tg.sort_by_batch(ev), 8, 64, 32, 1 << 18, 64)
     raise ValueError(name)
 
 
-def _worker(rank, world, port, name, q):
+def _words(t):
+    szl = (t.events["meta"] >> 2) & 7
+    return int(np.where(szl <= 2, 1, 1 << np.maximum(szl.astype(np.int64) - 2, 0)).sum())
+
+
+def _worker(rank, world, port, name, q, wire=False):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
@@ -101,7 +168,8 @@ def _worker(rank, world, port, name, q):
         mine = t.events[(blk % world) == rank]          # this rank's blocks, batch order kept
         ops = CpuTestOps(t, world, rank)
         ex = sharded.HostExchange(None)
-        n = sharded.run_sharded(_to_tensor(mine), ops, ex, None, dist)
+        run = sharded.run_sharded_wire if wire else sharded.run_sharded
+        n = run(_to_tensor(mine), ops, ex, None, dist)
         races = sharded.gather_races(ops.collect(), None, dist)
         tot = torch.tensor([n])
         dist.all_reduce(tot)
@@ -134,6 +202,44 @@ def test_sharded_exchange_reproduces_the_oracle(world, name):
     assert total == t.n                   # every event replayed exactly once
     assert keys == [int(x) for x in k]    # same words
     assert cls == [int(x) for x in c]     # same classes
+
+
+@pytest.mark.parametrize("world,name", [(2, "cfg2"), (3, "cfg4"), (2, "cfg3"), (3, "wide"), (2, "multi"),
+                                        (4, "multi")])
+def test_sharded_wire_pipeline_reproduces_the_oracle(world, name):
+    """8-byte wire records, one count-matrix exchange, async per-batch payloads."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, name, q, True)) for r in range(world)]
+    for p in procs:
+        p.start()
+    total, keys, cls = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    t = _make(name)
+    k, c, _ = oracle.races_of(t)
+    assert total == _words(t)              # every covered word replayed exactly once
+    assert keys == [int(x) for x in k]
+    assert cls == [int(x) for x in c]
+    assert len(k) > 0
+
+
+def test_wire_reference_roundtrip():
+    """The wire encoding is lossless for in-range records: decode(encode(e)) gives the event's
+    shard-local word, tid, kind and the batch's epochs."""
+    t = _make("multi")
+    offs = np.flatnonzero(np.concatenate(([True], np.diff(t.events["meta"] >> 5) != 0)))
+    offs = np.append(offs, t.n)
+    wire, counts = wire_bucket_np(t.events, offs, 1, 0)
+    assert int(counts.sum()) == _words(t) == wire.shape[0]
+    keys = t.events["meta"][offs[:-1]] >> 5
+    back = np.concatenate([wire_to_events(wire.numpy()[int(s):int(s + n)], int(k)) for s, n, k in
+                           zip(np.concatenate(([0], np.cumsum(counts.sum(1))[:-1])), counts.sum(1), keys)])
+    k1, c1, _ = oracle.races(back, t.block_threads, t.warp_size)
+    k0, c0, _ = oracle.races_of(t)
+    assert k1.tolist() == k0.tolist() and c1.tolist() == c0.tolist()
 
 
 def test_shard_geometry():
