@@ -225,7 +225,9 @@ hirace_status hirace_set_kernel_timing(hirace_ctx *ctx, void *start_event, void 
  * order is preserved — to DEVICE d_out (n records), with every global address rewritten to
  * the owner's shard-local word ((word >> 14) / nranks) << 14 | (word mod 2^14), so the owner's
  * context tracks ceil(global_words / (2^14 nranks)) * 2^14 words.  Per-owner counts go to HOST
- * h_counts[nranks].  Synchronises `stream` (the counts size the exchange).  nranks <= 32. */
+ * h_counts[nranks].  Synchronises `stream` (the counts size the exchange).  nranks <= 32.
+ * A global 8/16-byte access that straddles two owner chunks cannot be routed as one 16-byte
+ * event: it raises sticky BAD_TRACE (hirace_bucket_wire splits such accesses per word). */
 hirace_status hirace_bucket_events(hirace_ctx *ctx, const hirace_event *d_in, uint64_t n, int nranks, int my_rank,
                                    hirace_event *d_out, uint64_t *h_counts, void *stream);
 

@@ -245,7 +245,8 @@ __device__ __forceinline__ uint64_t shard_local_addr(uint64_t addr, int nranks)
 }
 
 __global__ void __launch_bounds__(kBucketThreads) k_bucket_hist(const hirace_event *__restrict__ in, uint32_t n,
-                                                                int nranks, int my_rank, uint32_t *tile_hist)
+                                                                int nranks, int my_rank, uint32_t *tile_hist,
+                                                                unsigned int *err)
 {
     __shared__ uint32_t s_h[kMaxRanks];
     if (threadIdx.x < kMaxRanks)
@@ -254,8 +255,18 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_hist(const hirace_eve
     const uint64_t base = (uint64_t)blockIdx.x * kBucketTile;
     for (int it = 0; it < kBucketTile / kBucketThreads; it++) {
         uint64_t i = base + (uint64_t)it * kBucketThreads + threadIdx.x;
-        if (i < n)
-            atomicAdd(&s_h[owner_of(in[i], nranks, my_rank)], 1u);
+        if (i < n) {
+            const hirace_event e = in[i];
+            atomicAdd(&s_h[owner_of(e, nranks, my_rank)], 1u);
+            /* a 16-byte event cannot be split: a global access straddling two owner chunks
+             * needs the wire format (hirace_bucket_wire) */
+            const uint32_t szl = (e.meta >> 2) & 7u;
+            if (nranks > 1 && !(e.addr & HIRACE_SHARED_BIT) && szl > 2) {
+                const uint64_t w0 = e.addr >> 2, w1 = w0 + (szl <= 4 ? (1u << (szl - 2)) : 1u) - 1;
+                if ((w0 >> kShardChunkLog2) != (w1 >> kShardChunkLog2))
+                    atomicOr(err, hirace::ERR_BAD_TRACE);
+            }
+        }
     }
     __syncthreads();
     if (threadIdx.x < (unsigned)nranks)
@@ -360,8 +371,7 @@ cudaError_t launch_bucket(const hirace_dev_ctx &c, const hirace_event *in, uint3
                           hirace_event *out, unsigned long long *d_counts, uint32_t *d_tile_hist, uint32_t ntiles,
                           cudaStream_t st)
 {
-    (void)c;
-    k_bucket_hist<<<ntiles, kBucketThreads, 0, st>>>(in, n, nranks, my_rank, d_tile_hist);
+    k_bucket_hist<<<ntiles, kBucketThreads, 0, st>>>(in, n, nranks, my_rank, d_tile_hist, c.error_flags);
     k_bucket_scan<<<1, 1024, 0, st>>>(d_tile_hist, ntiles, nranks, d_counts);
     k_bucket_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, n, nranks, my_rank, d_tile_hist, out);
     return cudaGetLastError();

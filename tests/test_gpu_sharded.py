@@ -210,3 +210,18 @@ def test_sharded_single_rank_nccl():
     assert races["key"].tolist() == [int(x) for x in k]
     assert (races["cls_and_epoch"] & 0xFF).tolist() == [int(x) for x in c]
     assert _to_events  # imported helper used by the CPU tests
+
+
+def test_bucket_events_flags_straddling_access():
+    """The 16-byte path cannot split an access across owners: it must say so (BAD_TRACE)."""
+    t = _make("multi")
+    c = hr.Checker(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words)
+    d = _to_tensor(t.events).cuda()
+    out = torch.empty_like(d)
+    c.bucket(d, t.n, 2, 0, out)
+    assert c.sync() == -6
+    c.close()
+    ok = hr.Checker(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words)
+    ok.bucket(d, t.n, 1, 0, out)  # one rank: nothing to split
+    assert ok.sync() == 0
+    ok.close()
