@@ -116,7 +116,8 @@ typedef struct hirace_ctx hirace_ctx;
  * All pointers are device pointers owned by the hirace_ctx. */
 typedef struct {
     unsigned long long *shadow;       /* [global_words | grid_blocks * smem_words] records   */
-    const unsigned char *table;       /* 2048-entry FSM transition table                      */
+    const unsigned char *table;       /* 2048-entry FSM transition table, followed by its
+                                         4096-entry raw-flag expansion (hirace_device.cuh)     */
     hirace_race *reports;             /* race-report ring                                     */
     unsigned long long *report_count; /* records appended (may exceed capacity)               */
     unsigned long long *stats;        /* [checked, cas_retries, cas_ops, no_write]            */

@@ -27,7 +27,7 @@ struct hirace_ctx {
     uint64_t global_words = 0, shadow_words = 0;
     unsigned long long *d_shadow = nullptr;
     unsigned char *d_table = nullptr;
-    unsigned char h_table[2048];
+    unsigned char h_table[2048 + hirace::RAW_TABLE_BYTES]; /* canonical | raw-flag expansion */
     int policy = HIRACE_POLICY_STRICT;
     hirace_race *d_reports = nullptr;
     unsigned long long *d_report_count = nullptr;
@@ -158,14 +158,14 @@ hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
         return fail(e);
     cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, c->device);
     c->replay_grid = replay_max_grid(c->device);
-    unsigned char table[2048];
+    unsigned char table[2048 + hirace::RAW_TABLE_BYTES];
     if (hirace_fsm_table(table) != HIRACE_OK) {
         hirace_shadow_free(c);
         return HIRACE_E_INVAL;
     }
     c->scr.collect_grid = collect_max_grid(c->device);
     if ((e = cudaMalloc(&c->d_shadow, c->shadow_words * 8)) != cudaSuccess ||
-        (e = cudaMalloc(&c->d_table, 2048)) != cudaSuccess ||
+        (e = cudaMalloc(&c->d_table, 2048 + hirace::RAW_TABLE_BYTES)) != cudaSuccess ||
         (e = cudaMalloc(&c->d_reports, c->cfg.report_capacity * sizeof(hirace_race))) != cudaSuccess ||
         (e = cudaMalloc(&c->d_report_count, sizeof(unsigned long long))) != cudaSuccess ||
         (e = cudaMalloc(&c->d_stats, 4 * sizeof(unsigned long long))) != cudaSuccess ||
@@ -178,7 +178,8 @@ hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
         (e = cudaMalloc(&c->scr.cta_cnt, kMaxCtas * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&c->d_total, sizeof(unsigned long long))) != cudaSuccess)
         return fail(e);
-    if ((e = cudaMemcpy(c->d_table, table, 2048, cudaMemcpyHostToDevice)) != cudaSuccess)
+    hirace::expand_raw_table(table, table + 2048); /* the replay kernel's label_raw layout */
+    if ((e = cudaMemcpy(c->d_table, table, sizeof(table), cudaMemcpyHostToDevice)) != cudaSuccess)
         return fail(e);
     hirace_dev_ctx &d = c->dev;
     d.shadow = c->d_shadow;
@@ -241,7 +242,9 @@ hirace_status hirace_set_policy(hirace_ctx *c, int policy, void *stream)
     HR_CUDA(c, cudaSetDevice(c->device));
     /* h_table is context-owned and only rewritten by a later policy change, which first waits */
     HR_CUDA(c, cudaStreamSynchronize((cudaStream_t)stream));
-    HR_CUDA(c, cudaMemcpyAsync(c->d_table, c->h_table, 2048, cudaMemcpyHostToDevice, (cudaStream_t)stream));
+    hirace::expand_raw_table(c->h_table, c->h_table + 2048);
+    HR_CUDA(c, cudaMemcpyAsync(c->d_table, c->h_table, sizeof(c->h_table), cudaMemcpyHostToDevice,
+                               (cudaStream_t)stream));
     HR_CUDA(c, cudaStreamSynchronize((cudaStream_t)stream));
     c->policy = policy;
     return HIRACE_OK;

@@ -87,6 +87,16 @@ __device__ __forceinline__ uint4 ld_event(const uint4 *p)
     return v;
 }
 
+/* predicated event load: v keeps its old contents when !pred (no zero-fill instructions;
+ * such lanes are masked by `valid`) */
+__device__ __forceinline__ void ld_event_if(const uint4 *p, bool pred, uint4 &v)
+{
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %5, 0;\n\t"
+                 "@q ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];\n\t}"
+                 : "+r"(v.x), "+r"(v.y), "+r"(v.z), "+r"(v.w)
+                 : "l"(p), "r"((uint32_t)pred));
+}
+
 /* race key (include/hirace.h) of word k of event e */
 __device__ __forceinline__ uint64_t key_of(const geom &G, const uint4 &e, uint32_t k)
 {
@@ -137,9 +147,8 @@ __device__ __forceinline__ uint32_t commit_groups(unsigned long long *p, uint64_
         if (pending) {
             if (n == o) {
                 pending = false;
-                cnt.nowrite++;
             } else {
-                cnt.cas++;
+                cnt.cas += first ? 1u : 0u; /* first attempt of this group, else a retry */
                 cnt.retry += first ? 0u : 1u;
                 const uint64_t prev = cas64(p, o, n);
                 if (prev == o) {
@@ -234,9 +243,12 @@ struct Lane {
 };
 
 /* a2: decode + validate one lane's event (sub-word accesses map to their word); 8/16-byte
- * accesses of the chunk are committed right here, word by word */
+ * accesses of the chunk are committed right here, word by word.  W32: the whole shadow has
+ * < 2^31 words and tracked byte offsets fit 32 bits, so index math and range checks are 32-bit
+ * (fewer instructions on the hot path); otherwise 64-bit. */
+template <bool W32>
 __device__ __forceinline__ Lane decode(const uint4 &e, bool valid, uint32_t keysz, const Batch &B,
-                                       uint64_t total_threads, const hirace_dev_ctx &c, const geom &G,
+                                       uint32_t tid_max, const hirace_dev_ctx &c, const geom &G,
                                        const unsigned char *tab, Counters &cnt, uint32_t &bad, uint32_t lane)
 {
     Lane L;
@@ -245,14 +257,23 @@ __device__ __forceinline__ Lane decode(const uint4 &e, bool valid, uint32_t keys
     const uint32_t meta = e.w;
     const bool sh = (int)e.y < 0;
     const bool key_ok = (meta >> 2) - keysz <= 2u; /* same batch, size <= 4 bytes */
-    const bool tid_ok = L.tid < total_threads;
-    const uint64_t word = ((uint64_t)(e.y & 0x7fffffffu) << 30) | (e.x >> 2);
-    const bool in_range = sh ? word < c.smem_words : word < c.global_words;
+    const bool tid_ok = L.tid <= tid_max;
+    uint64_t word;
+    bool in_range;
+    if (W32) {
+        const uint32_t w32 = e.x >> 2;
+        word = w32;
+        in_range = (e.y & 0x7fffffffu) == 0 && w32 < (sh ? c.smem_words : (uint32_t)c.global_words);
+    } else {
+        word = ((uint64_t)(e.y & 0x7fffffffu) << 30) | (e.x >> 2);
+        in_range = sh ? word < c.smem_words : word < c.global_words;
+    }
     L.ok = valid && key_ok && tid_ok && in_range;
     if (__any_sync(FULL, valid && !L.ok)) {
+        const uint64_t wfull = ((uint64_t)(e.y & 0x7fffffffu) << 30) | (e.x >> 2);
         const uint32_t szl = (meta >> 2) & 7u;
         const bool multi = valid && (meta >> 5) == B.key && (szl == 3 || szl == 4) && tid_ok &&
-                           (sh ? word + (1u << (szl - 2)) <= c.smem_words : word + (1u << (szl - 2)) <= c.global_words);
+                           (sh ? wfull + (1u << (szl - 2)) <= c.smem_words : wfull + (1u << (szl - 2)) <= c.global_words);
         if (valid && !L.ok && !multi)
             bad = 1;
         if (__any_sync(FULL, multi)) {
@@ -260,10 +281,14 @@ __device__ __forceinline__ Lane decode(const uint4 &e, bool valid, uint32_t keys
             cnt.checked += d.x;
             cnt.retry += d.y;
             cnt.cas += d.z;
-            cnt.nowrite += d.w;
         }
     }
-    L.idx = !L.ok ? NONE : (sh ? c.global_words + (uint64_t)block_of(L.tid, G) * c.smem_words + word : word);
+    if (W32)
+        L.idx = !L.ok ? NONE
+                      : (uint64_t)(sh ? (uint32_t)c.global_words + block_of(L.tid, G) * c.smem_words + (uint32_t)word
+                                      : (uint32_t)word);
+    else
+        L.idx = !L.ok ? NONE : (sh ? c.global_words + (uint64_t)block_of(L.tid, G) * c.smem_words + word : word);
     return L;
 }
 
@@ -291,12 +316,13 @@ __device__ __forceinline__ void process_decoded(const Lane &cur, const Batch &B,
                                                 const geom &G, const unsigned char *s_table, uint32_t tab_s,
                                                 Counters &cnt, uint32_t lane, uint32_t below);
 
+template <bool W32>
 __device__ __forceinline__ void process_chunk(const uint4 &e, bool valid, uint32_t keysz, const Batch &B,
-                                              uint64_t total_threads, const hirace_dev_ctx &c, const geom &G,
+                                              uint32_t tid_max, const hirace_dev_ctx &c, const geom &G,
                                               const unsigned char *s_table, uint32_t tab_s, Counters &cnt,
                                               uint32_t &bad, uint32_t lane, uint32_t below)
 {
-    const Lane cur = decode(e, valid, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+    const Lane cur = decode<W32>(e, valid, keysz, B, tid_max, c, G, s_table, cnt, bad, lane);
     process_decoded(cur, B, c, G, s_table, tab_s, cnt, lane, below);
 }
 
@@ -321,14 +347,13 @@ __device__ __forceinline__ void process_decoded(const Lane &cur, const Batch &B,
 
     /* a5: transition */
     const access a{cur.tid, cur.kind, B.g, B.b, B.w};
-    const uint32_t ent = lds_u8(tab_s + ((st_of(o) << 6) | label(o, a, G)));
+    const uint32_t ent = lds_u8(tab_s + 2048 + ((st_of(o) << 7) | label_raw(o, a, G)));
     const uint64_t n = (ent & E_KEEP) ? ((o & ~(uint64_t)31) | (ent & E_STATE))
                                       : (((uint64_t)cur.tid << SH_TID) | B.ep | (ent & E_STATE));
     /* a6: one CAS per changed word; unchanged = linearised at the load */
     const bool do_cas = cur.ok && n != o;
-    cnt.nowrite += cur.ok && !do_cas;
-    cnt.cas += do_cas;
-    const uint64_t prev = do_cas ? cas64(p, o, n) : o;
+    cnt.cas += do_cas; /* main-path no-write accesses = checked - first CASes (counted at the end) */
+    const uint64_t prev = cas64_if(p, o, n, do_cas);
     const bool failed = do_cas && prev != o;
     /* common case: no lane lost its CAS and no lane's transition reports -> one vote */
     const bool rep = (ent & E_REPORT) && do_cas && !failed;
@@ -350,8 +375,7 @@ __device__ __forceinline__ void process_decoded(const Lane &cur, const Batch &B,
          * leader folds its members' accesses from the record it observed */
         const uint32_t peers = __match_any_sync(FULL, failed ? cur.idx : NONE);
         const bool lead = failed && (peers & below) == 0;
-        cnt.retry += lead;
-        cls |= commit_groups(p, prev, lead ? peers : 0u, cur.tid, cur.kind, G, s_table, B, cnt, rtid, true);
+        cls |= commit_groups(p, prev, lead ? peers : 0u, cur.tid, cur.kind, G, s_table, B, cnt, rtid, false);
     }
     /* a7 */
     if (__any_sync(FULL, cls != 0))
@@ -386,12 +410,12 @@ struct Staged {
 };
 
 __device__ __forceinline__ Staged stage_chunk(const uint4 &e, bool valid, uint32_t keysz, const Batch &B,
-                                              uint64_t total_threads, const hirace_dev_ctx &c, const geom &G,
+                                              uint32_t tid_max, const hirace_dev_ctx &c, const geom &G,
                                               const unsigned char *s_table, Counters &cnt, uint32_t &bad,
                                               uint32_t lane)
 {
     Staged S;
-    S.L = decode(e, valid, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+    S.L = decode<false>(e, valid, keysz, B, tid_max, c, G, s_table, cnt, bad, lane);
     S.o = ld_coherent_if(c.shadow + S.L.idx, S.L.ok, 0); /* a4 */
     return S;
 }
@@ -413,7 +437,6 @@ __device__ __forceinline__ Issued issue_chunk(const Staged &S, const Batch &B, c
                            : (((uint64_t)S.L.tid << SH_TID) | B.ep | (I.ent & E_STATE));
     I.do_cas = S.L.ok && I.n != S.o;
     cnt.checked += S.L.ok;
-    cnt.nowrite += S.L.ok && !I.do_cas;
     cnt.cas += I.do_cas;
     I.prev = cas64_if(c.shadow + S.L.idx, S.o, I.n, I.do_cas);
     return I;
@@ -526,16 +549,16 @@ __device__ __forceinline__ int steal_back(uint32_t *s_rng, uint32_t nwib, uint32
 }
 #endif
 
-template <bool P2>
+template <bool P2, bool W32>
 __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     k_replay(hirace_dev_ctx c, const uint4 *__restrict__ ev, const uint32_t *__restrict__ off,
              const uint32_t *__restrict__ nbp, unsigned int *bar, uint64_t shadow_words, hirace_race *out,
              uint64_t cap, unsigned long long *d_total, uint32_t *cta_cnt)
 {
-    __shared__ __align__(16) unsigned char s_table[2048];
+    __shared__ __align__(16) unsigned char s_table[2048 + RAW_TABLE_BYTES]; /* canonical | raw-flag */
     __shared__ unsigned long long s_stats[4];
     const uint32_t lane = threadIdx.x & 31;
-    for (int i = threadIdx.x; i < 2048 / 16; i += blockDim.x)
+    for (int i = threadIdx.x; i < (2048 + RAW_TABLE_BYTES) / 16; i += blockDim.x)
         reinterpret_cast<uint4 *>(s_table)[i] = __ldg(reinterpret_cast<const uint4 *>(c.table) + i);
     if (threadIdx.x < 4)
         s_stats[threadIdx.x] = 0;
@@ -544,6 +567,7 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     G.pow2 = P2; /* compile-time geometry mode: shifts (P2) or fast division */
     const uint32_t nb = *nbp;
     const uint64_t total_threads = (uint64_t)c.grid_blocks * c.block_threads;
+    const uint32_t tid_max = total_threads > 0xffffffffull ? 0xffffffffu : (uint32_t)(total_threads - 1);
     const uint32_t below = (1u << lane) - 1;
     const uint32_t tab_s = smem_u32(s_table);
     const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -601,7 +625,7 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
                 cb = steal_back(rng, nwib, lane, nchunks, warp0, nwarps);
 #endif
             e1 = chunk_event(ev, cb, bstart, bend, lane);
-            process_chunk(e, valid, keysz, B, total_threads, c, G, s_table, tab_s, cnt, bad, lane, below);
+            process_chunk<W32>(e, valid, keysz, B, tid_max, c, G, s_table, tab_s, cnt, bad, lane, below);
         }
 #ifdef HIRACE_WARP_TRACE
         if (lane == 0 && bi < 16 && warp_global < 8192) {
@@ -624,14 +648,14 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
         for (;;) {
             if (i - lane >= iend)
                 break;
-            Lane cur = decode(e0, i < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
-            e0 = i + 64 < iend ? ld_event(ev + i + 64) : make_uint4(0, 0, 0, 0);
+            Lane cur = decode<W32>(e0, i < iend, keysz, B, tid_max, c, G, s_table, cnt, bad, lane);
+            ld_event_if(ev + i + 64, i + 64 < iend, e0);
             process_decoded(cur, B, c, G, s_table, tab_s, cnt, lane, below);
             i += 32;
             if (i - lane >= iend)
                 break;
-            cur = decode(e1, i < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
-            e1 = i + 64 < iend ? ld_event(ev + i + 64) : make_uint4(0, 0, 0, 0);
+            cur = decode<W32>(e1, i < iend, keysz, B, tid_max, c, G, s_table, cnt, bad, lane);
+            ld_event_if(ev + i + 64, i + 64 < iend, e1);
             process_decoded(cur, B, c, G, s_table, tab_s, cnt, lane, below);
             i += 32;
         }
@@ -643,7 +667,7 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
             const uint4 e = e0;
             const bool valid = i < iend;
             e0 = e1; /* a1: keep the next chunks' events in flight */
-            e1 = i + 64 < iend ? ld_event(ev + i + 64) : make_uint4(0, 0, 0, 0);
+            ld_event_if(ev + i + 64, i + 64 < iend, e1);
 #ifdef HIRACE_WARP_TRACE
             {
                 uint32_t dmy;
@@ -653,7 +677,7 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
                     t_evmax = t_ev - t_prev;
             }
 #endif
-            process_chunk(e, valid, keysz, B, total_threads, c, G, s_table, tab_s, cnt, bad, lane, below);
+            process_chunk<W32>(e, valid, keysz, B, tid_max, c, G, s_table, tab_s, cnt, bad, lane, below);
 #ifdef HIRACE_WARP_TRACE
             const unsigned long long t_now = gtimer();
             if (t_now - t_prev > t_max) {
@@ -665,7 +689,7 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
         }
 #else
         if (i - lane < iend) {
-            Staged cur = stage_chunk(e0, i < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+            Staged cur = stage_chunk(e0, i < iend, keysz, B, tid_max, c, G, s_table, cnt, bad, lane);
             e0 = e1; /* a1: keep the next chunks' events in flight */
             e1 = i + 64 < iend ? ld_event(ev + i + 64) : make_uint4(0, 0, 0, 0);
             for (;; i += 32) {
@@ -673,7 +697,7 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
                 const bool more = i + 32 - lane < iend; /* warp-uniform */
                 Staged nxt;
                 if (more) { /* next chunk's shadow loads go out behind this chunk's CASes */
-                    nxt = stage_chunk(e0, i + 32 < iend, keysz, B, total_threads, c, G, s_table, cnt, bad, lane);
+                    nxt = stage_chunk(e0, i + 32 < iend, keysz, B, tid_max, c, G, s_table, cnt, bad, lane);
                     e0 = e1;
                     e1 = i + 96 < iend ? ld_event(ev + i + 96) : make_uint4(0, 0, 0, 0);
                 }
@@ -723,6 +747,7 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
 
     if (__any_sync(FULL, bad) && lane == 0)
         atomicOr(c.error_flags, ERR_BAD_TRACE);
+    cnt.nowrite = cnt.checked - cnt.cas; /* accesses that issued no CAS of their own */
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) {
         cnt.checked += __shfl_xor_sync(FULL, cnt.checked, d);
@@ -749,10 +774,10 @@ template <bool P2>
 __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     k_replay_wire(hirace_dev_ctx c, const unsigned long long *__restrict__ wire, uint32_t n, uint32_t key)
 {
-    __shared__ __align__(16) unsigned char s_table[2048];
+    __shared__ __align__(16) unsigned char s_table[2048 + RAW_TABLE_BYTES]; /* canonical | raw-flag */
     __shared__ unsigned long long s_stats[4];
     const uint32_t lane = threadIdx.x & 31;
-    for (int i = threadIdx.x; i < 2048 / 16; i += blockDim.x)
+    for (int i = threadIdx.x; i < (2048 + RAW_TABLE_BYTES) / 16; i += blockDim.x)
         reinterpret_cast<uint4 *>(s_table)[i] = __ldg(reinterpret_cast<const uint4 *>(c.table) + i);
     if (threadIdx.x < 4)
         s_stats[threadIdx.x] = 0;
@@ -797,6 +822,7 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     }
     if ((__any_sync(FULL, bad) || B.g == 255u) && lane == 0)
         atomicOr(c.error_flags, ERR_BAD_TRACE);
+    cnt.nowrite = cnt.checked - cnt.cas; /* accesses that issued no CAS of their own */
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) {
         cnt.checked += __shfl_xor_sync(FULL, cnt.checked, d);
@@ -838,9 +864,14 @@ int replay_max_grid(int device)
 {
     int sms = 0, occ = 0, occ2 = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_replay<true>, kReplayThreads, 0);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_replay<false>, kReplayThreads, 0);
+    int occ3 = 0, occ4 = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_replay<true, false>, kReplayThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_replay<false, false>, kReplayThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ3, k_replay<true, true>, kReplayThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ4, k_replay<false, true>, kReplayThreads, 0);
     occ = occ < occ2 ? occ : occ2;
+    occ = occ < occ3 ? occ : occ3;
+    occ = occ < occ4 ? occ : occ4;
     if (occ < 1)
         occ = 1;
     return sms * occ;
@@ -888,7 +919,16 @@ cudaError_t launch_replay(const hirace_dev_ctx &c, const hirace_event *ev, const
     uint32_t *cnt = s.cta_cnt;
     void *args[] = {&cc, &evp, &offp, &nbp, &barp, &nw, &o, &cp, &dt, &cnt};
     const bool p2 = (c.block_threads & (c.block_threads - 1)) == 0 && (c.warp_size & (c.warp_size - 1)) == 0;
-    const void *fn = p2 ? (const void *)k_replay<true> : (const void *)k_replay<false>;
+    /* W32: every shadow index and tracked byte offset fits 32 bits (see decode) */
+    const uint64_t sw = c.global_words + (uint64_t)c.grid_blocks * c.smem_words;
+#ifdef HIRACE_NO_W32
+    const bool w32 = false;
+    (void)sw;
+#else
+    const bool w32 = sw < (1ull << 31) && c.global_words < (1ull << 30) && c.smem_words < (1u << 30);
+#endif
+    const void *fn = p2 ? (w32 ? (const void *)k_replay<true, true> : (const void *)k_replay<true, false>)
+                        : (w32 ? (const void *)k_replay<false, true> : (const void *)k_replay<false, false>);
     return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kReplayThreads), args, 0, st);
 }
 
