@@ -35,6 +35,11 @@ UNIT = "accesses/s"
 BYTES_PER_ACCESS = 32  # 16-B event + 8-B shadow read + 8-B shadow write
 
 
+def bytes_per_access(rec_bytes: int) -> int:
+    """16-B event + shadow read + shadow write of one record (8 B, or 4 B compact)."""
+    return 16 + 2 * rec_bytes
+
+
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -116,12 +121,12 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(rows), "samples_in_timed_region": len(inside)}
 
 
-def load_traffic(config: int, variant: str):
+def load_traffic(config: int, variant: str, compact: bool = False):
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(p):
         with open(p) as f:
             d = json.load(f)
-        return d.get(f"cfg{config}_{variant}")
+        return d.get(f"cfg{config}_{variant}" + ("_compact" if compact else ""))
     return None
 
 
@@ -172,7 +177,8 @@ def config_block(args, trace, world):
     return {"workload": f"config {args.config} ({trace.name}): {BASELINE_CFG.get(args.config, '')}",
             "events_per_rank": int(trace.n), "grid_blocks": trace.grid_blocks,
             "block_threads": trace.block_threads, "batches": trace.batch_count(),
-            "shadow_bytes": 8 * (trace.global_words + trace.grid_blocks * trace.smem_words),
+            "shadow_bytes": (4 if getattr(args, "compact", False) else 8) * (trace.global_words + trace.grid_blocks * trace.smem_words),
+            "shadow_record_bytes": 4 if getattr(args, "compact", False) else 8,
             "l2": "inputs larger than L2 (events %.0f MB > 126 MB L2)" % (trace.n * 16 / 1e6),
             "parallelism": f"replicas{world}" if world > 1 else "single"}
 
@@ -269,15 +275,21 @@ def run_sharded_bench(args, world, rank, local_rank):
     from paper_conf_sc_jacobsonbg24_b200 import sharded
     dev = local_rank % torch.cuda.device_count()
     torch.cuda.set_device(dev)
-    if args.transport == "nccl":
+    shared_gpu = world > torch.cuda.device_count()  # several ranks per GPU: NCCL cannot run there
+    if args.transport == "nccl" or (args.transport == "p2p" and not shared_gpu):
         dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
-        ex = sharded.NcclExchange(None, f"cuda:{dev}")
+        ex = sharded.NcclExchange(None, f"cuda:{dev}") if args.transport == "nccl" else \
+            sharded.PeerExchange(None, dist, device=dev)
+    elif args.transport == "p2p":  # control plane over gloo; the records still go peer to peer
+        dist.init_process_group("gloo")
+        ex = sharded.PeerExchange(None, dist, device=dev)
     else:
         dist.init_process_group("gloo")
         ex = sharded.HostExchange(None, device=f"cuda:{dev}")
     t = make_trace(5, args.variant, world, rank)
     n_local = word_accesses(t.events)
-    tot = torch.tensor([n_local], dtype=torch.int64, device=f"cuda:{dev}" if args.transport == "nccl" else "cpu")
+    nccl = dist.get_backend() == "nccl"
+    tot = torch.tensor([n_local], dtype=torch.int64, device=f"cuda:{dev}" if nccl else "cpu")
     dist.all_reduce(tot)
     n_total = int(tot.item())
     ops = sharded.GpuOps(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words, world, rank,
@@ -288,7 +300,10 @@ def run_sharded_bench(args, world, rank, local_rank):
     d_total = torch.zeros(1, dtype=torch.int64, device=f"cuda:{dev}")
 
     wire = sharded.wire_fits(t.grid_blocks * t.block_threads, t.global_words, t.smem_words, world)
-    run = sharded.run_sharded_wire if wire else sharded.run_sharded
+    if args.transport == "p2p" and not wire:
+        raise SystemExit("p2p transport needs the 8-byte wire format")
+    run = (sharded.run_sharded_p2p if args.transport == "p2p" else sharded.run_sharded_wire) if wire else \
+        sharded.run_sharded
 
     def step():
         ops.ctx.reset()
@@ -316,7 +331,7 @@ def run_sharded_bench(args, world, rank, local_rank):
     clocks.stop()
     ms = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64)
     fl = torch.tensor([flagged], dtype=torch.int64)
-    if args.transport == "nccl":
+    if nccl:
         ms, fl = ms.cuda(), fl.cuda()
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     dist.all_reduce(fl)
@@ -328,10 +343,14 @@ def run_sharded_bench(args, world, rank, local_rank):
                "steps": args.steps, "warmup": args.warmup, "ms_per_step": per_step, "higher_is_better": True,
                "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
                "config": {"workload": f"config 5: {BASELINE_CFG[5]}", "events_total": n_total,
-                          "parallelism": (f"address-sharded x{world} ({args.transport} all_to_all per batch, "
-                                          + ("8-byte wire records, async exchange overlapped with replay)" if wire
-                                             else "16-byte events)")),
-                          "l2": "inputs larger than L2"},
+                          "parallelism": (f"address-sharded x{world} (" + (
+                              "peer dispatch: bucketing kernel stores 8-byte wire records into the owners' "
+                              "IPC-mapped buffers over NVLink)" if args.transport == "p2p" else
+                              f"{args.transport} all_to_all per batch, "
+                              + ("8-byte wire records, async exchange overlapped with replay)" if wire
+                                 else "16-byte events)"))),
+                          "l2": "inputs larger than L2",
+                          "ranks_per_gpu": -(-world // torch.cuda.device_count())},
                "roofline": {"bound": "hbm", "achieved": BYTES_PER_ACCESS * n_total / world / (per_step / 1e3) / 1e9,
                             "peak": peak, "unit": "GB/s",
                             "frac": BYTES_PER_ACCESS * n_total / world / (per_step / 1e3) / 1e9 / peak,
@@ -339,6 +358,8 @@ def run_sharded_bench(args, world, rank, local_rank):
                "cpu_baseline": None, "e2e": None, "gpu_launches": None, "clocks": clocks.summary(),
                "check": {"flagged_words": flagged, "expected": len(t.info["expected"])}}
         print(json.dumps(out), flush=True)
+    if isinstance(ex, sharded.PeerExchange):
+        ex.close()
     dist.destroy_process_group()
 
 
@@ -353,8 +374,11 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-slowdown", action="store_true")
-    ap.add_argument("--transport", default="nccl", choices=["nccl", "host"],
-                    help="config-5 shard exchange: NCCL device all_to_all, or gloo host staging")
+    ap.add_argument("--compact", action="store_true",
+                    help="compact 4-byte shadow records (hirace_shadow_alloc_compact, SURVEY §8(f) f1)")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p", "host"],
+                    help="config-5 shard exchange: NCCL device all_to_all, peer-memory dispatch (CUDA IPC / "
+                         "NVLink stores from the bucketing kernel), or gloo host staging")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -379,7 +403,8 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
 
     n_acc = word_accesses(trace.events)
-    c = hr.Checker.for_trace(trace, device=local_rank)
+    c = hr.Checker.for_trace(trace, device=local_rank, compact=args.compact)
+    bpa = bytes_per_access(c.rec_bytes)
     d_ev = hr.events_to_device(trace.events, f"cuda:{local_rank}")
     cap = 1 << 20
     d_out = torch.empty(cap * 16, dtype=torch.uint8, device="cuda")
@@ -467,7 +492,7 @@ def main():
             dist.destroy_process_group()
         return
     peak, peak_kind = peaks()
-    achieved = BYTES_PER_ACCESS * n_acc / (kern_ms / 1e3) / 1e9
+    achieved = bpa * n_acc / (kern_ms / 1e3) / 1e9
     slow = None if args.no_slowdown else measure_slowdown(local_rank)
     cpu = None
     if not args.no_cpu_baseline and world == 1:
@@ -484,16 +509,16 @@ def main():
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "u64", "data": "synthetic", "config": config_block(args, trace, world),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": load_traffic(args.config, args.variant),
+                     "frac": achieved / peak, "traffic": load_traffic(args.config, args.variant, args.compact),
                      "kernel": "k_replay (incl. fused collect)", "kernel_ms": kern_ms, "kernel_share": kern_ms / ms_per_step,
-                     "bytes_per_access": BYTES_PER_ACCESS, "peak_kind": peak_kind},
+                     "bytes_per_access": bpa, "peak_kind": peak_kind},
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": 2 * K,  # k_batches + k_replay (fused collect) per step
         "clocks": clocks.summary(),
         "check": {"flagged_words": flagged, "per_step": st},  # stats are per step (reset clears them)
         "instrumented_slowdown": slow,
-        "shadow_overhead": {"bytes_per_tracked_word": 8, "ratio_to_tracked_bytes": 2.0,
+        "shadow_overhead": {"bytes_per_tracked_word": c.rec_bytes, "ratio_to_tracked_bytes": c.rec_bytes / 4,
                             "iguard_ratio_context": 4.0},
     }
     print(json.dumps(out), flush=True)

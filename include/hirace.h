@@ -130,6 +130,12 @@ typedef struct {
     unsigned int bt_magic, bt_s1, bt_s2; /* fast division by block_threads                    */
     unsigned int ws_magic, ws_s1, ws_s2; /* fast division by warp_size                        */
     unsigned int g;                   /* current grid epoch for inline hooks                  */
+    /* record layout: rec_bytes = 8 (the 64-bit record of hirace_device.cuh) or 4 (compact
+     * record of hirace_shadow_alloc_compact: state:5 | g | b | w | tid, fields starting at
+     * bits 5, c_sh_b, c_sh_w, c_sh_t; epochs up to c_max_g / c_max_b / c_max_w)            */
+    unsigned int rec_bytes;
+    unsigned int c_sh_b, c_sh_w, c_sh_t;
+    unsigned int c_max_g, c_max_b, c_max_w;
 } hirace_dev_ctx;
 
 /* ---- lifecycle (a11: shadow alloc/init, "Initially, all State values are set
@@ -139,6 +145,31 @@ typedef struct {
  * all INIT, plus the FSM table and report buffer on cfg->device.  Synchronous.
  * Errors: INVAL (NULL args, zero geometry, granularity != 2, tid space > 2^32), NOMEM, CUDA. */
 hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out);
+
+/* ---- compact 32-bit shadow ("the shadow-memory footprint
+ *      ... can be reduced", L419-423) ------------------------------------------------------ */
+
+/* Declared upper bounds of the epoch counters of the traces a compact context will replay:
+ * g <= max_g (grid epochs / kernel boundaries), b <= max_b (__syncthreads since the last g),
+ * w <= max_w (full-warp syncs since the last b).  0 = that barrier level never occurs. */
+typedef struct {
+    uint32_t max_g, max_b, max_w;
+} hirace_epoch_limits;
+
+/* hirace_shadow_alloc with 4-byte records: half the shadow footprint (4 B per tracked 4-byte
+ * word = 1.0x the tracked bytes, vs 2.0x for 8-byte records).  The record is
+ *     state:5 | g:Gb | b:Bb | w:Wb | tid:T     (bit 0 upward, all-zero = INIT)
+ * with Gb/Bb/Wb = bits needed for max_g/max_b/max_w and T = bits needed for the largest global
+ * thread id.  It holds exactly the fields of the 8-byte record, never truncated, so every
+ * transition is the same (same FSM table, same label); verdicts are identical.
+ * Replay only: inline hooks (hirace_get_dev_ctx) and hirace_barrier need the 8-byte record.
+ * A replayed batch whose (g,b,w) exceeds the declared limits is not checked and raises sticky
+ * HIRACE_E_CLOCK_OVERFLOW (races found in earlier batches stay valid).
+ * Errors: INVAL (as hirace_shadow_alloc; NULL lim; max_g > 254, max_b > 1023, max_w > 511;
+ * 5 + Gb + Bb + Wb + T > 32 — the trace does not fit 32 bits, use hirace_shadow_alloc),
+ * NOMEM, CUDA. */
+hirace_status hirace_shadow_alloc_compact(const hirace_config *cfg, const hirace_epoch_limits *lim,
+                                          hirace_ctx **out);
 
 /* Frees everything the context owns (synchronises the device first).  NULL is a no-op. */
 hirace_status hirace_shadow_free(hirace_ctx *ctx);
@@ -266,6 +297,51 @@ hirace_status hirace_bucket_wire(hirace_ctx *ctx, const hirace_event *d_in, cons
  * order.  Records with tid or word out of range -> sticky BAD_TRACE at the next sync.  Async. */
 hirace_status hirace_replay_wire(hirace_ctx *ctx, const uint64_t *d_wire, uint64_t n, uint32_t batch_key, void *stream);
 
+/* ---- sharded mode, peer-memory dispatch (a10 fused with the exchange) --------
+ * The bucketing kernel stores every wire record DIRECTLY into its owner's receive buffer — on
+ * the owner's GPU over NVLink/NVSwitch (CUDA IPC mapping + P2P), or in another process on the
+ * same GPU — so the exchange is the scatter itself: no local staging copy, no separate
+ * all_to_all.  Protocol per trace (sharded.run_sharded_p2p):
+ *   1. hirace_count_wire: per-batch per-owner record counts (no output);
+ *   2. the ranks all-gather their count matrices; every rank derives, for each batch b and
+ *      owner r, where its segment starts in r's buffer: batches in the global order, inside a
+ *      batch the senders in rank order;
+ *   3. hirace_dispatch_wire with the peer table (each rank's buffer from
+ *      hirace_peer_buffer_alloc, opened by the others with hirace_peer_open);
+ *   4. stream sync + a process barrier make the stores visible; each owner replays its buffer
+ *      batch by batch with hirace_replay_wire. */
+
+/* Per-batch per-owner wire-record counts of nb batches of DEVICE events (h_offsets as from
+ * hirace_find_batches): HOST h_counts[nb * nranks], row b = batch b.  Exactly the records
+ * hirace_dispatch_wire / hirace_bucket_wire produce.  Synchronises `stream`.
+ * Errors: as hirace_bucket_wire. */
+hirace_status hirace_count_wire(hirace_ctx *ctx, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
+                                int nranks, int my_rank, uint64_t *h_counts, void *stream);
+
+/* Buckets nb batches of DEVICE events into wire records and stores each one into its owner's
+ * receive buffer: h_peer[r] (HOST array of nranks device addresses valid in this process, 8-byte
+ * aligned) at record index h_dst[b * nranks + r] + k, k = 0 .. count(b, r) - 1 in unspecified
+ * order.  The caller owns the buffers and guarantees the index ranges are
+ * inside them and disjoint across senders.  Synchronises `stream` (stores are complete on
+ * return; visibility to other processes needs their own synchronisation).
+ * Errors: INVAL (NULL args, a NULL peer, nranks not in 1..32, geometry beyond the wire format),
+ * BAD_TRACE (sticky: access size > 16 B, shard-local word >= 2^31), CUDA. */
+hirace_status hirace_dispatch_wire(hirace_ctx *ctx, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
+                                   int nranks, int my_rank, void *const *h_peer, const uint64_t *h_dst,
+                                   void *stream);
+
+/* A receive buffer of `bytes` on `device` that other processes can map: *d_ptr = its device
+ * address here, handle = its 64-byte CUDA IPC handle (to be sent to the peers).  The caller
+ * frees it with hirace_peer_buffer_free after every peer closed it.  Errors: INVAL, NOMEM, CUDA. */
+hirace_status hirace_peer_buffer_alloc(int device, uint64_t bytes, void **d_ptr, unsigned char handle[64]);
+hirace_status hirace_peer_buffer_free(void *d_ptr);
+
+/* Maps a peer's receive buffer (handle from hirace_peer_buffer_alloc in ANOTHER process) into
+ * this process on `device`, enabling peer access when it lives on another GPU.  Unmap with
+ * hirace_peer_close.  Errors: INVAL, CUDA (e.g. no P2P path, or the handle is this process's). */
+hirace_status hirace_peer_open(int device, const unsigned char handle[64], void **d_ptr);
+hirace_status hirace_peer_close(void *d_ptr);
+
 /* ---- microbenchmarks for the roofline (diagnostics; not part of the checking path) -------- */
 
 /* Rate of 64-bit operations on `nwords` distinct words of a fresh device array (nwords*8 bytes;
@@ -303,6 +379,13 @@ uint64_t hirace_fsm_step(uint64_t old_shadow, uint32_t tid, uint32_t kind, uint3
 /* hirace_fsm_step under a given hirace_policy (unknown values select STRICT). */
 uint64_t hirace_fsm_step_policy(int policy, uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t b,
                                 uint32_t w, uint32_t block_threads, uint32_t warp_size, int *report);
+
+/* One FSM step on a compact 4-byte record (hirace_shadow_alloc_compact layout for grid_threads
+ * threads and limits *lim), with the same inline functions the compact replay kernels use.
+ * Inputs must lie within the limits.  Returns 0xffffffff if the layout does not fit 32 bits. */
+uint32_t hirace_fsm_step_compact(int policy, uint32_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t b,
+                                 uint32_t w, uint32_t block_threads, uint32_t warp_size, uint32_t grid_threads,
+                                 const hirace_epoch_limits *lim, int *report);
 
 const char *hirace_status_string(hirace_status s);
 

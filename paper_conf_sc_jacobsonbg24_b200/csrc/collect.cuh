@@ -2,7 +2,8 @@
  *
  * The flagged words are exactly the shadow records in a RACE state (RACE is sticky, one
  * record per word), so an order-preserving compaction of the shadow yields the unique,
- * key-sorted race set (global words first, then shared words block-major).  Each CTA owns a
+ * key-sorted race set (global words first, then shared words block-major).  Instantiated per
+ * record layout (record.cuh).  Each CTA owns a
  * contiguous range of 4096-word tiles: pass 1 counts its flagged words, one grid barrier
  * publishes the per-CTA counts, each CTA sums the counts before it, and pass 2 re-reads its
  * range (now L2-hot) and writes the records in order. */
@@ -14,24 +15,44 @@
 #include "hirace_device.cuh"
 #include "internal.h"
 #include "kernel_common.cuh"
+#include "record.cuh"
 
 namespace hirace_impl {
 
 constexpr int kCollectPerThread = 16; /* consecutive words per thread per tile */
 static_assert(kCollectTile == 256 * kCollectPerThread, "collect tile = 256 threads x 16 words");
 
-/* flagged-word count of the 16 words of this thread in tile t; words kept in v */
-__device__ __forceinline__ uint32_t collect_load(const unsigned long long *shadow, uint64_t nwords, uint64_t w0,
-                                                 ulonglong2 (&v)[kCollectPerThread / 2])
+/* flagged-word count of the 16 words of this thread in tile t; words kept in v (16-byte
+ * vector loads: 2 records of 8 bytes or 4 compact records each) */
+template <typename R>
+__device__ __forceinline__ uint32_t collect_load(const R *shadow, uint64_t nwords, uint64_t w0,
+                                                 R (&v)[kCollectPerThread])
 {
+    constexpr int per = 16 / sizeof(R);
     uint32_t n = 0;
 #pragma unroll
-    for (int k = 0; k < kCollectPerThread / 2; k++) {
-        const uint64_t wi = w0 + 2 * k;
-        v[k] = wi + 1 < nwords ? reinterpret_cast<const ulonglong2 *>(shadow + w0)[k]
-                               : make_ulonglong2(wi < nwords ? shadow[wi] : 0ull, 0ull);
-        n += (hirace::st_of(v[k].x) >= hirace::ST_RACE_W) + (hirace::st_of(v[k].y) >= hirace::ST_RACE_W);
+    for (int k = 0; k < kCollectPerThread / per; k++) {
+        const uint64_t wi = w0 + (uint64_t)per * k;
+        if (wi + per <= nwords) {
+            const uint4 q = reinterpret_cast<const uint4 *>(shadow + w0)[k];
+            if (sizeof(R) == 8) {
+                v[per * k] = (R)(((unsigned long long)q.y << 32) | q.x);
+                v[per * k + 1] = (R)(((unsigned long long)q.w << 32) | q.z);
+            } else {
+                v[per * k] = (R)q.x;
+                v[per * k + 1] = (R)q.y;
+                v[per * k + 2] = (R)q.z;
+                v[per * k + 3] = (R)q.w;
+            }
+        } else {
+#pragma unroll
+            for (int j = 0; j < per; j++)
+                v[per * k + j] = wi + j < nwords ? shadow[wi + j] : (R)0;
+        }
     }
+#pragma unroll
+    for (int k = 0; k < kCollectPerThread; k++)
+        n += hirace::st_of(v[k]) >= hirace::ST_RACE_W;
     return n;
 }
 
@@ -63,6 +84,7 @@ __device__ __forceinline__ uint32_t block_exclusive_scan(uint32_t mine, uint32_t
 
 /* grid-wide collect; every thread of every CTA of a cooperative launch must call it.
  * cta_cnt: gridDim.x words of scratch.  Writes min(cap, total) records and *d_total. */
+template <typename R>
 __device__ __forceinline__ void collect_phase(const hirace_dev_ctx &c, uint64_t nwords, hirace_race *out,
                                               uint64_t cap, unsigned long long *d_total, uint32_t *cta_cnt,
                                               unsigned int *bar, unsigned int &bar_epoch)
@@ -72,12 +94,14 @@ __device__ __forceinline__ void collect_phase(const hirace_dev_ctx &c, uint64_t 
     const uint64_t ntiles = (nwords + kCollectTile - 1) / kCollectTile;
     const uint64_t t0 = ntiles * blockIdx.x / gridDim.x, t1 = ntiles * (blockIdx.x + 1) / gridDim.x;
     const uint32_t tpb = blockDim.x; /* threads cover a tile in kCollectTile / tpb rounds */
-    ulonglong2 v[kCollectPerThread / 2];
+    R v[kCollectPerThread];
+    const R *const shadow = shadow_as<R>(c);
+    const Rec<R> rec(c);
     /* pass 1: count */
     uint32_t mine = 0;
     for (uint64_t t = t0; t < t1; t++)
         for (uint32_t r = threadIdx.x; r < kCollectTile / kCollectPerThread; r += tpb)
-            mine += collect_load(c.shadow, nwords, t * kCollectTile + (uint64_t)r * kCollectPerThread, v);
+            mine += collect_load<R>(shadow, nwords, t * kCollectTile + (uint64_t)r * kCollectPerThread, v);
     uint32_t cta_total;
     block_exclusive_scan(mine, s_w, &cta_total);
     if (threadIdx.x == 0)
@@ -107,14 +131,14 @@ __device__ __forceinline__ void collect_phase(const hirace_dev_ctx &c, uint64_t 
         for (uint32_t r0 = 0; r0 < kCollectTile / kCollectPerThread; r0 += tpb) {
             const uint32_t r = r0 + threadIdx.x;
             const uint64_t w0 = t * kCollectTile + (uint64_t)r * kCollectPerThread;
-            const uint32_t n = r < kCollectTile / kCollectPerThread ? collect_load(c.shadow, nwords, w0, v) : 0u;
+            const uint32_t n = r < kCollectTile / kCollectPerThread ? collect_load<R>(shadow, nwords, w0, v) : 0u;
             uint32_t round_total;
             const uint32_t excl = block_exclusive_scan(n, s_w, &round_total);
             uint64_t pos = base + excl;
             if (n) {
 #pragma unroll
                 for (int k = 0; k < kCollectPerThread; k++) {
-                    const uint64_t o = (k & 1) ? v[k / 2].y : v[k / 2].x;
+                    const R o = v[k];
                     if (hirace::st_of(o) >= hirace::ST_RACE_W) {
                         if (pos < cap) {
                             const uint64_t wi = w0 + k;
@@ -126,8 +150,8 @@ __device__ __forceinline__ void collect_phase(const hirace_dev_ctx &c, uint64_t 
                                 const uint64_t blk = sidx / smem_words;
                                 rr.key = HIRACE_SHARED_BIT | (blk << 32) | (sidx - blk * smem_words);
                             }
-                            rr.cls_and_epoch = hirace::race_class(hirace::st_of(o)) | (hirace::g_of(o) << 8);
-                            rr.detect_tid = hirace::tid_of(o);
+                            rr.cls_and_epoch = hirace::race_class(hirace::st_of(o)) | (rec.g(o) << 8);
+                            rr.detect_tid = rec.tid(o);
                             out[pos] = rr;
                         }
                         pos++;
@@ -137,6 +161,86 @@ __device__ __forceinline__ void collect_phase(const hirace_dev_ctx &c, uint64_t 
             base += round_total;
         }
     }
+}
+
+/* ---- report-buffer collection ("Collect = device sort + unique(key, max
+ * class); fallback = shadow scan") -------------------------------------------------------
+ * Every word that reaches RACE appends a report when its CAS enters RACE or upgrades the class
+ * (replay.cu append_reports, hirace_device.cuh report_one), so while the buffer has not
+ * overflowed the reported keys are exactly the flagged words.  For a large shadow with few
+ * races this replaces the full shadow scan (config 5: 32 GiB) by a sort of the reports: one
+ * CTA sorts the keys in shared memory, drops duplicates, and reads each word's final record
+ * (class, g*, detecting thread) from the shadow.  Output = the scan's output (unique keys in
+ * key order, which is shadow order). */
+constexpr uint32_t kReportSortCap = 16384; /* keys sorted in shared memory (128 KB) */
+constexpr int kReportThreads = 1024;
+
+/* the report path applies: report mode on, and every report fits the buffer and the sort */
+__device__ __forceinline__ bool reports_cover(const hirace_dev_ctx &c)
+{
+    const unsigned long long n = __ldcg(c.report_count);
+    return n <= kReportSortCap && n <= c.report_capacity;
+}
+
+template <typename R>
+__device__ __forceinline__ void collect_reports_cta(const hirace_dev_ctx &c, hirace_race *out, uint64_t cap,
+                                                    unsigned long long *d_total, unsigned long long *s_keys)
+{
+    __shared__ uint32_t s_w[32];
+    const unsigned long long n = __ldcg(c.report_count);
+    if (n > kReportSortCap || n > c.report_capacity)
+        return; /* the shadow scan collects */
+    uint32_t P = 1;
+    while (P < (uint32_t)n)
+        P <<= 1;
+    for (uint32_t i = threadIdx.x; i < P; i += blockDim.x)
+        s_keys[i] = i < n ? __ldcg(&c.reports[i].key) : ~0ull;
+    __syncthreads();
+    for (uint32_t k = 2; k <= P; k <<= 1) { /* bitonic sort, ascending */
+        for (uint32_t j = k >> 1; j > 0; j >>= 1) {
+            for (uint32_t i = threadIdx.x; i < P; i += blockDim.x) {
+                const uint32_t ixj = i ^ j;
+                if (ixj > i) {
+                    const unsigned long long x = s_keys[i], y = s_keys[ixj];
+                    if ((x > y) == ((i & k) == 0)) {
+                        s_keys[i] = y;
+                        s_keys[ixj] = x;
+                    }
+                }
+            }
+            __syncthreads();
+        }
+    }
+    /* each thread: a contiguous run of sorted keys; keep first occurrences whose record is RACE */
+    const uint32_t per = (P + blockDim.x - 1) / blockDim.x;
+    const uint32_t lo = threadIdx.x * per, hi = min(lo + per, (uint32_t)n);
+    const R *const shadow = shadow_as<R>(c);
+    const Rec<R> rec(c);
+    const uint64_t smem_words = c.smem_words ? c.smem_words : 1;
+    uint32_t mine = 0;
+    for (uint32_t i = lo; i < hi; i++)
+        mine += (i == 0 || s_keys[i] != s_keys[i - 1]) ? 1u : 0u;
+    uint32_t total;
+    uint64_t pos = block_exclusive_scan(mine, s_w, &total);
+    for (uint32_t i = lo; i < hi; i++) {
+        const unsigned long long key = s_keys[i];
+        if (i != 0 && key == s_keys[i - 1])
+            continue;
+        const uint64_t idx = (key & HIRACE_SHARED_BIT)
+                                 ? c.global_words + ((key >> 32) & 0x7fffffffull) * smem_words + (key & 0xffffffffull)
+                                 : key;
+        const R o = (R)__ldcg(shadow + idx);
+        if (pos < cap) {
+            hirace_race rr;
+            rr.key = key;
+            rr.cls_and_epoch = hirace::race_class(hirace::st_of(o)) | (rec.g(o) << 8);
+            rr.detect_tid = rec.tid(o);
+            out[pos] = rr;
+        }
+        pos++;
+    }
+    if (threadIdx.x == 0)
+        *d_total = total;
 }
 
 } // namespace hirace_impl

@@ -360,3 +360,34 @@ extern "C" uint64_t hirace_fsm_step(uint64_t old_shadow, uint32_t tid, uint32_t 
 {
     return hirace_fsm_step_policy(0, old_shadow, tid, kind, g, b, w, block_threads, warp_size, report);
 }
+
+/* compact 4-byte record (hirace_shadow_alloc_compact): the kernels' raw-flag table and
+ * label_raw_c / next_c, on the host */
+extern "C" uint32_t hirace_fsm_step_compact(int policy, uint32_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g,
+                                            uint32_t b, uint32_t w, uint32_t block_threads, uint32_t warp_size,
+                                            uint32_t grid_threads, const hirace_epoch_limits *lim, int *report)
+{
+    static unsigned char raw[2][2048 + hirace::RAW_TABLE_BYTES];
+    static bool built[2] = {false, false};
+    policy = policy == 1 ? 1 : 0;
+    if (!built[policy]) {
+        hirace_fsm_table_policy(policy, raw[policy]);
+        hirace::expand_raw_table(raw[policy], raw[policy] + 2048);
+        built[policy] = true;
+    }
+    hirace::clay L;
+    if (!lim || !hirace::make_clay(lim->max_g, lim->max_b, lim->max_w, grid_threads, &L))
+        return 0xffffffffu;
+    hirace_dev_ctx c{};
+    c.block_threads = block_threads ? block_threads : 1;
+    c.warp_size = warp_size ? warp_size : 1;
+    hirace::fastdiv_init(c.block_threads, &c.bt_magic, &c.bt_s1, &c.bt_s2);
+    hirace::fastdiv_init(c.warp_size, &c.ws_magic, &c.ws_s1, &c.ws_s2);
+    const hirace::geom G = hirace::make_geom(c);
+    uint32_t rep = 0;
+    const uint32_t n = hirace::step_c(old_shadow, tid, kind & 3u, hirace::c_epochs(L, g, b, w), raw[policy] + 2048, L,
+                                      G, &rep);
+    if (report)
+        *report = (int)rep;
+    return n;
+}

@@ -25,6 +25,7 @@ struct hirace_ctx {
     int sm_count = 0;
     int replay_grid = 0;
     uint64_t global_words = 0, shadow_words = 0;
+    uint32_t rec_bytes = 8; /* 8-byte records, or 4 (compact, hirace_shadow_alloc_compact) */
     unsigned long long *d_shadow = nullptr;
     unsigned char *d_table = nullptr;
     unsigned char h_table[2048 + hirace::RAW_TABLE_BYTES]; /* canonical | raw-flag expansion */
@@ -48,6 +49,9 @@ struct hirace_ctx {
     unsigned long long *d_wire_counts = nullptr; /* nb x nranks (+1: running total)    */
     uint64_t wire_counts_cap = 0;
     unsigned int *d_wire_flag = nullptr;
+    /* peer dispatch: [nranks peer buffer pointers | nb x nranks destination offsets] */
+    unsigned long long *d_peer_tab = nullptr;
+    uint64_t peer_tab_cap = 0;
     /* host-trace staging ring */
     hirace_event *d_stage[2] = {nullptr, nullptr};
     uint64_t stage_cap = 0;
@@ -81,6 +85,15 @@ hirace_status from_cuda(hirace_ctx *c, cudaError_t e)
         if (_e != cudaSuccess)                         \
             return from_cuda((c), _e);                 \
     } while (0)
+
+/* collect from the report buffer (falling back to the shadow scan on the device) when the
+ * shadow is large enough for a full scan to cost more than the sort (collect.cuh) */
+int report_mode(const hirace_ctx *c)
+{
+    if (const char *f = getenv("HIRACE_COLLECT")) /* "scan" / "reports": force a path (tests, A/B) */
+        return f[0] == 'r' ? 1 : 0;
+    return c->shadow_words * c->rec_bytes >= kReportModeMinBytes ? 1 : 0;
+}
 
 hirace_status device_errors(hirace_ctx *c)
 {
@@ -116,7 +129,10 @@ const char *hirace_status_string(hirace_status s)
     return "unknown";
 }
 
-hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
+namespace {
+
+/* shared by hirace_shadow_alloc (lim == NULL: 8-byte records) and hirace_shadow_alloc_compact */
+hirace_status shadow_alloc_impl(const hirace_config *cfg, const hirace_epoch_limits *lim, hirace_ctx **out)
 {
     if (!cfg || !out)
         return HIRACE_E_INVAL;
@@ -127,6 +143,13 @@ hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
         return HIRACE_E_INVAL;
     if ((cfg->smem_bytes_per_block & 3) || (cfg->global_bytes & 3))
         return HIRACE_E_INVAL;
+    hirace::clay lay{};
+    if (lim) {
+        if (lim->max_g > 254u || lim->max_b > 1023u || lim->max_w > 511u)
+            return HIRACE_E_INVAL;
+        if (!hirace::make_clay(lim->max_g, lim->max_b, lim->max_w, cfg->grid_blocks * cfg->block_threads, &lay))
+            return HIRACE_E_INVAL; /* the record would not fit 32 bits */
+    }
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0 || cfg->device < 0 || cfg->device >= ndev)
         return HIRACE_E_CUDA;
@@ -137,6 +160,7 @@ hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
     if (c->cfg.report_capacity == 0)
         c->cfg.report_capacity = 1ull << 20;
     c->device = cfg->device;
+    c->rec_bytes = lim ? 4u : 8u;
     c->global_words = cfg->global_bytes >> 2;
     const uint64_t smem_words = cfg->smem_bytes_per_block >> 2;
     c->shadow_words = c->global_words + (uint64_t)cfg->grid_blocks * smem_words;
@@ -164,7 +188,7 @@ hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
         return HIRACE_E_INVAL;
     }
     c->scr.collect_grid = collect_max_grid(c->device);
-    if ((e = cudaMalloc(&c->d_shadow, c->shadow_words * 8)) != cudaSuccess ||
+    if ((e = cudaMalloc(&c->d_shadow, c->shadow_words * c->rec_bytes)) != cudaSuccess ||
         (e = cudaMalloc(&c->d_table, 2048 + hirace::RAW_TABLE_BYTES)) != cudaSuccess ||
         (e = cudaMalloc(&c->d_reports, c->cfg.report_capacity * sizeof(hirace_race))) != cudaSuccess ||
         (e = cudaMalloc(&c->d_report_count, sizeof(unsigned long long))) != cudaSuccess ||
@@ -198,12 +222,33 @@ hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
     hirace::fastdiv_init(cfg->block_threads, &d.bt_magic, &d.bt_s1, &d.bt_s2);
     hirace::fastdiv_init(cfg->warp_size, &d.ws_magic, &d.ws_s1, &d.ws_s2);
     d.g = 0;
+    d.rec_bytes = c->rec_bytes;
+    d.c_sh_b = lay.sh_b;
+    d.c_sh_w = lay.sh_w;
+    d.c_sh_t = lay.sh_t;
+    d.c_max_g = lim ? lim->max_g : 254u;
+    d.c_max_b = lim ? lim->max_b : 1023u;
+    d.c_max_w = lim ? lim->max_w : 511u;
     if (hirace_shadow_reset(c, nullptr) != HIRACE_OK || cudaDeviceSynchronize() != cudaSuccess) {
         hirace_shadow_free(c);
         return HIRACE_E_CUDA;
     }
     *out = c;
     return HIRACE_OK;
+}
+
+} // namespace
+
+hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out)
+{
+    return shadow_alloc_impl(cfg, nullptr, out);
+}
+
+hirace_status hirace_shadow_alloc_compact(const hirace_config *cfg, const hirace_epoch_limits *lim, hirace_ctx **out)
+{
+    if (!lim)
+        return HIRACE_E_INVAL;
+    return shadow_alloc_impl(cfg, lim, out);
 }
 
 hirace_status hirace_shadow_free(hirace_ctx *c)
@@ -215,7 +260,8 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
     void *ptrs[] = {c->d_shadow, c->d_table, c->d_reports, c->d_report_count, c->d_stats, c->d_err,
                     c->scr.batch_off, c->scr.nbatches, c->scr.batch_ctr, c->scr.grid_bar,
                     c->scr.grid_bar2, c->scr.cta_cnt, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
-                    c->d_stage[0], c->d_stage[1], c->d_wire_off, c->d_wire_counts, c->d_wire_flag};
+                    c->d_stage[0], c->d_stage[1], c->d_wire_off, c->d_wire_counts, c->d_wire_flag,
+                    c->d_peer_tab};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
@@ -256,7 +302,7 @@ hirace_status hirace_shadow_reset(hirace_ctx *c, void *stream)
         return HIRACE_E_INVAL;
     cudaStream_t st = (cudaStream_t)stream;
     HR_CUDA(c, cudaSetDevice(c->device));
-    HR_CUDA(c, cudaMemsetAsync(c->d_shadow, 0, c->shadow_words * 8, st));
+    HR_CUDA(c, cudaMemsetAsync(c->d_shadow, 0, c->shadow_words * c->rec_bytes, st));
     HR_CUDA(c, cudaMemsetAsync(c->d_report_count, 0, sizeof(unsigned long long), st));
     HR_CUDA(c, cudaMemsetAsync(c->d_stats, 0, 4 * sizeof(unsigned long long), st));
     HR_CUDA(c, cudaMemsetAsync(c->d_err, 0, sizeof(unsigned int), st));
@@ -272,7 +318,7 @@ hirace_status hirace_barrier(hirace_ctx *c, hirace_scope scope, void *stream)
         return HIRACE_E_INVAL;
     if (c->sticky != HIRACE_OK)
         return c->sticky;
-    if (scope != HIRACE_SCOPE_GRID)
+    if (scope != HIRACE_SCOPE_GRID || c->rec_bytes != 8) /* compact contexts are replay-only */
         return set_sticky(c, HIRACE_E_INVAL);
     HR_CUDA(c, cudaSetDevice(c->device));
     if (c->g + 1 >= 255u) {
@@ -362,7 +408,8 @@ hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_eve
     HR_CUDA(c, launch_find_batches(d_events, (uint32_t)n, c->scr, c->d_err, c->sm_count, st));
     if (c->t_start)
         HR_CUDA(c, cudaEventRecord(c->t_start, st));
-    HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st, c->shadow_words, d_out, cap, d_n_total));
+    HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st, c->shadow_words, d_out, cap, d_n_total,
+                             report_mode(c)));
     if (c->t_stop)
         HR_CUDA(c, cudaEventRecord(c->t_stop, st));
     return HIRACE_OK;
@@ -374,7 +421,8 @@ hirace_status hirace_collect_races_device(hirace_ctx *c, hirace_race *d_out, uin
     if (!c || !d_n_total || (cap && !d_out))
         return HIRACE_E_INVAL;
     HR_CUDA(c, cudaSetDevice(c->device));
-    HR_CUDA(c, launch_collect(c->dev, c->shadow_words, c->scr, d_out, cap, d_n_total, (cudaStream_t)stream));
+    HR_CUDA(c, launch_collect(c->dev, c->shadow_words, c->scr, d_out, cap, d_n_total, (cudaStream_t)stream,
+                              report_mode(c)));
     return c->sticky;
 }
 
@@ -392,7 +440,7 @@ hirace_status hirace_collect_races(hirace_ctx *c, hirace_race *h_out, uint64_t c
         HR_CUDA(c, cudaMalloc(&c->d_collect, cap * sizeof(hirace_race)));
         c->collect_cap = cap;
     }
-    HR_CUDA(c, launch_collect(c->dev, c->shadow_words, c->scr, c->d_collect, cap, c->d_total, st));
+    HR_CUDA(c, launch_collect(c->dev, c->shadow_words, c->scr, c->d_collect, cap, c->d_total, st, report_mode(c)));
     unsigned long long total = 0;
     HR_CUDA(c, cudaMemcpyAsync(&total, c->d_total, sizeof(total), cudaMemcpyDeviceToHost, st));
     HR_CUDA(c, cudaStreamSynchronize(st));
@@ -487,7 +535,7 @@ hirace_status hirace_sync(hirace_ctx *c)
 
 hirace_status hirace_get_dev_ctx(hirace_ctx *c, const void *global_base, hirace_dev_ctx *out)
 {
-    if (!c || !out)
+    if (!c || !out || c->rec_bytes != 8) /* inline hooks use the 8-byte record */
         return HIRACE_E_INVAL;
     *out = c->dev;
     out->global_base = global_base;
@@ -532,26 +580,13 @@ hirace_status hirace_bucket_events(hirace_ctx *c, const hirace_event *d_in, uint
     return HIRACE_OK;
 }
 
-hirace_status hirace_bucket_wire(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
-                                 int nranks, int my_rank, uint64_t *d_out, uint64_t cap, uint64_t *h_counts,
-                                 uint64_t *n_words, void *stream)
+} /* extern "C" */
+
+namespace {
+
+/* scratch for per-batch wire bucketing of up to maxlen events into nranks owners */
+hirace_status wire_scratch(hirace_ctx *c, uint64_t nb, int nranks, uint32_t maxlen)
 {
-    if (!c || !h_offsets || !h_counts || !n_words || nranks < 1 || nranks > 32 || my_rank < 0 || my_rank >= nranks ||
-        nb > HIRACE_MAX_BATCHES || (nb && !d_in) || (cap && !d_out))
-        return HIRACE_E_INVAL;
-    if (c->sticky != HIRACE_OK)
-        return c->sticky;
-    const uint64_t threads = (uint64_t)c->cfg.grid_blocks * c->cfg.block_threads;
-    if (threads > HIRACE_WIRE_MAX_TIDS || (uint64_t)c->dev.smem_words > HIRACE_WIRE_MAX_WORDS)
-        return HIRACE_E_INVAL;
-    for (uint64_t b = 0; b < nb; b++)
-        if (h_offsets[b + 1] < h_offsets[b] || h_offsets[b + 1] >= 0xffffffffu)
-            return HIRACE_E_INVAL;
-    cudaStream_t st = (cudaStream_t)stream;
-    HR_CUDA(c, cudaSetDevice(c->device));
-    uint32_t maxlen = 0;
-    for (uint64_t b = 0; b < nb; b++)
-        maxlen = h_offsets[b + 1] - h_offsets[b] > maxlen ? h_offsets[b + 1] - h_offsets[b] : maxlen;
     const uint64_t ntiles = (maxlen + kWireTile - 1) / kWireTile;
     const uint64_t need_hist = ntiles * (uint64_t)nranks;
     if (need_hist > c->bucket_hist_cap) {
@@ -581,6 +616,148 @@ hirace_status hirace_bucket_wire(hirace_ctx *c, const hirace_event *d_in, const 
     }
     if (!c->d_wire_flag)
         HR_CUDA(c, cudaMalloc(&c->d_wire_flag, sizeof(unsigned int)));
+    return HIRACE_OK;
+}
+
+hirace_status wire_args_ok(hirace_ctx *c, const uint32_t *h_offsets, uint64_t nb, int nranks, int my_rank,
+                           uint32_t *maxlen)
+{
+    if (nranks < 1 || nranks > 32 || my_rank < 0 || my_rank >= nranks || nb > HIRACE_MAX_BATCHES)
+        return HIRACE_E_INVAL;
+    const uint64_t threads = (uint64_t)c->cfg.grid_blocks * c->cfg.block_threads;
+    if (threads > HIRACE_WIRE_MAX_TIDS || (uint64_t)c->dev.smem_words > HIRACE_WIRE_MAX_WORDS)
+        return HIRACE_E_INVAL;
+    *maxlen = 0;
+    for (uint64_t b = 0; b < nb; b++) {
+        if (h_offsets[b + 1] < h_offsets[b] || h_offsets[b + 1] >= 0xffffffffu)
+            return HIRACE_E_INVAL;
+        *maxlen = h_offsets[b + 1] - h_offsets[b] > *maxlen ? h_offsets[b + 1] - h_offsets[b] : *maxlen;
+    }
+    return HIRACE_OK;
+}
+
+} // namespace
+
+extern "C" {
+
+hirace_status hirace_count_wire(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
+                                int nranks, int my_rank, uint64_t *h_counts, void *stream)
+{
+    uint64_t n = 0;
+    if (!c || !h_counts || !h_offsets || (nb && !d_in))
+        return HIRACE_E_INVAL;
+    const hirace_status s = hirace_bucket_wire(c, d_in, h_offsets, nb, nranks, my_rank, nullptr, 0, h_counts, &n,
+                                               stream);
+    return (s == HIRACE_E_INVAL && n > 0) ? HIRACE_OK : s; /* count-only: no output buffer */
+}
+
+hirace_status hirace_dispatch_wire(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
+                                   int nranks, int my_rank, void *const *h_peer, const uint64_t *h_dst, void *stream)
+{
+    if (!c || !h_offsets || !h_peer || !h_dst || (nb && !d_in))
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    uint32_t maxlen = 0;
+    hirace_status s = wire_args_ok(c, h_offsets, nb, nranks, my_rank, &maxlen);
+    if (s != HIRACE_OK)
+        return s;
+    for (int r = 0; r < nranks; r++)
+        if (!h_peer[r])
+            return HIRACE_E_INVAL;
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    if ((s = wire_scratch(c, nb, nranks, maxlen)) != HIRACE_OK)
+        return s;
+    /* device copies of the peer table and every batch's per-owner destinations; the host
+     * arrays may be reused by the caller as soon as this call returns (staged, then synced) */
+    const uint64_t need = (uint64_t)nranks + nb * (uint64_t)nranks;
+    if (need > c->peer_tab_cap) {
+        if (c->d_peer_tab)
+            cudaFree(c->d_peer_tab);
+        c->d_peer_tab = nullptr;
+        c->peer_tab_cap = 0;
+        HR_CUDA(c, cudaMalloc(&c->d_peer_tab, need * sizeof(unsigned long long)));
+        c->peer_tab_cap = need;
+    }
+    HR_CUDA(c, cudaMemcpyAsync(c->d_peer_tab, h_peer, nranks * sizeof(void *), cudaMemcpyHostToDevice, st));
+    if (nb)
+        HR_CUDA(c, cudaMemcpyAsync(c->d_peer_tab + nranks, h_dst, nb * nranks * sizeof(uint64_t),
+                                   cudaMemcpyHostToDevice, st));
+    HR_CUDA(c, cudaMemsetAsync(c->d_wire_flag, 0, sizeof(unsigned int), st));
+    for (uint64_t b = 0; b < nb; b++)
+        HR_CUDA(c, launch_dispatch_wire(d_in, h_offsets[b], h_offsets[b + 1], nranks, my_rank,
+                                        reinterpret_cast<unsigned long long *const *>(c->d_peer_tab),
+                                        c->d_peer_tab + nranks + b * (uint64_t)nranks, c->d_bucket_hist,
+                                        c->d_wire_off, c->d_wire_flag, st));
+    unsigned int flag = 0;
+    HR_CUDA(c, cudaMemcpyAsync(&flag, c->d_wire_flag, sizeof(flag), cudaMemcpyDeviceToHost, st));
+    HR_CUDA(c, cudaStreamSynchronize(st));
+    if (flag & hirace::ERR_BAD_TRACE)
+        return set_sticky(c, HIRACE_E_BAD_TRACE);
+    return HIRACE_OK;
+}
+
+hirace_status hirace_peer_buffer_alloc(int device, uint64_t bytes, void **d_ptr, unsigned char handle[64])
+{
+    if (!d_ptr || !handle || bytes == 0)
+        return HIRACE_E_INVAL;
+    *d_ptr = nullptr;
+    if (cudaSetDevice(device) != cudaSuccess)
+        return HIRACE_E_CUDA;
+    void *p = nullptr;
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e != cudaSuccess)
+        return e == cudaErrorMemoryAllocation ? HIRACE_E_NOMEM : HIRACE_E_CUDA;
+    cudaIpcMemHandle_t h;
+    static_assert(sizeof(h) == 64, "CUDA IPC handles are 64 bytes");
+    if (cudaIpcGetMemHandle(&h, p) != cudaSuccess) {
+        cudaFree(p);
+        return HIRACE_E_CUDA;
+    }
+    memcpy(handle, &h, 64);
+    *d_ptr = p;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_peer_buffer_free(void *d_ptr)
+{
+    return cudaFree(d_ptr) == cudaSuccess ? HIRACE_OK : HIRACE_E_CUDA;
+}
+
+hirace_status hirace_peer_open(int device, const unsigned char handle[64], void **d_ptr)
+{
+    if (!handle || !d_ptr)
+        return HIRACE_E_INVAL;
+    *d_ptr = nullptr;
+    if (cudaSetDevice(device) != cudaSuccess)
+        return HIRACE_E_CUDA;
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle, 64);
+    return cudaIpcOpenMemHandle(d_ptr, h, cudaIpcMemLazyEnablePeerAccess) == cudaSuccess ? HIRACE_OK : HIRACE_E_CUDA;
+}
+
+hirace_status hirace_peer_close(void *d_ptr)
+{
+    return cudaIpcCloseMemHandle(d_ptr) == cudaSuccess ? HIRACE_OK : HIRACE_E_CUDA;
+}
+
+hirace_status hirace_bucket_wire(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
+                                 int nranks, int my_rank, uint64_t *d_out, uint64_t cap, uint64_t *h_counts,
+                                 uint64_t *n_words, void *stream)
+{
+    if (!c || !h_offsets || !h_counts || !n_words || (nb && !d_in) || (cap && !d_out))
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    uint32_t maxlen = 0;
+    hirace_status s = wire_args_ok(c, h_offsets, nb, nranks, my_rank, &maxlen);
+    if (s != HIRACE_OK)
+        return s;
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    if ((s = wire_scratch(c, nb, nranks, maxlen)) != HIRACE_OK)
+        return s;
     unsigned long long *running = c->d_wire_counts + nb * (uint64_t)nranks;
     HR_CUDA(c, cudaMemsetAsync(running, 0, sizeof(unsigned long long), st));
     HR_CUDA(c, cudaMemsetAsync(c->d_wire_flag, 0, sizeof(unsigned int), st));

@@ -165,32 +165,8 @@ cudaError_t launch_find_batches(const hirace_event *ev, uint32_t n, const Scratc
 /* words first, then shared words block-major)                                               */
 /* ---------------------------------------------------------------------------------------- */
 
-/* standalone collect: one cooperative kernel running collect_phase (collect.cuh) */
-__global__ void __launch_bounds__(256) k_collect(hirace_dev_ctx c, uint64_t nwords, hirace_race *out, uint64_t cap,
-                                                 unsigned long long *d_total, uint32_t *cta_cnt, unsigned int *bar)
-{
-    unsigned int epoch = 0;
-    collect_phase(c, nwords, out, cap, d_total, cta_cnt, bar, epoch);
-}
-
-cudaError_t launch_collect(const hirace_dev_ctx &c, uint64_t shadow_words, const Scratch &s, hirace_race *out,
-                           uint64_t cap, unsigned long long *d_total, cudaStream_t st)
-{
-    cudaError_t e = cudaMemsetAsync(s.grid_bar2, 0, sizeof(unsigned int), st);
-    if (e != cudaSuccess)
-        return e;
-    hirace_dev_ctx cc = c;
-    uint64_t nw = shadow_words;
-    hirace_race *o = out;
-    uint64_t cp = cap;
-    unsigned long long *dt = d_total;
-    uint32_t *cnt = s.cta_cnt;
-    unsigned int *bar = s.grid_bar2;
-    void *args[] = {&cc, &nw, &o, &cp, &dt, &cnt, &bar};
-    const uint64_t ntiles = (shadow_words + kCollectTile - 1) / kCollectTile;
-    const int grid = (int)(ntiles < (uint64_t)s.collect_grid ? ntiles : (uint64_t)s.collect_grid);
-    return cudaLaunchCooperativeKernel((const void *)k_collect, dim3(grid), dim3(256), args, 0, st);
-}
+/* the standalone collect kernel (k_collect<R>) and its launcher live in replay.cu, next to
+ * the fused collect, instantiated per record layout */
 
 /* ---------------------------------------------------------------------------------------- */
 /* a8: grid-epoch wrap — every access before a grid barrier happens-before every later one,  */
@@ -493,11 +469,16 @@ __global__ void __launch_bounds__(1024) k_wire_scan(uint32_t *tile_hist, uint32_
 
 /* scatter: each word gets a slot in its (owner) segment; order inside a batch is free
  * (PAPER.md L177), so slots are taken with warp-aggregated shared-memory counters */
+/* peer != nullptr (peer dispatch, hirace_dispatch_wire): the record goes straight to its
+ * owner's receive buffer peer[owner] (its own memory, or a peer GPU's / another process's
+ * buffer mapped through CUDA IPC, stores travelling over NVLink), at the slot given by the
+ * per-owner offsets in tile_off; no capacity check (the offsets come from exchanged counts) */
 __global__ void __launch_bounds__(kBucketThreads) k_wire_scatter(const hirace_event *__restrict__ in, uint32_t lo,
                                                                  uint32_t hi, int nranks, int my_rank,
                                                                  const unsigned long long *__restrict__ tile_off,
                                                                  unsigned long long *out, uint64_t cap,
-                                                                 unsigned int *err)
+                                                                 unsigned int *err,
+                                                                 unsigned long long *const *__restrict__ peer)
 {
     __shared__ unsigned long long s_run[kMaxRanks];
     const uint32_t lane = threadIdx.x & 31;
@@ -526,7 +507,9 @@ __global__ void __launch_bounds__(kBucketThreads) k_wire_scatter(const hirace_ev
                 slot = atomicAdd(&s_run[own], (unsigned long long)__popc(peers));
             slot = __shfl_sync(0xffffffffu, slot, leader) + __popc(peers & ((1u << lane) - 1));
             if (own != 0xffffffffu) {
-                if (slot < cap)
+                if (peer)
+                    __stcs(peer[own] + slot, (unsigned long long)w); /* streaming store to the owner */
+                else if (slot < cap)
                     out[slot] = w;
                 else
                     atomicOr(err, 8u); /* capacity exceeded: reported by the host call */
@@ -545,14 +528,79 @@ cudaError_t launch_bucket_wire(const hirace_event *in, uint32_t lo, uint32_t hi,
         return cudaMemsetAsync(d_counts_row, 0, nranks * sizeof(unsigned long long), st);
     k_wire_hist<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_hist, err);
     k_wire_scan<<<1, 1024, 0, st>>>(d_tile_hist, ntiles, nranks, d_running, d_counts_row, d_tile_off);
-    k_wire_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_off, out, cap, err);
+    if (out)
+        k_wire_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_off, out, cap, err,
+                                                          nullptr);
+    return cudaGetLastError();
+}
+
+/* per-owner exclusive scan of one batch's [owner][tile] histogram, each owner's slots starting
+ * at owner_base[owner] (its segment in that owner's receive buffer) */
+__global__ void __launch_bounds__(1024) k_wire_scan_peer(const uint32_t *tile_hist, uint32_t ntiles, int nranks,
+                                                         const unsigned long long *owner_base,
+                                                         unsigned long long *tile_off)
+{
+    __shared__ unsigned long long s_w[32];
+    __shared__ unsigned long long s_carry;
+    const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    for (int r = 0; r < nranks; r++) {
+        if (threadIdx.x == 0)
+            s_carry = owner_base[r];
+        __syncthreads();
+        for (uint32_t t0 = 0; t0 < ntiles; t0 += 1024) {
+            const uint32_t t = t0 + threadIdx.x;
+            const unsigned long long v = t < ntiles ? tile_hist[(uint64_t)r * ntiles + t] : 0;
+            unsigned long long x = v;
+            for (int o = 1; o < 32; o <<= 1) {
+                const unsigned long long y = __shfl_up_sync(0xffffffffu, x, o);
+                if ((int)lane >= o)
+                    x += y;
+            }
+            if (lane == 31)
+                s_w[wid] = x;
+            __syncthreads();
+            if (wid == 0) {
+                unsigned long long q = s_w[lane];
+                for (int o = 1; o < 32; o <<= 1) {
+                    const unsigned long long y = __shfl_up_sync(0xffffffffu, q, o);
+                    if ((int)lane >= o)
+                        q += y;
+                }
+                s_w[lane] = q;
+            }
+            __syncthreads();
+            if (t < ntiles)
+                tile_off[(uint64_t)r * ntiles + t] = s_carry + (wid ? s_w[wid - 1] : 0) + x - v;
+            __syncthreads();
+            if (threadIdx.x == 0)
+                s_carry += s_w[31];
+            __syncthreads();
+        }
+    }
+}
+
+cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, int my_rank,
+                                 unsigned long long *const *d_peer, const unsigned long long *d_owner_base,
+                                 uint32_t *d_tile_hist, unsigned long long *d_tile_off, unsigned int *err,
+                                 cudaStream_t st)
+{
+    const uint32_t ntiles = (hi - lo + kBucketTile - 1) / kBucketTile;
+    if (ntiles == 0)
+        return cudaSuccess;
+    k_wire_hist<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_hist, err);
+    k_wire_scan_peer<<<1, 1024, 0, st>>>(d_tile_hist, ntiles, nranks, d_owner_base, d_tile_off);
+    k_wire_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_off, nullptr, 0, err,
+                                                      d_peer);
     return cudaGetLastError();
 }
 
 cudaError_t kernels_init(int device)
 {
     (void)device;
-    return cudaFuncSetAttribute(k_batches, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(FindSmem));
+    cudaError_t e = cudaFuncSetAttribute(k_batches, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(FindSmem));
+    if (e != cudaSuccess)
+        return e;
+    return replay_init();
 }
 
 } // namespace hirace_impl

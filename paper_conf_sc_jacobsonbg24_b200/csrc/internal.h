@@ -33,16 +33,19 @@ cudaError_t launch_find_batches(const hirace_event *ev, uint32_t n, const Scratc
                                 int sm_count, cudaStream_t st);
 /* persistent cooperative replay over the discovered batches */
 /* optional fused collect at the end of the replay (out == nullptr: none) */
+/* report_mode: the fused collect uses the report buffer when it covers every flagged word
+ * (collect.cuh; k_collect_reports is launched right after), else the shadow scan */
 cudaError_t launch_replay(const hirace_dev_ctx &c, const hirace_event *ev, const Scratch &s, int grid,
                           cudaStream_t st, uint64_t shadow_words = 0, hirace_race *out = nullptr, uint64_t cap = 0,
-                          unsigned long long *d_total = nullptr);
+                          unsigned long long *d_total = nullptr, int report_mode = 0);
 int collect_max_grid(int device);
-__global__ void k_collect(hirace_dev_ctx c, uint64_t nwords, hirace_race *out, uint64_t cap,
-                          unsigned long long *d_total, uint32_t *cta_cnt, unsigned int *bar);
 int replay_max_grid(int device);
 /* order-preserving compaction of RACE records from the shadow */
 cudaError_t launch_collect(const hirace_dev_ctx &c, uint64_t shadow_words, const Scratch &s, hirace_race *out,
-                           uint64_t cap, unsigned long long *d_total, cudaStream_t st);
+                           uint64_t cap, unsigned long long *d_total, cudaStream_t st, int report_mode = 0);
+/* report mode pays off above this shadow size (a scan of it costs more than a launch + sort) */
+constexpr uint64_t kReportModeMinBytes = 64ull << 20;
+cudaError_t replay_init();
 cudaError_t launch_rebase(const hirace_dev_ctx &c, uint64_t shadow_words, cudaStream_t st);
 cudaError_t launch_bucket(const hirace_dev_ctx &c, const hirace_event *in, uint32_t n, int nranks, int my_rank,
                           hirace_event *out, unsigned long long *d_counts, uint32_t *d_tile_hist, uint32_t ntiles,
@@ -52,6 +55,13 @@ cudaError_t launch_bucket_wire(const hirace_event *in, uint32_t lo, uint32_t hi,
                                unsigned long long *out, uint64_t cap, uint32_t *d_tile_hist,
                                unsigned long long *d_tile_off, unsigned long long *d_running,
                                unsigned long long *d_counts_row, unsigned int *err, cudaStream_t st);
+/* one batch [lo, hi) -> wire records stored straight into their owners' receive buffers
+ * d_peer[owner] starting at d_owner_base[owner] (peer dispatch; d_peer / d_owner_base are
+ * device arrays of nranks entries) */
+cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, int my_rank,
+                                 unsigned long long *const *d_peer, const unsigned long long *d_owner_base,
+                                 uint32_t *d_tile_hist, unsigned long long *d_tile_off, unsigned int *err,
+                                 cudaStream_t st);
 /* single-batch replay of 8-byte wire records (batch key given) */
 cudaError_t launch_replay_wire(const hirace_dev_ctx &c, const unsigned long long *wire, uint32_t n, uint32_t batch_key,
                                int grid, cudaStream_t st);

@@ -28,11 +28,13 @@ STATUS = {0: "HIRACE_OK", -1: "HIRACE_E_INVAL", -2: "HIRACE_E_NOMEM", -3: "HIRAC
 POLICY_STRICT, POLICY_RELAXED_READ_ATOMIC = 0, 1
 
 # every symbol include/hirace.h declares (checked by tests/test_abi.py against the header)
-EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_free", "hirace_shadow_reset", "hirace_barrier",
+EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_free", "hirace_shadow_reset", "hirace_barrier",
            "hirace_replay_trace", "hirace_find_batches", "hirace_check_trace_device", "hirace_check_trace_host", "hirace_collect_races",
            "hirace_collect_races_device", "hirace_get_stats", "hirace_sync", "hirace_get_dev_ctx",
-           "hirace_bucket_events", "hirace_bucket_wire", "hirace_replay_wire", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_set_policy",
-           "hirace_fsm_table", "hirace_fsm_table_policy", "hirace_fsm_step", "hirace_fsm_step_policy", "hirace_status_string",
+           "hirace_bucket_events", "hirace_bucket_wire", "hirace_replay_wire", "hirace_count_wire",
+           "hirace_dispatch_wire", "hirace_peer_buffer_alloc", "hirace_peer_buffer_free", "hirace_peer_open",
+           "hirace_peer_close", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_set_policy",
+           "hirace_fsm_table", "hirace_fsm_table_policy", "hirace_fsm_step", "hirace_fsm_step_policy", "hirace_fsm_step_compact", "hirace_status_string",
            "hirace_version")
 
 
@@ -58,7 +60,14 @@ class DevCtx(ctypes.Structure):
                 ("block_threads", ctypes.c_uint32), ("warp_size", ctypes.c_uint32),
                 ("bt_magic", ctypes.c_uint32), ("bt_s1", ctypes.c_uint32), ("bt_s2", ctypes.c_uint32),
                 ("ws_magic", ctypes.c_uint32), ("ws_s1", ctypes.c_uint32), ("ws_s2", ctypes.c_uint32),
-                ("g", ctypes.c_uint32)]
+                ("g", ctypes.c_uint32), ("rec_bytes", ctypes.c_uint32), ("c_sh_b", ctypes.c_uint32),
+                ("c_sh_w", ctypes.c_uint32), ("c_sh_t", ctypes.c_uint32), ("c_max_g", ctypes.c_uint32),
+                ("c_max_b", ctypes.c_uint32), ("c_max_w", ctypes.c_uint32)]
+
+
+class EpochLimits(ctypes.Structure):
+    """hirace_epoch_limits: declared maxima of the g / b / w epoch counters (compact records)."""
+    _fields_ = [("max_g", ctypes.c_uint32), ("max_b", ctypes.c_uint32), ("max_w", ctypes.c_uint32)]
 
 
 _lib = None
@@ -76,6 +85,7 @@ def load():
     P, U64, U32, I32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int
     sig = {
         "hirace_shadow_alloc": (I32, [ctypes.POINTER(Config), ctypes.POINTER(P)]),
+        "hirace_shadow_alloc_compact": (I32, [ctypes.POINTER(Config), ctypes.POINTER(EpochLimits), ctypes.POINTER(P)]),
         "hirace_shadow_free": (I32, [P]),
         "hirace_shadow_reset": (I32, [P, P]),
         "hirace_barrier": (I32, [P, I32, P]),
@@ -91,6 +101,12 @@ def load():
         "hirace_bucket_events": (I32, [P, P, U64, I32, I32, P, ctypes.POINTER(U64), P]),
         "hirace_bucket_wire": (I32, [P, P, P, U64, I32, I32, P, U64, P, ctypes.POINTER(U64), P]),
         "hirace_replay_wire": (I32, [P, P, U64, U32, P]),
+        "hirace_count_wire": (I32, [P, P, P, U64, I32, I32, P, P]),
+        "hirace_dispatch_wire": (I32, [P, P, P, U64, I32, I32, P, P, P]),
+        "hirace_peer_buffer_alloc": (I32, [I32, U64, ctypes.POINTER(P), P]),
+        "hirace_peer_buffer_free": (I32, [P]),
+        "hirace_peer_open": (I32, [I32, P, ctypes.POINTER(P)]),
+        "hirace_peer_close": (I32, [P]),
         "hirace_set_kernel_timing": (I32, [P, P, P]),
         "hirace_microbench_atomics": (I32, [I32, U64, I32, I32, U64, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_microbench_grid_sync": (I32, [I32, I32, I32, ctypes.POINTER(ctypes.c_double), P]),
@@ -99,6 +115,8 @@ def load():
         "hirace_fsm_table_policy": (I32, [I32, P]),
         "hirace_fsm_step": (U64, [U64, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
         "hirace_fsm_step_policy": (U64, [I32, U64, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
+        "hirace_fsm_step_compact": (U32, [I32, U32, U32, U32, U32, U32, U32, U32, U32, U32,
+                                          ctypes.POINTER(EpochLimits), ctypes.POINTER(I32)]),
         "hirace_status_string": (ctypes.c_char_p, [I32]),
         "hirace_version": (ctypes.c_char_p, []),
     }
@@ -132,6 +150,24 @@ def fsm_step(old: int, tid: int, kind: int, g: int, b: int, w: int, block_thread
         n = load().hirace_fsm_step_policy(policy, old, tid, kind, g, b, w, block_threads, warp_size,
                                           ctypes.byref(rep))
     return int(n), int(rep.value)
+
+
+def fsm_step_compact(old: int, tid: int, kind: int, g: int, b: int, w: int, block_threads: int, warp_size: int,
+                     grid_threads: int, limits, policy: int = 0):
+    """One step on a compact 4-byte record (include/hirace.h hirace_fsm_step_compact)."""
+    rep = ctypes.c_int(0)
+    lim = EpochLimits(*limits)
+    n = load().hirace_fsm_step_compact(policy, old, tid, kind, g, b, w, block_threads, warp_size, grid_threads,
+                                       ctypes.byref(lim), ctypes.byref(rep))
+    return int(n), int(rep.value)
+
+
+def trace_epoch_limits(events: np.ndarray) -> tuple[int, int, int]:
+    """(max g, max b, max w) over a trace's events: the limits a compact context needs."""
+    meta = events["meta"]
+    if meta.shape[0] == 0:
+        return (0, 0, 0)
+    return (int((meta >> 24).max()), int(((meta >> 14) & 1023).max()), int(((meta >> 5) & 511).max()))
 
 
 def microbench_atomics(nwords: int, random: bool, op: int, nops: int, device: int = 0, stream=None) -> float:
@@ -168,16 +204,25 @@ def events_to_device(events: np.ndarray, device="cuda"):
 
 
 class Checker:
-    """One hirace_ctx: shadow (8 B per tracked 4-byte word), FSM table, report buffer."""
+    """One hirace_ctx: shadow (8 B per tracked 4-byte word, or 4 B with compact=(max_g, max_b,
+    max_w): hirace_shadow_alloc_compact), FSM table, report buffer."""
 
     def __init__(self, grid_blocks: int, block_threads: int, warp_size: int = 32, global_words: int = 0,
-                 smem_words: int = 0, report_capacity: int = 0, device: int = 0, policy: int = 0):
+                 smem_words: int = 0, report_capacity: int = 0, device: int = 0, policy: int = 0,
+                 compact=None):
         self.lib = load()
         cfg = Config(grid_blocks, block_threads, warp_size, 4 * smem_words, 4 * global_words, 2, device,
                      report_capacity)
         h = ctypes.c_void_p()
-        _check(self.lib.hirace_shadow_alloc(ctypes.byref(cfg), ctypes.byref(h)), "hirace_shadow_alloc")
+        if compact is None:
+            _check(self.lib.hirace_shadow_alloc(ctypes.byref(cfg), ctypes.byref(h)), "hirace_shadow_alloc")
+        else:
+            lim = EpochLimits(*compact)
+            _check(self.lib.hirace_shadow_alloc_compact(ctypes.byref(cfg), ctypes.byref(lim), ctypes.byref(h)),
+                   "hirace_shadow_alloc_compact")
         self.h = h
+        self.compact = None if compact is None else tuple(int(x) for x in compact)
+        self.rec_bytes = 8 if compact is None else 4
         self.geometry = dict(grid_blocks=grid_blocks, block_threads=block_threads, warp_size=warp_size,
                              global_words=global_words, smem_words=smem_words)
         self.device = device
@@ -186,9 +231,11 @@ class Checker:
             self.set_policy(policy)
 
     @classmethod
-    def for_trace(cls, trace, report_capacity: int = 0, device: int = 0, policy: int = 0):
+    def for_trace(cls, trace, report_capacity: int = 0, device: int = 0, policy: int = 0, compact: bool = False):
+        """compact=True: 4-byte records sized by the trace's own epoch maxima."""
+        lim = trace_epoch_limits(trace.events) if compact else None
         return cls(trace.grid_blocks, trace.block_threads, trace.warp_size, trace.global_words, trace.smem_words,
-                   report_capacity, device, policy)
+                   report_capacity, device, policy, compact=lim)
 
     def set_policy(self, policy: int, stream=None):
         """POLICY_STRICT or POLICY_RELAXED_READ_ATOMIC (include/hirace.h hirace_policy)."""
@@ -198,7 +245,7 @@ class Checker:
     @property
     def shadow_bytes(self) -> int:
         g = self.geometry
-        return 8 * (g["global_words"] + g["grid_blocks"] * g["smem_words"])
+        return self.rec_bytes * (g["global_words"] + g["grid_blocks"] * g["smem_words"])
 
     def close(self):
         if getattr(self, "h", None):
@@ -345,10 +392,68 @@ class Checker:
             _check(st, "hirace_bucket_wire")
             return out[: total.value], counts[:nb]
 
+    def count_wire(self, events_dev, offsets: np.ndarray, nranks: int, my_rank: int, stream=None) -> np.ndarray:
+        """Per-batch per-owner wire-record counts [nb, nranks] (hirace_count_wire)."""
+        offs = np.ascontiguousarray(offsets, dtype=np.uint32)
+        nb = max(len(offs) - 1, 0)
+        counts = np.zeros((max(nb, 1), nranks), np.uint64)
+        _check(self.lib.hirace_count_wire(self.h, ctypes.c_void_p(events_dev.data_ptr() if nb else 0),
+                                          offs.ctypes.data, nb, nranks, my_rank, counts.ctypes.data,
+                                          _stream_handle(stream)), "hirace_count_wire")
+        return counts[:nb]
+
+    def dispatch_wire(self, events_dev, offsets: np.ndarray, nranks: int, my_rank: int, peers, dst: np.ndarray,
+                      stream=None):
+        """Stores every batch's wire records into the owners' buffers (hirace_dispatch_wire).
+        peers: nranks device addresses; dst: uint64 [nb, nranks] record offsets."""
+        offs = np.ascontiguousarray(offsets, dtype=np.uint32)
+        nb = max(len(offs) - 1, 0)
+        if nb == 0:
+            return
+        tab = (ctypes.c_void_p * nranks)(*[ctypes.c_void_p(int(p)) for p in peers])
+        d = np.ascontiguousarray(dst, dtype=np.uint64).reshape(-1)
+        _check(self.lib.hirace_dispatch_wire(self.h, ctypes.c_void_p(events_dev.data_ptr() if nb else 0),
+                                             offs.ctypes.data, nb, nranks, my_rank, tab,
+                                             d.ctypes.data, _stream_handle(stream)),
+               "hirace_dispatch_wire")
+
     def replay_wire(self, wire_dev, n: int, batch_key: int, stream=None):
         """Replays n wire records of one batch (key g<<19 | b<<9 | w)."""
         _check(self.lib.hirace_replay_wire(self.h, ctypes.c_void_p(wire_dev.data_ptr() if n else 0), n, batch_key,
                                            _stream_handle(stream)), "hirace_replay_wire")
+
+    def replay_wire_ptr(self, ptr: int, n: int, batch_key: int, stream=None):
+        _check(self.lib.hirace_replay_wire(self.h, ctypes.c_void_p(ptr if n else 0), n, batch_key,
+                                           _stream_handle(stream)), "hirace_replay_wire")
+
+
+class PeerBuffer:
+    """A receive buffer other processes can map (hirace_peer_buffer_alloc): `ptr` here, `handle`
+    (64 bytes) for the peers, who map it with peer_open()."""
+
+    def __init__(self, nbytes: int, device: int = 0):
+        self.lib = load()
+        p = ctypes.c_void_p()
+        h = (ctypes.c_ubyte * 64)()
+        _check(self.lib.hirace_peer_buffer_alloc(device, max(int(nbytes), 8), ctypes.byref(p), h),
+               "hirace_peer_buffer_alloc")
+        self.ptr, self.handle, self.nbytes, self.device = int(p.value), bytes(h), max(int(nbytes), 8), device
+
+    def free(self):
+        if self.ptr:
+            self.lib.hirace_peer_buffer_free(ctypes.c_void_p(self.ptr))
+            self.ptr = 0
+
+
+def peer_open(handle: bytes, device: int = 0) -> int:
+    p = ctypes.c_void_p()
+    h = (ctypes.c_ubyte * 64).from_buffer_copy(handle)
+    _check(load().hirace_peer_open(device, h, ctypes.byref(p)), "hirace_peer_open")
+    return int(p.value)
+
+
+def peer_close(ptr: int):
+    _check(load().hirace_peer_close(ctypes.c_void_p(ptr)), "hirace_peer_close")
 
 
 def races_to_dict(races: np.ndarray) -> dict:

@@ -16,7 +16,13 @@ is exact for the words it owns; the union (keys mapped back to global words) is 
 Inside a batch any order is a linear extension of happens-before, so the
 received segments need no merge.
 
-`run_sharded_wire` is the default pipeline: ONE bucketing launch sequence over
+`run_sharded_p2p` fuses the bucketing with the exchange (the B200-native path): the dispatch
+kernel stores every wire record straight into its owner's receive buffer, mapped from the
+owner's GPU with CUDA IPC (NVLink/NVSwitch P2P stores; on one GPU, another process's buffer),
+at an offset every rank derives from one all-gather of the count matrices — no staging copy
+and no all_to_all (`PeerExchange`; include/hirace.h hirace_dispatch_wire).
+
+`run_sharded_wire` is the NCCL pipeline: ONE bucketing launch sequence over
 all local batches into 8-byte wire records (hirace_bucket_wire; g,b,w implied by the batch),
 ONE all_to_all of the [ranks x batches] count matrix, then every batch's payload
 all_to_all posted asynchronously up front while the replays (hirace_replay_wire) consume
@@ -127,6 +133,80 @@ class HostExchange(NcclExchange):
         return out.to(self.out_device) if self.out_device is not None else out
 
 
+class PeerExchange:
+    """Receive buffers in peer memory for run_sharded_p2p: this rank's buffer is a
+    hirace_peer_buffer_alloc allocation, the other ranks' are mapped with hirace_peer_open (CUDA
+    IPC; P2P over NVLink between GPUs).  Host-side agreement (count matrices, handles, the
+    completion barrier) goes through the process group (gloo or NCCL)."""
+
+    def __init__(self, group, dist, device: int = 0):
+        self.group, self.dist, self.device = group, dist, device
+        self.buf = None
+        self.opened = {}   # rank -> (handle, ptr)
+        self.ptrs = None
+
+    def _gather(self, obj):
+        objs = [None] * self.dist.get_world_size(self.group)
+        self.dist.all_gather_object(objs, obj, group=self.group)
+        return objs
+
+    def all_counts(self, counts):
+        """counts: int64 [nbg, P] of this rank -> [P_sender, nbg, P_owner] of all ranks."""
+        return np.stack([np.asarray(c, np.int64) for c in self._gather(np.asarray(counts, np.int64))])
+
+    def setup(self, need_bytes: int):
+        """Every rank's buffer holds at least its own need; returns the peer table (device
+        addresses in this process, index = owner rank)."""
+        from .hirace import PeerBuffer, peer_close, peer_open
+        me = self.dist.get_rank(self.group)
+        grow = self.buf is None or self.buf.nbytes < need_bytes
+        if any(self._gather(grow)):  # a remapped buffer: everyone drops stale mappings first
+            for _, (_, ptr) in self.opened.items():
+                peer_close(ptr)
+            self.opened = {}
+            self.dist.barrier(group=self.group)
+            if grow:
+                if self.buf is not None:
+                    self.buf.free()
+                self.buf = PeerBuffer(max(need_bytes, 1 << 20), self.device)
+        handles = self._gather(self.buf.handle)
+        ptrs = []
+        for r, h in enumerate(handles):
+            if r == me:
+                ptrs.append(self.buf.ptr)
+                continue
+            if r not in self.opened or self.opened[r][0] != h:
+                if r in self.opened:
+                    peer_close(self.opened[r][1])
+                self.opened[r] = (h, peer_open(h, self.device))
+            ptrs.append(self.opened[r][1])
+        self.ptrs = ptrs
+        return ptrs
+
+    def fence(self):
+        """All stores of every rank's dispatch are complete and visible before any replay."""
+        import torch
+        torch.cuda.synchronize(self.device)
+        self.dist.barrier(group=self.group)
+
+    def dispatch(self, ops, events, offs, dst_local):
+        ops.dispatch_wire(events, offs, self.ptrs, dst_local)
+
+    def received(self, ops, start: int, n: int, key: int):
+        """Replays records [start, start + n) of this rank's buffer as batch `key`."""
+        ops.replay_wire_ptr(self.buf.ptr + 8 * start, n, key)
+
+    def close(self):
+        from .hirace import peer_close
+        for _, (_, ptr) in self.opened.items():
+            peer_close(ptr)
+        self.opened = {}
+        self.dist.barrier(group=self.group)
+        if self.buf is not None:
+            self.buf.free()
+            self.buf = None
+
+
 # ---------------------------------------------------------------------------------------------
 # GPU ops (the library's kernels)
 # ---------------------------------------------------------------------------------------------
@@ -171,6 +251,19 @@ class GpuOps:
     def replay_wire(self, wire, key: int):
         if wire.shape[0]:
             self.ctx.replay_wire(wire, int(wire.shape[0]), key)
+
+    def count_wire(self, events, offsets):
+        """Per-batch per-owner wire-record counts [nb, P] (hirace_count_wire)."""
+        if len(offsets) <= 1:
+            return np.zeros((0, self.nranks), np.uint64)
+        return self.ctx.count_wire(events, offsets, self.nranks, self.rank)
+
+    def dispatch_wire(self, events, offsets, peers, dst):
+        self.ctx.dispatch_wire(events, offsets, self.nranks, self.rank, peers, dst)
+
+    def replay_wire_ptr(self, ptr: int, n: int, key: int):
+        if n:
+            self.ctx.replay_wire_ptr(ptr, n, key)
 
     def collect(self):
         r = self.ctx.collect()
@@ -246,6 +339,45 @@ def run_sharded_wire(local_events, ops, exchange, group, dist, on_batch=None):
         received += int(got.shape[0])
         if on_batch is not None:
             on_batch(int(k), int(got.shape[0]))
+    return received
+
+
+def p2p_layout(all_counts: np.ndarray, me: int):
+    """Receive-buffer layout of run_sharded_p2p from every rank's count matrix
+    all_counts[s, j, r] (sender s, global batch j, owner r): owner r's buffer holds batch 0's
+    records, then batch 1's, ...; inside a batch the senders in rank order.  Returns
+    (dst [nbg, P]: where this rank's segment of batch j starts in owner r's buffer,
+     base [nbg]: where batch j starts in this rank's own buffer, n_recv [nbg])."""
+    per_batch = all_counts.sum(axis=0)                                   # [nbg, P]
+    base_all = np.cumsum(per_batch, axis=0) - per_batch                  # exclusive over batches
+    before = all_counts[:me].sum(axis=0) if me else np.zeros_like(per_batch)
+    return base_all + before, base_all[:, me], per_batch[:, me]
+
+
+def run_sharded_p2p(local_events, ops, exchange, group, dist, on_batch=None):
+    """Fused bucket + exchange over peer memory (module docstring).  Returns the number of wire
+    records (word accesses) replayed on this rank."""
+    offs, keys = ops.find_batches(local_events)
+    order = all_batch_keys(keys, group, dist)
+    P = dist.get_world_size(group)
+    me = dist.get_rank(group)
+    counts = np.asarray(ops.count_wire(local_events, offs), dtype=np.int64).reshape(-1, P)
+    gidx = np.array([int(np.searchsorted(order, k)) for k in keys], dtype=np.int64)
+    nbg = len(order)
+    mine = np.zeros((nbg, P), np.int64)
+    if len(keys):
+        mine[gidx] = counts
+    dst, base, n_recv = p2p_layout(exchange.all_counts(mine), me)
+    exchange.setup(8 * int(n_recv.sum()))
+    exchange.dispatch(ops, local_events, offs, dst[gidx] if len(keys) else np.zeros((0, P), np.int64))
+    exchange.fence()
+    received = 0
+    for j, k in enumerate(order):
+        n = int(n_recv[j])
+        exchange.received(ops, int(base[j]), n, int(k))
+        received += n
+        if on_batch is not None:
+            on_batch(int(k), n)
     return received
 
 

@@ -119,9 +119,16 @@ def _gpu_worker(rank, world, port, name, q, wire=False):
         mine = t.events[(blk % world) == rank]
         ops = sharded.GpuOps(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words, world,
                              rank, device=0)
-        ex = sharded.HostExchange(None, device="cuda:0")
-        run = sharded.run_sharded_wire if wire else sharded.run_sharded
+        if wire == "p2p":   # peer dispatch into CUDA-IPC-mapped buffers of the other processes
+            ex, run = sharded.PeerExchange(None, dist, device=0), sharded.run_sharded_p2p
+        else:
+            ex = sharded.HostExchange(None, device="cuda:0")
+            run = sharded.run_sharded_wire if wire else sharded.run_sharded
         n = run(_to_tensor(mine).cuda(), ops, ex, None, dist)
+        if wire == "p2p":   # a second trace on the same buffers (handles cached, no regrowth)
+            n2 = run(_to_tensor(mine).cuda(), ops, ex, None, dist)
+            assert n2 == n
+            ex.close()
         races = sharded.gather_races(ops.collect(), None, dist)
         tot = torch.tensor([n])
         dist.all_reduce(tot)
@@ -173,6 +180,51 @@ def test_sharded_wire_gpu_ranks_reproduce_the_oracle(world, name):
     assert total == _words(t)
     assert keys == [int(x) for x in k]
     assert cls == [int(x) for x in c]
+
+
+@pytest.mark.parametrize("world,name", [(1, "multi"), (2, "cfg2"), (3, "multi"), (2, "cfg3"), (4, "cfg4")])
+def test_sharded_p2p_gpu_ranks_reproduce_the_oracle(world, name):
+    """Peer dispatch with the real kernels: `world` processes share the GPU, each maps the
+    others' receive buffers through CUDA IPC and the dispatch kernel stores straight into them.
+    The trace is replayed twice (RACE is sticky, so the race set is unchanged)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_gpu_worker, args=(r, world, port, name, q, "p2p")) for r in range(world)]
+    for p in procs:
+        p.start()
+    total, keys, cls = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    t = _make(name)
+    k, c, _ = oracle.races_of(t)
+    assert total == _words(t)
+    assert keys == [int(x) for x in k]
+    assert cls == [int(x) for x in c]
+
+
+def test_dispatch_wire_matches_bucket_wire():
+    """One process: the dispatch kernel's stores (own buffer as every owner's destination,
+    at disjoint offsets) hold exactly hirace_bucket_wire's (batch, owner) segments."""
+    t = _make("multi")
+    P, me = 4, 1
+    c = hr.Checker(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words)
+    d = _to_tensor(t.events).cuda()
+    offs, _ = c.find_batches(d)
+    counts = c.count_wire(d, offs, P, me).astype(np.int64)
+    wire, counts2 = c.bucket_wire(d, offs, P, me)
+    assert np.array_equal(counts, counts2.astype(np.int64))
+    flat = counts.reshape(-1)
+    dst = (np.cumsum(flat) - flat).reshape(counts.shape)          # segment (b, r) at its bucket_wire position
+    buf = torch.full((int(flat.sum()),), -1, dtype=torch.int64, device="cuda")
+    c.dispatch_wire(d, offs, P, me, [buf.data_ptr()] * P, dst)
+    got, ref = buf.cpu().numpy(), wire.cpu().numpy()
+    assert (got != -1).all()
+    for i in range(len(flat)):
+        a, b = int(dst.reshape(-1)[i]), int(dst.reshape(-1)[i] + flat[i])
+        assert np.array_equal(np.sort(got[a:b]), np.sort(ref[a:b]))
+    c.close()
 
 
 def test_sharded_wire_single_rank_nccl():

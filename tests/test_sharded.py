@@ -68,6 +68,9 @@ class CpuTestOps:
     def replay_wire(self, wire, key):
         self.got.append(wire_to_events(np.asarray(wire), key))
 
+    def count_wire(self, events, offsets):
+        return wire_bucket_np(_to_events(events), offsets, self.P, self.r)[1]
+
     def collect(self):
         ev = np.concatenate(self.got) if self.got else np.empty(0, tg.EVENT_DTYPE)
         k, c, g = oracle.races(ev, self.t.block_threads, self.t.warp_size)
@@ -76,6 +79,53 @@ class CpuTestOps:
         out["cls_and_epoch"] = c.astype(np.uint32) | (g.astype(np.uint32) << 8)
         out["detect_tid"] = 0
         return out
+
+
+class CpuPeerExchange:
+    """Test double of sharded.PeerExchange: the receive buffer is a numpy array, and the
+    "remote stores" of the dispatch travel as (offset, records) messages over gloo; the layout
+    arithmetic (sharded.p2p_layout) and the orchestration are the product's."""
+
+    def __init__(self, group, dist_mod):
+        self.group, self.dist = group, dist_mod
+        self.buf = None
+
+    def _gather(self, obj):
+        objs = [None] * self.dist.get_world_size(self.group)
+        self.dist.all_gather_object(objs, obj, group=self.group)
+        return objs
+
+    def all_counts(self, counts):
+        return np.stack([np.asarray(c, np.int64) for c in self._gather(np.asarray(counts, np.int64))])
+
+    def setup(self, need_bytes):
+        self.buf = np.full(need_bytes // 8, -1, np.int64)
+        return None
+
+    def dispatch(self, ops, events, offs, dst_local):
+        wire, counts = ops.bucket_wire(events, offs)
+        w = wire.numpy()
+        flat = np.asarray(counts, np.int64).reshape(-1)
+        pos = np.concatenate(([0], np.cumsum(flat)))
+        P = self.dist.get_world_size(self.group)
+        msgs = [[] for _ in range(P)]
+        for i in range(len(flat)):            # segment (local batch i // P, owner i % P)
+            b, r = divmod(i, P)
+            if flat[i]:
+                msgs[r].append((int(dst_local[b, r]), w[pos[i]:pos[i + 1]].copy()))
+        me = self.dist.get_rank(self.group)
+        for src, m in enumerate(self._gather(msgs)):
+            for off, recs in m[me]:
+                assert (self.buf[off:off + len(recs)] == -1).all()   # disjoint segments
+                self.buf[off:off + len(recs)] = recs
+
+    def fence(self):
+        self.dist.barrier(group=self.group)
+        assert (self.buf != -1).all()                                # every slot written once
+
+    def received(self, ops, start, n, key):
+        if n:
+            ops.replay_wire(torch.from_numpy(self.buf[start:start + n]), key)
 
 
 def wire_bucket_np(ev, offsets, P, r):
@@ -160,6 +210,7 @@ def _words(t):
 
 
 def _worker(rank, world, port, name, q, wire=False):
+    """wire: False = 16-byte events, True = 8-byte wire + all_to_all, "p2p" = peer dispatch."""
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
@@ -167,8 +218,11 @@ def _worker(rank, world, port, name, q, wire=False):
         blk = t.events["tid"] // t.block_threads
         mine = t.events[(blk % world) == rank]          # this rank's blocks, batch order kept
         ops = CpuTestOps(t, world, rank)
-        ex = sharded.HostExchange(None)
-        run = sharded.run_sharded_wire if wire else sharded.run_sharded
+        if wire == "p2p":
+            ex, run = CpuPeerExchange(None, dist), sharded.run_sharded_p2p
+        else:
+            ex = sharded.HostExchange(None)
+            run = sharded.run_sharded_wire if wire else sharded.run_sharded
         n = run(_to_tensor(mine), ops, ex, None, dist)
         races = sharded.gather_races(ops.collect(), None, dist)
         tot = torch.tensor([n])
@@ -224,6 +278,41 @@ def test_sharded_wire_pipeline_reproduces_the_oracle(world, name):
     assert keys == [int(x) for x in k]
     assert cls == [int(x) for x in c]
     assert len(k) > 0
+
+
+@pytest.mark.parametrize("world,name", [(2, "cfg2"), (3, "cfg4"), (2, "cfg3"), (3, "wide"), (4, "multi")])
+def test_sharded_p2p_pipeline_reproduces_the_oracle(world, name):
+    """Peer-memory dispatch (run_sharded_p2p): count matrices all-gathered once, every rank
+    stores its records at sharded.p2p_layout offsets of the owners' buffers (disjoint, every
+    slot written), owners replay batch by batch."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, name, q, "p2p")) for r in range(world)]
+    for p in procs:
+        p.start()
+    total, keys, cls = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    t = _make(name)
+    k, c, _ = oracle.races_of(t)
+    assert total == _words(t)
+    assert keys == [int(x) for x in k]
+    assert cls == [int(x) for x in c]
+
+
+def test_p2p_layout_closed_form():
+    # 3 ranks, 2 batches: owner r's buffer = batch-major, sender-minor segments
+    a = np.arange(18).reshape(3, 2, 3) % 5
+    for me in range(3):
+        dst, base, n = sharded.p2p_layout(a, me)
+        for j in range(2):
+            for r in range(3):
+                want = sum(a[s, jj, r] for s in range(3) for jj in range(j)) + sum(a[s, j, r] for s in range(me))
+                assert dst[j, r] == want
+            assert base[j] == sum(a[s, jj, me] for s in range(3) for jj in range(j))
+            assert n[j] == a[:, j, me].sum()
 
 
 def test_wire_reference_roundtrip():
