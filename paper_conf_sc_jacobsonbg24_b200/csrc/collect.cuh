@@ -97,11 +97,49 @@ __device__ __forceinline__ void collect_phase(const hirace_dev_ctx &c, uint64_t 
     R v[kCollectPerThread];
     const R *const shadow = shadow_as<R>(c);
     const Rec<R> rec(c);
-    /* pass 1: count */
+    /* pass 1: count — a streaming read of the CTA's range: each warp takes 4 KB blocks, lane l
+     * loading 16-byte vectors l, l+32, ... (every load instruction fully coalesced, 8 in flight
+     * per lane); the order of the words does not matter for a count */
     uint32_t mine = 0;
-    for (uint64_t t = t0; t < t1; t++)
-        for (uint32_t r = threadIdx.x; r < kCollectTile / kCollectPerThread; r += tpb)
-            mine += collect_load<R>(shadow, nwords, t * kCollectTile + (uint64_t)r * kCollectPerThread, v);
+    {
+        constexpr uint32_t kVec = 16 / sizeof(R);            /* records per 16-byte vector    */
+        constexpr uint32_t kBlockWords = 32 * 8 * kVec;      /* words per warp block (4 KB)   */
+        const uint64_t wb = t0 * (uint64_t)kCollectTile;
+        const uint64_t we = min(t1 * (uint64_t)kCollectTile, nwords);
+        const uint32_t lane = threadIdx.x & 31, nwarp = blockDim.x >> 5;
+        for (uint64_t b0 = wb + (uint64_t)(threadIdx.x >> 5) * kBlockWords; b0 < we;
+             b0 += (uint64_t)nwarp * kBlockWords) {
+            uint4 q[8];
+            const uint4 *src = reinterpret_cast<const uint4 *>(shadow + b0);
+            if (b0 + kBlockWords <= we) {
+#pragma unroll
+                for (int k = 0; k < 8; k++)
+                    q[k] = __ldcs(src + k * 32 + lane);
+            } else {
+#pragma unroll
+                for (int k = 0; k < 8; k++) {
+                    const uint64_t w = b0 + (uint64_t)(k * 32 + lane) * kVec;
+                    q[k] = w + kVec <= we ? __ldcs(src + k * 32 + lane) : make_uint4(0, 0, 0, 0);
+                    if (w < we && w + kVec > we) { /* ragged tail: scalar records */
+                        __align__(16) R t[kVec];
+#pragma unroll
+                        for (uint32_t j = 0; j < kVec; j++)
+                            t[j] = w + j < we ? shadow[w + j] : (R)0;
+                        q[k] = *reinterpret_cast<const uint4 *>(t);
+                    }
+                }
+            }
+#pragma unroll
+            for (int k = 0; k < 8; k++) {
+                const uint32_t xs[4] = {q[k].x, q[k].y, q[k].z, q[k].w};
+#pragma unroll
+                for (int j = 0; j < 4; j++) /* the state is in the low 5 bits of each record's
+                                             * low word (u64: words 0 and 2; u32: every word) */
+                    if (sizeof(R) == 4 || (j & 1) == 0)
+                        mine += (xs[j] & 31u) >= hirace::ST_RACE_W;
+            }
+        }
+    }
     uint32_t cta_total;
     block_exclusive_scan(mine, s_w, &cta_total);
     if (threadIdx.x == 0)
