@@ -73,8 +73,12 @@ typedef enum { HIRACE_POLICY_STRICT = 0, HIRACE_POLICY_RELAXED_READ_ATOMIC = 1 }
 #define HIRACE_SHARED_BIT (1ull << 63)
 
 /* Tracked geometry.  warp_size may be any value >= 1 (2 reproduces the paper's Fig. 1 toy
- * hierarchy).  Tracking granularity is the 4-byte word (per array element,
- * PAPER.md L162): granularity_log2 must be 2.  report_capacity = device race-report records
+ * hierarchy).  One shadow record per tracked element ("for each element",
+ * PAPER.md L162) of 1 << granularity_log2 bytes: 2 = 4-byte words (default, every sharded /
+ * wire entry point requires it), 1 = half-words, 0 = bytes (arrays of char: neighbouring bytes
+ * written by different threads do not race).  Race keys and "word" indices below count elements.
+ * Accesses smaller than an element map to their element; larger ones cover size >> granularity
+ * elements.  report_capacity = device race-report records
  * (16 B each); 0 selects a default of 1<<20. */
 typedef struct {
     uint32_t grid_blocks;          /* blocks of the checked kernel                        */
@@ -82,7 +86,7 @@ typedef struct {
     uint32_t warp_size;            /* threads per warp (32 on NVIDIA hardware)             */
     uint32_t smem_bytes_per_block; /* tracked shared-memory window per block, bytes        */
     uint64_t global_bytes;         /* tracked global extent, bytes from the tracked base   */
-    uint32_t granularity_log2;     /* must be 2                                            */
+    uint32_t granularity_log2;     /* 0, 1 or 2: element = 1, 2 or 4 bytes                  */
     int32_t device;                /* CUDA device ordinal                                  */
     uint64_t report_capacity;      /* race-report ring entries (0 = default)               */
 } hirace_config;
@@ -136,6 +140,7 @@ typedef struct {
     unsigned int rec_bytes;
     unsigned int c_sh_b, c_sh_w, c_sh_t;
     unsigned int c_max_g, c_max_b, c_max_w;
+    unsigned int gran_log2;           /* tracked element = 1 << gran_log2 bytes               */
 } hirace_dev_ctx;
 
 /* ---- lifecycle (a11: shadow alloc/init, "Initially, all State values are set
@@ -143,7 +148,8 @@ typedef struct {
 
 /* Allocates shadow = 8 B per tracked word (global_bytes/4 + grid_blocks*smem_bytes/4 words),
  * all INIT, plus the FSM table and report buffer on cfg->device.  Synchronous.
- * Errors: INVAL (NULL args, zero geometry, granularity != 2, tid space > 2^32), NOMEM, CUDA. */
+ * Errors: INVAL (NULL args, zero geometry, granularity_log2 > 2, extents not multiples of 4
+ * bytes, tid space > 2^32), NOMEM, CUDA. */
 hirace_status hirace_shadow_alloc(const hirace_config *cfg, hirace_ctx **out);
 
 /* ---- compact 32-bit shadow ("the shadow-memory footprint

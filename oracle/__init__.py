@@ -43,13 +43,18 @@ def _load():
         lib.oracle_races_policy.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                             ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
                                             ctypes.c_int]
+        lib.oracle_races_gran.restype = ctypes.c_int64
+        lib.oracle_races_gran.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                                          ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                                          ctypes.c_int, ctypes.c_uint32]
         _lib = lib
     return _lib
 
 
-def races(events: np.ndarray, block_threads: int, warp_size: int, policy: int = 0):
+def races(events: np.ndarray, block_threads: int, warp_size: int, policy: int = 0, granularity_log2: int = 2):
     """Oracle-D.  Returns (keys u64[], cls u8[], gstar u8[]) sorted by key.  policy 0 = strict
-    conflict rule (C1.3), 1 = relaxed read-vs-atomic (R2b)."""
+    conflict rule (C1.3), 1 = relaxed read-vs-atomic (R2b).  granularity_log2: the
+    tracked element is 1 << granularity_log2 bytes (2 = 4-byte words; keys are element indices)."""
     lib = _load()
     ev = np.ascontiguousarray(events)
     n = int(ev.shape[0])
@@ -58,8 +63,8 @@ def races(events: np.ndarray, block_threads: int, warp_size: int, policy: int = 
         keys = np.empty(cap, np.uint64)
         cls = np.empty(cap, np.uint8)
         gs = np.empty(cap, np.uint8)
-        r = lib.oracle_races_policy(ev.ctypes.data if n else None, n, block_threads, warp_size,
-                                    keys.ctypes.data, cls.ctypes.data, gs.ctypes.data, cap, policy)
+        r = lib.oracle_races_gran(ev.ctypes.data if n else None, n, block_threads, warp_size,
+                                  keys.ctypes.data, cls.ctypes.data, gs.ctypes.data, cap, policy, granularity_log2)
         if r < 0:
             raise RuntimeError(f"oracle_races failed ({r})")
         if r <= cap:
@@ -68,7 +73,7 @@ def races(events: np.ndarray, block_threads: int, warp_size: int, policy: int = 
 
 
 def races_of(trace, policy: int = 0):
-    return races(trace.events, trace.block_threads, trace.warp_size, policy)
+    return races(trace.events, trace.block_threads, trace.warp_size, policy, getattr(trace, "granularity_log2", 2))
 
 
 def races_dict(trace, policy: int = 0) -> dict:

@@ -11,16 +11,18 @@ WARP, BLOCK, GRID = 1, 2, 3
 SHARED = 1 << 63
 
 
-def accesses(events, block_threads, warp_size):
-    """C1.1: word-level accesses (key, tid, kind, g, b, w, block, warp)."""
+def accesses(events, block_threads, warp_size, gran_log2=2):
+    """C1.1: element-level accesses (key, tid, kind, g, b, w, block, warp); an element is
+    1 << gran_log2 bytes (4-byte words by default)."""
     out = []
+    granule = 1 << gran_log2
     for e in events:
         addr, tid, meta = int(e["addr"]), int(e["tid"]), int(e["meta"])
         kind, size = meta & 3, 1 << ((meta >> 2) & 7)
         w, b, g = (meta >> 5) & 511, (meta >> 14) & 1023, (meta >> 24) & 255
         block, warp = tid // block_threads, (tid % block_threads) // warp_size
-        word0 = (addr & ~SHARED) >> 2
-        for k in range(1 if size <= 4 else size // 4):
+        word0 = (addr & ~SHARED) >> gran_log2
+        for k in range(1 if size <= granule else size // granule):
             word = word0 + k
             key = (SHARED | (block << 32) | word) if addr & SHARED else word
             out.append((key, tid, kind, g, b, w, block, warp))
@@ -63,9 +65,9 @@ def level(a, c):
     return WARP
 
 
-def races(events, block_threads, warp_size, policy=0):
+def races(events, block_threads, warp_size, policy=0, gran_log2=2):
     """Returns {key: (class, g*)} by literal enumeration of all pairs (C1.4-C1.6)."""
-    acc = accesses(events, block_threads, warp_size)
+    acc = accesses(events, block_threads, warp_size, gran_log2)
     pairs = {}
     for i in range(len(acc)):
         for j in range(i + 1, len(acc)):

@@ -12,7 +12,8 @@
  *         warp = (tid mod blockDim) / warpSize                         PAPER.md L164 (T_bwt), L259
  *         key: global -> word index; shared -> 1<<63 | block<<32 | word (shared memory is per
  *         block); 8/16-byte accesses cover 2/4 words, sub-word accesses their
- *         containing word (per-element shadow; reading R8).
+ *         containing word (per-element shadow; reading R8).  With
+ *         element size 1 << gran_log2 < 4 (oracle_races_gran) "word" reads "element".
  *   C1.2  Concurrent(e1,e2) <=> tid1 != tid2 and g1 == g2 and
  *         [block1 != block2 or (b1 == b2 and (warp1 != warp2 or w1 == w2))]
  *         (barrier semantics PAPER.md L122, L211-213; grid epoch PAPER.md L221, reading R4)
@@ -139,18 +140,22 @@ static int masks_push(masks_t *s, uint8_t v)
  * by C1.2/C1.3 and is reported so a test can pin it).
  * out_g receives g* (the grid epoch of the first racing pair).
  */
-int64_t oracle_races_policy(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
-                            uint64_t *out_key, uint8_t *out_cls, uint8_t *out_g, uint64_t cap, int policy)
+int64_t oracle_races_gran(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
+                          uint64_t *out_key, uint8_t *out_cls, uint8_t *out_g, uint64_t cap, int policy,
+                          uint32_t gran_log2)
 {
     if (policy != 0 && policy != 1)
         return -1;
-    if (block_threads == 0 || warp_size == 0 || (n && !ev))
+    if (block_threads == 0 || warp_size == 0 || (n && !ev) || gran_log2 > 2)
         return -1;
-    /* C1.1: expand to word-level accesses */
+    /* C1.1: expand to element-level accesses; an element ("granule") is 1 << gran_log2 bytes
+     * (per-element shadow; reading R8: 4-byte words by default, bytes
+     * or half-words for arrays of such elements) */
+    const uint32_t granule = 1u << gran_log2;
     uint64_t nacc = 0;
     for (uint64_t i = 0; i < n; i++) {
         uint32_t sz = 1u << ((ev[i].meta >> 2) & 7);
-        nacc += sz <= 4 ? 1 : sz / 4;
+        nacc += sz <= granule ? 1 : sz / granule;
     }
     access_t *acc = (access_t *)malloc((nacc ? nacc : 1) * sizeof(access_t));
     if (!acc)
@@ -164,8 +169,8 @@ int64_t oracle_races_policy(const oracle_event *ev, uint64_t n, uint32_t block_t
         uint32_t block = tid / block_threads;
         uint32_t warp = (tid % block_threads) / warp_size;
         int shared = (ev[i].addr & SHARED) != 0;
-        uint64_t word0 = (ev[i].addr & ~SHARED) >> 2;
-        uint32_t nw = sz <= 4 ? 1 : sz / 4;
+        uint64_t word0 = (ev[i].addr & ~SHARED) >> gran_log2;
+        uint32_t nw = sz <= granule ? 1 : sz / granule;
         for (uint32_t k = 0; k < nw; k++) {
             access_t *a = &acc[j++];
             uint64_t word = word0 + k;
@@ -289,6 +294,12 @@ int64_t oracle_races_policy(const oracle_event *ev, uint64_t n, uint32_t block_t
     free(threads.m);
     free(acc);
     return err ? err : nflag;
+}
+
+int64_t oracle_races_policy(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
+                            uint64_t *out_key, uint8_t *out_cls, uint8_t *out_g, uint64_t cap, int policy)
+{
+    return oracle_races_gran(ev, n, block_threads, warp_size, out_key, out_cls, out_g, cap, policy, 2);
 }
 
 int64_t oracle_races(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,

@@ -137,7 +137,7 @@ hirace_status shadow_alloc_impl(const hirace_config *cfg, const hirace_epoch_lim
     if (!cfg || !out)
         return HIRACE_E_INVAL;
     *out = nullptr;
-    if (cfg->grid_blocks == 0 || cfg->block_threads == 0 || cfg->warp_size == 0 || cfg->granularity_log2 != 2)
+    if (cfg->grid_blocks == 0 || cfg->block_threads == 0 || cfg->warp_size == 0 || cfg->granularity_log2 > 2)
         return HIRACE_E_INVAL;
     if ((uint64_t)cfg->grid_blocks * cfg->block_threads > 0xffffffffull)
         return HIRACE_E_INVAL;
@@ -161,8 +161,8 @@ hirace_status shadow_alloc_impl(const hirace_config *cfg, const hirace_epoch_lim
         c->cfg.report_capacity = 1ull << 20;
     c->device = cfg->device;
     c->rec_bytes = lim ? 4u : 8u;
-    c->global_words = cfg->global_bytes >> 2;
-    const uint64_t smem_words = cfg->smem_bytes_per_block >> 2;
+    c->global_words = cfg->global_bytes >> cfg->granularity_log2;
+    const uint64_t smem_words = cfg->smem_bytes_per_block >> cfg->granularity_log2;
     c->shadow_words = c->global_words + (uint64_t)cfg->grid_blocks * smem_words;
     if (c->shadow_words == 0)
         c->shadow_words = 1;
@@ -223,6 +223,7 @@ hirace_status shadow_alloc_impl(const hirace_config *cfg, const hirace_epoch_lim
     hirace::fastdiv_init(cfg->warp_size, &d.ws_magic, &d.ws_s1, &d.ws_s2);
     d.g = 0;
     d.rec_bytes = c->rec_bytes;
+    d.gran_log2 = cfg->granularity_log2;
     d.c_sh_b = lay.sh_b;
     d.c_sh_w = lay.sh_w;
     d.c_sh_t = lay.sh_t;
@@ -547,7 +548,7 @@ hirace_status hirace_bucket_events(hirace_ctx *c, const hirace_event *d_in, uint
                                    hirace_event *d_out, uint64_t *h_counts, void *stream)
 {
     if (!c || !h_counts || nranks < 1 || nranks > 32 || my_rank < 0 || my_rank >= nranks || n >= 0xffffffffull ||
-        (n && (!d_in || !d_out)))
+        (n && (!d_in || !d_out)) || c->cfg.granularity_log2 != 2)
         return HIRACE_E_INVAL;
     if (c->sticky != HIRACE_OK)
         return c->sticky;
@@ -622,7 +623,8 @@ hirace_status wire_scratch(hirace_ctx *c, uint64_t nb, int nranks, uint32_t maxl
 hirace_status wire_args_ok(hirace_ctx *c, const uint32_t *h_offsets, uint64_t nb, int nranks, int my_rank,
                            uint32_t *maxlen)
 {
-    if (nranks < 1 || nranks > 32 || my_rank < 0 || my_rank >= nranks || nb > HIRACE_MAX_BATCHES)
+    if (nranks < 1 || nranks > 32 || my_rank < 0 || my_rank >= nranks || nb > HIRACE_MAX_BATCHES ||
+        c->cfg.granularity_log2 != 2)
         return HIRACE_E_INVAL;
     const uint64_t threads = (uint64_t)c->cfg.grid_blocks * c->cfg.block_threads;
     if (threads > HIRACE_WIRE_MAX_TIDS || (uint64_t)c->dev.smem_words > HIRACE_WIRE_MAX_WORDS)
@@ -789,7 +791,7 @@ hirace_status hirace_replay_wire(hirace_ctx *c, const uint64_t *d_wire, uint64_t
         return c->sticky;
     if (n == 0)
         return HIRACE_OK;
-    if (!d_wire || n >= 0xffffffffull || batch_key >= (1u << 27))
+    if (!d_wire || n >= 0xffffffffull || batch_key >= (1u << 27) || c->cfg.granularity_log2 != 2)
         return set_sticky(c, HIRACE_E_INVAL);
     cudaStream_t st = (cudaStream_t)stream;
     HR_CUDA(c, cudaSetDevice(c->device));

@@ -103,11 +103,11 @@ __device__ __forceinline__ void ld_event_if(const uint4 *p, bool pred, uint4 &v)
                  : "l"(p), "r"((uint32_t)pred));
 }
 
-/* race key (include/hirace.h) of word k of event e */
-__device__ __forceinline__ uint64_t key_of(const geom &G, const uint4 &e, uint32_t k)
+/* race key (include/hirace.h) of element k of event e (elements of 1 << gran bytes) */
+__device__ __forceinline__ uint64_t key_of(const geom &G, const uint4 &e, uint32_t k, uint32_t gran)
 {
     const uint64_t addr = ((uint64_t)e.y << 32) | e.x;
-    const uint64_t word = ((addr & ~HIRACE_SHARED_BIT) >> 2) + k;
+    const uint64_t word = ((addr & ~HIRACE_SHARED_BIT) >> gran) + k;
     if (addr & HIRACE_SHARED_BIT)
         return HIRACE_SHARED_BIT | ((uint64_t)block_of(e.z, G) << 32) | word;
     return word;
@@ -207,9 +207,9 @@ __device__ __noinline__ uint4 chunk_multiword(const hirace_dev_ctx c, const geom
     const Rec<R> rec(c);
     Counters cnt{0, 0, 0, 0};
     const uint64_t addr = ((uint64_t)e.y << 32) | e.x;
-    const uint32_t szl = (e.w >> 2) & 7u;
-    const uint32_t nw = szl <= 2 ? 1u : (1u << (szl - 2));
-    const uint64_t word = (addr & ~HIRACE_SHARED_BIT) >> 2;
+    const uint32_t szl = (e.w >> 2) & 7u, gran = c.gran_log2;
+    const uint32_t nw = szl <= gran ? 1u : (1u << (szl - gran));
+    const uint64_t word = (addr & ~HIRACE_SHARED_BIT) >> gran;
     const bool sh = (addr & HIRACE_SHARED_BIT) != 0;
     const uint64_t base = sh ? c.global_words + (uint64_t)block_of(e.z, G) * c.smem_words + word : word;
     R *const shadow = shadow_as<R>(c);
@@ -225,7 +225,7 @@ __device__ __noinline__ uint4 chunk_multiword(const hirace_dev_ctx c, const geom
         const uint32_t cls = commit_groups<R>(shadow + my, o, lead ? peers : 0u, e.z, e.w & 3u, G, raw, B, rec, cnt,
                                               rtid, true);
         if (__any_sync(FULL, cls != 0))
-            append_reports(c, cls, key_of(G, e, k), B.g, rtid, lane);
+            append_reports(c, cls, key_of(G, e, k, gran), B.g, rtid, lane);
     }
     return make_uint4(cnt.checked, cnt.retry, cnt.cas, cnt.nowrite);
 }
@@ -244,6 +244,7 @@ __device__ __forceinline__ void warp_share(uint32_t bstart, uint32_t bend, uint3
     iend = min(bend, bstart + c1 * 32);
 }
 
+
 /* one lane's decoded access */
 struct Lane {
     uint64_t idx;
@@ -251,8 +252,9 @@ struct Lane {
     bool ok;
 };
 
-/* a2: decode + validate one lane's event (sub-word accesses map to their word); 8/16-byte
- * accesses of the chunk are committed right here, word by word.  W32: the whole shadow has
+/* a2: decode + validate one lane's event (sub-element accesses map to their element; the
+ * element is 1 << gran_log2 bytes, a 4-byte word by default); accesses covering several
+ * elements are committed right here, element by element.  W32: the whole shadow has
  * < 2^31 words and tracked byte offsets fit 32 bits, so index math and range checks are 32-bit
  * (fewer instructions on the hot path); otherwise 64-bit. */
 template <bool W32, typename R>
@@ -265,24 +267,26 @@ __device__ __forceinline__ Lane decode(const uint4 &e, bool valid, uint32_t keys
     L.kind = e.w & 3u;
     const uint32_t meta = e.w;
     const bool sh = (int)e.y < 0;
-    const bool key_ok = (meta >> 2) - keysz <= 2u; /* same batch, size <= 4 bytes */
+    const uint32_t gran = c.gran_log2;
+    const bool key_ok = (meta >> 2) - keysz <= gran; /* same batch, size <= one element */
     const bool tid_ok = L.tid <= tid_max;
     uint64_t word;
     bool in_range;
     if (W32) {
-        const uint32_t w32 = e.x >> 2;
+        const uint32_t w32 = e.x >> gran;
         word = w32;
         in_range = (e.y & 0x7fffffffu) == 0 && w32 < (sh ? c.smem_words : (uint32_t)c.global_words);
     } else {
-        word = ((uint64_t)(e.y & 0x7fffffffu) << 30) | (e.x >> 2);
+        word = ((((uint64_t)(e.y & 0x7fffffffu)) << 32) | e.x) >> gran;
         in_range = sh ? word < c.smem_words : word < c.global_words;
     }
     L.ok = valid && key_ok && tid_ok && in_range;
     if (__any_sync(FULL, valid && !L.ok)) {
-        const uint64_t wfull = ((uint64_t)(e.y & 0x7fffffffu) << 30) | (e.x >> 2);
+        const uint64_t wfull = ((((uint64_t)(e.y & 0x7fffffffu)) << 32) | e.x) >> gran;
         const uint32_t szl = (meta >> 2) & 7u;
-        const bool multi = valid && (meta >> 5) == B.key && (szl == 3 || szl == 4) && tid_ok &&
-                           (sh ? wfull + (1u << (szl - 2)) <= c.smem_words : wfull + (1u << (szl - 2)) <= c.global_words);
+        const bool multi = valid && (meta >> 5) == B.key && szl > gran && szl <= 4 && tid_ok &&
+                           (sh ? wfull + (1u << (szl - gran)) <= c.smem_words
+                               : wfull + (1u << (szl - gran)) <= c.global_words);
         if (valid && !L.ok && !multi)
             bad = 1;
         if (__any_sync(FULL, multi)) {

@@ -62,7 +62,7 @@ class DevCtx(ctypes.Structure):
                 ("ws_magic", ctypes.c_uint32), ("ws_s1", ctypes.c_uint32), ("ws_s2", ctypes.c_uint32),
                 ("g", ctypes.c_uint32), ("rec_bytes", ctypes.c_uint32), ("c_sh_b", ctypes.c_uint32),
                 ("c_sh_w", ctypes.c_uint32), ("c_sh_t", ctypes.c_uint32), ("c_max_g", ctypes.c_uint32),
-                ("c_max_b", ctypes.c_uint32), ("c_max_w", ctypes.c_uint32)]
+                ("c_max_b", ctypes.c_uint32), ("c_max_w", ctypes.c_uint32), ("gran_log2", ctypes.c_uint32)]
 
 
 class EpochLimits(ctypes.Structure):
@@ -209,10 +209,12 @@ class Checker:
 
     def __init__(self, grid_blocks: int, block_threads: int, warp_size: int = 32, global_words: int = 0,
                  smem_words: int = 0, report_capacity: int = 0, device: int = 0, policy: int = 0,
-                 compact=None):
+                 compact=None, granularity_log2: int = 2):
+        """Extents are given in 4-byte words (global_words, smem_words per block); the shadow has
+        one record per element of 1 << granularity_log2 bytes."""
         self.lib = load()
-        cfg = Config(grid_blocks, block_threads, warp_size, 4 * smem_words, 4 * global_words, 2, device,
-                     report_capacity)
+        cfg = Config(grid_blocks, block_threads, warp_size, 4 * smem_words, 4 * global_words, granularity_log2,
+                     device, report_capacity)
         h = ctypes.c_void_p()
         if compact is None:
             _check(self.lib.hirace_shadow_alloc(ctypes.byref(cfg), ctypes.byref(h)), "hirace_shadow_alloc")
@@ -225,6 +227,7 @@ class Checker:
         self.rec_bytes = 8 if compact is None else 4
         self.geometry = dict(grid_blocks=grid_blocks, block_threads=block_threads, warp_size=warp_size,
                              global_words=global_words, smem_words=smem_words)
+        self.granularity_log2 = granularity_log2
         self.device = device
         self.policy = POLICY_STRICT
         if policy != POLICY_STRICT:
@@ -235,7 +238,8 @@ class Checker:
         """compact=True: 4-byte records sized by the trace's own epoch maxima."""
         lim = trace_epoch_limits(trace.events) if compact else None
         return cls(trace.grid_blocks, trace.block_threads, trace.warp_size, trace.global_words, trace.smem_words,
-                   report_capacity, device, policy, compact=lim)
+                   report_capacity, device, policy, compact=lim,
+                   granularity_log2=getattr(trace, "granularity_log2", 2))
 
     def set_policy(self, policy: int, stream=None):
         """POLICY_STRICT or POLICY_RELAXED_READ_ATOMIC (include/hirace.h hirace_policy)."""
@@ -245,7 +249,8 @@ class Checker:
     @property
     def shadow_bytes(self) -> int:
         g = self.geometry
-        return self.rec_bytes * (g["global_words"] + g["grid_blocks"] * g["smem_words"])
+        per_word = 4 >> self.granularity_log2   # records per 4-byte word
+        return self.rec_bytes * per_word * (g["global_words"] + g["grid_blocks"] * g["smem_words"])
 
     def close(self):
         if getattr(self, "h", None):

@@ -197,3 +197,52 @@ def test_cfg5_construction_and_rank_partition():
     key = lambda e: np.sort(e.view(np.dtype((np.void, 16))))  # noqa: E731
     assert np.array_equal(key(allev), key(t.events))
     assert all(p.batch_count() == 32 for p in parts)
+
+
+# ---- element granularity (per-element shadow; reading R8) ----------
+
+@pytest.mark.parametrize("gran", [0, 1, 2])
+def test_granularity_oracle_vs_brute_force(gran):
+    for seed in range(300):
+        t = tg.random_tiny_bytes(seed, gran)
+        want = {k: c for k, (c, _) in brute.races(t.events, t.block_threads, t.warp_size, 0, gran).items()}
+        k, c, _ = oracle.races_of(t)
+        assert {int(a): int(b) for a, b in zip(k, c)} == want, (gran, seed)
+
+
+def _two_threads(off1, sz1, off2, sz2, kind1=1, kind2=1):
+    """thread 0 and thread 32 (another warp of block 0) access bytes of one shared window,
+    concurrently (same epochs)."""
+    ev = np.empty(2, dtype=tg.EVENT_DTYPE)
+    ev["addr"] = np.array([off1, off2], np.uint64) | tg.SHARED_BIT
+    ev["tid"] = [0, 32]
+    ev["meta"] = tg.pack_meta(np.array([kind1, kind2]), np.array([sz1, sz2]), 0, 0, 0)
+    return ev
+
+
+@pytest.mark.parametrize("off1,sz1,off2,sz2,flagged", [
+    # (byte offset, size_log2) of two concurrent writes -> flagged elements per granularity 0/1/2
+    (0, 0, 1, 0, ([], [0], [0])),            # adjacent bytes: race only when they share an element
+    (1, 0, 2, 0, ([], [], [0])),             # bytes 1 and 2: different half-words
+    (0, 2, 2, 0, ([2], [1], [0])),           # a word write and a byte write inside it
+    (0, 3, 6, 1, ([6, 7], [3], [1])),        # 8-byte write vs half-word at bytes 6-7
+    (4, 2, 8, 2, ([], [], [])),              # disjoint words never race
+])
+def test_granularity_closed_forms(off1, sz1, off2, sz2, flagged):
+    ev = _two_threads(off1, sz1, off2, sz2)
+    for gran in (0, 1, 2):
+        k, c, _ = oracle.races(ev, 64, 32, 0, gran)
+        assert [int(x) & 0xFFFFFFFF for x in k] == flagged[gran], gran
+        assert all(int(x) == 2 for x in c)   # two warps of one block: BLOCK class
+
+
+def test_finer_granularity_only_removes_races():
+    """A racing pair on an element is a racing pair on the word holding it, so the words of the
+    byte-granularity race set are a subset of the word-granularity race set."""
+    for seed in range(300):
+        t = tg.random_tiny_bytes(seed, 0)
+        k0, _, _ = oracle.races(t.events, t.block_threads, t.warp_size, 0, 0)
+        k2, _, _ = oracle.races(t.events, t.block_threads, t.warp_size, 0, 2)
+        hi = np.uint64(0xFFFFFFFF00000000)
+        words0 = {int((x & hi) | ((x & ~hi) >> np.uint64(2))) for x in k0}
+        assert words0 <= {int(x) for x in k2}, seed
