@@ -141,6 +141,11 @@ typedef struct {
     unsigned int c_sh_b, c_sh_w, c_sh_t;
     unsigned int c_max_g, c_max_b, c_max_w;
     unsigned int gran_log2;           /* tracked element = 1 << gran_log2 bytes               */
+    /* selective tracking (hirace_set_filter): an access is checked iff f_active == 0, or
+     * (tid & f_tid_mask) == f_tid_match and its space is enabled in f_spaces (bit 0 global,
+     * bit 1 shared) and, for global, its first element index lies in [f_glo, f_ghi)          */
+    unsigned int f_active, f_tid_mask, f_tid_match, f_spaces;
+    unsigned long long f_glo, f_ghi;
 } hirace_dev_ctx;
 
 /* ---- lifecycle (a11: shadow alloc/init, "Initially, all State values are set
@@ -360,6 +365,22 @@ hirace_status hirace_microbench_atomics(int device, uint64_t nwords, int random,
 /* Cost of one grid barrier at the persistent replay kernel's grid size, microseconds.
  * mode 0 = the library's barrier; 1 = busy polling; 2 = generation flag set by the last CTA. */
 hirace_status hirace_microbench_grid_sync(int device, int iters, int mode, double *us_per_barrier, void *stream);
+
+/* Selective tracking ("Individual threads or test data
+ * addresses may have their instrumentation enabled or disabled dynamically.  The memory
+ * footprint can be reduced by tracking only representative threads from a symmetric group").
+ * Later replays (hirace_replay_trace / hirace_check_trace_*) and inline launches (the device
+ * context copied after this call) check an access only if
+ *     (tid & tid_mask) == tid_match                 -- e.g. mask 31, match 0: lane 0 of every warp
+ *     and its space is in `spaces` (1 = global, 2 = shared, 3 = both)
+ *     and, for a global access, its first element index is in [global_lo, global_hi).
+ * Unselected accesses are skipped (not counted as checked, never BAD_TRACE).  Races are then
+ * those among the selected accesses.  hirace_set_filter(ctx, 0, 0, 3, 0, UINT64_MAX) selects
+ * everything (the default).  Host-side; takes effect at the next launch.  The wire replay
+ * (sharded mode) ignores the filter.  Errors: INVAL (NULL ctx, tid_match outside tid_mask,
+ * spaces > 3, global_lo > global_hi). */
+hirace_status hirace_set_filter(hirace_ctx *ctx, uint32_t tid_mask, uint32_t tid_match, uint32_t spaces,
+                                uint64_t global_lo, uint64_t global_hi);
 
 /* Selects the conflict policy of a context by uploading that policy's FSM table (stream-ordered
  * on `stream`).  Takes effect for later replays and inline launches; call it on a reset shadow

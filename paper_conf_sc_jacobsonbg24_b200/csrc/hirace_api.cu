@@ -224,6 +224,12 @@ hirace_status shadow_alloc_impl(const hirace_config *cfg, const hirace_epoch_lim
     d.g = 0;
     d.rec_bytes = c->rec_bytes;
     d.gran_log2 = cfg->granularity_log2;
+    d.f_active = 0;
+    d.f_tid_mask = 0;
+    d.f_tid_match = 0;
+    d.f_spaces = 3;
+    d.f_glo = 0;
+    d.f_ghi = ~0ull;
     d.c_sh_b = lay.sh_b;
     d.c_sh_w = lay.sh_w;
     d.c_sh_t = lay.sh_t;
@@ -275,6 +281,21 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
     if (c->copy_stream)
         cudaStreamDestroy(c->copy_stream);
     delete c;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_set_filter(hirace_ctx *c, uint32_t tid_mask, uint32_t tid_match, uint32_t spaces,
+                                uint64_t global_lo, uint64_t global_hi)
+{
+    if (!c || (tid_match & ~tid_mask) || spaces > 3 || global_lo > global_hi)
+        return HIRACE_E_INVAL;
+    hirace_dev_ctx &d = c->dev;
+    d.f_tid_mask = tid_mask;
+    d.f_tid_match = tid_match;
+    d.f_spaces = spaces;
+    d.f_glo = global_lo;
+    d.f_ghi = global_hi;
+    d.f_active = (tid_mask != 0 || spaces != 3 || global_lo != 0 || global_hi < c->global_words) ? 1u : 0u;
     return HIRACE_OK;
 }
 

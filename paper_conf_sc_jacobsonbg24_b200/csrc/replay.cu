@@ -258,11 +258,12 @@ struct Lane {
  * < 2^31 words and tracked byte offsets fit 32 bits, so index math and range checks are 32-bit
  * (fewer instructions on the hot path); otherwise 64-bit. */
 template <bool W32, typename R>
-__device__ __forceinline__ Lane decode(const uint4 &e, bool valid, uint32_t keysz, const Batch &B,
+__device__ __forceinline__ Lane decode(const uint4 &e, bool valid_in, uint32_t keysz, const Batch &B,
                                        uint32_t tid_max, const hirace_dev_ctx &c, const geom &G,
                                        const unsigned char *raw, Counters &cnt, uint32_t &bad, uint32_t lane)
 {
     Lane L;
+    bool valid = valid_in;
     L.tid = e.z;
     L.kind = e.w & 3u;
     const uint32_t meta = e.w;
@@ -279,6 +280,11 @@ __device__ __forceinline__ Lane decode(const uint4 &e, bool valid, uint32_t keys
     } else {
         word = ((((uint64_t)(e.y & 0x7fffffffu)) << 32) | e.x) >> gran;
         in_range = sh ? word < c.smem_words : word < c.global_words;
+    }
+    if (c.f_active) { /* selective tracking (hirace_set_filter): unselected accesses are skipped */
+        const uint64_t wsel = ((((uint64_t)(e.y & 0x7fffffffu)) << 32) | e.x) >> gran;
+        valid = valid && (L.tid & c.f_tid_mask) == c.f_tid_match &&
+                (sh ? (c.f_spaces & 2u) != 0 : ((c.f_spaces & 1u) != 0 && wsel >= c.f_glo && wsel < c.f_ghi));
     }
     L.ok = valid && key_ok && tid_ok && in_range;
     if (__any_sync(FULL, valid && !L.ok)) {

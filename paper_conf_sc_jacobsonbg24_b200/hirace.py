@@ -33,7 +33,7 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_collect_races_device", "hirace_get_stats", "hirace_sync", "hirace_get_dev_ctx",
            "hirace_bucket_events", "hirace_bucket_wire", "hirace_replay_wire", "hirace_count_wire",
            "hirace_dispatch_wire", "hirace_peer_buffer_alloc", "hirace_peer_buffer_free", "hirace_peer_open",
-           "hirace_peer_close", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_set_policy",
+           "hirace_peer_close", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_set_policy", "hirace_set_filter",
            "hirace_fsm_table", "hirace_fsm_table_policy", "hirace_fsm_step", "hirace_fsm_step_policy", "hirace_fsm_step_compact", "hirace_status_string",
            "hirace_version")
 
@@ -62,7 +62,9 @@ class DevCtx(ctypes.Structure):
                 ("ws_magic", ctypes.c_uint32), ("ws_s1", ctypes.c_uint32), ("ws_s2", ctypes.c_uint32),
                 ("g", ctypes.c_uint32), ("rec_bytes", ctypes.c_uint32), ("c_sh_b", ctypes.c_uint32),
                 ("c_sh_w", ctypes.c_uint32), ("c_sh_t", ctypes.c_uint32), ("c_max_g", ctypes.c_uint32),
-                ("c_max_b", ctypes.c_uint32), ("c_max_w", ctypes.c_uint32), ("gran_log2", ctypes.c_uint32)]
+                ("c_max_b", ctypes.c_uint32), ("c_max_w", ctypes.c_uint32), ("gran_log2", ctypes.c_uint32),
+                ("f_active", ctypes.c_uint32), ("f_tid_mask", ctypes.c_uint32), ("f_tid_match", ctypes.c_uint32),
+                ("f_spaces", ctypes.c_uint32), ("f_glo", ctypes.c_uint64), ("f_ghi", ctypes.c_uint64)]
 
 
 class EpochLimits(ctypes.Structure):
@@ -111,6 +113,7 @@ def load():
         "hirace_microbench_atomics": (I32, [I32, U64, I32, I32, U64, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_microbench_grid_sync": (I32, [I32, I32, I32, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_set_policy": (I32, [P, I32, P]),
+        "hirace_set_filter": (I32, [P, U32, U32, U32, U64, U64]),
         "hirace_fsm_table": (I32, [P]),
         "hirace_fsm_table_policy": (I32, [I32, P]),
         "hirace_fsm_step": (U64, [U64, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
@@ -240,6 +243,12 @@ class Checker:
         return cls(trace.grid_blocks, trace.block_threads, trace.warp_size, trace.global_words, trace.smem_words,
                    report_capacity, device, policy, compact=lim,
                    granularity_log2=getattr(trace, "granularity_log2", 2))
+
+    def set_filter(self, tid_mask: int = 0, tid_match: int = 0, spaces: int = 3, global_lo: int = 0,
+                   global_hi: int = (1 << 64) - 1):
+        """Selective tracking (include/hirace.h hirace_set_filter); defaults select everything."""
+        _check(self.lib.hirace_set_filter(self.h, tid_mask, tid_match, spaces, global_lo, global_hi),
+               "hirace_set_filter")
 
     def set_policy(self, policy: int, stream=None):
         """POLICY_STRICT or POLICY_RELAXED_READ_ATOMIC (include/hirace.h hirace_policy)."""

@@ -56,3 +56,24 @@ def test_status_strings_and_version():
     lib = hirace.load()
     assert lib.hirace_status_string(-6) == b"bad trace"
     assert b"sm_100a" in lib.hirace_version()
+
+
+def test_ctypes_structs_match_the_c_header(tmp_path):
+    """The binding's ctypes mirrors of hirace_config / hirace_dev_ctx / hirace_epoch_limits have
+    the C layout (the library writes whole structs into them)."""
+    import ctypes
+    import subprocess
+
+    from paper_conf_sc_jacobsonbg24_b200 import hirace as hb
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    src = tmp_path / "sz.c"
+    fields = [f for f, _ in hb.DevCtx._fields_]
+    src.write_text("#include <stdio.h>\n#include <stddef.h>\n#include \"hirace.h\"\nint main(){\n"
+                   "printf(\"%zu %zu %zu\\n\", sizeof(hirace_config), sizeof(hirace_dev_ctx), sizeof(hirace_epoch_limits));\n"
+                   + "".join(f"printf(\"%zu\\n\", offsetof(hirace_dev_ctx, {f}));\n" for f in fields) + "return 0;}\n")
+    exe = tmp_path / "sz"
+    subprocess.check_call(["gcc", "-I", os.path.join(root, "include"), str(src), "-o", str(exe)])
+    out = subprocess.check_output([str(exe)], text=True).split()
+    assert [int(x) for x in out[:3]] == [ctypes.sizeof(hb.Config), ctypes.sizeof(hb.DevCtx),
+                                        ctypes.sizeof(hb.EpochLimits)]
+    assert [int(x) for x in out[3:]] == [getattr(hb.DevCtx, f).offset for f in fields]
