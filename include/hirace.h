@@ -143,9 +143,12 @@ typedef struct {
     unsigned int gran_log2;           /* tracked element = 1 << gran_log2 bytes               */
     /* selective tracking (hirace_set_filter): an access is checked iff f_active == 0, or
      * (tid & f_tid_mask) == f_tid_match and its space is enabled in f_spaces (bit 0 global,
-     * bit 1 shared) and, for global, its first element index lies in [f_glo, f_ghi)          */
+     * bit 1 shared) and, for global, its first element index lies in [f_glo, f_ghi) (an empty
+     * range when global memory is disabled).  f_smem_words = smem_words, or 0 when shared
+     * memory is disabled (the inline hook's bound).                                          */
     unsigned int f_active, f_tid_mask, f_tid_match, f_spaces;
     unsigned long long f_glo, f_ghi;
+    unsigned int f_smem_words, f_pad;
 } hirace_dev_ctx;
 
 /* ---- lifecycle (a11: shadow alloc/init, "Initially, all State values are set

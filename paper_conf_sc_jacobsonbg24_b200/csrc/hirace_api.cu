@@ -230,6 +230,8 @@ hirace_status shadow_alloc_impl(const hirace_config *cfg, const hirace_epoch_lim
     d.f_spaces = 3;
     d.f_glo = 0;
     d.f_ghi = ~0ull;
+    d.f_smem_words = d.smem_words;
+    d.f_pad = 0;
     d.c_sh_b = lay.sh_b;
     d.c_sh_w = lay.sh_w;
     d.c_sh_t = lay.sh_t;
@@ -293,8 +295,9 @@ hirace_status hirace_set_filter(hirace_ctx *c, uint32_t tid_mask, uint32_t tid_m
     d.f_tid_mask = tid_mask;
     d.f_tid_match = tid_match;
     d.f_spaces = spaces;
-    d.f_glo = global_lo;
-    d.f_ghi = global_hi;
+    d.f_glo = (spaces & 1u) ? global_lo : 0;
+    d.f_ghi = (spaces & 1u) ? global_hi : 0;
+    d.f_smem_words = (spaces & 2u) ? d.smem_words : 0;
     d.f_active = (tid_mask != 0 || spaces != 3 || global_lo != 0 || global_hi < c->global_words) ? 1u : 0u;
     return HIRACE_OK;
 }

@@ -64,7 +64,8 @@ class DevCtx(ctypes.Structure):
                 ("c_sh_w", ctypes.c_uint32), ("c_sh_t", ctypes.c_uint32), ("c_max_g", ctypes.c_uint32),
                 ("c_max_b", ctypes.c_uint32), ("c_max_w", ctypes.c_uint32), ("gran_log2", ctypes.c_uint32),
                 ("f_active", ctypes.c_uint32), ("f_tid_mask", ctypes.c_uint32), ("f_tid_match", ctypes.c_uint32),
-                ("f_spaces", ctypes.c_uint32), ("f_glo", ctypes.c_uint64), ("f_ghi", ctypes.c_uint64)]
+                ("f_spaces", ctypes.c_uint32), ("f_glo", ctypes.c_uint64), ("f_ghi", ctypes.c_uint64),
+                ("f_smem_words", ctypes.c_uint32), ("f_pad", ctypes.c_uint32)]
 
 
 class EpochLimits(ctypes.Structure):

@@ -96,3 +96,17 @@ def test_sharded_entry_points_need_word_granularity():
     c.close()
     with pytest.raises(hr.HiraceError):
         hr.Checker(4, 64, 32, 64, 16, granularity_log2=3)
+
+
+def test_inline_hook_granularity_must_match_its_build():
+    # the examples are built with the default inline element size (4-byte words): a context at
+    # byte granularity disables their tracking and reports BAD_TRACE instead of mis-keying
+    from paper_conf_sc_jacobsonbg24_b200 import examples as ex
+    n, steps = 64, 2
+    t = tg.cfg2(True, n=n, steps=steps)
+    c = hr.Checker(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words, granularity_log2=0)
+    c.reset()
+    buf = torch.rand(2 * n * n, device="cuda")
+    ex.stencil(c, buf, n, steps, True)
+    assert c.sync() == -6
+    c.close()
