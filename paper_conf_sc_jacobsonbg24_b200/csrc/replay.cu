@@ -330,6 +330,57 @@ __device__ __noinline__ unsigned int collect_call(const hirace_dev_ctx c, uint64
     return epoch;
 }
 
+/* a5 + a6 issue for one chunk whose records o were loaded: transition, then the CAS of every
+ * changed word (the result is awaited in chunk_finish, so other work can overlap it) */
+template <typename R> struct Issued {
+    R n, prev;
+    uint32_t ent;
+    bool do_cas;
+};
+
+template <typename R>
+__device__ __forceinline__ Issued<R> chunk_issue(const Lane &cur, R o, const Batch &B, const hirace_dev_ctx &c,
+                                                 const geom &G, const Rec<R> &rec, uint32_t tab_s, Counters &cnt)
+{
+    Issued<R> I;
+    I.ent = lds_u8(tab_s + 2048 + (((uint32_t)(o & 31u) << 7) | rec.label(o, cur.tid, cur.kind, B.ep, G)));
+    I.n = rec.next(o, I.ent, cur.tid, B.ep);
+    /* a6: one CAS per changed word; unchanged = linearised at the load */
+    I.do_cas = cur.ok && I.n != o;
+    cnt.cas += I.do_cas; /* main-path no-write accesses = checked - first CASes (counted at the end) */
+    I.prev = Rec<R>::cas_if(shadow_as<R>(c) + cur.idx, o, I.n, I.do_cas);
+    return I;
+}
+
+/* a6 result, a3 fold of the lost CASes, a7 report (warp-collective) */
+template <typename R>
+__device__ __forceinline__ void chunk_finish(const Lane &cur, R o, const Issued<R> &I, const Batch &B,
+                                             const hirace_dev_ctx &c, const geom &G, const Rec<R> &rec,
+                                             const unsigned char *raw, Counters &cnt, uint32_t lane, uint32_t below)
+{
+    const bool failed = I.do_cas && I.prev != o;
+    /* common case: no lane lost its CAS and no lane's transition reports -> one vote */
+    const bool rep = (I.ent & E_REPORT) && I.do_cas && !failed;
+    if (!__any_sync(FULL, failed || rep))
+        return;
+    uint32_t cls = 0, rtid = cur.tid;
+    if (rep) {
+        const uint32_t cn = race_class(st_of(I.n)), co = race_class(st_of(o));
+        cls = cn > co ? cn : 0u;
+    }
+    if (__any_sync(FULL, failed)) {
+        /* Algorithm 1's retry for the lanes whose CAS lost: group them by word, the group
+         * leader folds its members' accesses from the record it observed */
+        const uint32_t peers = __match_any_sync(FULL, failed ? cur.idx : NONE);
+        const bool lead = failed && (peers & below) == 0;
+        cls |= commit_groups<R>(shadow_as<R>(c) + cur.idx, I.prev, lead ? peers : 0u, cur.tid, cur.kind, G, raw, B,
+                                rec, cnt, rtid, false);
+    }
+    /* a7 */
+    if (__any_sync(FULL, cls != 0))
+        append_reports(c, cls, key_of_idx(cur, c, G), B.g, rtid, lane);
+}
+
 /* One 32-event chunk (one event per lane) after decode: a4 load, a5 transition, a6 CAS, a3
  * collision fold, a7 report.  All lanes of the warp call it (warp-collective).  tab_s = shared
  * address of the canonical table; the raw-flag table follows it at +2048. */
@@ -339,38 +390,11 @@ __device__ __forceinline__ void process_decoded(const Lane &cur, const Batch &B,
                                                 uint32_t tab_s, Counters &cnt, uint32_t lane, uint32_t below)
 {
     /* a4: optimistic: every lane reads its own word (coherent load); lanes that share a word
-     * are grouped only if their CAS collides (below) */
-    R *const p = shadow_as<R>(c) + cur.idx;
-    const R o = cur.ok ? Rec<R>::load(p) : (R)0;
+     * are grouped only if their CAS collides (chunk_finish) */
+    const R o = cur.ok ? Rec<R>::load(shadow_as<R>(c) + cur.idx) : (R)0;
     cnt.checked += cur.ok;
-
-    /* a5: transition */
-    const uint32_t ent = lds_u8(tab_s + 2048 + (((uint32_t)(o & 31u) << 7) | rec.label(o, cur.tid, cur.kind, B.ep, G)));
-    const R n = rec.next(o, ent, cur.tid, B.ep);
-    /* a6: one CAS per changed word; unchanged = linearised at the load */
-    const bool do_cas = cur.ok && n != o;
-    cnt.cas += do_cas; /* main-path no-write accesses = checked - first CASes (counted at the end) */
-    const R prev = Rec<R>::cas_if(p, o, n, do_cas);
-    const bool failed = do_cas && prev != o;
-    /* common case: no lane lost its CAS and no lane's transition reports -> one vote */
-    const bool rep = (ent & E_REPORT) && do_cas && !failed;
-    if (!__any_sync(FULL, failed || rep))
-        return;
-    uint32_t cls = 0, rtid = cur.tid;
-    if (rep) {
-        const uint32_t cn = race_class(st_of(n)), co = race_class(st_of(o));
-        cls = cn > co ? cn : 0u;
-    }
-    if (__any_sync(FULL, failed)) {
-        /* Algorithm 1's retry for the lanes whose CAS lost: group them by word, the group
-         * leader folds its members' accesses from the record it observed */
-        const uint32_t peers = __match_any_sync(FULL, failed ? cur.idx : NONE);
-        const bool lead = failed && (peers & below) == 0;
-        cls |= commit_groups<R>(p, prev, lead ? peers : 0u, cur.tid, cur.kind, G, raw, B, rec, cnt, rtid, false);
-    }
-    /* a7 */
-    if (__any_sync(FULL, cls != 0))
-        append_reports(c, cls, key_of_idx(cur, c, G), B.g, rtid, lane);
+    const Issued<R> I = chunk_issue<R>(cur, o, B, c, G, rec, tab_s, cnt);
+    chunk_finish<R>(cur, o, I, B, c, G, rec, raw, cnt, lane, below);
 }
 
 __device__ __forceinline__ void flush_stats(const hirace_dev_ctx &c, Counters cnt, unsigned long long *s_stats,
