@@ -327,10 +327,8 @@ hirace_status hirace_shadow_reset(hirace_ctx *c, void *stream)
         return HIRACE_E_INVAL;
     cudaStream_t st = (cudaStream_t)stream;
     HR_CUDA(c, cudaSetDevice(c->device));
-    HR_CUDA(c, cudaMemsetAsync(c->d_shadow, 0, c->shadow_words * c->rec_bytes, st));
-    HR_CUDA(c, cudaMemsetAsync(c->d_report_count, 0, sizeof(unsigned long long), st));
-    HR_CUDA(c, cudaMemsetAsync(c->d_stats, 0, 4 * sizeof(unsigned long long), st));
-    HR_CUDA(c, cudaMemsetAsync(c->d_err, 0, sizeof(unsigned int), st));
+    HR_CUDA(c, launch_reset(c->d_shadow, c->shadow_words * c->rec_bytes, c->d_report_count, c->d_stats, c->d_err,
+                            c->sm_count, st));
     c->g = 0;
     c->dev.g = 0;
     c->sticky = HIRACE_OK;

@@ -52,11 +52,13 @@ struct FindSmem {
  * batch_off[0..nb], zero the per-batch claim counters, check keys strictly increase. */
 __global__ void __launch_bounds__(kFindThreads) k_batches(const hirace_event *__restrict__ ev, uint32_t n,
                                                           uint32_t *off, uint32_t *nbatches, uint32_t *batch_ctr,
-                                                          unsigned int *err)
+                                                          unsigned int *err, unsigned int *grid_bar)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     FindSmem &S = *reinterpret_cast<FindSmem *>(smem_raw);
     const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    if (threadIdx.x == 0)
+        *grid_bar = 0; /* the replay kernel's grid-barrier counter (stream-ordered before it) */
     if (threadIdx.x == 0) {
         S.count = 1;
         S.list[0] = 0;
@@ -156,7 +158,8 @@ cudaError_t launch_find_batches(const hirace_event *ev, uint32_t n, const Scratc
                                 int sm_count, cudaStream_t st)
 {
     (void)sm_count;
-    k_batches<<<1, kFindThreads, sizeof(FindSmem), st>>>(ev, n, s.batch_off, s.nbatches, s.batch_ctr, err);
+    k_batches<<<1, kFindThreads, sizeof(FindSmem), st>>>(ev, n, s.batch_off, s.nbatches, s.batch_ctr, err,
+                                                         s.grid_bar);
     return cudaGetLastError();
 }
 
@@ -592,6 +595,36 @@ cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t h
     k_wire_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_off, nullptr, 0, err,
                                                       d_peer);
     return cudaGetLastError();
+}
+
+/* a11 + counters: the whole context reset as ONE launch (shadow := INIT, reports, stats and
+ * error flags := 0) instead of four memsets */
+__global__ void __launch_bounds__(256) k_reset(uint4 *shadow, uint64_t n16, unsigned long long *report_count,
+                                               unsigned long long *stats, unsigned int *err)
+{
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n16; i += stride)
+        __stcs(shadow + i, make_uint4(0, 0, 0, 0));
+    if (blockIdx.x == 0 && threadIdx.x < 4)
+        stats[threadIdx.x] = 0;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        *report_count = 0;
+        *err = 0;
+    }
+}
+
+cudaError_t launch_reset(void *shadow, uint64_t bytes, unsigned long long *report_count, unsigned long long *stats,
+                         unsigned int *err, int sm_count, cudaStream_t st)
+{
+    const uint64_t n16 = bytes / 16;
+    uint64_t blocks = (n16 + 255) / 256;
+    const uint64_t cap = (uint64_t)(sm_count > 0 ? sm_count : 148) * 8;
+    blocks = blocks < 1 ? 1 : (blocks > cap ? cap : blocks);
+    k_reset<<<(unsigned)blocks, 256, 0, st>>>(reinterpret_cast<uint4 *>(shadow), n16, report_count, stats, err);
+    cudaError_t e = cudaGetLastError();
+    if (e == cudaSuccess && (bytes & 15)) /* shadow sizes are multiples of 4: a ragged 4/8/12-byte tail */
+        e = cudaMemsetAsync(static_cast<char *>(shadow) + n16 * 16, 0, bytes & 15, st);
+    return e;
 }
 
 cudaError_t kernels_init(int device)

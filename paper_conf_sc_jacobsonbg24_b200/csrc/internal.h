@@ -47,6 +47,9 @@ cudaError_t launch_collect(const hirace_dev_ctx &c, uint64_t shadow_words, const
 constexpr uint64_t kReportModeMinBytes = 64ull << 20;
 cudaError_t replay_init();
 cudaError_t launch_rebase(const hirace_dev_ctx &c, uint64_t shadow_words, cudaStream_t st);
+/* shadow := INIT and report count, stats, error flags := 0, in one launch */
+cudaError_t launch_reset(void *shadow, uint64_t bytes, unsigned long long *report_count, unsigned long long *stats,
+                         unsigned int *err, int sm_count, cudaStream_t st);
 cudaError_t launch_bucket(const hirace_dev_ctx &c, const hirace_event *in, uint32_t n, int nranks, int my_rank,
                           hirace_event *out, unsigned long long *d_counts, uint32_t *d_tile_hist, uint32_t ntiles,
                           cudaStream_t st);
