@@ -35,3 +35,18 @@ for b in range(min(nb - 1, 12)):
     print(f"batch {b}: work {(a0 - start) / 1e3:7.2f}..{(a1 - start) / 1e3:7.2f} us (first..last CTA arrival), "
           f"spread {(a1 - a0) / 1e3:6.2f} us, p50 {(np.median(arr) - start) / 1e3:7.2f}, release {(r1 - a1) / 1e3:5.2f} us")
     prev_rel = rel.min()
+
+# persistence of lateness: rank correlation of per-CTA arrival order between batches, and the
+# arrival spread by SM die half (CTA i runs on SM ~ i mod #SMs for a 2-CTA/SM persistent grid)
+ranks = []
+for b in range(min(nb - 1, 12)):
+    arr = buf[b, :grid, 0]
+    ranks.append(np.argsort(np.argsort(arr)))
+ranks = np.array(ranks, dtype=np.float64)
+if len(ranks) > 2:
+    cc = np.corrcoef(ranks)
+    off = cc[np.triu_indices(len(ranks), 1)]
+    print(f"rank correlation of CTA arrival order across batches: mean {off.mean():.3f} "
+          f"(min {off.min():.3f}, max {off.max():.3f})")
+    mean_rank = ranks.mean(axis=0)
+    print("latest 10 CTAs on average:", np.argsort(-mean_rank)[:10].tolist())
