@@ -192,6 +192,22 @@ BASELINE_CFG = {
 }
 
 
+def l2_roofline(st: dict, n_acc: int, kern_ms: float, rec_bytes: int, dev: int) -> dict:
+    """the L2-atomic roofline of this workload, from microbenchmarks run in the same
+    process on L2-resident words (coalesced, the replay's access shape): every access is one
+    coherent load, the ones that change their record add a CAS.  t = loads / load_rate +
+    CASes / cas_rate; the binding roofline is the lower of this and the HBM one."""
+    from paper_conf_sc_jacobsonbg24_b200 import hirace as h
+    nwords = 1 << 22  # 32 MiB of 8-byte words: L2-resident
+    load_rate = h.microbench_atomics(nwords, False, 2, 1 << 27, device=dev)
+    cas_rate = h.microbench_atomics(nwords, False, 0, 1 << 27, device=dev)
+    t = n_acc / load_rate + st["cas_ops"] / cas_rate
+    return {"bound": "l2_atomic", "accesses_per_s_peak": n_acc / t, "achieved": n_acc / (kern_ms / 1e3),
+            "frac": (n_acc / (kern_ms / 1e3)) / (n_acc / t), "coalesced_load_ops_per_s": load_rate,
+            "coalesced_cas_ops_per_s": cas_rate, "cas_ops": st["cas_ops"], "loads": n_acc,
+            "note": "64-bit microbenchmark rates; min(HBM, this) binds (SURVEY 8(d))"}
+
+
 def measure_slowdown(dev: int, reps: int = 5) -> dict:
     """Instrumented slowdown (BASELINE.json metric): native CUDA programs timed uninstrumented
     and with every tracked access / barrier checked inline by the HiRace device hooks
@@ -493,6 +509,12 @@ def main():
         return
     peak, peak_kind = peaks()
     achieved = bpa * n_acc / (kern_ms / 1e3) / 1e9
+    try:
+        l2 = l2_roofline(st, n_acc, kern_ms, c.rec_bytes, local_rank)
+        l2["hbm_accesses_per_s_peak"] = peak * 1e9 / bpa
+        l2["binding"] = "hbm" if peak * 1e9 / bpa <= l2["accesses_per_s_peak"] else "l2_atomic"
+    except Exception as exc:  # diagnostics only; never fails the bench line
+        l2 = {"error": str(exc)}
     slow = None if args.no_slowdown else measure_slowdown(local_rank)
     cpu = None
     if not args.no_cpu_baseline and world == 1:
@@ -512,6 +534,7 @@ def main():
                      "frac": achieved / peak, "traffic": load_traffic(args.config, args.variant, args.compact),
                      "kernel": "k_replay (incl. fused collect)", "kernel_ms": kern_ms, "kernel_share": kern_ms / ms_per_step,
                      "bytes_per_access": bpa, "peak_kind": peak_kind},
+        "roofline_l2": l2,
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": 2 * K,  # k_batches + k_replay (fused collect) per step

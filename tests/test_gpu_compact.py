@@ -220,3 +220,24 @@ def test_report_collect_overflow_falls_back_to_scan(monkeypatch):
     assert as_dict(c.collect()) == want
     assert c.stats()["dropped_reports"] > 0
     c.close()
+
+
+def test_compact_cfg5_medium_by_construction():
+    """Config 5 shape at 2^28 words and 2^21 threads fits the compact record (5 + 2 + 2 + 1 + 21
+    bits): 1.3e8 events, report-buffer collect on a 1 GiB compact shadow; the flagged set is known
+    by construction (tracegen; pinned against the oracle at reduced scale in the CPU suite)."""
+    from tests.helpers import CLS
+    t = tg.cfg5(grid_blocks=8192, words_log2=28)
+    want = {w: CLS[c] for w, c in t.info["expected"].items()}
+    r, st = compact_races(t, fused=True)
+    assert as_dict(r) == want
+    assert st["dropped_reports"] == 0
+
+
+def test_compact_host_entry_point():
+    t = tg.cfg4("B", 8, 128, 34)
+    c = hr.Checker.for_trace(t, compact=True)
+    c.reset()
+    got = as_dict(c.check_host(t.events))
+    c.close()
+    assert got == oracle_dict(t)
