@@ -414,9 +414,16 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_sc_jacobsonbg24_b200 as hr
+    ngpu = torch.cuda.device_count()
+    local_rank = local_rank % ngpu  # several ranks per GPU only in single-GPU functional runs
     torch.cuda.set_device(local_rank)
+    red_dev = "cuda"
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if world <= ngpu:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        else:  # ranks share a GPU: NCCL cannot run there; timing reductions go through gloo
+            dist.init_process_group("gloo")
+            red_dev = "cpu"
 
     n_acc = word_accesses(trace.events)
     c = hr.Checker.for_trace(trace, device=local_rank, compact=args.compact)
@@ -467,7 +474,7 @@ def main():
     kern_ms = sum(a.elapsed_time(b) for a, b in zip(ks, ke)) / K
     c.set_kernel_timing(None, None)
     if world > 1:
-        tt = torch.tensor([ms, kern_ms], dtype=torch.float64, device="cuda")
+        tt = torch.tensor([ms, kern_ms], dtype=torch.float64, device=red_dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms, kern_ms = float(tt[0]), float(tt[1])
     ms_per_step = ms / K
@@ -495,7 +502,7 @@ def main():
         torch.cuda.synchronize()
         e2e_s = (time.perf_counter() - we0) / ke2
         if world > 1:
-            tt = torch.tensor([e2e_s], dtype=torch.float64, device="cuda")
+            tt = torch.tensor([e2e_s], dtype=torch.float64, device=red_dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             e2e_s = float(tt[0])
         e2e = {"value": n_acc * world / e2e_s, "unit": UNIT, "h2d_bytes_per_step": int(trace.n * 16),
