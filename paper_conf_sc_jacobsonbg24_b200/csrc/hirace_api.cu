@@ -642,6 +642,10 @@ hirace_status wire_scratch(hirace_ctx *c, uint64_t nb, int nranks, uint32_t maxl
     return HIRACE_OK;
 }
 
+hirace_status bucket_wire_impl(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
+                               int nranks, int my_rank, uint64_t *d_out, uint64_t cap, uint64_t *h_counts,
+                               uint64_t *n_words, void *stream);
+
 hirace_status wire_args_ok(hirace_ctx *c, const uint32_t *h_offsets, uint64_t nb, int nranks, int my_rank,
                            uint32_t *maxlen)
 {
@@ -670,9 +674,7 @@ hirace_status hirace_count_wire(hirace_ctx *c, const hirace_event *d_in, const u
     uint64_t n = 0;
     if (!c || !h_counts || !h_offsets || (nb && !d_in))
         return HIRACE_E_INVAL;
-    const hirace_status s = hirace_bucket_wire(c, d_in, h_offsets, nb, nranks, my_rank, nullptr, 0, h_counts, &n,
-                                               stream);
-    return (s == HIRACE_E_INVAL && n > 0) ? HIRACE_OK : s; /* count-only: no output buffer */
+    return bucket_wire_impl(c, d_in, h_offsets, nb, nranks, my_rank, nullptr, 0, h_counts, &n, stream);
 }
 
 hirace_status hirace_dispatch_wire(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
@@ -766,9 +768,14 @@ hirace_status hirace_peer_close(void *d_ptr)
     return cudaIpcCloseMemHandle(d_ptr) == cudaSuccess ? HIRACE_OK : HIRACE_E_CUDA;
 }
 
-hirace_status hirace_bucket_wire(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
-                                 int nranks, int my_rank, uint64_t *d_out, uint64_t cap, uint64_t *h_counts,
-                                 uint64_t *n_words, void *stream)
+} /* extern "C" */
+
+namespace {
+
+/* hirace_bucket_wire; d_out == NULL counts only (hirace_count_wire: no capacity check) */
+hirace_status bucket_wire_impl(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
+                               int nranks, int my_rank, uint64_t *d_out, uint64_t cap, uint64_t *h_counts,
+                               uint64_t *n_words, void *stream)
 {
     if (!c || !h_offsets || !h_counts || !n_words || (nb && !d_in) || (cap && !d_out))
         return HIRACE_E_INVAL;
@@ -800,9 +807,27 @@ hirace_status hirace_bucket_wire(hirace_ctx *c, const hirace_event *d_in, const 
     *n_words = total;
     if (flag & hirace::ERR_BAD_TRACE)
         return set_sticky(c, HIRACE_E_BAD_TRACE);
-    if (total > cap)
+    if (d_out && total > cap)
         return HIRACE_E_INVAL;
     return HIRACE_OK;
+}
+
+} // namespace
+
+extern "C" {
+
+hirace_status hirace_bucket_wire(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
+                                 int nranks, int my_rank, uint64_t *d_out, uint64_t cap, uint64_t *h_counts,
+                                 uint64_t *n_words, void *stream)
+{
+    if (cap && !d_out)
+        return HIRACE_E_INVAL;
+    uint64_t dummy = 0;
+    const hirace_status s = bucket_wire_impl(c, d_in, h_offsets, nb, nranks, my_rank, d_out, cap, h_counts,
+                                             n_words ? n_words : &dummy, stream);
+    if (s == HIRACE_OK && !d_out && n_words && *n_words > 0)
+        return HIRACE_E_INVAL; /* not sticky: call again with a buffer of *n_words records */
+    return s;
 }
 
 hirace_status hirace_replay_wire(hirace_ctx *c, const uint64_t *d_wire, uint64_t n, uint32_t batch_key, void *stream)
