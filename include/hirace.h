@@ -322,8 +322,9 @@ hirace_status hirace_replay_wire(hirace_ctx *ctx, const uint64_t *d_wire, uint64
  *      batch the senders in rank order;
  *   3. hirace_dispatch_wire with the peer table (each rank's buffer from
  *      hirace_peer_buffer_alloc, opened by the others with hirace_peer_open);
- *   4. stream sync + a process barrier make the stores visible; each owner replays its buffer
- *      batch by batch with hirace_replay_wire. */
+ *   4. every rank records an interprocess CUDA event after its dispatch; after a host barrier
+ *      (which only orders the records) each owner's stream waits on all the peers' events and
+ *      replays its buffer batch by batch with hirace_replay_wire — no stream drains. */
 
 /* Per-batch per-owner wire-record counts of nb batches of DEVICE events (h_offsets as from
  * hirace_find_batches): HOST h_counts[nb * nranks], row b = batch b.  Exactly the records
@@ -336,10 +337,12 @@ hirace_status hirace_count_wire(hirace_ctx *ctx, const hirace_event *d_in, const
  * receive buffer: h_peer[r] (HOST array of nranks device addresses valid in this process, 8-byte
  * aligned) at record index h_dst[b * nranks + r] + k, k = 0 .. count(b, r) - 1 in unspecified
  * order.  The caller owns the buffers and guarantees the index ranges are
- * inside them and disjoint across senders.  Synchronises `stream` (stores are complete on
- * return; visibility to other processes needs their own synchronisation).
+ * inside them and disjoint across senders.  Asynchronous on `stream`; the host arrays may be
+ * reused on return.  The owners may read the records once the stream has passed this call
+ * (e.g. an interprocess CUDA event recorded after it, waited on by the owners' streams).
  * Errors: INVAL (NULL args, a NULL peer, nranks not in 1..32, geometry beyond the wire format),
- * BAD_TRACE (sticky: access size > 16 B, shard-local word >= 2^31), CUDA. */
+ * CUDA; a record beyond the wire format (access size > 16 B, shard-local word >= 2^31) is
+ * dropped and raises sticky BAD_TRACE at the next synchronising call. */
 hirace_status hirace_dispatch_wire(hirace_ctx *ctx, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
                                    int nranks, int my_rank, void *const *h_peer, const uint64_t *h_dst,
                                    void *stream);

@@ -710,17 +710,13 @@ hirace_status hirace_dispatch_wire(hirace_ctx *c, const hirace_event *d_in, cons
     if (nb)
         HR_CUDA(c, cudaMemcpyAsync(c->d_peer_tab + nranks, h_dst, nb * nranks * sizeof(uint64_t),
                                    cudaMemcpyHostToDevice, st));
-    HR_CUDA(c, cudaMemsetAsync(c->d_wire_flag, 0, sizeof(unsigned int), st));
+    /* asynchronous: a bad record raises the context's sticky device error (BAD_TRACE at the
+     * next synchronising call), so the dispatch -> replay path never drains the stream */
     for (uint64_t b = 0; b < nb; b++)
         HR_CUDA(c, launch_dispatch_wire(d_in, h_offsets[b], h_offsets[b + 1], nranks, my_rank,
                                         reinterpret_cast<unsigned long long *const *>(c->d_peer_tab),
                                         c->d_peer_tab + nranks + b * (uint64_t)nranks, c->d_bucket_hist,
-                                        c->d_wire_off, c->d_wire_flag, st));
-    unsigned int flag = 0;
-    HR_CUDA(c, cudaMemcpyAsync(&flag, c->d_wire_flag, sizeof(flag), cudaMemcpyDeviceToHost, st));
-    HR_CUDA(c, cudaStreamSynchronize(st));
-    if (flag & hirace::ERR_BAD_TRACE)
-        return set_sticky(c, HIRACE_E_BAD_TRACE);
+                                        c->d_wire_off, c->d_err, st));
     return HIRACE_OK;
 }
 

@@ -137,13 +137,22 @@ class PeerExchange:
     """Receive buffers in peer memory for run_sharded_p2p: this rank's buffer is a
     hirace_peer_buffer_alloc allocation, the other ranks' are mapped with hirace_peer_open (CUDA
     IPC; P2P over NVLink between GPUs).  Host-side agreement (count matrices, handles, the
-    completion barrier) goes through the process group (gloo or NCCL)."""
+    barrier that orders the completion events) goes through the process group (gloo or NCCL).
+    Reusing the buffers run after run is safe: run_sharded_p2p's count pass synchronises each
+    rank's stream before the count all-gather, so every owner has finished replaying the
+    previous run before any rank dispatches into its buffer again."""
 
     def __init__(self, group, dist, device: int = 0):
+        import torch
         self.group, self.dist, self.device = group, dist, device
         self.buf = None
         self.opened = {}   # rank -> (handle, ptr)
         self.ptrs = None
+        # completion: an interprocess event per rank, recorded after its dispatch; the owners'
+        # streams wait on the peers' events (GPU-side ordering, no stream drain)
+        with torch.cuda.device(device):
+            self.done = torch.cuda.Event(interprocess=True)
+        self.peer_done = None
 
     def _gather(self, obj):
         objs = [None] * self.dist.get_world_size(self.group)
@@ -184,10 +193,21 @@ class PeerExchange:
         return ptrs
 
     def fence(self):
-        """All stores of every rank's dispatch are complete and visible before any replay."""
+        """Every rank's dispatch stores are complete and visible before any replay: each rank
+        records its interprocess event after its dispatch, a host barrier orders those records
+        before the waits, and this rank's stream waits on every peer's event."""
         import torch
-        torch.cuda.synchronize(self.device)
+        stream = torch.cuda.current_stream(self.device)
+        if self.peer_done is None:
+            handles = self._gather(self.done.ipc_handle())
+            me = self.dist.get_rank(self.group)
+            self.peer_done = [None if r == me else torch.cuda.Event.from_ipc_handle(self.device, h)
+                              for r, h in enumerate(handles)]
+        self.done.record(stream)
         self.dist.barrier(group=self.group)
+        for ev in self.peer_done:
+            if ev is not None:
+                stream.wait_event(ev)
 
     def dispatch(self, ops, events, offs, dst_local):
         ops.dispatch_wire(events, offs, self.ptrs, dst_local)
