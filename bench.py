@@ -170,7 +170,7 @@ def run_reference(args, trace, world):
            "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True, "scaling": "weak",
            "vs_baseline": None, "dtype": "u64", "data": "synthetic", "impl": "reference",
            "config": config_block(args, trace, world),
-           "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+           "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample, **host_cpu()},
            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
 
@@ -192,6 +192,20 @@ BASELINE_CFG = {
     4: "cooperative multi-phase kernel, 592 x 256, 64 grid phases, racy-B",
     5: "1.07e9 accesses over 2^32 tracked words (16 GiB tracked, 32 GiB shadow), 65536 x 256 threads, 32 batches",
 }
+
+
+def host_cpu() -> dict:
+    """The box's host CPU (report the oracle's core count, nproc and CPU model)."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count()}
 
 
 def l2_roofline(st: dict, n_acc: int, kern_ms: float, rec_bytes: int, dev: int) -> dict:
@@ -574,7 +588,8 @@ def main():
         dt = time.perf_counter() - t
         na = word_accesses(sub.events)
         cpu = {"value": na / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"events of blocks [0,{m}) of {trace.name} ({na} word accesses), one run, 1 thread"}
+               "sample": f"events of blocks [0,{m}) of {trace.name} ({na} word accesses), one run, 1 thread",
+               **host_cpu()}
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": W,
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
