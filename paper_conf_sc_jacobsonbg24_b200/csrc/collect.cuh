@@ -201,6 +201,101 @@ __device__ __forceinline__ void collect_phase(const hirace_dev_ctx &c, uint64_t 
     }
 }
 
+/* Single-load variant of collect_phase for small shadows (every warp's share of its CTA's word
+ * range is at most kRowsMax rows of 32 words): each warp reads its rows once, coalesced, keeps
+ * them in registers with their ballot masks across the grid barrier, and writes its flagged
+ * records in order after the CTA prefix — one shadow read and no block-wide scans.  Same
+ * output as collect_phase.  Returns false (nothing done) when the shadow is too large. */
+constexpr uint32_t kRowsMax = 8;
+
+template <typename R>
+__device__ __forceinline__ bool collect_phase_small(const hirace_dev_ctx &c, uint64_t nwords, hirace_race *out,
+                                                    uint64_t cap, unsigned long long *d_total, uint32_t *cta_cnt,
+                                                    unsigned int *bar, unsigned int &bar_epoch)
+{
+    const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
+    const uint64_t w0 = nwords * blockIdx.x / gridDim.x, w1 = nwords * (blockIdx.x + 1) / gridDim.x;
+    const uint64_t rows = (w1 - w0 + 31) / 32;
+    /* uniform across the grid (both paths must agree on every CTA's range): the largest CTA
+     * range, in rows of 32 words, must fit kRowsMax rows per warp */
+    const uint64_t max_rows = ((nwords + gridDim.x - 1) / gridDim.x + 31) / 32;
+    if (max_rows > (uint64_t)kRowsMax * nwarp)
+        return false;
+    __shared__ uint32_t s_wc[32];
+    __shared__ unsigned long long s_base;
+    const R *const shadow = shadow_as<R>(c);
+    const Rec<R> rec(c);
+    const uint32_t r0 = (uint32_t)(rows * wid / nwarp), r1 = (uint32_t)(rows * (wid + 1) / nwarp);
+    R v[kRowsMax];
+    uint32_t m[kRowsMax];
+    uint32_t mine = 0;
+#pragma unroll
+    for (uint32_t k = 0; k < kRowsMax; k++) {
+        const uint64_t idx = w0 + (uint64_t)(r0 + k) * 32 + lane;
+        v[k] = (r0 + k < r1 && idx < w1) ? __ldcg(shadow + idx) : (R)0;
+    }
+#pragma unroll
+    for (uint32_t k = 0; k < kRowsMax; k++) {
+        m[k] = __ballot_sync(0xffffffffu, hirace::st_of(v[k]) >= hirace::ST_RACE_W);
+        mine += __popc(m[k]);
+    }
+    if (lane == 0)
+        s_wc[wid] = mine;
+    __syncthreads();
+    uint32_t before = 0, total = 0;
+    for (uint32_t w = 0; w < nwarp; w++) {
+        const uint32_t x = s_wc[w];
+        before += w < wid ? x : 0u;
+        total += x;
+    }
+    if (threadIdx.x == 0)
+        cta_cnt[blockIdx.x] = total;
+    grid_sync(bar, gridDim.x, bar_epoch);
+    /* prefix of the CTAs before this one */
+    unsigned long long part = 0;
+    for (uint32_t k = threadIdx.x; k < blockIdx.x; k += blockDim.x)
+        part += __ldcg(&cta_cnt[k]);
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1)
+        part += __shfl_xor_sync(0xffffffffu, part, d);
+    if (threadIdx.x == 0)
+        s_base = 0;
+    __syncthreads();
+    if (lane == 0 && part)
+        atomicAdd(&s_base, part);
+    __syncthreads();
+    const unsigned long long base = s_base;
+    if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
+        *d_total = base + total;
+    if (!total)
+        return true;
+    uint64_t pos = base + before;
+    const uint64_t global_words = c.global_words;
+    const uint64_t smem_words = c.smem_words ? c.smem_words : 1;
+#pragma unroll
+    for (uint32_t k = 0; k < kRowsMax; k++) {
+        if ((m[k] >> lane) & 1u) {
+            const uint64_t at = pos + __popc(m[k] & ((1u << lane) - 1u));
+            if (at < cap) {
+                const uint64_t wi = w0 + (uint64_t)(r0 + k) * 32 + lane;
+                hirace_race rr;
+                if (wi < global_words) {
+                    rr.key = wi;
+                } else {
+                    const uint64_t sidx = wi - global_words;
+                    const uint64_t blk = sidx / smem_words;
+                    rr.key = HIRACE_SHARED_BIT | (blk << 32) | (sidx - blk * smem_words);
+                }
+                rr.cls_and_epoch = hirace::race_class(hirace::st_of(v[k])) | (rec.g(v[k]) << 8);
+                rr.detect_tid = rec.tid(v[k]);
+                out[at] = rr;
+            }
+        }
+        pos += __popc(m[k]);
+    }
+    return true;
+}
+
 /* ---- report-buffer collection ("Collect = device sort + unique(key, max
  * class); fallback = shadow scan") -------------------------------------------------------
  * Every word that reaches RACE appends a report when its CAS enters RACE or upgrades the class

@@ -326,7 +326,8 @@ __device__ __noinline__ unsigned int collect_call(const hirace_dev_ctx c, uint64
                                                   uint64_t cap, unsigned long long *d_total, uint32_t *cta_cnt,
                                                   unsigned int *bar, unsigned int epoch)
 {
-    collect_phase<R>(c, nwords, out, cap, d_total, cta_cnt, bar, epoch);
+    if (!collect_phase_small<R>(c, nwords, out, cap, d_total, cta_cnt, bar, epoch))
+        collect_phase<R>(c, nwords, out, cap, d_total, cta_cnt, bar, epoch);
     return epoch;
 }
 
