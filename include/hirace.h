@@ -232,6 +232,14 @@ hirace_status hirace_check_trace_host(hirace_ctx *ctx, const hirace_event *h_eve
 
 /* ---- results (a7) -------------------------------------------------------------------- */
 
+/* How the flagged words are gathered (same output either way): every word entering RACE or
+ * upgrading its class appends a report, so for a shadow of >= 64 MiB whose report buffer did
+ * not overflow and holds <= 16,384 reports, one CTA sorts the reported keys in shared memory and
+ * reads each word's final record ("device sort + unique"); otherwise an
+ * order-preserving compaction of the RACE records of the whole shadow runs (single-read,
+ * register-resident for small shadows).  Keys come out sorted (global words, then shared words
+ * block-major) because the shadow is laid out in key order. */
+
 /* Copies min(cap, n_total) flagged words, sorted by key, unique, to HOST memory h_out and sets
  * *n_total (call again with a bigger buffer if n_total > cap).  Synchronises `stream`.
  * Returns the sticky status (e.g. BAD_TRACE) after copying. */
