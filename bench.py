@@ -593,7 +593,7 @@ def main():
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": W,
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-        "dtype": "u64", "data": "synthetic", "config": config_block(args, trace, world),
+        "dtype": "u64" if c.rec_bytes == 8 else "u32", "data": "synthetic", "config": config_block(args, trace, world),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": load_traffic(args.config, args.variant, args.compact),
                      "kernel": "k_replay (incl. fused collect)", "kernel_ms": kern_ms, "kernel_share": kern_ms / ms_per_step,
