@@ -78,15 +78,17 @@ def test_bucket_wire_capacity_and_bad_sizes():
     c.close()
 
 
-def test_replay_wire_matches_replay_trace():
-    """Single rank: wire replay of every batch == the 16-byte replay (same race set)."""
+@pytest.mark.parametrize("compact", [False, True])
+def test_replay_wire_matches_replay_trace(compact):
+    """Single rank: wire replay of every batch == the 16-byte replay (same race set), with the
+    8-byte and the compact 4-byte record."""
     for name in ("cfg2", "multi", "cfg4"):
         t = _make(name)
         d = _to_tensor(t.events).cuda()
         a = hr.Checker.for_trace(t)
         a.replay(d, t.n)
         want = a.collect()
-        b = hr.Checker.for_trace(t)
+        b = hr.Checker.for_trace(t, compact=compact)
         offs, keys = b.find_batches(d)
         wire, counts = b.bucket_wire(d, offs, 1, 0)
         start = 0
