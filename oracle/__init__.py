@@ -7,6 +7,8 @@ two share no code.
 
   oracle_d.c  Oracle-D: the race definition, sort + per-level scan, C.
   brute.py    literal O(n^2) pairwise enumeration of C1, for tiny traces.
+  races_cluster / brute.races_cluster: the definition with a thread-block-cluster level
+              (reading R16); class CLUSTER = 4.
 
 Pins (tests/test_oracle_pins.py): brute force on random tiny traces, the paper's listings
 (closed forms, tests/golden/), configs 1/2/4 closed forms, read-only invariants.
@@ -24,8 +26,8 @@ _SRC = os.path.join(_HERE, "oracle_d.c")
 _SO = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
-WARP, BLOCK, GRID = 1, 2, 3
-CLASS_NAMES = {1: "WARP", 2: "BLOCK", 3: "GRID"}
+WARP, BLOCK, GRID, CLUSTER = 1, 2, 3, 4
+CLASS_NAMES = {1: "WARP", 2: "BLOCK", 3: "GRID", 4: "CLUSTER"}
 
 
 def build(force: bool = False) -> str:
@@ -47,6 +49,10 @@ def _load():
         lib.oracle_races_gran.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                           ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
                                           ctypes.c_int, ctypes.c_uint32]
+        lib.oracle_races_cluster.restype = ctypes.c_int64
+        lib.oracle_races_cluster.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                                             ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                             ctypes.c_uint64]
         _lib = lib
     return _lib
 
@@ -78,4 +84,29 @@ def races_of(trace, policy: int = 0):
 
 def races_dict(trace, policy: int = 0) -> dict:
     k, c, _ = races_of(trace, policy)
+    return {int(a): int(b) for a, b in zip(k, c)}
+
+
+def races_cluster(events: np.ndarray, block_threads: int, warp_size: int, cluster_blocks: int):
+    """Oracle-D with the cluster level (C1.1'-C1.6' in oracle_d.c; strict conflict rule, 4-byte
+    words).  Returns (keys u64[], cls u8[], gstar u8[]) sorted by key; cls 4 = CLUSTER."""
+    lib = _load()
+    ev = np.ascontiguousarray(events)
+    n = int(ev.shape[0])
+    cap = max(1024, n)
+    while True:
+        keys = np.empty(cap, np.uint64)
+        cls = np.empty(cap, np.uint8)
+        gs = np.empty(cap, np.uint8)
+        r = lib.oracle_races_cluster(ev.ctypes.data if n else None, n, block_threads, warp_size, cluster_blocks,
+                                     keys.ctypes.data, cls.ctypes.data, gs.ctypes.data, cap)
+        if r < 0:
+            raise RuntimeError(f"oracle_races_cluster failed ({r})")
+        if r <= cap:
+            return keys[:r], cls[:r], gs[:r]
+        cap = int(r)
+
+
+def races_cluster_dict(trace) -> dict:
+    k, c, _ = races_cluster(trace.events, trace.block_threads, trace.warp_size, trace.cluster_blocks)
     return {int(a): int(b) for a, b in zip(k, c)}

@@ -86,3 +86,86 @@ def races(events, block_threads, warp_size, policy=0, gran_log2=2):
         in_b = [p for p in in_g if p[1] == bstar]
         out[key] = (BLOCK if any(p[2] == BLOCK for p in in_b) else WARP, gstar)
     return out
+
+
+# ---------------------------------------------------------------------------------------------
+# Cluster level (reading R16): the literal pair
+# loop over C1.1'-C1.6' (see oracle_d.c).  Event encoding: addr bits 56..62 = cluster epoch c,
+# shared addr bits 48..55 = DSMEM target (0 own block, r+1 = cluster rank r).
+# ---------------------------------------------------------------------------------------------
+CLUSTER = 4
+
+
+def accesses_cluster(events, block_threads, warp_size, cluster_blocks):
+    """C1.1': (key, tid, kind, g, c, b, w, cluster, block, warp) per word."""
+    out = []
+    for e in events:
+        addr, tid, meta = int(e["addr"]), int(e["tid"]), int(e["meta"])
+        kind, size = meta & 3, 1 << ((meta >> 2) & 7)
+        w, b, g = (meta >> 5) & 511, (meta >> 14) & 1023, (meta >> 24) & 255
+        c = (addr >> 56) & 127
+        target = (addr >> 48) & 255
+        block, warp = tid // block_threads, (tid % block_threads) // warp_size
+        cl = block // cluster_blocks
+        shared = bool(addr & SHARED)
+        owner = cl * cluster_blocks + target - 1 if (shared and target) else block
+        word0 = (addr & ((1 << 48) - 1)) >> 2
+        for k in range(1 if size <= 4 else size // 4):
+            word = word0 + k
+            key = (SHARED | (owner << 32) | word) if shared else word
+            out.append(dict(key=key, tid=tid, kind=kind, g=g, c=c, b=b, w=w, cl=cl, block=block, warp=warp))
+    return out
+
+
+def concurrent_cluster(a, d):
+    """C1.2': a cluster barrier orders everything inside one cluster; __syncthreads orders a
+    block; a full-warp sync a warp."""
+    if a["tid"] == d["tid"] or a["g"] != d["g"]:
+        return False
+    if a["cl"] != d["cl"]:
+        return True
+    if a["c"] != d["c"]:
+        return False
+    if a["block"] != d["block"]:
+        return True
+    if a["b"] != d["b"]:
+        return False
+    return a["warp"] != d["warp"] or a["w"] == d["w"]
+
+
+def races_cluster(events, block_threads, warp_size, cluster_blocks):
+    """{key: (class, g*)} by enumeration of all pairs (C1.4'-C1.6'), strict conflict rule."""
+    acc = accesses_cluster(events, block_threads, warp_size, cluster_blocks)
+    pairs = {}
+    for i in range(len(acc)):
+        for j in range(i + 1, len(acc)):
+            a, d = acc[i], acc[j]
+            if a["key"] != d["key"] or not concurrent_cluster(a, d):
+                continue
+            if not conflict((0, 0, a["kind"], 0, 0, 0, a["block"]), (0, 0, d["kind"], 0, 0, 0, d["block"])):
+                continue
+            if a["cl"] != d["cl"]:
+                lvl = GRID
+            elif a["block"] != d["block"]:
+                lvl = CLUSTER
+            elif a["warp"] != d["warp"]:
+                lvl = BLOCK
+            else:
+                lvl = WARP
+            pairs.setdefault(a["key"], []).append((a["g"], a["c"], a["b"], lvl))
+    out = {}
+    for key, ps in pairs.items():
+        gstar = min(p[0] for p in ps)
+        in_g = [p for p in ps if p[0] == gstar]
+        if any(p[3] == GRID for p in in_g):
+            out[key] = (GRID, gstar)
+            continue
+        cstar = min(p[1] for p in in_g)
+        in_c = [p for p in in_g if p[1] == cstar]
+        if any(p[3] == CLUSTER for p in in_c):
+            out[key] = (CLUSTER, gstar)
+            continue
+        bstar = min(p[2] for p in in_c)
+        in_b = [p for p in in_c if p[2] == bstar]
+        out[key] = (BLOCK if any(p[3] == BLOCK for p in in_b) else WARP, gstar)
+    return out

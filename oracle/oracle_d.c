@@ -307,3 +307,259 @@ int64_t oracle_races(const oracle_event *ev, uint64_t n, uint32_t block_threads,
 {
     return oracle_races_policy(ev, n, block_threads, warp_size, out_key, out_cls, out_g, cap, 0);
 }
+
+/*
+ * ---------------------------------------------------------------------------------------------
+ * Cluster level (reading R16): thread < warp < block < CLUSTER < grid.
+ * PAPER.md L134 ("easily extended to ... deeper hierarchies"), L431, L490; the thread-block
+ * cluster is the level sm_90+/sm_100 adds between the block and the grid.
+ *
+ *   C1.1'  cluster(e) = block(e) / cluster_blocks (consecutive block ids form a cluster);
+ *          epochs g > c > b > w are nested: c = cluster barriers (barrier.cluster arrive+wait)
+ *          passed since the last g, b = __syncthreads passed since the last c (a cluster barrier
+ *          is also a rendezvous of every block of the cluster), w as before.
+ *          Event encoding (tracegen.pack_cluster_addr): addr bits 56..62 = c; for shared
+ *          accesses addr bits 48..55 = DSMEM target (0 = own block, r+1 = the block of cluster
+ *          rank r); bits 0..47 = byte offset.  Shared key = 1<<63 | target_block<<32 | word.
+ *   C1.2'  Concurrent <=> tid1 != tid2 and g1 == g2 and [cluster1 != cluster2 or (c1 == c2 and
+ *          (block1 != block2 or (b1 == b2 and (warp1 != warp2 or w1 == w2))))]
+ *   C1.3   Conflict as above (strict policy only), same_block = the ACCESSING threads' blocks.
+ *   C1.4'  level GRID (clusters differ) / CLUSTER (blocks differ) / BLOCK (warps differ) / WARP
+ *   C1.6'  class: g* = smallest racing g; GRID if a racing pair of g* is GRID-level; else c* =
+ *          smallest c with a racing pair in g*, CLUSTER if a racing pair in (g*, c*) is
+ *          CLUSTER-level; else b*, BLOCK / WARP as in C1.6 inside (g*, c*).
+ * Class codes: WARP 1, BLOCK 2, GRID 3, CLUSTER 4 (coarseness WARP < BLOCK < CLUSTER < GRID).
+ * ---------------------------------------------------------------------------------------------
+ */
+enum { CLS_CLUSTER = 4 };
+
+typedef struct {
+    uint64_t key;
+    uint32_t g, cl, c, block, b, warp, w, tid, kind;
+} caccess_t;
+
+static int cmp_caccess(const void *pa, const void *pb)
+{
+    const caccess_t *a = (const caccess_t *)pa, *b = (const caccess_t *)pb;
+#define CMP(f)                  \
+    if (a->f != b->f)           \
+        return a->f < b->f ? -1 : 1;
+    CMP(key) CMP(g) CMP(cl) CMP(c) CMP(block) CMP(b) CMP(warp) CMP(w) CMP(tid)
+#undef CMP
+    return 0;
+}
+
+/* Returns the flagged-key count (first `cap` written in key order), -1 bad argument / out of
+ * memory, -2 a C1.6' premise failed, -3 a DSMEM target outside the cluster. */
+int64_t oracle_races_cluster(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
+                             uint32_t cluster_blocks, uint64_t *out_key, uint8_t *out_cls, uint8_t *out_g,
+                             uint64_t cap)
+{
+    if (block_threads == 0 || warp_size == 0 || cluster_blocks == 0 || cluster_blocks > 255 || (n && !ev))
+        return -1;
+    const uint64_t OFF_MASK = (1ull << 48) - 1;
+    uint64_t nacc = 0;
+    for (uint64_t i = 0; i < n; i++) {
+        uint32_t sz = 1u << ((ev[i].meta >> 2) & 7);
+        nacc += sz <= 4 ? 1 : sz / 4;
+    }
+    caccess_t *acc = (caccess_t *)malloc((nacc ? nacc : 1) * sizeof(caccess_t));
+    if (!acc)
+        return -1;
+    uint64_t j = 0;
+    for (uint64_t i = 0; i < n; i++) {
+        uint32_t meta = ev[i].meta;
+        uint32_t kind = meta & 3, sz = 1u << ((meta >> 2) & 7);
+        uint32_t w = (meta >> 5) & 511, b = (meta >> 14) & 1023, g = (meta >> 24) & 255;
+        uint64_t addr = ev[i].addr;
+        uint32_t c = (uint32_t)((addr >> 56) & 127);
+        uint32_t tid = ev[i].tid;
+        uint32_t block = tid / block_threads;
+        uint32_t warp = (tid % block_threads) / warp_size;
+        uint32_t cl = block / cluster_blocks;
+        int shared = (addr & SHARED) != 0;
+        uint32_t target = block;
+        if (shared) {
+            uint32_t t = (uint32_t)((addr >> 48) & 255);
+            if (t) {
+                if (t - 1 >= cluster_blocks) {
+                    free(acc);
+                    return -3;
+                }
+                target = cl * cluster_blocks + (t - 1);
+            }
+        } else if ((addr >> 48) & 255) {
+            free(acc);
+            return -1; /* DSMEM target on a global access */
+        }
+        uint64_t word0 = (addr & OFF_MASK) >> 2;
+        uint32_t nw = sz <= 4 ? 1 : sz / 4;
+        for (uint32_t k = 0; k < nw; k++) {
+            caccess_t *a = &acc[j++];
+            uint64_t word = word0 + k;
+            a->key = shared ? (SHARED | ((uint64_t)target << 32) | (word & 0xffffffffull)) : word;
+            a->g = g;
+            a->cl = cl;
+            a->c = c;
+            a->block = block;
+            a->b = b;
+            a->warp = warp;
+            a->w = w;
+            a->tid = tid;
+            a->kind = kind;
+        }
+    }
+    qsort(acc, nacc, sizeof(caccess_t), cmp_caccess);
+
+    masks_t clusters = {0}, blocks = {0}, warps = {0}, threads = {0};
+    int64_t nflag = 0;
+    int err = 0;
+    uint64_t i = 0;
+    while (i < nacc && !err) {
+        uint64_t key = acc[i].key, kend = i;
+        while (kend < nacc && acc[kend].key == key)
+            kend++;
+        int cls = CLS_NONE;
+        uint32_t gstar = 0;
+        for (uint64_t gs = i; gs < kend && cls == CLS_NONE;) {
+            uint32_t g = acc[gs].g;
+            uint64_t ge = gs;
+            while (ge < kend && acc[ge].g == g)
+                ge++;
+            /* GRID level: groups = clusters of g */
+            clusters.n = 0;
+            int have_c = 0, cl_race_at_c = 0, have_b = 0, blk_race_at_b = 0;
+            uint32_t min_c = 0;
+            uint32_t nclusters_touching = 0;
+            for (uint64_t ks = gs; ks < ge;) {
+                uint32_t cl = acc[ks].cl;
+                uint64_t ke = ks;
+                uint8_t kmask = 0;
+                while (ke < ge && acc[ke].cl == cl)
+                    kmask |= (uint8_t)(1u << acc[ke].kind), ke++;
+                if (masks_push(&clusters, kmask))
+                    err = -1;
+                nclusters_touching++;
+                /* per cluster epoch c */
+                for (uint64_t cs = ks; cs < ke;) {
+                    uint32_t c = acc[cs].c;
+                    uint64_t ce = cs;
+                    while (ce < ke && acc[ce].c == c)
+                        ce++;
+                    /* CLUSTER level: groups = blocks of (cluster, c) */
+                    blocks.n = 0;
+                    int lower_race = 0, c_have_b = 0, c_blk_race_at_b = 0;
+                    uint32_t c_min_b = 0;
+                    for (uint64_t bs = cs; bs < ce;) {
+                        uint32_t blk = acc[bs].block;
+                        uint64_t be = bs;
+                        uint8_t bmask = 0;
+                        while (be < ce && acc[be].block == blk)
+                            bmask |= (uint8_t)(1u << acc[be].kind), be++;
+                        if (masks_push(&blocks, bmask))
+                            err = -1;
+                        for (uint64_t es = bs; es < be;) {
+                            uint32_t b = acc[es].b;
+                            uint64_t ee = es;
+                            while (ee < be && acc[ee].b == b)
+                                ee++;
+                            /* BLOCK level: groups = warps of (block, b) */
+                            warps.n = 0;
+                            int warp_race = 0;
+                            for (uint64_t ws = es; ws < ee;) {
+                                uint32_t wp = acc[ws].warp;
+                                uint64_t we = ws;
+                                uint8_t wmask = 0;
+                                while (we < ee && acc[we].warp == wp)
+                                    wmask |= (uint8_t)(1u << acc[we].kind), we++;
+                                if (masks_push(&warps, wmask))
+                                    err = -1;
+                                /* WARP level: groups = threads of (block, b, warp, w) */
+                                for (uint64_t xs = ws; xs < we;) {
+                                    uint32_t w = acc[xs].w;
+                                    uint64_t xe = xs;
+                                    while (xe < we && acc[xe].w == w)
+                                        xe++;
+                                    threads.n = 0;
+                                    for (uint64_t ts = xs; ts < xe;) {
+                                        uint32_t t = acc[ts].tid;
+                                        uint8_t tmask = 0;
+                                        while (ts < xe && acc[ts].tid == t)
+                                            tmask |= (uint8_t)(1u << acc[ts].kind), ts++;
+                                        if (masks_push(&threads, tmask))
+                                            err = -1;
+                                    }
+                                    if (distinct_conflict(threads.m, threads.n, 1, 0))
+                                        warp_race = 1;
+                                    xs = xe;
+                                }
+                                ws = we;
+                            }
+                            int block_race = distinct_conflict(warps.m, warps.n, 1, 0);
+                            if (block_race || warp_race) {
+                                lower_race = 1;
+                                if (!c_have_b || b < c_min_b) {
+                                    c_have_b = 1;
+                                    c_min_b = b;
+                                    c_blk_race_at_b = block_race;
+                                } else if (b == c_min_b && block_race) {
+                                    c_blk_race_at_b = 1;
+                                }
+                            }
+                            es = ee;
+                        }
+                        bs = be;
+                    }
+                    int cluster_race = distinct_conflict(blocks.m, blocks.n, 0, 0);
+                    if (cluster_race || lower_race) {
+                        if (!have_c || c < min_c) { /* c ascends inside a cluster; a second
+                                                       * racing cluster fails the premise below */
+                            have_c = 1;
+                            min_c = c;
+                            cl_race_at_c = cluster_race;
+                            if (!cluster_race && blocks.n >= 2)
+                                err = -2; /* only one block may touch the key in (g*, c*) */
+                            have_b = c_have_b;
+                            blk_race_at_b = c_blk_race_at_b;
+                        }
+                    }
+                    cs = ce;
+                }
+                ks = ke;
+            }
+            int grid_race = distinct_conflict(clusters.m, clusters.n, 0, 0);
+            if (grid_race) {
+                cls = CLS_GRID;
+            } else if (have_c) {
+                if (nclusters_touching >= 2)
+                    err = -2; /* C1.6' premise: only one cluster can touch the key in g* */
+                if (cl_race_at_c)
+                    cls = CLS_CLUSTER;
+                else if (have_b)
+                    cls = blk_race_at_b ? CLS_BLOCK : CLS_WARP;
+                else
+                    err = -2;
+            }
+            gstar = g;
+            gs = ge;
+        }
+        if (cls != CLS_NONE) {
+            if ((uint64_t)nflag < cap) {
+                if (out_key)
+                    out_key[nflag] = key;
+                if (out_cls)
+                    out_cls[nflag] = (uint8_t)cls;
+                if (out_g)
+                    out_g[nflag] = (uint8_t)gstar;
+            }
+            nflag++;
+        }
+        i = kend;
+    }
+    free(clusters.m);
+    free(blocks.m);
+    free(warps.m);
+    free(threads.m);
+    free(acc);
+    return err ? err : nflag;
+}
