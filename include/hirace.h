@@ -428,6 +428,20 @@ uint32_t hirace_fsm_step_compact(int policy, uint32_t old_shadow, uint32_t tid, 
                                  uint32_t w, uint32_t block_threads, uint32_t warp_size, uint32_t grid_threads,
                                  const hirace_epoch_limits *lim, int *report);
 
+/* Cluster level (reading R16): host model of the
+ * derived cluster-level FSM (hirace_device.cuh, namespace hirace::cluster).  Not yet a replay path.
+ * hirace_fsm_table_cluster writes the 16384-byte table (entry[state<<8 | kind<<6 | sync<<3 | rel]
+ * = next:6 | keep:1 | report:1) and the number of live states.  Errors: INVAL (NULL out, or the
+ * rules reaching more than 64 states).
+ * hirace_fsm_cluster_class: race class of a state code (0 = not RACE; 4 = CLUSTER).
+ * hirace_fsm_step_cluster: one step on the record state:6 | g:8 | c:7 | b:8 | w:8 | tid:27;
+ * returns ~0 for a zero geometry or an epoch / tid beyond its field. */
+hirace_status hirace_fsm_table_cluster(unsigned char out[16384], uint32_t *n_states);
+uint32_t hirace_fsm_cluster_class(uint32_t state);
+uint64_t hirace_fsm_step_cluster(uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t c, uint32_t b,
+                                 uint32_t w, uint32_t block_threads, uint32_t warp_size, uint32_t cluster_blocks,
+                                 int *report);
+
 const char *hirace_status_string(hirace_status s);
 
 /* Library version string and the compile target ("sm_100a"). */

@@ -297,6 +297,134 @@ Out rules(int s, uint32_t k, uint32_t sync, uint32_t rel)
 
 } // namespace relaxed
 
+/* ---- cluster level (reading R16) ---------------------------------
+ * thread < warp < block < cluster < grid.  Across blocks (of one cluster or of two clusters)
+ * the grid classes apply (clsG); inside a block the low classes (cls).  States:
+ *   T(KT,KB,KC,KG)  one thread in the current warp epoch; KC = its block's kinds in the cluster
+ *                   epoch, KG = its cluster's kinds in the grid epoch (grid classes)
+ *   W(c,KB,KC,KG)   >= 2 threads of one warp;   B(c,KC,KG) >= 2 warps of one block
+ *   C(c,KG)         >= 2 blocks of one cluster in the cluster epoch, all of grid class c
+ *   G(c)            >= 2 clusters in the grid epoch
+ *   RACE_W/B/G/C    class codes 1/2/3/4 (the oracle's), sticky, frozen record
+ * Rules, first match wins (record := the accessor unless "keep"); KB' = join(KB, cls k),
+ * KC' = join(KC, clsG k), KG' = join(KG, clsG k):
+ *   0 RACE: Gs keep; RACE_W & rel B & Us -> RACE_B; RACE_W/B & rel C & Us -> RACE_C;
+ *     RACE_W/B/C & rel G & !Gs -> RACE_G (upgrades report, keep); otherwise keep
+ *   1 INIT or Gs -> T(cls k, cls k, clsG k, clsG k)
+ *   2 G(c): compatG(c,k) -> keep, else RACE_G          3 rel G: compatG(KG,k) -> G(KG), else RACE_G
+ *   4 Cs -> T(cls k, cls k, clsG k, KG')
+ *   5 C(c,KG): compatG(c,k) -> C(c,KG') keep, else RACE_C
+ *   6 rel C: compatG(KC,k) -> C(KC,KG'), else RACE_C
+ *   7 Bs -> T(cls k, cls k, KC', KG')
+ *   8 B(c,KC,KG): compat(c,k) -> B(c,KC',KG') keep, else RACE_B
+ *   9 rel B: compat(KB,k) -> B(KB,KC',KG'), else RACE_B
+ *  10 Ws -> T(cls k, KB', KC', KG')
+ *  11 W(c,..): compat(c,k) -> W(c,KB',KC',KG') keep, else RACE_W
+ *  12 rel W: compat(KT,k) -> W(KT,KB',KC',KG'), else RACE_W
+ *  13 rel S: T(join(KT, cls k), KB', KC', KG') keep
+ * The state list is the set reachable from INIT, sorted by (group, fields), RACE states last. */
+namespace clus {
+
+using namespace hirace::cluster;
+enum CGroup { Q_INIT = 0, Q_T, Q_W, Q_B, Q_C, Q_G, Q_RACE };
+struct CD {
+    int grp, a, b, c, d; /* T: KT,KB,KC,KG  W: c,KB,KC,KG  B: c,-,KC,KG  C: c,-,-,KG  G: c  RACE: class */
+    bool operator==(const CD &o) const { return grp == o.grp && a == o.a && b == o.b && c == o.c && d == o.d; }
+    bool operator<(const CD &o) const
+    {
+        if (grp != o.grp) return grp < o.grp;
+        if (a != o.a) return a < o.a;
+        if (b != o.b) return b < o.b;
+        if (c != o.c) return c < o.c;
+        return d < o.d;
+    }
+};
+struct COut {
+    CD next;
+    bool keep, report;
+};
+const CD INIT{Q_INIT, 0, 0, 0, 0};
+CD T(int kt, int kb, int kc, int kg) { return {Q_T, kt, kb, kc, kg}; }
+CD Wq(int c, int kb, int kc, int kg) { return {Q_W, c, kb, kc, kg}; }
+CD Bq(int c, int kc, int kg) { return {Q_B, c, 0, kc, kg}; }
+CD Cq(int c, int kg) { return {Q_C, c, 0, 0, kg}; }
+CD Gq(int c) { return {Q_G, c, 0, 0, 0}; }
+CD RACE(int cls) { return {Q_RACE, cls, 0, 0, 0}; }
+enum { RW = 1, RB = 2, RG = 3, RC = 4 };
+
+COut rules(const CD &d, uint32_t k, uint32_t sync, uint32_t rel)
+{
+    const int ck = cls_low(k), gk = cls_grid(k);
+    if (d.grp == Q_RACE) { /* rule 0 */
+        if (sync == SYNC_GS)
+            return {d, true, false};
+        if (d.a == RW && rel == REL_B && sync == SYNC_US)
+            return {RACE(RB), true, true};
+        if ((d.a == RW || d.a == RB) && rel == REL_C && sync == SYNC_US)
+            return {RACE(RC), true, true};
+        if (d.a != RG && rel == REL_G)
+            return {RACE(RG), true, true};
+        return {d, true, false};
+    }
+    if (d.grp == Q_INIT || sync == SYNC_GS) /* rule 1 */
+        return {T(ck, ck, gk, gk), false, false};
+    if (d.grp == Q_G) /* rule 2 */
+        return compatG(d.a, k) ? COut{d, true, false} : COut{RACE(RG), false, true};
+    const int KT = d.a, KB = d.grp == Q_B ? d.a : d.b, KC = d.grp == Q_C ? d.a : d.c, KG = d.d;
+    const int KBp = join(KB, ck), KCp = join(KC, gk), KGp = join(KG, gk);
+    if (rel == REL_G) /* rule 3 */
+        return compatG(KG, k) ? COut{Gq(KG), false, false} : COut{RACE(RG), false, true};
+    if (sync == SYNC_CS) /* rule 4 */
+        return {T(ck, ck, gk, KGp), false, false};
+    if (d.grp == Q_C) /* rule 5 */
+        return compatG(d.a, k) ? COut{Cq(d.a, KGp), true, false} : COut{RACE(RC), false, true};
+    if (rel == REL_C) /* rule 6 */
+        return compatG(KC, k) ? COut{Cq(KC, KGp), false, false} : COut{RACE(RC), false, true};
+    if (sync == SYNC_BS) /* rule 7 */
+        return {T(ck, ck, KCp, KGp), false, false};
+    if (d.grp == Q_B) /* rule 8 */
+        return compat(d.a, k) ? COut{Bq(d.a, KCp, KGp), true, false} : COut{RACE(RB), false, true};
+    if (rel == REL_B) /* rule 9 */
+        return compat(KB, k) ? COut{Bq(KB, KCp, KGp), false, false} : COut{RACE(RB), false, true};
+    if (sync == SYNC_WS) /* rule 10 */
+        return {T(ck, KBp, KCp, KGp), false, false};
+    if (d.grp == Q_W) /* rule 11 */
+        return compat(d.a, k) ? COut{Wq(d.a, KBp, KCp, KGp), true, false} : COut{RACE(RW), false, true};
+    if (rel == REL_W) /* rule 12 */
+        return compat(KT, k) ? COut{Wq(KT, KBp, KCp, KGp), false, false} : COut{RACE(RW), false, true};
+    return {T(join(KT, ck), KBp, KCp, KGp), true, false}; /* rule 13 */
+}
+
+/* reachable states from INIT under every label, sorted; RACE states sort last by group */
+int states(CD *out, int cap)
+{
+    int n = 0;
+    out[n++] = INIT;
+    for (int i = 0; i < n; i++)
+        for (uint32_t k = 0; k < 4; k++)
+            for (uint32_t y = 0; y < 5; y++)
+                for (uint32_t r = 0; r < 5; r++) {
+                    const CD nx = rules(out[i], k, y, r).next;
+                    bool seen = false;
+                    for (int j = 0; j < n && !seen; j++)
+                        seen = out[j] == nx;
+                    if (!seen) {
+                        if (n == cap)
+                            return -1;
+                        out[n++] = nx;
+                    }
+                }
+    for (int i = 1; i < n; i++) /* insertion sort (INIT stays first: group 0) */
+        for (int j = i; j > 0 && out[j] < out[j - 1]; j--) {
+            CD t = out[j];
+            out[j] = out[j - 1];
+            out[j - 1] = t;
+        }
+    return n;
+}
+
+} // namespace clus
+
 } // namespace
 
 extern "C" hirace_status hirace_fsm_table_policy(int policy, unsigned char out[2048])
@@ -387,6 +515,72 @@ extern "C" uint32_t hirace_fsm_step_compact(int policy, uint32_t old_shadow, uin
     uint32_t rep = 0;
     const uint32_t n = hirace::step_c(old_shadow, tid, kind & 3u, hirace::c_epochs(L, g, b, w), raw[policy] + 2048, L,
                                       G, &rep);
+    if (report)
+        *report = (int)rep;
+    return n;
+}
+
+/* Cluster-level table (hirace::cluster layout): 64 states x 256 labels. */
+extern "C" hirace_status hirace_fsm_table_cluster(unsigned char out[16384], uint32_t *n_states)
+{
+    using namespace clus;
+    if (!out)
+        return HIRACE_E_INVAL;
+    CD st[64];
+    const int n = states(st, 64);
+    if (n < 0)
+        return HIRACE_E_INVAL; /* more than 64 states: a rule bug */
+    memset(out, 0, 16384);
+    for (int s = 0; s < 64; s++)
+        for (uint32_t lab = 0; lab < 256; lab++) {
+            const uint32_t k = lab >> 6, y = (lab >> 3) & 7u, r = lab & 7u;
+            const uint32_t idx = ((uint32_t)s << 8) | lab;
+            if (s >= n || y > 4 || r > 4) {
+                out[idx] = (unsigned char)(s | E_KEEP); /* unused codes */
+                continue;
+            }
+            const COut o = rules(st[s], k, y, r);
+            int nx = -1;
+            for (int j = 0; j < n; j++)
+                if (st[j] == o.next)
+                    nx = j;
+            if (nx < 0)
+                return HIRACE_E_INVAL;
+            out[idx] = (unsigned char)(nx | (o.keep ? E_KEEP : 0) | (o.report ? E_REPORT : 0));
+        }
+    if (n_states)
+        *n_states = (uint32_t)n;
+    return HIRACE_OK;
+}
+
+/* Race class of a cluster-table state code (0 if not RACE): WARP 1, BLOCK 2, GRID 3, CLUSTER 4. */
+extern "C" uint32_t hirace_fsm_cluster_class(uint32_t state)
+{
+    using namespace clus;
+    CD st[64];
+    const int n = states(st, 64);
+    if (n < 0 || state >= (uint32_t)n || st[state].grp != Q_RACE)
+        return 0;
+    return (uint32_t)st[state].a;
+}
+
+extern "C" uint64_t hirace_fsm_step_cluster(uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t c,
+                                            uint32_t b, uint32_t w, uint32_t block_threads, uint32_t warp_size,
+                                            uint32_t cluster_blocks, int *report)
+{
+    static unsigned char table[16384];
+    static bool built = false;
+    if (!built) {
+        hirace_fsm_table_cluster(table, nullptr);
+        built = true;
+    }
+    if (!block_threads || !warp_size || !cluster_blocks || g > hirace::cluster::MAX_G ||
+        c > hirace::cluster::MAX_C || b > hirace::cluster::MAX_B || w > hirace::cluster::MAX_W ||
+        tid > hirace::cluster::MAX_TID)
+        return ~0ull;
+    uint32_t rep = 0;
+    const uint64_t n = hirace::cluster::step(old_shadow, tid, kind & 3u, g, c, b, w, table, block_threads, warp_size,
+                                             cluster_blocks, &rep);
     if (report)
         *report = (int)rep;
     return n;

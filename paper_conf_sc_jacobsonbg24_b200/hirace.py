@@ -34,7 +34,8 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_bucket_events", "hirace_bucket_wire", "hirace_replay_wire", "hirace_count_wire",
            "hirace_dispatch_wire", "hirace_peer_buffer_alloc", "hirace_peer_buffer_free", "hirace_peer_open",
            "hirace_peer_close", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_set_policy", "hirace_set_filter",
-           "hirace_fsm_table", "hirace_fsm_table_policy", "hirace_fsm_step", "hirace_fsm_step_policy", "hirace_fsm_step_compact", "hirace_status_string",
+           "hirace_fsm_table", "hirace_fsm_table_policy", "hirace_fsm_step", "hirace_fsm_step_policy", "hirace_fsm_step_compact",
+           "hirace_fsm_table_cluster", "hirace_fsm_cluster_class", "hirace_fsm_step_cluster", "hirace_status_string",
            "hirace_version")
 
 
@@ -121,6 +122,9 @@ def load():
         "hirace_fsm_step_policy": (U64, [I32, U64, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
         "hirace_fsm_step_compact": (U32, [I32, U32, U32, U32, U32, U32, U32, U32, U32, U32,
                                           ctypes.POINTER(EpochLimits), ctypes.POINTER(I32)]),
+        "hirace_fsm_table_cluster": (I32, [P, ctypes.POINTER(U32)]),
+        "hirace_fsm_cluster_class": (U32, [U32]),
+        "hirace_fsm_step_cluster": (U64, [U64, U32, U32, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
         "hirace_status_string": (ctypes.c_char_p, [I32]),
         "hirace_version": (ctypes.c_char_p, []),
     }
@@ -163,6 +167,29 @@ def fsm_step_compact(old: int, tid: int, kind: int, g: int, b: int, w: int, bloc
     lim = EpochLimits(*limits)
     n = load().hirace_fsm_step_compact(policy, old, tid, kind, g, b, w, block_threads, warp_size, grid_threads,
                                        ctypes.byref(lim), ctypes.byref(rep))
+    return int(n), int(rep.value)
+
+
+def fsm_table_cluster():
+    """(16384-byte cluster-level table, number of live states) (hirace_fsm_table_cluster)."""
+    t = np.zeros(16384, np.uint8)
+    n = ctypes.c_uint32(0)
+    _check(load().hirace_fsm_table_cluster(t.ctypes.data, ctypes.byref(n)), "hirace_fsm_table_cluster")
+    return t, int(n.value)
+
+
+def fsm_cluster_class(state: int) -> int:
+    return int(load().hirace_fsm_cluster_class(state))
+
+
+def fsm_step_cluster(old: int, tid: int, kind: int, g: int, c: int, b: int, w: int, block_threads: int,
+                     warp_size: int, cluster_blocks: int):
+    """One cluster-level FSM step on the host (include/hirace.h hirace_fsm_step_cluster)."""
+    rep = ctypes.c_int(0)
+    n = load().hirace_fsm_step_cluster(old, tid, kind, g, c, b, w, block_threads, warp_size, cluster_blocks,
+                                       ctypes.byref(rep))
+    if n == (1 << 64) - 1:
+        raise HiraceError(-1, "hirace_fsm_step_cluster")
     return int(n), int(rep.value)
 
 
