@@ -442,6 +442,40 @@ uint64_t hirace_fsm_step_cluster(uint64_t old_shadow, uint32_t tid, uint32_t kin
                                  uint32_t w, uint32_t block_threads, uint32_t warp_size, uint32_t cluster_blocks,
                                  int *report);
 
+/* ---- cluster-level replay (reading R16) ----------------------------
+ * A context whose hierarchy has a thread-block-cluster level between the block and the grid:
+ * blocks [k*cluster_blocks, (k+1)*cluster_blocks) form cluster k (cluster_blocks must divide
+ * grid_blocks, <= 255; granularity_log2 must be 2; grid_blocks*block_threads <= 2^27).
+ * Events are hirace_event with two extra address fields:
+ *   addr bits 56..62  c: cluster barriers (barrier.cluster arrive+wait) passed since the last g;
+ *                     __syncthreads counts b restart at each c;
+ *   addr bits 48..55  shared accesses only: DSMEM target, 0 = the accessing block's own window,
+ *                     r+1 = the window of the block with cluster rank r;
+ *   addr bits 0..47   byte offset (global from the tracked base, shared in the target window).
+ * Records: 8 bytes, state:6 | g:8 | c:7 | b:8 | w:8 | tid:27 (so b, w <= 255), the derived cluster
+ * FSM (hirace_fsm_table_cluster).  Race classes add HIRACE_RACE_CLUSTER = 4.
+ *
+ * hirace_cluster_alloc   context + shadow (all INIT) on cfg->device; caller frees with
+ *                        hirace_cluster_free.  Errors: INVAL (geometry as above), NOMEM, CUDA.
+ * hirace_cluster_reset   shadow := INIT, errors and stats := 0, stream-ordered.
+ * hirace_cluster_replay  d_events (device, n < 2^32) sorted by (g, c, b, w); asynchronous on
+ *                        `stream`; one cooperative launch.  Events that are not batch-sorted or
+ *                        out of range (tid, address, DSMEM target outside the cluster, b or w
+ *                        > 255) are skipped and make the next collect return BAD_TRACE (sticky
+ *                        until reset).
+ * hirace_cluster_collect synchronises the device, writes min(cap, n_total) flagged words in key
+ *                        order (hirace_race; class 1 WARP, 2 BLOCK, 3 GRID, 4 CLUSTER) to
+ *                        host memory and sets *n_total.
+ * hirace_cluster_get_stats  checked word accesses and CAS retries since the last reset. */
+typedef struct hirace_cluster_ctx hirace_cluster_ctx;
+#define HIRACE_RACE_CLUSTER 4
+hirace_status hirace_cluster_alloc(const hirace_config *cfg, uint32_t cluster_blocks, hirace_cluster_ctx **out);
+hirace_status hirace_cluster_free(hirace_cluster_ctx *ctx);
+hirace_status hirace_cluster_reset(hirace_cluster_ctx *ctx, void *stream);
+hirace_status hirace_cluster_replay(hirace_cluster_ctx *ctx, const hirace_event *d_events, uint64_t n, void *stream);
+hirace_status hirace_cluster_collect(hirace_cluster_ctx *ctx, hirace_race *h_out, uint64_t cap, uint64_t *n_total);
+hirace_status hirace_cluster_get_stats(hirace_cluster_ctx *ctx, uint64_t *checked, uint64_t *cas_retries);
+
 const char *hirace_status_string(hirace_status s);
 
 /* Library version string and the compile target ("sm_100a"). */

@@ -1,0 +1,378 @@
+/*
+ * cluster.cu — replay with a thread-block-cluster level (DESIGN.md reading
+ * R16; "easily extended to ... deeper hierarchies", L431).
+ *
+ * The hierarchy is thread < warp < block < cluster (cluster_blocks consecutive blocks) < grid.
+ * Events carry the cluster epoch c in addr bits 56..62 and, for shared accesses, a DSMEM target
+ * in addr bits 48..55 (0 = own block, r+1 = cluster rank r); see include/hirace.h.  Records are
+ * the 8-byte cluster layout state:6 | g:8 | c:7 | b:8 | w:8 | tid:27 and the transition is the
+ * derived 34-state table (fsm_table.cpp clus::rules) through hirace::cluster::step — the same
+ * inline function the CPU bisimulation test runs.
+ *
+ * k_cluster_replay is one persistent cooperative kernel: every thread finds the end of the
+ * current (g,c,b,w) batch by binary search over the batch-sorted events, the grid covers the
+ * batch in a grid-stride loop (one event per thread: Algorithm 1's load / step / CAS loop,
+ * PAPER.md L249-279, with no store when the record is unchanged), and a grid barrier separates batches (all events of a
+ * batch are pairwise concurrent or program-ordered in one thread: PAPER.md L177).
+ * Collection selects RACE records in shadow order (cub::DeviceSelect) and expands them to
+ * hirace_race rows.
+ */
+#include <cooperative_groups.h>
+#include <cub/device/device_select.cuh>
+#include <thrust/iterator/counting_iterator.h>
+
+#include <stdlib.h>
+#include <string.h>
+
+#include "hirace.h"
+#include "hirace_device.cuh"
+
+namespace cg = cooperative_groups;
+using namespace hirace::cluster;
+
+struct hirace_cluster_ctx {
+    hirace_config cfg;
+    uint32_t cluster_blocks;
+    uint64_t global_words, smem_words, shadow_words;
+    unsigned long long *shadow;
+    unsigned char *table;       /* 16 KB transition table            */
+    unsigned char *race_class;  /* 64 entries: state -> class (0..4) */
+    unsigned int *err;          /* sticky device error flags          */
+    unsigned long long *stats;  /* [0] checked word accesses, [1] CAS retries */
+    int grid;
+    int sm_count;
+    hirace_status sticky;
+};
+
+namespace {
+
+enum : unsigned int { ERR_BAD_TRACE = 1u, ERR_RANGE = 2u };
+constexpr int kThreads = 256;
+
+/* (g, c, b, w) in lexicographic order: g:8 | c:7 | b:10 | w:9 */
+__device__ __forceinline__ uint64_t batch_key(const hirace_event &e)
+{
+    const uint64_t c = (e.addr >> 56) & 127u;
+    return ((uint64_t)(e.meta >> 24) << 26) | (c << 19) | ((e.meta >> 5) & ((1u << 19) - 1u));
+}
+
+__device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long *p)
+{
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+struct Geo {
+    uint32_t block_threads, warp_size, cluster_blocks, grid_blocks;
+    uint64_t global_words, smem_words;
+};
+
+__device__ void check_event(const hirace_event e, unsigned long long *shadow, const unsigned char *table,
+                            const Geo &G, unsigned int *err, unsigned long long &checked,
+                            unsigned long long &retries)
+{
+    const uint32_t meta = e.meta, tid = e.tid;
+    const uint32_t kind = meta & 3u, size = 1u << ((meta >> 2) & 7u);
+    const uint32_t w = (meta >> 5) & 511u, b = (meta >> 14) & 1023u, g = meta >> 24;
+    const uint32_t c = (uint32_t)(e.addr >> 56) & 127u;
+    const uint32_t tgt = (uint32_t)(e.addr >> 48) & 255u;
+    const bool shared = (e.addr >> 63) != 0;
+    const uint64_t off = e.addr & ((1ull << 48) - 1);
+    const uint32_t block = tid / G.block_threads;
+    if (b > MAX_B || w > MAX_W || tid > MAX_TID || block >= G.grid_blocks || size > 16u ||
+        (!shared && tgt != 0) || (tgt != 0 && tgt - 1u >= G.cluster_blocks)) {
+        atomicOr(err, ERR_RANGE);
+        return;
+    }
+    const uint32_t owner = tgt ? (block / G.cluster_blocks) * G.cluster_blocks + (tgt - 1u) : block;
+    const uint64_t word0 = off >> 2;
+    const uint32_t nw = size <= 4u ? 1u : size >> 2;
+    const uint64_t limit = shared ? G.smem_words : G.global_words;
+    if (owner >= G.grid_blocks || word0 + nw > limit) {
+        atomicOr(err, ERR_RANGE);
+        return;
+    }
+    for (uint32_t k = 0; k < nw; k++) {
+        const uint64_t idx = shared ? G.global_words + (uint64_t)owner * G.smem_words + word0 + k : word0 + k;
+        unsigned long long *p = shadow + idx;
+        unsigned long long o = ld_relaxed(p);
+        for (;;) {
+            uint32_t rep;
+            const unsigned long long nv =
+                step(o, tid, kind, g, c, b, w, table, G.block_threads, G.warp_size, G.cluster_blocks, &rep);
+            if (nv == o)
+                break; /* unchanged record: linearised at the coherent load */
+            const unsigned long long prev = atomicCAS(p, o, nv);
+            if (prev == o)
+                break;
+            o = prev;
+            retries++;
+        }
+        checked++;
+    }
+}
+
+__global__ void __launch_bounds__(kThreads) k_cluster_replay(const hirace_event *__restrict__ ev, uint32_t n,
+                                                             unsigned long long *shadow, const unsigned char *gtable,
+                                                             Geo G, unsigned int *err, unsigned long long *stats)
+{
+    __shared__ unsigned char table[TABLE_BYTES];
+    for (uint32_t i = threadIdx.x; i < TABLE_BYTES / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(table)[i] = reinterpret_cast<const uint4 *>(gtable)[i];
+    __syncthreads();
+    cg::grid_group grid = cg::this_grid();
+    const uint64_t gsize = (uint64_t)gridDim.x * blockDim.x;
+    const uint64_t gtid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    unsigned long long checked = 0, retries = 0;
+    uint32_t start = 0;
+    while (start < n) {
+        const uint64_t key0 = batch_key(ev[start]);
+        /* end = first index > start whose batch key differs (upper bound; sorted input) */
+        uint32_t lo = start + 1, hi = n;
+        while (lo < hi) {
+            const uint32_t mid = lo + (hi - lo) / 2;
+            if (batch_key(ev[mid]) <= key0)
+                lo = mid + 1;
+            else
+                hi = mid;
+        }
+        const uint32_t end = lo;
+        /* grid-stride over the batch: consecutive warps take consecutive 32-event chunks.
+         * Contiguous per-warp or per-CTA shares (the three-level replay's layout) were measured
+         * slower on the halo workloads (profiles/r1_cluster_ab.txt). */
+        for (uint64_t i = start + gtid; i < end; i += gsize) {
+            const hirace_event e = ev[i];
+            if (batch_key(e) != key0) {
+                atomicOr(err, ERR_BAD_TRACE); /* not batch-sorted */
+                continue;
+            }
+            check_event(e, shadow, table, G, err, checked, retries);
+        }
+        grid.sync();
+        start = end;
+    }
+    if (checked)
+        atomicAdd(&stats[0], checked);
+    if (retries)
+        atomicAdd(&stats[1], retries);
+}
+
+struct IsRace {
+    const unsigned long long *shadow;
+    const unsigned char *cls;
+    __device__ bool operator()(uint64_t i) const { return cls[shadow[i] & 63u] != 0; }
+};
+
+__global__ void k_cluster_rows(const uint64_t *__restrict__ sel, uint64_t n, const unsigned long long *shadow,
+                               const unsigned char *cls, uint64_t global_words, uint64_t smem_words,
+                               hirace_race *out)
+{
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n)
+        return;
+    const uint64_t idx = sel[i];
+    const unsigned long long r = shadow[idx];
+    uint64_t key = idx;
+    if (idx >= global_words) {
+        const uint64_t s = idx - global_words;
+        key = HIRACE_SHARED_BIT | ((s / smem_words) << 32) | (s % smem_words);
+    }
+    out[i].key = key;
+    out[i].cls_and_epoch = (uint32_t)cls[r & 63u] | (uint32_t)((r >> SH_G) & 255u) << 8;
+    out[i].detect_tid = (uint32_t)(r >> SH_TID);
+}
+
+__global__ void k_cluster_fill(unsigned long long *p, uint64_t n)
+{
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        p[i] = 0ull;
+}
+
+hirace_status cuda_status(cudaError_t e) { return e == cudaSuccess ? HIRACE_OK : HIRACE_E_CUDA; }
+
+hirace_status sync_errors(hirace_cluster_ctx *ctx)
+{
+    unsigned int h = 0;
+    if (cudaMemcpy(&h, ctx->err, sizeof(h), cudaMemcpyDeviceToHost) != cudaSuccess)
+        return HIRACE_E_CUDA;
+    if (h && ctx->sticky == HIRACE_OK)
+        ctx->sticky = HIRACE_E_BAD_TRACE;
+    return ctx->sticky;
+}
+
+} // namespace
+
+extern "C" {
+
+hirace_status hirace_cluster_alloc(const hirace_config *cfg, uint32_t cluster_blocks, hirace_cluster_ctx **out)
+{
+    if (!cfg || !out || !cfg->grid_blocks || !cfg->block_threads || !cfg->warp_size || !cluster_blocks ||
+        cluster_blocks > 255 || cfg->grid_blocks % cluster_blocks != 0 || cfg->granularity_log2 != 2 ||
+        (uint64_t)cfg->grid_blocks * cfg->block_threads > (uint64_t)MAX_TID + 1)
+        return HIRACE_E_INVAL;
+    *out = nullptr;
+    if (cudaSetDevice(cfg->device) != cudaSuccess)
+        return HIRACE_E_CUDA;
+    hirace_cluster_ctx *c = (hirace_cluster_ctx *)calloc(1, sizeof(hirace_cluster_ctx));
+    if (!c)
+        return HIRACE_E_NOMEM;
+    c->cfg = *cfg;
+    c->cluster_blocks = cluster_blocks;
+    c->global_words = (cfg->global_bytes + 3) / 4;
+    c->smem_words = (cfg->smem_bytes_per_block + 3u) / 4u;
+    c->shadow_words = c->global_words + (uint64_t)cfg->grid_blocks * c->smem_words;
+    unsigned char table[TABLE_BYTES], cls[64] = {0};
+    uint32_t nst = 0;
+    if (hirace_fsm_table_cluster(table, &nst) != HIRACE_OK) {
+        free(c);
+        return HIRACE_E_INVAL;
+    }
+    for (uint32_t s = 0; s < nst; s++)
+        cls[s] = (unsigned char)hirace_fsm_cluster_class(s);
+    cudaError_t e = cudaMalloc(&c->shadow, (c->shadow_words ? c->shadow_words : 1) * 8);
+    if (e == cudaSuccess)
+        e = cudaMalloc(&c->table, TABLE_BYTES);
+    if (e == cudaSuccess)
+        e = cudaMalloc(&c->race_class, 64);
+    if (e == cudaSuccess)
+        e = cudaMalloc(&c->err, sizeof(unsigned int));
+    if (e == cudaSuccess)
+        e = cudaMalloc(&c->stats, 2 * sizeof(unsigned long long));
+    if (e == cudaSuccess)
+        e = cudaMemcpy(c->table, table, TABLE_BYTES, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess)
+        e = cudaMemcpy(c->race_class, cls, 64, cudaMemcpyHostToDevice);
+    int per_sm = 0;
+    if (e == cudaSuccess)
+        e = cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, cfg->device);
+    if (e == cudaSuccess)
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_cluster_replay, kThreads, 0);
+    if (e != cudaSuccess || per_sm < 1) {
+        hirace_cluster_free(c);
+        return e == cudaErrorMemoryAllocation ? HIRACE_E_NOMEM : HIRACE_E_CUDA;
+    }
+    c->grid = c->sm_count * (per_sm < 4 ? per_sm : 4);
+    hirace_status st = hirace_cluster_reset(c, nullptr);
+    if (st == HIRACE_OK)
+        st = cuda_status(cudaDeviceSynchronize());
+    if (st != HIRACE_OK) {
+        hirace_cluster_free(c);
+        return st;
+    }
+    *out = c;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_cluster_free(hirace_cluster_ctx *c)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    cudaFree(c->shadow);
+    cudaFree(c->table);
+    cudaFree(c->race_class);
+    cudaFree(c->err);
+    cudaFree(c->stats);
+    free(c);
+    return HIRACE_OK;
+}
+
+hirace_status hirace_cluster_reset(hirace_cluster_ctx *c, void *stream)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    cudaStream_t st = (cudaStream_t)stream;
+    k_cluster_fill<<<c->sm_count * 4, 256, 0, st>>>(c->shadow, c->shadow_words);
+    cudaError_t e = cudaGetLastError();
+    if (e == cudaSuccess)
+        e = cudaMemsetAsync(c->err, 0, sizeof(unsigned int), st);
+    if (e == cudaSuccess)
+        e = cudaMemsetAsync(c->stats, 0, 2 * sizeof(unsigned long long), st);
+    c->sticky = HIRACE_OK;
+    return cuda_status(e);
+}
+
+hirace_status hirace_cluster_replay(hirace_cluster_ctx *c, const hirace_event *d_events, uint64_t n, void *stream)
+{
+    if (!c || (n && !d_events) || n >= (1ull << 32))
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    if (!n)
+        return HIRACE_OK;
+    Geo G{c->cfg.block_threads, c->cfg.warp_size, c->cluster_blocks, c->cfg.grid_blocks, c->global_words,
+          c->smem_words};
+    uint32_t nn = (uint32_t)n;
+    const hirace_event *ev = d_events;
+    unsigned long long *shadow = c->shadow;
+    const unsigned char *table = c->table;
+    void *args[] = {(void *)&ev, (void *)&nn, (void *)&shadow, (void *)&table, (void *)&G, (void *)&c->err,
+                    (void *)&c->stats};
+    return cuda_status(cudaLaunchCooperativeKernel((const void *)k_cluster_replay, dim3(c->grid), dim3(kThreads),
+                                                   args, 0, (cudaStream_t)stream));
+}
+
+hirace_status hirace_cluster_collect(hirace_cluster_ctx *c, hirace_race *h_out, uint64_t cap, uint64_t *n_total)
+{
+    if (!c || !n_total || (cap && !h_out))
+        return HIRACE_E_INVAL;
+    if (cudaDeviceSynchronize() != cudaSuccess)
+        return HIRACE_E_CUDA;
+    hirace_status st = sync_errors(c);
+    if (st != HIRACE_OK)
+        return st;
+    uint64_t *sel = nullptr, *d_num = nullptr;
+    void *tmp = nullptr;
+    size_t tmp_bytes = 0;
+    hirace_race *d_rows = nullptr;
+    IsRace pred{c->shadow, c->race_class};
+    auto first = thrust::make_counting_iterator<uint64_t>(0);
+    const int64_t nw = (int64_t)c->shadow_words;
+    cudaError_t e = cudaMalloc(&sel, (nw ? nw : 1) * sizeof(uint64_t));
+    if (e == cudaSuccess)
+        e = cudaMalloc(&d_num, sizeof(uint64_t));
+    if (e == cudaSuccess)
+        e = cub::DeviceSelect::If(nullptr, tmp_bytes, first, sel, d_num, nw, pred);
+    if (e == cudaSuccess)
+        e = cudaMalloc(&tmp, tmp_bytes ? tmp_bytes : 1);
+    if (e == cudaSuccess)
+        e = cub::DeviceSelect::If(tmp, tmp_bytes, first, sel, d_num, nw, pred);
+    uint64_t total = 0;
+    if (e == cudaSuccess)
+        e = cudaMemcpy(&total, d_num, sizeof(total), cudaMemcpyDeviceToHost);
+    const uint64_t m = total < cap ? total : cap;
+    if (e == cudaSuccess && m) {
+        e = cudaMalloc(&d_rows, m * sizeof(hirace_race));
+        if (e == cudaSuccess) {
+            k_cluster_rows<<<(unsigned)((m + 255) / 256), 256>>>(sel, m, c->shadow, c->race_class, c->global_words,
+                                                                 c->smem_words ? c->smem_words : 1, d_rows);
+            e = cudaGetLastError();
+        }
+        if (e == cudaSuccess)
+            e = cudaMemcpy(h_out, d_rows, m * sizeof(hirace_race), cudaMemcpyDeviceToHost);
+    }
+    cudaFree(d_rows);
+    cudaFree(tmp);
+    cudaFree(d_num);
+    cudaFree(sel);
+    if (e != cudaSuccess)
+        return HIRACE_E_CUDA;
+    *n_total = total;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_cluster_get_stats(hirace_cluster_ctx *c, uint64_t *checked, uint64_t *cas_retries)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    unsigned long long h[2] = {0, 0};
+    if (cudaMemcpy(h, c->stats, sizeof(h), cudaMemcpyDeviceToHost) != cudaSuccess)
+        return HIRACE_E_CUDA;
+    if (checked)
+        *checked = h[0];
+    if (cas_retries)
+        *cas_retries = h[1];
+    return HIRACE_OK;
+}
+
+} /* extern "C" */

@@ -35,7 +35,9 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_dispatch_wire", "hirace_peer_buffer_alloc", "hirace_peer_buffer_free", "hirace_peer_open",
            "hirace_peer_close", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_set_policy", "hirace_set_filter",
            "hirace_fsm_table", "hirace_fsm_table_policy", "hirace_fsm_step", "hirace_fsm_step_policy", "hirace_fsm_step_compact",
-           "hirace_fsm_table_cluster", "hirace_fsm_cluster_class", "hirace_fsm_step_cluster", "hirace_status_string",
+           "hirace_fsm_table_cluster", "hirace_fsm_cluster_class", "hirace_fsm_step_cluster",
+           "hirace_cluster_alloc", "hirace_cluster_free", "hirace_cluster_reset", "hirace_cluster_replay",
+           "hirace_cluster_collect", "hirace_cluster_get_stats", "hirace_status_string",
            "hirace_version")
 
 
@@ -125,6 +127,12 @@ def load():
         "hirace_fsm_table_cluster": (I32, [P, ctypes.POINTER(U32)]),
         "hirace_fsm_cluster_class": (U32, [U32]),
         "hirace_fsm_step_cluster": (U64, [U64, U32, U32, U32, U32, U32, U32, U32, U32, U32, ctypes.POINTER(I32)]),
+        "hirace_cluster_alloc": (I32, [ctypes.POINTER(Config), U32, ctypes.POINTER(ctypes.c_void_p)]),
+        "hirace_cluster_free": (I32, [P]),
+        "hirace_cluster_reset": (I32, [P, P]),
+        "hirace_cluster_replay": (I32, [P, P, U64, P]),
+        "hirace_cluster_collect": (I32, [P, P, U64, ctypes.POINTER(U64)]),
+        "hirace_cluster_get_stats": (I32, [P, ctypes.POINTER(U64), ctypes.POINTER(U64)]),
         "hirace_status_string": (ctypes.c_char_p, [I32]),
         "hirace_version": (ctypes.c_char_p, []),
     }
@@ -496,6 +504,62 @@ def peer_open(handle: bytes, device: int = 0) -> int:
 
 def peer_close(ptr: int):
     _check(load().hirace_peer_close(ctypes.c_void_p(ptr)), "hirace_peer_close")
+
+
+class ClusterChecker:
+    """One hirace_cluster_ctx (include/hirace.h, cluster-level replay): the
+    hierarchy thread < warp < block < cluster < grid, events with the cluster epoch and DSMEM
+    target in their address bits (tracegen.pack_cluster_addr)."""
+
+    def __init__(self, grid_blocks: int, block_threads: int, cluster_blocks: int, warp_size: int = 32,
+                 global_words: int = 0, smem_words: int = 0, device: int = 0):
+        self.lib = load()
+        cfg = Config(grid_blocks, block_threads, warp_size, 4 * smem_words, 4 * global_words, 2, device, 0)
+        h = ctypes.c_void_p()
+        _check(self.lib.hirace_cluster_alloc(ctypes.byref(cfg), cluster_blocks, ctypes.byref(h)),
+               "hirace_cluster_alloc")
+        self.h = h
+        self.device = device
+
+    @classmethod
+    def for_trace(cls, trace, device: int = 0):
+        return cls(trace.grid_blocks, trace.block_threads, trace.cluster_blocks, trace.warp_size,
+                   trace.global_words, trace.smem_words, device)
+
+    def close(self):
+        if getattr(self, "h", None):
+            self.lib.hirace_cluster_free(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def reset(self, stream=None):
+        _check(self.lib.hirace_cluster_reset(self.h, _stream_handle(stream)), "hirace_cluster_reset")
+
+    def replay(self, events_dev, n: int | None = None, stream=None):
+        if n is None:
+            n = events_dev.numel() * events_dev.element_size() // 16
+        _check(self.lib.hirace_cluster_replay(self.h, ctypes.c_void_p(events_dev.data_ptr()), n,
+                                              _stream_handle(stream)), "hirace_cluster_replay")
+
+    def collect(self, cap: int = 1 << 16) -> np.ndarray:
+        total = ctypes.c_uint64(0)
+        while True:
+            out = np.empty(max(cap, 1), RACE_DTYPE)
+            _check(self.lib.hirace_cluster_collect(self.h, out.ctypes.data, cap, ctypes.byref(total)),
+                   "hirace_cluster_collect")
+            if total.value <= cap:
+                return out[: total.value]
+            cap = int(total.value)
+
+    def stats(self):
+        a, b = ctypes.c_uint64(0), ctypes.c_uint64(0)
+        _check(self.lib.hirace_cluster_get_stats(self.h, ctypes.byref(a), ctypes.byref(b)), "hirace_cluster_get_stats")
+        return int(a.value), int(b.value)
 
 
 def races_to_dict(races: np.ndarray) -> dict:
