@@ -9,9 +9,10 @@
  * derived 34-state table (fsm_table.cpp clus::rules) through hirace::cluster::step — the same
  * inline function the CPU bisimulation test runs.
  *
- * k_cluster_replay is one persistent cooperative kernel: every thread finds the end of the
- * current (g,c,b,w) batch by binary search over the batch-sorted events, the grid covers the
- * batch in a grid-stride loop (one event per thread: Algorithm 1's load / step / CAS loop,
+ * k_cluster_replay is one persistent cooperative kernel: every warp finds the end of the
+ * current (g,c,b,w) batch by a 32-ary search over the batch-sorted events, the grid covers the
+ * batch in a grid-stride loop (kU = 4 events per thread per iteration, loads issued together;
+ * Algorithm 1's load / step / CAS loop per event,
  * PAPER.md L249-279, with no store when the record is unchanged), and a grid barrier separates batches (all events of a
  * batch are pairwise concurrent or program-ordered in one thread: PAPER.md L177).
  * Collection selects RACE records in shadow order (cub::DeviceSelect) and expands them to
@@ -66,54 +67,73 @@ __device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long lon
 struct Geo {
     uint32_t block_threads, warp_size, cluster_blocks, grid_blocks;
     uint64_t global_words, smem_words;
+    uint32_t bt_log2, ws_log2, cb_log2; /* valid when all three sizes are powers of two (P2) */
 };
 
-__device__ void check_event(const hirace_event e, unsigned long long *shadow, const unsigned char *table,
-                            const Geo &G, unsigned int *err, unsigned long long &checked,
-                            unsigned long long &retries)
+/* Decode one event: range checks, DSMEM owner, first shadow index and word count.  Returns
+ * false (and sets ERR_RANGE) for an out-of-range event. */
+template <bool P2>
+__device__ __forceinline__ bool decode_event(const hirace_event &e, const Geo &G, unsigned int *err, uint64_t &idx0,
+                                             uint32_t &nw)
 {
     const uint32_t meta = e.meta, tid = e.tid;
-    const uint32_t kind = meta & 3u, size = 1u << ((meta >> 2) & 7u);
-    const uint32_t w = (meta >> 5) & 511u, b = (meta >> 14) & 1023u, g = meta >> 24;
-    const uint32_t c = (uint32_t)(e.addr >> 56) & 127u;
+    const uint32_t size = 1u << ((meta >> 2) & 7u);
+    const uint32_t w = (meta >> 5) & 511u, b = (meta >> 14) & 1023u;
     const uint32_t tgt = (uint32_t)(e.addr >> 48) & 255u;
     const bool shared = (e.addr >> 63) != 0;
     const uint64_t off = e.addr & ((1ull << 48) - 1);
-    const uint32_t block = tid / G.block_threads;
+    const uint32_t block = P2 ? tid >> G.bt_log2 : tid / G.block_threads;
     if (b > MAX_B || w > MAX_W || tid > MAX_TID || block >= G.grid_blocks || size > 16u ||
         (!shared && tgt != 0) || (tgt != 0 && tgt - 1u >= G.cluster_blocks)) {
         atomicOr(err, ERR_RANGE);
-        return;
+        return false;
     }
-    const uint32_t owner = tgt ? (block / G.cluster_blocks) * G.cluster_blocks + (tgt - 1u) : block;
+    const uint32_t cl = P2 ? block >> G.cb_log2 : block / G.cluster_blocks;
+    const uint32_t owner = tgt ? cl * G.cluster_blocks + (tgt - 1u) : block;
     const uint64_t word0 = off >> 2;
-    const uint32_t nw = size <= 4u ? 1u : size >> 2;
+    nw = size <= 4u ? 1u : size >> 2;
     const uint64_t limit = shared ? G.smem_words : G.global_words;
     if (owner >= G.grid_blocks || word0 + nw > limit) {
         atomicOr(err, ERR_RANGE);
-        return;
+        return false;
     }
-    for (uint32_t k = 0; k < nw; k++) {
-        const uint64_t idx = shared ? G.global_words + (uint64_t)owner * G.smem_words + word0 + k : word0 + k;
-        unsigned long long *p = shadow + idx;
-        unsigned long long o = ld_relaxed(p);
-        for (;;) {
-            uint32_t rep;
-            const unsigned long long nv =
-                step(o, tid, kind, g, c, b, w, table, G.block_threads, G.warp_size, G.cluster_blocks, &rep);
-            if (nv == o)
-                break; /* unchanged record: linearised at the coherent load */
-            const unsigned long long prev = atomicCAS(p, o, nv);
-            if (prev == o)
-                break;
-            o = prev;
-            retries++;
-        }
-        checked++;
+    idx0 = shared ? G.global_words + (uint64_t)owner * G.smem_words + word0 : word0;
+    return true;
+}
+
+/* Algorithm 1's load / step / CAS loop on one record whose value o was
+ * already loaded; no store when the record is unchanged (linearised at the coherent load).
+ * P2: power-of-two geometry, label by shifts (label_p2); else the generic step(). */
+template <bool P2>
+__device__ __forceinline__ void commit(const hirace_event &e, unsigned long long *p, unsigned long long o,
+                                       const unsigned char *table, const Geo &G, unsigned long long &retries)
+{
+    const uint32_t meta = e.meta;
+    const uint32_t kind = meta & 3u, w = (meta >> 5) & 511u, b = (meta >> 14) & 1023u, g = meta >> 24;
+    const uint32_t c = (uint32_t)(e.addr >> 56) & 127u;
+    for (;;) {
+        uint32_t rep;
+        const unsigned long long nv =
+            P2 ? step_labelled(o, label_p2(o, e.tid, kind, g, c, b, w, G.bt_log2, G.ws_log2, G.cb_log2), e.tid, g,
+                               c, b, w, table)
+               : step(o, e.tid, kind, g, c, b, w, table, G.block_threads, G.warp_size, G.cluster_blocks, &rep);
+        if (nv == o)
+            break;
+        const unsigned long long prev = atomicCAS(p, o, nv);
+        if (prev == o)
+            break;
+        o = prev;
+        retries++;
     }
 }
 
-__global__ void __launch_bounds__(kThreads) k_cluster_replay(const hirace_event *__restrict__ ev, uint32_t n,
+/* kU events per thread per iteration of the grid-stride loop: their event loads, then their
+ * record loads, are issued back to back so kU L2/HBM round trips overlap (the chain event ->
+ * record -> CAS is latency-bound with one event in flight). */
+constexpr int kU = 4;
+
+template <bool P2>
+__global__ void __launch_bounds__(kThreads, 4) k_cluster_replay(const hirace_event *__restrict__ ev, uint32_t n,
                                                              unsigned long long *shadow, const unsigned char *gtable,
                                                              Geo G, unsigned int *err, unsigned long long *stats)
 {
@@ -128,26 +148,66 @@ __global__ void __launch_bounds__(kThreads) k_cluster_replay(const hirace_event 
     uint32_t start = 0;
     while (start < n) {
         const uint64_t key0 = batch_key(ev[start]);
-        /* end = first index > start whose batch key differs (upper bound; sorted input) */
+        /* end = first index > start whose batch key differs (upper bound; sorted input), by a
+         * 32-ary search: each lane probes one of 32 evenly spaced events, the ballot's prefix of
+         * "key <= key0" lanes narrows the range 32x per round (5 dependent loads for 16M events
+         * instead of 24 for a binary search).  The loop is grid-uniform, so all lanes are here. */
+        const uint32_t lane = threadIdx.x & 31u;
         uint32_t lo = start + 1, hi = n;
         while (lo < hi) {
-            const uint32_t mid = lo + (hi - lo) / 2;
-            if (batch_key(ev[mid]) <= key0)
-                lo = mid + 1;
-            else
-                hi = mid;
+            const uint32_t stride = (uint32_t)(((uint64_t)(hi - lo) + 31u) / 32u);
+            const uint64_t q = (uint64_t)lo + (uint64_t)lane * stride;
+            const bool le = q < hi && batch_key(ev[q]) <= key0;
+            const uint32_t t = __popc(__ballot_sync(0xffffffffu, le));
+            if (t == 0) {
+                hi = lo;
+            } else {
+                const uint64_t nhi = (uint64_t)lo + (uint64_t)t * stride;
+                lo = lo + (t - 1u) * stride + 1u;
+                hi = nhi < hi ? (uint32_t)nhi : hi;
+            }
         }
         const uint32_t end = lo;
-        /* grid-stride over the batch: consecutive warps take consecutive 32-event chunks.
-         * Contiguous per-warp or per-CTA shares (the three-level replay's layout) were measured
-         * slower on the halo workloads (profiles/r1_cluster_ab.txt). */
-        for (uint64_t i = start + gtid; i < end; i += gsize) {
-            const hirace_event e = ev[i];
-            if (batch_key(e) != key0) {
-                atomicOr(err, ERR_BAD_TRACE); /* not batch-sorted */
-                continue;
+        /* grid-stride over the batch: consecutive warps take consecutive 32-event chunks, each
+         * thread kU of them per iteration (i, i + gsize, ...).  Contiguous per-warp or per-CTA
+         * shares (the three-level replay's layout) were measured slower on the halo workloads
+         * (profiles/r1_cluster_ab.txt).  Events of one batch are pairwise concurrent or
+         * program-ordered in one thread, so the order in which a thread commits
+         * its kU events does not change the flagged set. */
+        for (uint64_t i = start + gtid; i < end; i += kU * gsize) {
+            hirace_event e[kU];
+            bool v[kU];
+#pragma unroll
+            for (int k = 0; k < kU; k++) {
+                v[k] = i + k * gsize < end;
+                if (v[k])
+                    e[k] = ev[i + k * gsize];
             }
-            check_event(e, shadow, table, G, err, checked, retries);
+            uint64_t idx[kU];
+            uint32_t nw[kU];
+#pragma unroll
+            for (int k = 0; k < kU; k++) {
+                if (v[k] && batch_key(e[k]) != key0) {
+                    atomicOr(err, ERR_BAD_TRACE); /* not batch-sorted */
+                    v[k] = false;
+                }
+                if (v[k])
+                    v[k] = decode_event<P2>(e[k], G, err, idx[k], nw[k]);
+            }
+            unsigned long long o[kU];
+#pragma unroll
+            for (int k = 0; k < kU; k++)
+                if (v[k])
+                    o[k] = ld_relaxed(shadow + idx[k]);
+#pragma unroll
+            for (int k = 0; k < kU; k++) {
+                if (!v[k])
+                    continue;
+                commit<P2>(e[k], shadow + idx[k], o[k], table, G, retries);
+                for (uint32_t j = 1; j < nw[k]; j++) /* wide access: one record per word */
+                    commit<P2>(e[k], shadow + idx[k] + j, ld_relaxed(shadow + idx[k] + j), table, G, retries);
+                checked += nw[k];
+            }
         }
         grid.sync();
         start = end;
@@ -247,7 +307,7 @@ hirace_status hirace_cluster_alloc(const hirace_config *cfg, uint32_t cluster_bl
     if (e == cudaSuccess)
         e = cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, cfg->device);
     if (e == cudaSuccess)
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_cluster_replay, kThreads, 0);
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_cluster_replay<false>, kThreads, 0);
     if (e != cudaSuccess || per_sm < 1) {
         hirace_cluster_free(c);
         return e == cudaErrorMemoryAllocation ? HIRACE_E_NOMEM : HIRACE_E_CUDA;
@@ -301,14 +361,21 @@ hirace_status hirace_cluster_replay(hirace_cluster_ctx *c, const hirace_event *d
     if (!n)
         return HIRACE_OK;
     Geo G{c->cfg.block_threads, c->cfg.warp_size, c->cluster_blocks, c->cfg.grid_blocks, c->global_words,
-          c->smem_words};
+          c->smem_words, 0, 0, 0};
+    const auto pow2 = [](uint32_t x) { return x && !(x & (x - 1)); };
+    const bool p2 = pow2(G.block_threads) && pow2(G.warp_size) && pow2(G.cluster_blocks);
+    if (p2) {
+        G.bt_log2 = __builtin_ctz(G.block_threads);
+        G.ws_log2 = __builtin_ctz(G.warp_size);
+        G.cb_log2 = __builtin_ctz(G.cluster_blocks);
+    }
     uint32_t nn = (uint32_t)n;
     const hirace_event *ev = d_events;
     unsigned long long *shadow = c->shadow;
     const unsigned char *table = c->table;
     void *args[] = {(void *)&ev, (void *)&nn, (void *)&shadow, (void *)&table, (void *)&G, (void *)&c->err,
                     (void *)&c->stats};
-    return cuda_status(cudaLaunchCooperativeKernel((const void *)k_cluster_replay, dim3(c->grid), dim3(kThreads),
+    return cuda_status(cudaLaunchCooperativeKernel(p2 ? (const void *)k_cluster_replay<true> : (const void *)k_cluster_replay<false>, dim3(c->grid), dim3(kThreads),
                                                    args, 0, (cudaStream_t)stream));
 }
 
