@@ -64,6 +64,21 @@ __device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long lon
     return v;
 }
 
+/* 16-byte event, streaming: read once, so no L1 allocation (the records are what should stay
+ * cached) */
+__device__ __forceinline__ hirace_event ld_event_stream(const hirace_event *p)
+{
+    uint32_t x, y, z, w;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(x), "=r"(y), "=r"(z), "=r"(w)
+                 : "l"(p));
+    hirace_event e;
+    e.addr = (uint64_t)x | ((uint64_t)y << 32);
+    e.tid = z;
+    e.meta = w;
+    return e;
+}
+
 struct Geo {
     uint32_t block_threads, warp_size, cluster_blocks, grid_blocks;
     uint64_t global_words, smem_words;
@@ -181,7 +196,7 @@ __global__ void __launch_bounds__(kThreads, 4) k_cluster_replay(const hirace_eve
             for (int k = 0; k < kU; k++) {
                 v[k] = i + k * gsize < end;
                 if (v[k])
-                    e[k] = ev[i + k * gsize];
+                    e[k] = ld_event_stream(ev + i + k * gsize);
             }
             uint64_t idx[kU];
             uint32_t nw[kU];
