@@ -379,6 +379,12 @@ hirace_status hirace_microbench_atomics(int device, uint64_t nwords, int random,
 /* Cost of one grid barrier at the persistent replay kernel's grid size, microseconds.
  * mode 0 = the library's barrier; 1 = busy polling; 2 = generation flag set by the last CTA. */
 hirace_status hirace_microbench_grid_sync(int device, int iters, int mode, double *us_per_barrier, void *stream);
+/* Diagnostics: op 2 (coherent load) or 3 (load + CAS) on the 8-byte words words[idx[i]],
+ * i < n, grid-stride over the list with ctas_per_sm x 256-thread CTAs per SM; the list order is
+ * the access pattern.  *ms_out = kernel time (CUDA events on `stream`).  Caller owns both
+ * device buffers.  HIRACE_E_INVAL on null pointers or another op. */
+hirace_status hirace_microbench_indexed(int device, void *words, const void *idx, uint64_t n, int op,
+                                        int ctas_per_sm, double *ms_out, void *stream);
 
 /* Selective tracking ("Individual threads or test data
  * addresses may have their instrumentation enabled or disabled dynamically.  The memory

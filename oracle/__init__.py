@@ -6,6 +6,9 @@ TEST INFRASTRUCTURE ONLY.  Only `tests/`, `__graft_entry__.smoke()` and `bench.p
 two share no code.
 
   oracle_d.c  Oracle-D: the race definition, sort + per-level scan, C.
+  oracle_par.c  all-core driver: splits the element-level accesses by key into shards and runs
+              oracle_d.c's oracle_races_gran on each (a key's verdict depends only on its own
+              accesses); pinned against the single-thread function.
   brute.py    literal O(n^2) pairwise enumeration of C1, for tiny traces.
   races_cluster / brute.races_cluster: the definition with a thread-block-cluster level
               (reading R16); class CLUSTER = 4.
@@ -23,6 +26,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "oracle_d.c")
+_SRCS = [_SRC, os.path.join(_HERE, "oracle_par.c")]
 _SO = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
@@ -31,8 +35,9 @@ CLASS_NAMES = {1: "WARP", 2: "BLOCK", 3: "GRID", 4: "CLUSTER"}
 
 
 def build(force: bool = False) -> str:
-    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", _SRC, "-o", _SO])
+    if force or not os.path.exists(_SO) or any(os.path.getmtime(_SO) < os.path.getmtime(p) for p in _SRCS):
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", "-pthread", *_SRCS, "-o", _SO + ".tmp"])
+        os.replace(_SO + ".tmp", _SO)
     return _SO
 
 
@@ -49,6 +54,10 @@ def _load():
         lib.oracle_races_gran.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                           ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
                                           ctypes.c_int, ctypes.c_uint32]
+        lib.oracle_races_par.restype = ctypes.c_int64
+        lib.oracle_races_par.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                                         ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                                         ctypes.c_int, ctypes.c_uint32, ctypes.c_int, ctypes.c_int]
         lib.oracle_races_cluster.restype = ctypes.c_int64
         lib.oracle_races_cluster.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                              ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
@@ -73,6 +82,37 @@ def races(events: np.ndarray, block_threads: int, warp_size: int, policy: int = 
                                   keys.ctypes.data, cls.ctypes.data, gs.ctypes.data, cap, policy, granularity_log2)
         if r < 0:
             raise RuntimeError(f"oracle_races failed ({r})")
+        if r <= cap:
+            return keys[:r], cls[:r], gs[:r]
+        cap = int(r)
+
+
+def hardware_threads() -> int:
+    """std::thread::hardware_concurrency() equivalent: the CPUs this process may run on."""
+    try:
+        return len(os.sched_getaffinity(0))
+    except (AttributeError, OSError):
+        return os.cpu_count() or 1
+
+
+def races_parallel(events: np.ndarray, block_threads: int, warp_size: int, policy: int = 0,
+                   granularity_log2: int = 2, threads: int | None = None, shards: int | None = None):
+    """Oracle-D over address shards on `threads` cores (default: all).  Same result as races()
+    (oracle_par.c; pinned by tests/test_oracle_par.py)."""
+    lib = _load()
+    ev = np.ascontiguousarray(events)
+    n = int(ev.shape[0])
+    t = int(threads or hardware_threads())
+    s = int(shards or max(4 * t, min(4096, n // (1 << 22) + 1)))
+    cap = 1 << 16
+    while True:
+        keys = np.empty(cap, np.uint64)
+        cls = np.empty(cap, np.uint8)
+        gs = np.empty(cap, np.uint8)
+        r = lib.oracle_races_par(ev.ctypes.data if n else None, n, block_threads, warp_size, keys.ctypes.data,
+                                 cls.ctypes.data, gs.ctypes.data, cap, policy, granularity_log2, t, s)
+        if r < 0:
+            raise RuntimeError(f"oracle_races_par failed ({r})")
         if r <= cap:
             return keys[:r], cls[:r], gs[:r]
         cap = int(r)

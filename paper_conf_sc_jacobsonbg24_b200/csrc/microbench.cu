@@ -96,10 +96,56 @@ __global__ void __launch_bounds__(kReplayThreads) k_mb_grid_sync(unsigned int *b
         grid_sync_variant(bar, gridDim.x, epoch, mode);
 }
 
+/* the words listed in idx[0..n), grid-stride (consecutive threads take consecutive list
+ * entries): op 2 = coherent load, 3 = load + CAS.  The list's order is the access pattern
+ * (random, sorted, window-major ...), chosen by the caller. */
+__global__ void __launch_bounds__(256) k_mb_indexed(unsigned long long *a, const unsigned long long *__restrict__ idx,
+                                                    uint64_t n, int op, unsigned long long *sink)
+{
+    unsigned long long acc = 0;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        unsigned long long *p = a + __ldcs(idx + i);
+        const unsigned long long o = hirace::ld_coherent(p);
+        if (op == 3)
+            acc += atomicCAS(p, o, o + 1);
+        else
+            acc += o;
+    }
+    if (acc == 0x123456789ull)
+        *sink = acc;
+}
+
 } // namespace
 } // namespace hirace_impl
 
 using namespace hirace_impl;
+
+extern "C" hirace_status hirace_microbench_indexed(int device, void *words, const void *idx, uint64_t n, int op,
+                                                   int ctas_per_sm, double *ms_out, void *stream)
+{
+    if (!ms_out || !words || (n && !idx) || (op != 2 && op != 3) || ctas_per_sm < 1)
+        return HIRACE_E_INVAL;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (cudaSetDevice(device) != cudaSuccess)
+        return HIRACE_E_CUDA;
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    cudaEventRecord(e0, st);
+    k_mb_indexed<<<sms * ctas_per_sm, 256, 0, st>>>((unsigned long long *)words, (const unsigned long long *)idx, n, op,
+                                                    (unsigned long long *)words);
+    cudaEventRecord(e1, st);
+    float ms = 0;
+    hirace_status s = HIRACE_OK;
+    if (cudaEventSynchronize(e1) != cudaSuccess || cudaEventElapsedTime(&ms, e0, e1) != cudaSuccess)
+        s = HIRACE_E_CUDA;
+    *ms_out = ms;
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    return s;
+}
 
 extern "C" hirace_status hirace_microbench_atomics(int device, uint64_t nwords, int random, int op, uint64_t nops,
                                                    double *ops_per_s, void *stream)

@@ -33,7 +33,7 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_collect_races_device", "hirace_get_stats", "hirace_sync", "hirace_get_dev_ctx",
            "hirace_bucket_events", "hirace_bucket_wire", "hirace_replay_wire", "hirace_count_wire",
            "hirace_dispatch_wire", "hirace_peer_buffer_alloc", "hirace_peer_buffer_free", "hirace_peer_open",
-           "hirace_peer_close", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_set_policy", "hirace_set_filter",
+           "hirace_peer_close", "hirace_set_kernel_timing", "hirace_microbench_atomics", "hirace_microbench_grid_sync", "hirace_microbench_indexed", "hirace_set_policy", "hirace_set_filter",
            "hirace_fsm_table", "hirace_fsm_table_policy", "hirace_fsm_step", "hirace_fsm_step_policy", "hirace_fsm_step_compact",
            "hirace_fsm_table_cluster", "hirace_fsm_cluster_class", "hirace_fsm_step_cluster",
            "hirace_cluster_alloc", "hirace_cluster_free", "hirace_cluster_reset", "hirace_cluster_replay",
@@ -116,6 +116,7 @@ def load():
         "hirace_set_kernel_timing": (I32, [P, P, P]),
         "hirace_microbench_atomics": (I32, [I32, U64, I32, I32, U64, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_microbench_grid_sync": (I32, [I32, I32, I32, ctypes.POINTER(ctypes.c_double), P]),
+        "hirace_microbench_indexed": (I32, [I32, P, P, U64, I32, I32, ctypes.POINTER(ctypes.c_double), P]),
         "hirace_set_policy": (I32, [P, I32, P]),
         "hirace_set_filter": (I32, [P, U32, U32, U32, U64, U64]),
         "hirace_fsm_table": (I32, [P]),
@@ -223,6 +224,15 @@ def microbench_grid_sync(iters: int = 200, mode: int = 0, device: int = 0, strea
     _check(load().hirace_microbench_grid_sync(device, iters, mode, ctypes.byref(r), _stream_handle(stream)),
            "hirace_microbench_grid_sync")
     return r.value
+
+
+def microbench_indexed(words_ptr: int, idx_ptr: int, n: int, op: int = 3, ctas_per_sm: int = 8, device: int = 0,
+                       stream=None) -> float:
+    """ms of one load (op 2) / load+CAS (op 3) pass over words[idx[i]] (diagnostics)."""
+    ms = ctypes.c_double()
+    _check(load().hirace_microbench_indexed(device, words_ptr, idx_ptr, n, op, ctas_per_sm, ctypes.byref(ms),
+                                            _stream_handle(stream)), "microbench_indexed")
+    return ms.value
 
 
 def _stream_handle(stream):
