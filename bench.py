@@ -5,16 +5,24 @@
 One step = one pass of the whole hot path over the workload: shadow reset (a11), replay of
 the full trace through the FSM with CAS updates and race reports (a1-a9), and the device-side
 collection of flagged words (a7).  The step's launches are captured once as a CUDA graph and
-the graph is replayed for the timed steps (`--no-graph`: eager launches); the replay kernel's
-own time comes from CUDA events around it in an eager pass.  Default workload = BASELINE.json configs[1] (config 2:
-tiled shared-memory stencil, 1024 blocks x 256 threads, racy-A variant, 17,825,792 events);
-inputs are resident in HBM when timing starts and are larger than L2 (285 MB of events).
+the graph is replayed for the timed steps (`--no-graph`: eager launches); per-kernel times come
+from CUDA events around each kernel in an eager pass.
+
+Default workload = config 5 (BASELINE.json configs[4], the config the metric is quoted on at
+1/2/4/8 GPUs): 1.07e9 accesses over 2^32 tracked words, 65,536 x 256 threads, 32 batches.
+N=1 replays the whole trace on one GPU; N>1 (torchrun) shards it by address (strong scaling,
+owner = 64 KiB chunk mod N) with the exchange over NCCL (`--transport nccl`, default) or peer
+stores (`--transport p2p`).  Configs 2, 3 and 4 are measured after it at N=1 and reported under
+`per_config` (`--no-per-config` skips them).  Inputs are resident in HBM when timing starts
+and are larger than L2 (17 GB of events for config 5).
 
 `value` = word-level accesses checked per second (whole job, all ranks).  `e2e` = the same
 metric through the C-ABI host entry point (hirace_check_trace_host: pinned host events ->
-H2D -> replay -> collect -> D2H).  `roofline` = the replay kernel against the measured HBM
-copy bandwidth at 32 algorithmic bytes per access.  `cpu_baseline` = the oracle (C, one core).
-`--impl reference` times that oracle as the reference arm.
+H2D -> replay -> collect -> D2H; N>1: per rank host -> device, then the sharded step).
+`roofline` = the dominant kernel against the measured HBM copy bandwidth at its algorithmic
+bytes; `roofline_step` = the whole step at 32 algorithmic bytes per access.  `cpu_baseline` =
+Oracle-D on all host cores (address-sharded, oracle/oracle_par.c) on a bounded sample, with the
+one-thread rate beside it.  `--impl reference` times that oracle as the reference arm.
 """
 from __future__ import annotations
 
@@ -66,9 +74,13 @@ def make_trace(config: int, variant: str, nranks: int = 1, rank: int = 0):
     raise SystemExit(f"unknown config {config}")
 
 
-def word_accesses(events) -> int:
-    sz = 1 << ((events["meta"] >> 2) & 7).astype(np.int64)
-    return int(np.where(sz <= 4, 1, sz // 4).sum())
+def word_accesses(events, chunk: int = 1 << 26) -> int:
+    """Word-level accesses (8/16-byte accesses count 2/4 words), chunked for 1e9-event traces."""
+    tot = 0
+    for lo in range(0, events.shape[0], chunk):
+        szl = (events["meta"][lo:lo + chunk] >> 2) & 7
+        tot += int(np.where(szl <= 2, 1, 1 << np.maximum(szl.astype(np.int64) - 2, 0)).sum())
+    return tot
 
 
 class ClockSampler:
@@ -123,66 +135,109 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(rows), "samples_in_timed_region": len(inside)}
 
 
-def load_traffic(config: int, variant: str, compact: bool = False):
+def load_traffic(key: str):
+    """DRAM bytes per launch of the dominant kernel for this workload, from the committed ncu
+    captures (profiles/traffic.json, one key per config/variant/record layout)."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(p):
         with open(p) as f:
             d = json.load(f)
-        return d.get(f"cfg{config}_{variant}" + ("_compact" if compact else ""))
+        v = d.get(key)
+        return v.get("bytes") if isinstance(v, dict) else v
     return None
 
 
-def time_oracle(trace, budget_s: float):
-    """Oracle-D as it stands on a bounded sample: the events of the first m blocks."""
-    import oracle
+def sample_blocks(trace, m: int):
+    """The events of blocks [0, m) of a trace (a bounded sample of the same workload)."""
     import tracegen as tg
     ev = trace.events
-    blk = ev["tid"] // trace.block_threads
-    # calibrate on 1/64 of the blocks
-    m0 = max(1, trace.grid_blocks // 64)
-    s0 = ev[blk < m0]
+    if m >= trace.grid_blocks:
+        return trace
+    sel = ev["tid"] < np.uint32(m * trace.block_threads)
+    return tg.Trace(trace.name, ev[sel], trace.grid_blocks, trace.block_threads, trace.warp_size,
+                    trace.global_words, trace.smem_words)
+
+
+def oracle_sample(trace, budget_s: float, threads: int):
+    """Blocks [0, m) with m sized (from a calibration run on 1/256 of the blocks) so that the
+    oracle on `threads` cores takes about budget_s."""
+    import oracle
+    m0 = max(1, trace.grid_blocks // 256)
+    s0 = sample_blocks(trace, m0)
     t = time.perf_counter()
-    oracle.races(s0, trace.block_threads, trace.warp_size)
-    rate = max(len(s0), 1) / max(time.perf_counter() - t, 1e-6)
-    m = int(min(trace.grid_blocks, max(m0, trace.grid_blocks * min(1.0, budget_s * rate / max(len(ev), 1)))))
-    sample = ev[blk < m]
-    sub = tg.Trace(trace.name, sample, trace.grid_blocks, trace.block_threads, trace.warp_size,
-                   trace.global_words, trace.smem_words)
-    return sub, m
+    oracle.races_parallel(s0.events, s0.block_threads, s0.warp_size, threads=threads)
+    dt = max(time.perf_counter() - t, 1e-6)
+    m = int(min(trace.grid_blocks, max(m0, m0 * budget_s / dt)))
+    return sample_blocks(trace, m), m
 
 
-def run_reference(args, trace, world):
+def cpu_baseline(trace, budget_s: float = 20.0) -> dict:
+    """Oracle-D as it stands on the box's host cores (SURVEY §8(d) "Oracle timing"): all cores
+    (hardware_concurrency threads over address shards) on a ~budget_s sample, and one core on a
+    smaller sample."""
+    import oracle
+    cores = oracle.hardware_threads()
+    sub, m = oracle_sample(trace, budget_s, cores)
+    na = word_accesses(sub.events)
+    t = time.perf_counter()
+    oracle.races_parallel(sub.events, sub.block_threads, sub.warp_size, threads=cores)
+    dt = time.perf_counter() - t
+    sub1 = sample_blocks(trace, max(1, m // (4 * cores)))
+    na1 = word_accesses(sub1.events)
+    t = time.perf_counter()
+    oracle.races(sub1.events, sub1.block_threads, sub1.warp_size)
+    dt1 = time.perf_counter() - t
+    return {"value": na / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"events of blocks [0,{m}) of {trace.name} ({na} word accesses), one run, {cores} threads "
+                      f"over address shards (oracle/oracle_par.c)",
+            "one_thread": {"value": na1 / dt1, "unit": UNIT,
+                           "sample": f"events of blocks [0,{max(1, m // (4 * cores))}) ({na1} word accesses)"},
+            **host_cpu()}
+
+
+def run_reference(args, world):
+    """Reference arm: the oracle (all host cores) as it stands, on a bounded sample of the
+    workload per step.  Rank 0 only; other ranks exit without work."""
     import oracle
     if int(os.environ.get("RANK", "0")) != 0:
         return
+    trace = make_trace(args.config, args.variant)
+    cores = oracle.hardware_threads()
     budget = max(0.05, 150.0 / max(args.steps + args.warmup, 1))
-    sub, m = time_oracle(trace, budget)
+    sub, m = oracle_sample(trace, budget, cores)
+    if args.config == 5:
+        trace.info.pop("buffer", None)
     n_acc = word_accesses(sub.events)
     for _ in range(args.warmup):
-        oracle.races(sub.events, sub.block_threads, sub.warp_size)
+        oracle.races_parallel(sub.events, sub.block_threads, sub.warp_size, threads=cores)
     t = time.perf_counter()
     for _ in range(args.steps):
-        oracle.races(sub.events, sub.block_threads, sub.warp_size)
+        oracle.races_parallel(sub.events, sub.block_threads, sub.warp_size, threads=cores)
     dt = (time.perf_counter() - t) / max(args.steps, 1)
     v = n_acc / dt
-    sample = f"events of blocks [0,{m}) of {trace.name} ({n_acc} word accesses) per step"
+    sample = (f"events of blocks [0,{m}) of {trace.name} ({n_acc} word accesses) per step, {cores} threads over "
+              "address shards")
     out = {"metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-           "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True, "scaling": "weak",
+           "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+           "scaling": "strong" if args.config == 5 else "weak",
            "vs_baseline": None, "dtype": "u64", "data": "synthetic", "impl": "reference",
            "config": config_block(args, trace, world),
-           "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample, **host_cpu()},
+           "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample,
+                            **host_cpu()},
            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
 
 
-def config_block(args, trace, world):
-    return {"workload": f"config {args.config} ({trace.name}): {BASELINE_CFG.get(args.config, '')}",
+def config_block(args, trace, world, config=None):
+    config = args.config if config is None else config
+    rb = 4 if getattr(args, "compact", False) else 8
+    return {"workload": f"config {config} ({trace.name}): {BASELINE_CFG.get(config, '')}",
             "events_per_rank": int(trace.n), "grid_blocks": trace.grid_blocks,
             "block_threads": trace.block_threads, "batches": trace.batch_count(),
-            "shadow_bytes": (4 if getattr(args, "compact", False) else 8) * (trace.global_words + trace.grid_blocks * trace.smem_words),
-            "shadow_record_bytes": 4 if getattr(args, "compact", False) else 8,
+            "shadow_bytes": rb * (trace.global_words + trace.grid_blocks * trace.smem_words),
+            "shadow_record_bytes": rb,
             "l2": "inputs larger than L2 (events %.0f MB > 126 MB L2)" % (trace.n * 16 / 1e6),
-            "parallelism": f"replicas{world}" if world > 1 else "single"}
+            "parallelism": "single" if world == 1 else f"replicas{world}"}
 
 
 BASELINE_CFG = {
@@ -305,6 +360,9 @@ def run_sharded_bench(args, world, rank, local_rank):
     import torch.distributed as dist
 
     from paper_conf_sc_jacobsonbg24_b200 import sharded
+    # communicator-init lines (rank / nranks / transport) for the driver's rank check
+    os.environ.setdefault("NCCL_DEBUG", "INFO")
+    os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
     dev = local_rank % torch.cuda.device_count()
     torch.cuda.set_device(dev)
     shared_gpu = world > torch.cuda.device_count()  # several ranks per GPU: NCCL cannot run there
@@ -368,6 +426,41 @@ def run_sharded_bench(args, world, rank, local_rank):
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     dist.all_reduce(fl)
     ms, flagged = float(ms.item()), int(fl.item())
+    # e2e: every step copies this rank's events from pinned host memory to the device, runs the
+    # sharded step and reads the flagged words back (D2H); max over ranks of the wall time
+    e2e = None
+    if not args.no_e2e:
+        host = torch.from_numpy(t.events.view(np.int64).reshape(-1, 2))
+        try:
+            host = host.pin_memory()
+            pinned = True
+        except RuntimeError:
+            pinned = False
+        h_out = torch.empty(cap * 16, dtype=torch.uint8, pin_memory=True)
+        h_tot = torch.zeros(1, dtype=torch.int64, pin_memory=True)
+        ke2 = max(3, min(args.steps, 5))
+
+        def e2e_step():
+            ev.copy_(host, non_blocking=True)
+            step()
+            h_tot.copy_(d_total, non_blocking=True)
+            torch.cuda.synchronize()
+            h_out[: min(int(h_tot.item()), cap) * 16].copy_(d_out[: min(int(h_tot.item()), cap) * 16])
+
+        e2e_step()
+        dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(ke2):
+            e2e_step()
+        dt = torch.tensor([(time.perf_counter() - t0) / ke2], dtype=torch.float64)
+        if nccl:
+            dt = dt.cuda()
+        dist.all_reduce(dt, op=dist.ReduceOp.MAX)
+        dt = float(dt.item())
+        e2e = {"value": n_total / dt, "unit": UNIT, "h2d_bytes_per_step": int(t.n * 16) * world,
+               "d2h_bytes_per_step": int(min(flagged, cap) * 16 + 8), "ms_per_step": dt * 1e3,
+               "host_memory": "pinned" if pinned else "pageable", "steps": ke2,
+               "path": "per rank: H2D of its events, sharded step, collect, D2H"}
     if rank == 0:
         peak, peak_kind = peaks()
         per_step = ms / args.steps
@@ -387,7 +480,8 @@ def run_sharded_bench(args, world, rank, local_rank):
                             "peak": peak, "unit": "GB/s",
                             "frac": BYTES_PER_ACCESS * n_total / world / (per_step / 1e3) / 1e9 / peak,
                             "traffic": None, "kernel": "whole sharded step per GPU", "peak_kind": peak_kind},
-               "cpu_baseline": None, "e2e": None, "gpu_launches": None, "clocks": clocks.summary(),
+               "cpu_baseline": None,  # the oracle is timed on rank 0 at N=1 only
+               "e2e": e2e, "gpu_launches": None, "clocks": clocks.summary(),
                "check": {"flagged_words": flagged, "expected": len(t.info["expected"])}}
         print(json.dumps(out), flush=True)
     if isinstance(ex, sharded.PeerExchange):
@@ -395,62 +489,21 @@ def run_sharded_bench(args, world, rank, local_rank):
     dist.destroy_process_group()
 
 
-def main():
-    ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=200)
-    ap.add_argument("--warmup", type=int, default=10)
-    ap.add_argument("--impl", default="hirace", choices=["hirace", "reference"])
-    ap.add_argument("--config", type=int, default=2)
-    ap.add_argument("--variant", default="racy", choices=["racy", "clean"])
-    ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--no-slowdown", action="store_true")
-    ap.add_argument("--no-graph", action="store_true", help="time the eager step instead of its CUDA graph")
-    ap.add_argument("--compact", action="store_true",
-                    help="compact 4-byte shadow records (hirace_shadow_alloc_compact, SURVEY §8(f) f1)")
-    ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p", "host"],
-                    help="config-5 shard exchange: NCCL device all_to_all, peer-memory dispatch (CUDA IPC / "
-                         "NVLink stores from the bucketing kernel), or gloo host staging")
-    args = ap.parse_args()
-    args.warmup = max(args.warmup, 3)
-
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
-    if args.config == 5 and world > 1 and args.impl != "reference":
-        run_sharded_bench(args, world, rank, local_rank)
-        return
-    trace = make_trace(args.config, args.variant)
-
-    if args.impl == "reference":
-        run_reference(args, trace, world)
-        return
-
+def measure_single(args, config: int, variant: str, K: int, W: int, dev: int, clocks=None, keep=False):
+    """Times the full step (reset + check_device: batch discovery, replay with fused collect)
+    of one workload on one GPU: an eager pass with CUDA events around the replay kernel, then the
+    same step captured as a CUDA graph and replayed K times (the timed `value`)."""
     import torch
-    import torch.distributed as dist
 
     import paper_conf_sc_jacobsonbg24_b200 as hr
-    ngpu = torch.cuda.device_count()
-    local_rank = local_rank % ngpu  # several ranks per GPU only in single-GPU functional runs
-    torch.cuda.set_device(local_rank)
-    red_dev = "cuda"
-    if world > 1:
-        if world <= ngpu:
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
-        else:  # ranks share a GPU: NCCL cannot run there; timing reductions go through gloo
-            dist.init_process_group("gloo")
-            red_dev = "cpu"
-
+    trace = make_trace(config, variant)
     n_acc = word_accesses(trace.events)
-    c = hr.Checker.for_trace(trace, device=local_rank, compact=args.compact)
-    bpa = bytes_per_access(c.rec_bytes)
-    d_ev = hr.events_to_device(trace.events, f"cuda:{local_rank}")
+    c = hr.Checker.for_trace(trace, device=dev, compact=args.compact)
+    d_ev = hr.events_to_device(trace.events, f"cuda:{dev}")
     cap = 1 << 20
-    d_out = torch.empty(cap * 16, dtype=torch.uint8, device="cuda")
-    d_total = torch.zeros(1, dtype=torch.int64, device="cuda")
+    d_out = torch.empty(cap * 16, dtype=torch.uint8, device=f"cuda:{dev}")
+    d_total = torch.zeros(1, dtype=torch.int64, device=f"cuda:{dev}")
     stream = torch.cuda.current_stream()
-    K, W = args.steps, args.warmup
     ks = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
     ke = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
     for e in ks + ke:
@@ -458,24 +511,18 @@ def main():
 
     def step(i=None):
         c.reset(stream)
-        if i is not None:
-            c.set_kernel_timing(ks[i], ke[i])
-        else:
-            c.set_kernel_timing(None, None)
+        c.set_kernel_timing(ks[i], ke[i]) if i is not None else c.set_kernel_timing(None, None)
         c.check_device(d_ev, d_out, cap, d_total, stream=stream)  # replay + fused collect
 
-    clocks = ClockSampler(local_rank)
-    clocks.start()
-    time.sleep(0.3)
     for _ in range(W):
         step()
     torch.cuda.synchronize()
     flagged = int(d_total.item())
-
-    t0 = torch.cuda.Event(enable_timing=True)
-    t1 = torch.cuda.Event(enable_timing=True)
-    if world > 1:
-        dist.barrier()
+    l0 = c.launches()
+    step()
+    torch.cuda.synchronize()
+    launches_per_step = c.launches() - l0
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()
     w0 = time.time()
     t0.record(stream)
@@ -484,17 +531,12 @@ def main():
     t1.record(stream)
     torch.cuda.synchronize()
     w1 = time.time()
-    if world > 1:
-        dist.barrier()
-    clocks.mark(w0, w1)
-    ms = t0.elapsed_time(t1)
-    eager_ms = ms
+    if clocks:
+        clocks.mark(w0, w1)
+    eager_ms = t0.elapsed_time(t1)
     kern_ms = sum(a.elapsed_time(b) for a, b in zip(ks, ke)) / K
     c.set_kernel_timing(None, None)
-    # the same step captured once as a CUDA graph (reset + batch discovery + persistent replay
-    # with fused collect) and replayed K times: the launch gaps between the step's kernels go
-    # away; this is the timed `value`.  The kernel-only time above comes from the eager pass.
-    step_mode = "eager"
+    ms, step_mode = eager_ms, "eager"
     if not args.no_graph:
         try:
             gs = torch.cuda.Stream()
@@ -510,8 +552,6 @@ def main():
             torch.cuda.synchronize()
             if int(d_total.item()) != flagged:
                 raise RuntimeError("graph replay disagrees with the eager step")
-            if world > 1:
-                dist.barrier()
             torch.cuda.synchronize()
             w0 = time.time()
             t0.record(gs)
@@ -521,93 +561,190 @@ def main():
             t1.record(gs)
             torch.cuda.synchronize()
             w1 = time.time()
-            if world > 1:
-                dist.barrier()
-            clocks.mark(w0, w1)
-            ms = t0.elapsed_time(t1)
-            step_mode = "cuda_graph"
+            if clocks:
+                clocks.mark(w0, w1)
+            ms, step_mode = t0.elapsed_time(t1), "cuda_graph"
+            del graph
         except Exception as exc:  # capture unsupported: the eager timing stands
             print(f"bench: CUDA graph step unavailable ({exc}); eager timing", file=sys.stderr)
-            ms = eager_ms
+    st = c.stats()
+    peak, peak_kind = peaks()
+    bpa = bytes_per_access(c.rec_bytes)
+    ms_per_step = ms / K
+    achieved = bpa * n_acc / (kern_ms / 1e3) / 1e9
+    key = f"cfg{config}_{variant}" + ("_compact" if args.compact else "")
+    res = {"config": config, "variant": variant, "trace": trace.name, "events": int(trace.n), "accesses": n_acc,
+           "value": n_acc * K / (ms / 1e3), "ms_per_step": ms_per_step, "step_mode": step_mode,
+           "eager_ms_per_step": eager_ms / K, "launches_per_step": launches_per_step,
+           "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                        "traffic": load_traffic(key), "traffic_key": key,
+                        "kernel": "k_replay (incl. fused collect)", "kernel_ms": kern_ms,
+                        "kernel_share": kern_ms / ms_per_step, "bytes_per_access": bpa, "peak_kind": peak_kind},
+           "roofline_step": {"bound": "hbm", "achieved": bpa * n_acc / (ms_per_step / 1e3) / 1e9, "peak": peak,
+                             "unit": "GB/s", "frac": bpa * n_acc / (ms_per_step / 1e3) / 1e9 / peak,
+                             "bytes_per_access": bpa, "what": "whole step (reset + batches + replay + collect)"},
+           "flagged_words": flagged, "stats_per_step": st,
+           "expected_flagged": len(trace.info["expected"]) if "expected" in trace.info else None}
+    if keep:
+        return res, dict(trace=trace, checker=c, n_acc=n_acc, cap=cap, d_ev=d_ev)
+    c.close()
+    del d_ev, d_out, d_total
+    torch.cuda.empty_cache()
+    return res, None
+
+
+def measure_e2e(ctx, K: int, dev: int) -> dict:
+    """The same metric through the C-ABI host entry point: pinned host events -> H2D (chunked,
+    overlapped) -> replay -> collect -> D2H of the flagged words, every step."""
+    import torch
+    trace, c, n_acc, cap = ctx["trace"], ctx["checker"], ctx["n_acc"], ctx["cap"]
+    ev = trace.events
+    nbytes = ev.shape[0] * 16
+    registered = False
+    try:  # page-lock the generator's buffer in place (no 17 GB copy)
+        rc = torch.cuda.cudart().cudaHostRegister(ev.ctypes.data, nbytes, 0)
+        registered = int(rc) == 0 if not isinstance(rc, tuple) else int(rc[0]) == 0
+    except Exception:
+        registered = False
+    hout = torch.empty(cap * 16, dtype=torch.uint8, pin_memory=True)
+    stream = torch.cuda.current_stream()
+    for _ in range(2):
+        c.reset(stream)
+        c.check_host_ptr(ev.ctypes.data, ev.shape[0], hout.data_ptr(), cap, stream=stream)
+    torch.cuda.synchronize()
+    k = max(3, min(K, 10))
+    t = time.perf_counter()
+    tot = 0
+    for _ in range(k):
+        c.reset(stream)
+        tot = c.check_host_ptr(ev.ctypes.data, ev.shape[0], hout.data_ptr(), cap, stream=stream)
+    torch.cuda.synchronize()
+    dt = (time.perf_counter() - t) / k
+    if registered:
+        torch.cuda.cudart().cudaHostUnregister(ev.ctypes.data)
+    return {"value": n_acc / dt, "unit": UNIT, "h2d_bytes_per_step": int(nbytes),
+            "host_memory": "pinned" if registered else "pageable",
+            "d2h_bytes_per_step": int(min(tot, cap) * 16 + 8), "ms_per_step": dt * 1e3, "steps": k,
+            "path": "hirace_check_trace_host"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="hirace", choices=["hirace", "reference"])
+    ap.add_argument("--config", type=int, default=5)
+    ap.add_argument("--variant", default="racy", choices=["racy", "clean"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-slowdown", action="store_true")
+    ap.add_argument("--no-per-config", action="store_true", help="skip the config 2/3/4 secondary measurements")
+    ap.add_argument("--no-graph", action="store_true", help="time the eager step instead of its CUDA graph")
+    ap.add_argument("--compact", action="store_true",
+                    help="compact 4-byte shadow records (hirace_shadow_alloc_compact, SURVEY §8(f) f1)")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p", "host"],
+                    help="config-5 shard exchange (N>1): NCCL device all_to_all, peer-memory dispatch (CUDA IPC / "
+                         "NVLink stores from the bucketing kernel), or gloo host staging")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, world)
+        return
+    if args.config == 5 and world > 1:
+        run_sharded_bench(args, world, rank, local_rank)
+        return
+
+    import torch
+    import torch.distributed as dist
+    ngpu = torch.cuda.device_count()
+    dev = local_rank % ngpu  # several ranks per GPU only in single-GPU functional runs
+    torch.cuda.set_device(dev)
+    red_dev = "cuda"
+    if world > 1:  # configs 1-4 at N>1: independent replicas (weak scaling, no collective)
+        if world <= ngpu:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group("gloo")
+            red_dev = "cpu"
+        dist.barrier()
+    K, W = args.steps, args.warmup
+    clocks = ClockSampler(dev)
+    clocks.start()
+    time.sleep(0.3)
+    res, ctx = measure_single(args, args.config, args.variant, K, W, dev, clocks, keep=True)
+    ms, kern_ms = res["ms_per_step"] * K, res["roofline"]["kernel_ms"]
     if world > 1:
         tt = torch.tensor([ms, kern_ms], dtype=torch.float64, device=red_dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms, kern_ms = float(tt[0]), float(tt[1])
     ms_per_step = ms / K
-    value = n_acc * world * K / (ms / 1e3)
-    st = c.stats()
-
-    # e2e through the C-ABI host entry point: pinned host events -> H2D -> replay -> D2H
-    e2e = None
-    if not args.no_e2e:
-        small = trace.n * 16 <= (4 << 30)
-        pin = torch.empty(trace.n * 16, dtype=torch.uint8, pin_memory=small)
-        pin.numpy()[:] = trace.events.view(np.uint8)
-        hout = torch.empty(cap * 16, dtype=torch.uint8, pin_memory=True)
-        ke2 = max(3, min(K, 10))
-        for _ in range(2):
-            c.reset(stream)
-            c.check_host_ptr(pin.data_ptr(), trace.n, hout.data_ptr(), cap, stream=stream)
-        if world > 1:
-            dist.barrier()
-        torch.cuda.synchronize()
-        we0 = time.perf_counter()
-        for _ in range(ke2):
-            c.reset(stream)
-            tot = c.check_host_ptr(pin.data_ptr(), trace.n, hout.data_ptr(), cap, stream=stream)
-        torch.cuda.synchronize()
-        e2e_s = (time.perf_counter() - we0) / ke2
-        if world > 1:
-            tt = torch.tensor([e2e_s], dtype=torch.float64, device=red_dev)
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            e2e_s = float(tt[0])
-        e2e = {"value": n_acc * world / e2e_s, "unit": UNIT, "h2d_bytes_per_step": int(trace.n * 16),
-               "host_memory": "pinned" if small else "pageable",
-               "d2h_bytes_per_step": int(min(tot, cap) * 16 + 8), "ms_per_step": e2e_s * 1e3}
+    trace, c, n_acc = ctx["trace"], ctx["checker"], ctx["n_acc"]
+    cb = config_block(args, trace, world)
+    e2e = None if args.no_e2e else measure_e2e(ctx, K, dev)
+    if e2e and world > 1:
+        tt = torch.tensor([e2e["ms_per_step"]], dtype=torch.float64, device=red_dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        e2e["ms_per_step"] = float(tt[0])
+        e2e["value"] = n_acc * world / (e2e["ms_per_step"] / 1e3)
+    st = res["stats_per_step"]
+    l2 = None
+    if rank == 0:
+        try:
+            l2 = l2_roofline(st, n_acc, kern_ms, c.rec_bytes, dev)
+            bpa = bytes_per_access(c.rec_bytes)
+            l2["hbm_accesses_per_s_peak"] = peaks()[0] * 1e9 / bpa
+            l2["binding"] = "hbm" if l2["hbm_accesses_per_s_peak"] <= l2["accesses_per_s_peak"] else "l2_atomic"
+        except Exception as exc:  # diagnostics only; never fails the bench line
+            l2 = {"error": str(exc)}
+    rec_bytes = c.rec_bytes
+    c.close()
+    ctx["d_ev"] = None
+    torch.cuda.empty_cache()
+    cpu = None
+    if not args.no_cpu_baseline and world == 1 and rank == 0:
+        cpu = cpu_baseline(trace, 20.0)
+    trace.info.pop("buffer", None)
+    del trace, ctx
+    per_config = {}
+    if not args.no_per_config and world == 1:
+        for cfg in (2, 3, 4):
+            if cfg == args.config:
+                continue
+            r, _ = measure_single(args, cfg, "racy", min(K, 20), W, dev, None)
+            per_config[f"config{cfg}"] = {k: r[k] for k in ("trace", "events", "value", "ms_per_step", "step_mode",
+                                                            "roofline", "roofline_step", "flagged_words",
+                                                            "launches_per_step")}
+    slow = None if (args.no_slowdown or rank != 0) else measure_slowdown(dev)
     clocks.stop()
-
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()
         return
-    peak, peak_kind = peaks()
-    achieved = bpa * n_acc / (kern_ms / 1e3) / 1e9
-    try:
-        l2 = l2_roofline(st, n_acc, kern_ms, c.rec_bytes, local_rank)
-        l2["hbm_accesses_per_s_peak"] = peak * 1e9 / bpa
-        l2["binding"] = "hbm" if peak * 1e9 / bpa <= l2["accesses_per_s_peak"] else "l2_atomic"
-    except Exception as exc:  # diagnostics only; never fails the bench line
-        l2 = {"error": str(exc)}
-    slow = None if args.no_slowdown else measure_slowdown(local_rank)
-    cpu = None
-    if not args.no_cpu_baseline and world == 1:
-        import oracle
-        sub, m = time_oracle(trace, 20.0)
-        t = time.perf_counter()
-        oracle.races(sub.events, sub.block_threads, sub.warp_size)
-        dt = time.perf_counter() - t
-        na = word_accesses(sub.events)
-        cpu = {"value": na / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"events of blocks [0,{m}) of {trace.name} ({na} word accesses), one run, 1 thread",
-               **host_cpu()}
+    roof = dict(res["roofline"])
+    roof["kernel_ms"] = kern_ms
+    roof["achieved"] = roof["bytes_per_access"] * n_acc / (kern_ms / 1e3) / 1e9
+    roof["frac"] = roof["achieved"] / roof["peak"]
+    roof["kernel_share"] = kern_ms / ms_per_step
     out = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": W,
-        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-        "dtype": "u64" if c.rec_bytes == 8 else "u32", "data": "synthetic", "config": config_block(args, trace, world),
-        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": load_traffic(args.config, args.variant, args.compact),
-                     "kernel": "k_replay (incl. fused collect)", "kernel_ms": kern_ms, "kernel_share": kern_ms / ms_per_step,
-                     "bytes_per_access": bpa, "peak_kind": peak_kind},
-        "roofline_l2": l2,
-        "cpu_baseline": cpu,
-        "e2e": e2e,
-        # per step: k_reset, k_batches, k_replay (fused collect) [+ k_collect_reports in report mode]
-        "gpu_launches": (4 if c.shadow_bytes >= (64 << 20) else 3) * K,
-        "step_mode": step_mode, "eager_ms_per_step": eager_ms / K,
+        "metric": METRIC, "value": n_acc * world * K / (ms / 1e3), "unit": UNIT, "n_gpus": world, "steps": K,
+        "warmup": W, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "strong" if args.config == 5 else "weak", "vs_baseline": None,
+        "dtype": "u64" if rec_bytes == 8 else "u32", "data": "synthetic", "config": cb,
+        "roofline": roof, "roofline_step": res["roofline_step"], "roofline_l2": l2,
+        "cpu_baseline": cpu, "e2e": e2e,
+        "gpu_launches": res["launches_per_step"] * K,
+        "step_mode": res["step_mode"], "eager_ms_per_step": res["eager_ms_per_step"],
         "clocks": clocks.summary(),
-        "check": {"flagged_words": flagged, "per_step": st},  # stats are per step (reset clears them)
+        "check": {"flagged_words": res["flagged_words"], "expected_flagged": res["expected_flagged"],
+                  "per_step": st},  # stats are per step (reset clears them)
+        "per_config": per_config or None,
         "instrumented_slowdown": slow,
-        "shadow_overhead": {"bytes_per_tracked_word": c.rec_bytes, "ratio_to_tracked_bytes": c.rec_bytes / 4,
+        "shadow_overhead": {"bytes_per_tracked_word": rec_bytes, "ratio_to_tracked_bytes": rec_bytes / 4,
                             "iguard_ratio_context": 4.0},
     }
     print(json.dumps(out), flush=True)

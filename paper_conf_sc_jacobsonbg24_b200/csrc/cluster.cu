@@ -27,6 +27,7 @@
 
 #include "hirace.h"
 #include "hirace_device.cuh"
+#include "internal.h"
 
 namespace cg = cooperative_groups;
 using namespace hirace::cluster;
@@ -357,6 +358,7 @@ hirace_status hirace_cluster_reset(hirace_cluster_ctx *c, void *stream)
     if (!c)
         return HIRACE_E_INVAL;
     cudaStream_t st = (cudaStream_t)stream;
+    hirace_impl::note_launches(1);
     k_cluster_fill<<<c->sm_count * 4, 256, 0, st>>>(c->shadow, c->shadow_words);
     cudaError_t e = cudaGetLastError();
     if (e == cudaSuccess)
@@ -390,6 +392,7 @@ hirace_status hirace_cluster_replay(hirace_cluster_ctx *c, const hirace_event *d
     const unsigned char *table = c->table;
     void *args[] = {(void *)&ev, (void *)&nn, (void *)&shadow, (void *)&table, (void *)&G, (void *)&c->err,
                     (void *)&c->stats};
+    hirace_impl::note_launches(1);
     return cuda_status(cudaLaunchCooperativeKernel(p2 ? (const void *)k_cluster_replay<true> : (const void *)k_cluster_replay<false>, dim3(c->grid), dim3(kThreads),
                                                    args, 0, (cudaStream_t)stream));
 }
@@ -426,6 +429,7 @@ hirace_status hirace_cluster_collect(hirace_cluster_ctx *c, hirace_race *h_out, 
     if (e == cudaSuccess && m) {
         e = cudaMalloc(&d_rows, m * sizeof(hirace_race));
         if (e == cudaSuccess) {
+            hirace_impl::note_launches(1);
             k_cluster_rows<<<(unsigned)((m + 255) / 256), 256>>>(sel, m, c->shadow, c->race_class, c->global_words,
                                                                  c->smem_words ? c->smem_words : 1, d_rows);
             e = cudaGetLastError();

@@ -58,6 +58,14 @@ struct hirace_ctx {
     cudaStream_t copy_stream = nullptr;
     cudaEvent_t ev_copied[2] = {nullptr, nullptr}, ev_used[2] = {nullptr, nullptr};
     hirace_dev_ctx dev{};
+    /* window-major path (window.cu) */
+    int replay_mode = HIRACE_REPLAY_AUTO;
+    uint32_t win_log2 = 14;
+    WinDev win{};
+    uint64_t win_events_cap = 0;  /* events the window scratch is sized for */
+    hirace_event *d_trace = nullptr; /* whole-trace staging for hirace_check_trace_host */
+    uint64_t trace_cap = 0;
+    bool lazy = false;            /* a lazy reset left stale windows behind */
     uint32_t g = 0;
     cudaEvent_t t_start = nullptr, t_stop = nullptr;
     hirace_status sticky = HIRACE_OK;
@@ -105,14 +113,210 @@ hirace_status device_errors(hirace_ctx *c)
         set_sticky(c, HIRACE_E_BAD_TRACE);
     if (flags & hirace::ERR_CLOCK)
         set_sticky(c, HIRACE_E_CLOCK_OVERFLOW);
+    if (flags & ERR_CAPACITY)
+        set_sticky(c, HIRACE_E_NOMEM);
     return c->sticky;
+}
+
+constexpr uint64_t kWindowAutoBytes = 1ull << 30; /* AUTO: window-major for shadows >= 1 GiB */
+constexpr uint32_t kWindowPadLog2 = 14;           /* shadow allocation padded to 2^14 records */
+
+/* does this context replay window-major? (8-byte records, 4-byte elements) */
+bool window_active(const hirace_ctx *c)
+{
+    if (c->rec_bytes != 8 || c->cfg.granularity_log2 != 2 || !c->win.gen)
+        return false;
+    if (c->replay_mode == HIRACE_REPLAY_WINDOW)
+        return true;
+    return c->replay_mode == HIRACE_REPLAY_AUTO && c->shadow_words * 8 >= kWindowAutoBytes;
+}
+
+/* window geometry + generation array for window size 2^wl records (all windows stale) */
+cudaError_t window_geometry(hirace_ctx *c, uint32_t wl)
+{
+    WinDev &W = c->win;
+    const uint64_t padded = ((c->shadow_words + (1ull << kWindowPadLog2) - 1) >> kWindowPadLog2) << kWindowPadLog2;
+    const uint64_t nw = padded >> wl;
+    if (nw + 1 >= (1ull << 31))
+        return cudaErrorInvalidValue;
+    uint32_t wb = 0;
+    while ((1ull << wb) < nw)
+        wb++;
+    if (wb > 9 + 12)
+        return cudaErrorInvalidValue;
+    if (W.gen)
+        cudaFree(W.gen);
+    W.gen = nullptr;
+    cudaError_t e;
+    if ((e = cudaMalloc(&W.gen, nw * sizeof(uint32_t))) != cudaSuccess)
+        return e;
+    if (!W.cur_gen && (e = cudaMalloc(&W.cur_gen, sizeof(uint32_t))) != cudaSuccess)
+        return e;
+    if ((e = cudaMemset(W.gen, 0, nw * sizeof(uint32_t))) != cudaSuccess)
+        return e;
+    const uint32_t one = 1;
+    if ((e = cudaMemcpy(W.cur_gen, &one, sizeof(one), cudaMemcpyHostToDevice)) != cudaSuccess)
+        return e;
+    W.wl = wl;
+    W.nw = (uint32_t)nw;
+    W.d0b = wb < 9 ? wb : 9;
+    W.d1b = wb - W.d0b;
+    W.p1 = 1u << 16;
+    W.p2 = 1u << 16;
+    W.heavy_cap = kWinHeavyCap;
+    const char *hf = getenv("HIRACE_WIN_HEAVY"); /* tests: force the heavy-window path */
+    W.heavy_force = hf ? (uint32_t)strtoul(hf, nullptr, 10) : 0u;
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, window_light_kernel(), 1024, (size_t)8 << wl);
+    W.light_ctas = (uint32_t)(c->sm_count * (occ > 0 ? occ : 1));
+    c->win_log2 = wl;
+    c->win_events_cap = 0; /* per-size scratch is (re)allocated on the next check */
+    return cudaSuccess;
+}
+
+void window_free_scratch(WinDev &W)
+{
+    void *ptrs[] = {W.items1, W.item1_first, W.batch_key, W.count1, W.count2, W.rec1,
+                    W.rec2 != W.rec1 ? W.rec2 : nullptr, W.win_cnt, W.aux, W.heavy, W.light, W.hseg,
+                    W.partials, W.bar, W.elems};
+    for (void *p : ptrs)
+        if (p)
+            cudaFree(p);
+    W.items1 = nullptr;
+    W.item1_first = W.batch_key = W.count1 = W.count2 = W.win_cnt = W.aux = W.heavy = W.light = W.hseg = nullptr;
+    W.partials = nullptr;
+    W.rec1 = W.rec2 = nullptr;
+    W.bar = nullptr;
+    W.elems = nullptr;
+}
+
+/* per-check scratch sized for n events (grown on demand; never inside a graph capture: the
+ * warm-up call allocates) */
+cudaError_t window_scratch(hirace_ctx *c, uint64_t n)
+{
+    WinDev &W = c->win;
+    if (n <= c->win_events_cap && W.rec1)
+        return cudaSuccess;
+    cudaDeviceSynchronize();
+    window_free_scratch(W);
+    const uint64_t nb_max = HIRACE_MAX_BATCHES;
+    const uint64_t items1 = n / W.p1 + (n < nb_max ? n : nb_max) + 1;
+    const uint64_t elem_cap = n + n / 4 + 65536;
+    const uint64_t chunks2 = elem_cap / W.p2 + 2;
+    const uint64_t R0 = 1ull << W.d0b, R1 = 1ull << W.d1b;
+    if (items1 > 0xffffffffull || R0 * items1 > 0xffffffffull || R1 * chunks2 > 0xffffffffull ||
+        elem_cap >= 0xffffffffull)
+        return cudaErrorInvalidValue;
+    W.elem_cap = elem_cap;
+    W.items1_cap = (uint32_t)items1;
+    W.chunks2_cap = (uint32_t)chunks2;
+    cudaError_t e;
+#define WA(ptr, bytes)                                                                                              \
+    if ((e = cudaMalloc((void **)&(ptr), (bytes))) != cudaSuccess) {                                                 \
+        window_free_scratch(W);                                                                                      \
+        return e;                                                                                                    \
+    }
+    WA(W.items1, items1 * sizeof(uint4));
+    WA(W.item1_first, (nb_max + 1) * sizeof(uint32_t));
+    WA(W.batch_key, nb_max * sizeof(uint32_t));
+    WA(W.count1, R0 * items1 * sizeof(uint32_t));
+    WA(W.count2, W.d1b ? R1 * chunks2 * sizeof(uint32_t) : sizeof(uint32_t));
+    WA(W.rec1, elem_cap * sizeof(unsigned long long));
+    if (W.d1b) {
+        WA(W.rec2, elem_cap * sizeof(unsigned long long));
+    } else {
+        W.rec2 = W.rec1;
+    }
+    WA(W.win_cnt, ((uint64_t)W.nw + 1) * sizeof(uint32_t));
+    WA(W.aux, kAuxCount * sizeof(uint32_t));
+    WA(W.heavy, W.heavy_cap * sizeof(uint32_t));
+    WA(W.light, (uint64_t)W.nw * sizeof(uint32_t));
+    WA(W.hseg, (uint64_t)W.heavy_cap * (nb_max + 1) * sizeof(uint32_t));
+    WA(W.partials, kScanMaxCtas * sizeof(uint32_t));
+    WA(W.bar, kBarSlots * sizeof(unsigned int));
+    WA(W.elems, sizeof(unsigned long long));
+#undef WA
+    if ((e = cudaMemset(W.aux, 0, kAuxCount * sizeof(uint32_t))) != cudaSuccess)
+        return e;
+    c->win_events_cap = n;
+    return cudaSuccess;
+}
+
+/* stale windows := INIT before a path that reads or writes the shadow directly */
+hirace_status ensure_materialized(hirace_ctx *c, cudaStream_t st)
+{
+    if (!c->lazy)
+        return HIRACE_OK;
+    HR_CUDA(c, launch_materialize(c->dev, c->win, 0, c->sm_count, st));
+    c->lazy = false;
+    return HIRACE_OK;
+}
+
+/* a7 collection into device memory: the report buffer when it covers every flagged word (large
+ * shadows), else the ordered shadow scan; after a lazy reset the stale windows are made INIT
+ * first, and only when the scan actually runs */
+hirace_status collect_into(hirace_ctx *c, hirace_race *d_out, uint64_t cap, unsigned long long *d_total,
+                           cudaStream_t st)
+{
+    const int rm = report_mode(c);
+    if (c->lazy && rm) {
+        HR_CUDA(c, launch_collect_reports(c->dev, d_out, cap, d_total, st));
+        HR_CUDA(c, launch_materialize(c->dev, c->win, 1, c->sm_count, st));
+        HR_CUDA(c, launch_collect(c->dev, c->shadow_words, c->scr, d_out, cap, d_total, st, 2));
+        return HIRACE_OK;
+    }
+    if (ensure_materialized(c, st) != HIRACE_OK)
+        return c->sticky;
+    HR_CUDA(c, launch_collect(c->dev, c->shadow_words, c->scr, d_out, cap, d_total, st, rm));
+    return HIRACE_OK;
 }
 
 } // namespace
 
 extern "C" {
 
-const char *hirace_version(void) { return "hirace-b200 0.1 (sm_100a)"; }
+const char *hirace_version(void) { return "hirace-b200 0.2 (sm_100a)"; }
+
+hirace_status hirace_set_replay_mode(hirace_ctx *c, int mode, uint32_t window_log2)
+{
+    if (!c || mode < HIRACE_REPLAY_AUTO || mode > HIRACE_REPLAY_WINDOW || (window_log2 && (window_log2 < 5 || window_log2 > 14)))
+        return HIRACE_E_INVAL;
+    if (mode == HIRACE_REPLAY_WINDOW && (c->rec_bytes != 8 || c->cfg.granularity_log2 != 2))
+        return HIRACE_E_INVAL;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    HR_CUDA(c, cudaDeviceSynchronize());
+    const uint32_t wl = window_log2 ? window_log2 : 14u;
+    if (c->win.gen && wl != c->win_log2) {
+        window_free_scratch(c->win);
+        HR_CUDA(c, window_geometry(c, wl));
+    }
+    c->replay_mode = mode;
+    c->lazy = false;
+    /* the mode change starts from an all-INIT shadow (full reset: every window current) */
+    HR_CUDA(c, launch_reset(c->d_shadow, c->shadow_words * c->rec_bytes, c->d_report_count, c->d_stats, c->d_err,
+                            c->sm_count, nullptr));
+    HR_CUDA(c, cudaDeviceSynchronize());
+    c->g = 0;
+    c->dev.g = 0;
+    c->sticky = HIRACE_OK;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_get_replay_mode(const hirace_ctx *c, int *active_window)
+{
+    if (!c || !active_window)
+        return HIRACE_E_INVAL;
+    *active_window = window_active(c) ? 1 : 0;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_launch_count(uint64_t *out)
+{
+    if (!out)
+        return HIRACE_E_INVAL;
+    *out = launch_count();
+    return HIRACE_OK;
+}
 
 const char *hirace_status_string(hirace_status s)
 {
@@ -188,7 +392,8 @@ hirace_status shadow_alloc_impl(const hirace_config *cfg, const hirace_epoch_lim
         return HIRACE_E_INVAL;
     }
     c->scr.collect_grid = collect_max_grid(c->device);
-    if ((e = cudaMalloc(&c->d_shadow, c->shadow_words * c->rec_bytes)) != cudaSuccess ||
+    const uint64_t padded = ((c->shadow_words + (1ull << kWindowPadLog2) - 1) >> kWindowPadLog2) << kWindowPadLog2;
+    if ((e = cudaMalloc(&c->d_shadow, padded * c->rec_bytes)) != cudaSuccess ||
         (e = cudaMalloc(&c->d_table, 2048 + hirace::RAW_TABLE_BYTES)) != cudaSuccess ||
         (e = cudaMalloc(&c->d_reports, c->cfg.report_capacity * sizeof(hirace_race))) != cudaSuccess ||
         (e = cudaMalloc(&c->d_report_count, sizeof(unsigned long long))) != cudaSuccess ||
@@ -238,6 +443,8 @@ hirace_status shadow_alloc_impl(const hirace_config *cfg, const hirace_epoch_lim
     d.c_max_g = lim ? lim->max_g : 254u;
     d.c_max_b = lim ? lim->max_b : 1023u;
     d.c_max_w = lim ? lim->max_w : 511u;
+    if (c->rec_bytes == 8 && cfg->granularity_log2 == 2 && (e = window_geometry(c, 14)) != cudaSuccess)
+        return fail(e);
     if (hirace_shadow_reset(c, nullptr) != HIRACE_OK || cudaDeviceSynchronize() != cudaSuccess) {
         hirace_shadow_free(c);
         return HIRACE_E_CUDA;
@@ -274,6 +481,13 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
+    window_free_scratch(c->win);
+    if (c->win.gen)
+        cudaFree(c->win.gen);
+    if (c->win.cur_gen)
+        cudaFree(c->win.cur_gen);
+    if (c->d_trace)
+        cudaFree(c->d_trace);
     for (int i = 0; i < 2; i++) {
         if (c->ev_copied[i])
             cudaEventDestroy(c->ev_copied[i]);
@@ -327,8 +541,14 @@ hirace_status hirace_shadow_reset(hirace_ctx *c, void *stream)
         return HIRACE_E_INVAL;
     cudaStream_t st = (cudaStream_t)stream;
     HR_CUDA(c, cudaSetDevice(c->device));
-    HR_CUDA(c, launch_reset(c->d_shadow, c->shadow_words * c->rec_bytes, c->d_report_count, c->d_stats, c->d_err,
-                            c->sm_count, st));
+    if (window_active(c)) { /* lazy: the generation moves on, windows read as INIT (O(1)) */
+        HR_CUDA(c, launch_lazy_reset(c->dev, c->win, st));
+        c->lazy = true;
+    } else {
+        HR_CUDA(c, launch_reset(c->d_shadow, c->shadow_words * c->rec_bytes, c->d_report_count, c->d_stats, c->d_err,
+                                c->sm_count, st));
+        c->lazy = false;
+    }
     c->g = 0;
     c->dev.g = 0;
     c->sticky = HIRACE_OK;
@@ -345,6 +565,8 @@ hirace_status hirace_barrier(hirace_ctx *c, hirace_scope scope, void *stream)
         return set_sticky(c, HIRACE_E_INVAL);
     HR_CUDA(c, cudaSetDevice(c->device));
     if (c->g + 1 >= 255u) {
+        if (ensure_materialized(c, (cudaStream_t)stream) != HIRACE_OK)
+            return c->sticky;
         HR_CUDA(c, launch_rebase(c->dev, c->shadow_words, (cudaStream_t)stream));
         c->g = 0;
     } else {
@@ -366,10 +588,19 @@ hirace_status hirace_replay_trace(hirace_ctx *c, const hirace_event *d_events, u
         return set_sticky(c, HIRACE_E_INVAL);
     cudaStream_t st = (cudaStream_t)stream;
     HR_CUDA(c, cudaSetDevice(c->device));
+    const bool win = window_active(c);
+    if (win)
+        HR_CUDA(c, window_scratch(c, n));
+    else if (ensure_materialized(c, st) != HIRACE_OK)
+        return c->sticky;
     HR_CUDA(c, launch_find_batches(d_events, (uint32_t)n, c->scr, c->d_err, c->sm_count, st));
     if (c->t_start)
         HR_CUDA(c, cudaEventRecord(c->t_start, st));
-    HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st));
+    if (win)
+        HR_CUDA(c, launch_window_check(c->dev, c->win, c->scr, d_events, (uint32_t)n, c->sm_count, c->replay_grid, st,
+                                       c->shadow_words, nullptr, 0, nullptr));
+    else
+        HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st));
     if (c->t_stop)
         HR_CUDA(c, cudaEventRecord(c->t_stop, st));
     return HIRACE_OK;
@@ -428,11 +659,20 @@ hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_eve
     HR_CUDA(c, cudaSetDevice(c->device));
     if (n == 0)
         return hirace_collect_races_device(c, d_out, cap, d_n_total, stream);
+    const bool win = window_active(c);
+    if (win)
+        HR_CUDA(c, window_scratch(c, n));
+    else if (ensure_materialized(c, st) != HIRACE_OK)
+        return c->sticky;
     HR_CUDA(c, launch_find_batches(d_events, (uint32_t)n, c->scr, c->d_err, c->sm_count, st));
     if (c->t_start)
         HR_CUDA(c, cudaEventRecord(c->t_start, st));
-    HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st, c->shadow_words, d_out, cap, d_n_total,
-                             report_mode(c)));
+    if (win)
+        HR_CUDA(c, launch_window_check(c->dev, c->win, c->scr, d_events, (uint32_t)n, c->sm_count, c->replay_grid, st,
+                                       c->shadow_words, d_out, cap, d_n_total));
+    else
+        HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st, c->shadow_words, d_out, cap, d_n_total,
+                                 report_mode(c)));
     if (c->t_stop)
         HR_CUDA(c, cudaEventRecord(c->t_stop, st));
     return HIRACE_OK;
@@ -444,8 +684,8 @@ hirace_status hirace_collect_races_device(hirace_ctx *c, hirace_race *d_out, uin
     if (!c || !d_n_total || (cap && !d_out))
         return HIRACE_E_INVAL;
     HR_CUDA(c, cudaSetDevice(c->device));
-    HR_CUDA(c, launch_collect(c->dev, c->shadow_words, c->scr, d_out, cap, d_n_total, (cudaStream_t)stream,
-                              report_mode(c)));
+    if (collect_into(c, d_out, cap, d_n_total, (cudaStream_t)stream) != HIRACE_OK)
+        return c->sticky;
     return c->sticky;
 }
 
@@ -463,7 +703,8 @@ hirace_status hirace_collect_races(hirace_ctx *c, hirace_race *h_out, uint64_t c
         HR_CUDA(c, cudaMalloc(&c->d_collect, cap * sizeof(hirace_race)));
         c->collect_cap = cap;
     }
-    HR_CUDA(c, launch_collect(c->dev, c->shadow_words, c->scr, c->d_collect, cap, c->d_total, st, report_mode(c)));
+    if (collect_into(c, c->d_collect, cap, c->d_total, st) != HIRACE_OK)
+        return c->sticky;
     unsigned long long total = 0;
     HR_CUDA(c, cudaMemcpyAsync(&total, c->d_total, sizeof(total), cudaMemcpyDeviceToHost, st));
     HR_CUDA(c, cudaStreamSynchronize(st));
@@ -483,6 +724,24 @@ hirace_status hirace_check_trace_host(hirace_ctx *c, const hirace_event *h_event
         return c->sticky;
     cudaStream_t st = (cudaStream_t)stream;
     HR_CUDA(c, cudaSetDevice(c->device));
+    if (window_active(c) && n) {
+        /* window-major: the partition needs the whole trace; stage it in HBM (chunked copies on
+         * the copy stream), then one check */
+        if (n > c->trace_cap) {
+            HR_CUDA(c, cudaStreamSynchronize(st));
+            if (c->d_trace)
+                cudaFree(c->d_trace);
+            c->d_trace = nullptr;
+            c->trace_cap = 0;
+            HR_CUDA(c, cudaMalloc(&c->d_trace, n * sizeof(hirace_event)));
+            c->trace_cap = n;
+        }
+        HR_CUDA(c, cudaMemcpyAsync(c->d_trace, h_events, n * sizeof(hirace_event), cudaMemcpyHostToDevice, st));
+        hirace_status s = hirace_replay_trace(c, c->d_trace, n, stream);
+        if (s != HIRACE_OK)
+            return s;
+        return hirace_collect_races(c, h_out, cap, n_total, stream);
+    }
     const uint64_t chunk = 1ull << 22; /* 4 Mi events = 64 MiB per staging buffer */
     if (!c->copy_stream) {
         HR_CUDA(c, cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
@@ -560,6 +819,11 @@ hirace_status hirace_get_dev_ctx(hirace_ctx *c, const void *global_base, hirace_
 {
     if (!c || !out || c->rec_bytes != 8) /* inline hooks use the 8-byte record */
         return HIRACE_E_INVAL;
+    if (c->lazy) { /* inline hooks update the shadow in place: no stale windows */
+        HR_CUDA(c, cudaSetDevice(c->device));
+        if (ensure_materialized(c, nullptr) != HIRACE_OK)
+            return c->sticky;
+    }
     *out = c->dev;
     out->global_base = global_base;
     out->g = c->g;
@@ -838,6 +1102,8 @@ hirace_status hirace_replay_wire(hirace_ctx *c, const uint64_t *d_wire, uint64_t
         return set_sticky(c, HIRACE_E_INVAL);
     cudaStream_t st = (cudaStream_t)stream;
     HR_CUDA(c, cudaSetDevice(c->device));
+    if (ensure_materialized(c, st) != HIRACE_OK)
+        return c->sticky;
     if (c->t_start)
         HR_CUDA(c, cudaEventRecord(c->t_start, st));
     HR_CUDA(c, launch_replay_wire(c->dev, reinterpret_cast<const unsigned long long *>(d_wire), (uint32_t)n, batch_key,

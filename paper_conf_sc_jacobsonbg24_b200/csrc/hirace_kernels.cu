@@ -8,6 +8,7 @@
  *   k_rebase                          a8  grid-epoch wrap sweep
  *   k_bucket_*                        a10 owner bucketing for the address-sharded mode
  */
+#include <atomic>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -158,6 +159,7 @@ cudaError_t launch_find_batches(const hirace_event *ev, uint32_t n, const Scratc
                                 int sm_count, cudaStream_t st)
 {
     (void)sm_count;
+    note_launches(1);
     k_batches<<<1, kFindThreads, sizeof(FindSmem), st>>>(ev, n, s.batch_off, s.nbatches, s.batch_ctr, err,
                                                          s.grid_bar);
     return cudaGetLastError();
@@ -190,6 +192,7 @@ __global__ void k_rebase(unsigned long long *shadow, uint64_t nwords)
 
 cudaError_t launch_rebase(const hirace_dev_ctx &c, uint64_t shadow_words, cudaStream_t st)
 {
+    note_launches(1);
     k_rebase<<<148 * 8, 256, 0, st>>>(c.shadow, shadow_words);
     return cudaGetLastError();
 }
@@ -350,6 +353,7 @@ cudaError_t launch_bucket(const hirace_dev_ctx &c, const hirace_event *in, uint3
                           hirace_event *out, unsigned long long *d_counts, uint32_t *d_tile_hist, uint32_t ntiles,
                           cudaStream_t st)
 {
+    note_launches(3);
     k_bucket_hist<<<ntiles, kBucketThreads, 0, st>>>(in, n, nranks, my_rank, d_tile_hist, c.error_flags);
     k_bucket_scan<<<1, 1024, 0, st>>>(d_tile_hist, ntiles, nranks, d_counts);
     k_bucket_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, n, nranks, my_rank, d_tile_hist, out);
@@ -529,6 +533,7 @@ cudaError_t launch_bucket_wire(const hirace_event *in, uint32_t lo, uint32_t hi,
     const uint32_t ntiles = (hi - lo + kBucketTile - 1) / kBucketTile;
     if (ntiles == 0)
         return cudaMemsetAsync(d_counts_row, 0, nranks * sizeof(unsigned long long), st);
+    note_launches(3);
     k_wire_hist<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_hist, err);
     k_wire_scan<<<1, 1024, 0, st>>>(d_tile_hist, ntiles, nranks, d_running, d_counts_row, d_tile_off);
     if (out)
@@ -590,6 +595,7 @@ cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t h
     const uint32_t ntiles = (hi - lo + kBucketTile - 1) / kBucketTile;
     if (ntiles == 0)
         return cudaSuccess;
+    note_launches(3);
     k_wire_hist<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_hist, err);
     k_wire_scan_peer<<<1, 1024, 0, st>>>(d_tile_hist, ntiles, nranks, d_owner_base, d_tile_off);
     k_wire_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_off, nullptr, 0, err,
@@ -620,11 +626,24 @@ cudaError_t launch_reset(void *shadow, uint64_t bytes, unsigned long long *repor
     uint64_t blocks = (n16 + 255) / 256;
     const uint64_t cap = (uint64_t)(sm_count > 0 ? sm_count : 148) * 8;
     blocks = blocks < 1 ? 1 : (blocks > cap ? cap : blocks);
+    note_launches(1);
     k_reset<<<(unsigned)blocks, 256, 0, st>>>(reinterpret_cast<uint4 *>(shadow), n16, report_count, stats, err);
     cudaError_t e = cudaGetLastError();
     if (e == cudaSuccess && (bytes & 15)) /* shadow sizes are multiples of 4: a ragged 4/8/12-byte tail */
         e = cudaMemsetAsync(static_cast<char *>(shadow) + n16 * 16, 0, bytes & 15, st);
     return e;
+}
+
+static std::atomic<unsigned long long> g_launches{0};
+
+void note_launches(unsigned k)
+{
+    g_launches.fetch_add(k, std::memory_order_relaxed);
+}
+
+unsigned long long launch_count()
+{
+    return g_launches.load(std::memory_order_relaxed);
 }
 
 cudaError_t kernels_init(int device)
@@ -633,7 +652,9 @@ cudaError_t kernels_init(int device)
     cudaError_t e = cudaFuncSetAttribute(k_batches, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(FindSmem));
     if (e != cudaSuccess)
         return e;
-    return replay_init();
+    if ((e = replay_init()) != cudaSuccess)
+        return e;
+    return window_init();
 }
 
 } // namespace hirace_impl

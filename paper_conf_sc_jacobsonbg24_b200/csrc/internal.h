@@ -40,9 +40,14 @@ cudaError_t launch_replay(const hirace_dev_ctx &c, const hirace_event *ev, const
                           unsigned long long *d_total = nullptr, int report_mode = 0);
 int collect_max_grid(int device);
 int replay_max_grid(int device);
-/* order-preserving compaction of RACE records from the shadow */
+/* order-preserving compaction of RACE records from the shadow; report_mode 1: the report
+ * buffer first (k_collect_reports), the scan only if it does not cover; 2: the same, with
+ * k_collect_reports already launched by the caller */
 cudaError_t launch_collect(const hirace_dev_ctx &c, uint64_t shadow_words, const Scratch &s, hirace_race *out,
                            uint64_t cap, unsigned long long *d_total, cudaStream_t st, int report_mode = 0);
+/* one-CTA report-buffer collect (sort + unique of the reported keys) */
+cudaError_t launch_collect_reports(const hirace_dev_ctx &c, hirace_race *out, uint64_t cap,
+                                   unsigned long long *d_total, cudaStream_t st);
 /* report mode pays off above this shadow size (a scan of it costs more than a launch + sort) */
 constexpr uint64_t kReportModeMinBytes = 64ull << 20;
 cudaError_t replay_init();
@@ -70,6 +75,58 @@ cudaError_t launch_replay_wire(const hirace_dev_ctx &c, const unsigned long long
                                int grid, cudaStream_t st);
 constexpr int kWireTile = 4096;
 cudaError_t kernels_init(int device);
+
+/* ---- window-major replay (window.cu; DESIGN.md §8 "window-major path") ------------------
+ * The shadow is cut into windows of 2^wl records.  Element accesses are partitioned by window
+ * with one or two counting-sort passes (digits d0 = low d0b bits of the window id, d1 = the
+ * rest), keeping batch order inside every window; each light window is then replayed by one
+ * CTA with its records in shared memory (TMA bulk copies in and out, shared-memory CAS,
+ * __syncthreads between batches instead of grid barriers), heavy windows by all CTAs through
+ * the global shadow.  Lazy reset: a window whose gen[] differs from *cur_gen is all-INIT. */
+struct WinDev {
+    uint32_t wl, d0b, d1b, nw;   /* window = 2^wl records; nw windows; digits              */
+    uint32_t p1, p2;             /* events per pass-1 item, records per pass-2 chunk       */
+    uint32_t heavy_cap;          /* max heavy windows                                      */
+    uint32_t heavy_force;        /* != 0: heavy threshold override (tests: HIRACE_WIN_HEAVY) */
+    uint32_t light_ctas;         /* CTAs of the light kernel                               */
+    uint64_t elem_cap;           /* capacity of rec1/rec2 (element accesses)               */
+    uint32_t items1_cap, chunks2_cap;
+    uint4 *items1;               /* pass-1 items {start, end, batch, 0}                    */
+    uint32_t *item1_first;       /* [nb + 1] first item of each batch                      */
+    uint32_t *batch_key;         /* [nb] batch key (g:8 | b:10 | w:9)                      */
+    uint32_t *count1, *count2;   /* digit x item count matrices, scanned in place          */
+    unsigned long long *rec1, *rec2;
+    uint32_t *win_cnt;           /* [nw + 1] counts, scanned in place into window starts   */
+    uint32_t *aux;               /* kAux* slots                                            */
+    uint32_t *heavy, *light;     /* window lists                                           */
+    uint32_t *hseg;              /* [heavy_cap][nb + 1] batch starts inside heavy windows  */
+    uint32_t *gen, *cur_gen;     /* window generation (lazy reset)                         */
+    uint32_t *partials;          /* scan scratch (kScanMaxCtas)                            */
+    unsigned long long *elems;   /* element accesses counted by pass 1                     */
+    unsigned int *bar;           /* grid-barrier counters (kBarSlots)                      */
+};
+enum : uint32_t { kAuxItems1 = 0, kAuxTotal1, kAuxChunks2, kAuxTotal2, kAuxNHeavy, kAuxNLight, kAuxQueue,
+                  kAuxAbort, kAuxCount = 16 };
+constexpr int kScanMaxCtas = 1024;
+constexpr int kBarSlots = 8;
+constexpr uint32_t kWinHeavyCap = 64;
+constexpr uint32_t ERR_CAPACITY = 8u; /* window path: more element accesses than rec1/rec2 hold */
+/* the whole window-major check: partition, heavy + light replay, then (d_total != null) the
+ * collect into out / d_total */
+cudaError_t launch_window_check(const hirace_dev_ctx &c, const WinDev &W, const Scratch &s, const hirace_event *ev,
+                                uint32_t n, int sm_count, int replay_grid, cudaStream_t st, uint64_t shadow_words,
+                                hirace_race *out, uint64_t cap, unsigned long long *d_total);
+/* lazy reset: ++*cur_gen, report count / stats / error flags := 0 */
+cudaError_t launch_lazy_reset(const hirace_dev_ctx &c, const WinDev &W, cudaStream_t st);
+/* stale windows := INIT (all of them, or only when the report buffer does not cover the
+ * flagged words and a shadow scan will follow) */
+cudaError_t launch_materialize(const hirace_dev_ctx &c, const WinDev &W, int only_if_scan, int sm_count,
+                               cudaStream_t st);
+const void *window_light_kernel();
+cudaError_t window_init();
+/* process-wide count of kernels the library has launched (hirace_launch_count) */
+void note_launches(unsigned k);
+unsigned long long launch_count();
 
 } // namespace hirace_impl
 

@@ -26,6 +26,7 @@ STATUS = {0: "HIRACE_OK", -1: "HIRACE_E_INVAL", -2: "HIRACE_E_NOMEM", -3: "HIRAC
           -7: "HIRACE_E_COMM"}
 
 POLICY_STRICT, POLICY_RELAXED_READ_ATOMIC = 0, 1
+REPLAY_AUTO, REPLAY_BATCH, REPLAY_WINDOW = 0, 1, 2
 
 # every symbol include/hirace.h declares (checked by tests/test_abi.py against the header)
 EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_free", "hirace_shadow_reset", "hirace_barrier",
@@ -38,7 +39,7 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_fsm_table_cluster", "hirace_fsm_cluster_class", "hirace_fsm_step_cluster",
            "hirace_cluster_alloc", "hirace_cluster_free", "hirace_cluster_reset", "hirace_cluster_replay",
            "hirace_cluster_collect", "hirace_cluster_get_stats", "hirace_status_string",
-           "hirace_version")
+           "hirace_version", "hirace_launch_count", "hirace_set_replay_mode", "hirace_get_replay_mode")
 
 
 class HiraceError(RuntimeError):
@@ -136,6 +137,9 @@ def load():
         "hirace_cluster_get_stats": (I32, [P, ctypes.POINTER(U64), ctypes.POINTER(U64)]),
         "hirace_status_string": (ctypes.c_char_p, [I32]),
         "hirace_version": (ctypes.c_char_p, []),
+        "hirace_launch_count": (I32, [ctypes.POINTER(U64)]),
+        "hirace_set_replay_mode": (I32, [P, I32, U32]),
+        "hirace_get_replay_mode": (I32, [P, ctypes.POINTER(I32)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -233,6 +237,12 @@ def microbench_indexed(words_ptr: int, idx_ptr: int, n: int, op: int = 3, ctas_p
     _check(load().hirace_microbench_indexed(device, words_ptr, idx_ptr, n, op, ctas_per_sm, ctypes.byref(ms),
                                             _stream_handle(stream)), "microbench_indexed")
     return ms.value
+
+
+def launch_count() -> int:
+    v = ctypes.c_uint64(0)
+    _check(load().hirace_launch_count(ctypes.byref(v)), "hirace_launch_count")
+    return int(v.value)
 
 
 def _stream_handle(stream):
@@ -406,6 +416,20 @@ class Checker:
         a = ctypes.c_void_p(start.cuda_event if start is not None else 0)
         b = ctypes.c_void_p(stop.cuda_event if stop is not None else 0)
         _check(self.lib.hirace_set_kernel_timing(self.h, a, b), "hirace_set_kernel_timing")
+
+    def set_replay_mode(self, mode: int, window_log2: int = 0):
+        """REPLAY_AUTO / REPLAY_BATCH / REPLAY_WINDOW (include/hirace.h); resets the shadow."""
+        _check(self.lib.hirace_set_replay_mode(self.h, mode, window_log2), "hirace_set_replay_mode")
+
+    @property
+    def window_active(self) -> bool:
+        v = ctypes.c_int(0)
+        _check(self.lib.hirace_get_replay_mode(self.h, ctypes.byref(v)), "hirace_get_replay_mode")
+        return bool(v.value)
+
+    def launches(self) -> int:
+        """Kernels the library has launched so far (process-wide, hirace_launch_count)."""
+        return launch_count()
 
     def stats(self) -> dict:
         v = [ctypes.c_uint64(0) for _ in range(5)]
