@@ -499,6 +499,9 @@ def measure_single(args, config: int, variant: str, K: int, W: int, dev: int, cl
     trace = make_trace(config, variant)
     n_acc = word_accesses(trace.events)
     c = hr.Checker.for_trace(trace, device=dev, compact=args.compact)
+    if args.replay_mode != "auto":
+        c.set_replay_mode({"batch": hr.REPLAY_BATCH, "window": hr.REPLAY_WINDOW}[args.replay_mode], args.window_log2)
+    window = c.window_active
     d_ev = hr.events_to_device(trace.events, f"cuda:{dev}")
     cap = 1 << 20
     d_out = torch.empty(cap * 16, dtype=torch.uint8, device=f"cuda:{dev}")
@@ -574,6 +577,7 @@ def measure_single(args, config: int, variant: str, K: int, W: int, dev: int, cl
     achieved = bpa * n_acc / (kern_ms / 1e3) / 1e9
     key = f"cfg{config}_{variant}" + ("_compact" if args.compact else "")
     res = {"config": config, "variant": variant, "trace": trace.name, "events": int(trace.n), "accesses": n_acc,
+           "replay": "window-major" if window else "batch-major",
            "value": n_acc * K / (ms / 1e3), "ms_per_step": ms_per_step, "step_mode": step_mode,
            "eager_ms_per_step": eager_ms / K, "launches_per_step": launches_per_step,
            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
@@ -641,6 +645,9 @@ def main():
     ap.add_argument("--no-slowdown", action="store_true")
     ap.add_argument("--no-per-config", action="store_true", help="skip the config 2/3/4 secondary measurements")
     ap.add_argument("--no-graph", action="store_true", help="time the eager step instead of its CUDA graph")
+    ap.add_argument("--replay-mode", default="auto", choices=["auto", "batch", "window"],
+                    help="hirace_set_replay_mode: batch-major k_replay or window-major (auto: window for >= 1 GiB)")
+    ap.add_argument("--window-log2", type=int, default=0, help="records per window (log2; 0 = 14)")
     ap.add_argument("--compact", action="store_true",
                     help="compact 4-byte shadow records (hirace_shadow_alloc_compact, SURVEY §8(f) f1)")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p", "host"],

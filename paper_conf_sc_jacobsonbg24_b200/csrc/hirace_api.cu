@@ -167,7 +167,8 @@ cudaError_t window_geometry(hirace_ctx *c, uint32_t wl)
     const char *hf = getenv("HIRACE_WIN_HEAVY"); /* tests: force the heavy-window path */
     W.heavy_force = hf ? (uint32_t)strtoul(hf, nullptr, 10) : 0u;
     int occ = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, window_light_kernel(), 1024, (size_t)8 << wl);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, window_light_kernel(), window_light_threads(),
+                                                  window_light_smem(wl));
     W.light_ctas = (uint32_t)(c->sm_count * (occ > 0 ? occ : 1));
     c->win_log2 = wl;
     c->win_events_cap = 0; /* per-size scratch is (re)allocated on the next check */
@@ -221,9 +222,9 @@ cudaError_t window_scratch(hirace_ctx *c, uint64_t n)
     WA(W.batch_key, nb_max * sizeof(uint32_t));
     WA(W.count1, R0 * items1 * sizeof(uint32_t));
     WA(W.count2, W.d1b ? R1 * chunks2 * sizeof(uint32_t) : sizeof(uint32_t));
-    WA(W.rec1, elem_cap * sizeof(unsigned long long));
+    WA(W.rec1, (elem_cap + 2) * sizeof(unsigned long long)); /* +2: 16-byte aligned bulk reads */
     if (W.d1b) {
-        WA(W.rec2, elem_cap * sizeof(unsigned long long));
+        WA(W.rec2, (elem_cap + 2) * sizeof(unsigned long long));
     } else {
         W.rec2 = W.rec1;
     }
@@ -670,6 +671,14 @@ hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_eve
     if (win)
         HR_CUDA(c, launch_window_check(c->dev, c->win, c->scr, d_events, (uint32_t)n, c->sm_count, c->replay_grid, st,
                                        c->shadow_words, d_out, cap, d_n_total));
+    if (win && getenv("HIRACE_WIN_VALIDATE")) { /* diagnostics: synchronous */
+        uint32_t aux[kAuxCount];
+        HR_CUDA(c, cudaStreamSynchronize(st));
+        HR_CUDA(c, cudaMemcpy(aux, c->win.aux, sizeof(aux), cudaMemcpyDeviceToHost));
+        fprintf(stderr, "window check: items1 %u total1 %u chunks2 %u heavy %u light %u abort %u violations %u\n",
+                aux[kAuxItems1], aux[kAuxTotal1], aux[kAuxChunks2], aux[kAuxNHeavy], aux[kAuxNLight], aux[kAuxAbort],
+                aux[kAuxViolations]);
+    }
     else
         HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st, c->shadow_words, d_out, cap, d_n_total,
                                  report_mode(c)));

@@ -106,7 +106,7 @@ struct WinDev {
     unsigned int *bar;           /* grid-barrier counters (kBarSlots)                      */
 };
 enum : uint32_t { kAuxItems1 = 0, kAuxTotal1, kAuxChunks2, kAuxTotal2, kAuxNHeavy, kAuxNLight, kAuxQueue,
-                  kAuxAbort, kAuxCount = 16 };
+                  kAuxAbort, kAuxViolations, kAuxCount = 16 };
 constexpr int kScanMaxCtas = 1024;
 constexpr int kBarSlots = 8;
 constexpr uint32_t kWinHeavyCap = 64;
@@ -123,6 +123,8 @@ cudaError_t launch_lazy_reset(const hirace_dev_ctx &c, const WinDev &W, cudaStre
 cudaError_t launch_materialize(const hirace_dev_ctx &c, const WinDev &W, int only_if_scan, int sm_count,
                                cudaStream_t st);
 const void *window_light_kernel();
+int window_light_threads();
+size_t window_light_smem(uint32_t wl);
 cudaError_t window_init();
 /* process-wide count of kernels the library has launched (hirace_launch_count) */
 void note_launches(unsigned k);

@@ -34,6 +34,7 @@
  */
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "collect.cuh"
 #include "hirace_device.cuh"
@@ -47,7 +48,8 @@ namespace hirace_impl {
 namespace {
 
 constexpr int kPassThreads = 512;
-constexpr int kLightThreads = 1024;
+constexpr int kLightThreads = 512;
+constexpr uint32_t kRing = 2048; /* records per ring buffer (16 KB) */
 constexpr uint32_t kMaxD0 = 512, kMaxD1 = 4096;
 using u64 = unsigned long long;
 
@@ -101,17 +103,22 @@ __device__ __forceinline__ Elems elems_of(const uint4 &e, uint32_t key, const hi
     return E;
 }
 
-/* ---- device-sized exclusive scan (cooperative: one grid barrier) --------------------------
- * a[0 .. rows * (*cols) + extra) in place; *total_out = the sum; optional derived slot
- * *ceil_out = ceil(sum / ceil_div); sum > cap raises ERR_CAPACITY and sets *abort. */
-__global__ void __launch_bounds__(1024) k_w_scan(uint32_t *a, uint32_t rows, const uint32_t *cols, uint32_t extra,
-                                                 uint32_t *partials, unsigned int *bar, uint32_t *total_out,
-                                                 uint32_t *ceil_out, uint32_t ceil_div,
-                                                 const unsigned long long *check_total, uint64_t cap,
-                                                 uint32_t *abort, unsigned int *err)
+/* ---- device-sized exclusive scan: three plain launches (reduce, scan of the partials, apply).
+ * a[0 .. rows * (*cols) + extra) in place (cols null: extra elements); *total_out = the sum;
+ * optional *ceil_out = ceil(sum / ceil_div); a check_total above cap raises ERR_CAPACITY and
+ * sets *abort (every later window kernel then stands down).  G = the grid of the reduce and
+ * apply launches (a kernel argument, so every launch splits the array the same way). */
+__device__ __forceinline__ uint64_t scan_n(uint32_t rows, const uint32_t *cols, uint32_t extra)
+{
+    return (cols ? (uint64_t)rows * *cols : 0ull) + extra;
+}
+
+__global__ void __launch_bounds__(1024) k_w_scan_reduce(const uint32_t *a, uint32_t rows, const uint32_t *cols,
+                                                        uint32_t extra, uint32_t G, uint32_t *partials,
+                                                        const unsigned long long *check_total, uint64_t cap,
+                                                        uint32_t *abort, unsigned int *err)
 {
     __shared__ uint32_t s_w[32];
-    __shared__ uint32_t s_pre;
     if (*abort)
         return;
     if (check_total && *check_total > cap) { /* the records would not fit rec1 / rec2 */
@@ -121,29 +128,45 @@ __global__ void __launch_bounds__(1024) k_w_scan(uint32_t *a, uint32_t rows, con
         }
         return;
     }
-    const uint64_t n = (uint64_t)rows * (cols ? *cols : 1u) + extra;
-    const uint32_t G = gridDim.x, cta = blockIdx.x;
-    const uint64_t lo = n * cta / G, hi = n * (cta + 1) / G;
+    const uint64_t n = scan_n(rows, cols, extra), chunk = (n + G - 1) / G;
+    const uint64_t lo = min(n, chunk * blockIdx.x), hi = min(n, lo + chunk);
     uint32_t sum = 0;
     for (uint64_t i = lo + threadIdx.x; i < hi; i += blockDim.x)
         sum += a[i];
     uint32_t tot;
     block_exclusive_scan(sum, s_w, &tot);
     if (threadIdx.x == 0)
-        partials[cta] = tot;
-    unsigned int epoch = 0;
-    grid_sync(bar, G, epoch);
-    uint32_t pre = 0;
-    for (uint32_t k = threadIdx.x; k < cta; k += blockDim.x)
-        pre += __ldcg(&partials[k]);
-    __syncthreads();
-    uint32_t dummy;
-    const uint32_t pe = block_exclusive_scan(pre, s_w, &dummy);
-    (void)pe;
-    if (threadIdx.x == 0)
-        s_pre = dummy;
-    __syncthreads();
-    uint32_t run = s_pre;
+        partials[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(1024) k_w_scan_partials(uint32_t *partials, uint32_t G, uint32_t *total_out,
+                                                          uint32_t *ceil_out, uint32_t ceil_div, const uint32_t *abort)
+{
+    __shared__ uint32_t s_w[32];
+    if (*abort)
+        return;
+    const uint32_t v = threadIdx.x < G ? partials[threadIdx.x] : 0u;
+    uint32_t tot;
+    const uint32_t ex = block_exclusive_scan(v, s_w, &tot);
+    if (threadIdx.x < G)
+        partials[threadIdx.x] = ex;
+    if (threadIdx.x == 0) {
+        if (total_out)
+            *total_out = tot;
+        if (ceil_out)
+            *ceil_out = (uint32_t)(((uint64_t)tot + ceil_div - 1) / ceil_div);
+    }
+}
+
+__global__ void __launch_bounds__(1024) k_w_scan_apply(uint32_t *a, uint32_t rows, const uint32_t *cols, uint32_t extra,
+                                                       uint32_t G, const uint32_t *partials, const uint32_t *abort)
+{
+    __shared__ uint32_t s_w[32];
+    if (*abort)
+        return;
+    const uint64_t n = scan_n(rows, cols, extra), chunk = (n + G - 1) / G;
+    const uint64_t lo = min(n, chunk * blockIdx.x), hi = min(n, lo + chunk);
+    uint32_t run = partials[blockIdx.x];
     constexpr int PER = 4;
     for (uint64_t base = lo; base < hi; base += (uint64_t)blockDim.x * PER) {
         uint32_t v[PER], mine = 0;
@@ -153,7 +176,6 @@ __global__ void __launch_bounds__(1024) k_w_scan(uint32_t *a, uint32_t rows, con
             v[k] = i0 + k < hi ? a[i0 + k] : 0u;
             mine += v[k];
         }
-        __syncthreads();
         uint32_t tile;
         uint32_t ex = block_exclusive_scan(mine, s_w, &tile) + run;
 #pragma unroll
@@ -163,13 +185,7 @@ __global__ void __launch_bounds__(1024) k_w_scan(uint32_t *a, uint32_t rows, con
             ex += v[k];
         }
         run += tile;
-    }
-    if (cta == G - 1 && threadIdx.x == 0) {
-        const uint64_t total = (uint64_t)run;
-        if (total_out)
-            *total_out = run;
-        if (ceil_out)
-            *ceil_out = (uint32_t)((total + ceil_div - 1) / ceil_div);
+        __syncthreads(); /* s_w reuse */
     }
 }
 
@@ -335,6 +351,176 @@ __global__ void __launch_bounds__(kPassThreads) k_w_pass2(WinDev W, const uint32
         if (!SCATTER)
             for (uint32_t d = threadIdx.x; d < R1; d += blockDim.x)
                 W.count2[(uint64_t)d * nc + ch] = s_cnt[d];
+        __syncthreads();
+    }
+}
+
+
+/* ---- scatter with per-digit sector buffers ------------------------------------------------
+ * Records go to their digit's output run through an 8-record shared-memory buffer; a flush
+ * writes only whole 32-byte sectors (4 records) of the run, so DRAM never sees a partial-sector
+ * write (which ECC turns into a read-modify-write) except at the two ends of each run of an
+ * item.  A digit that receives more than 8 records between flushes writes the excess straight
+ * to its final position (hot digits; still exact). */
+constexpr uint32_t kMaxBufDigits = 1024;
+template <uint32_t BUF, uint32_t RMAX> struct ScatterSmem {
+    u64 buf[RMAX * BUF];
+    uint32_t cnt[RMAX], done[RMAX], base[RMAX];
+};
+
+template <uint32_t BUF, uint32_t RMAX>
+__device__ __forceinline__ void sc_put(ScatterSmem<BUF, RMAX> &S, u64 *out, uint32_t d, u64 rec)
+{
+    const uint32_t slot = atomicAdd(&S.cnt[d], 1u);
+    if (slot - S.done[d] < BUF)
+        S.buf[d * BUF + (slot & (BUF - 1))] = rec;
+    else
+        out[S.base[d] + slot] = rec;
+}
+
+/* thread per digit: write the buffered records up to the last whole sector (all if final);
+ * 16-byte stores where the destination is 16-byte aligned */
+template <uint32_t BUF, uint32_t RMAX>
+__device__ __forceinline__ void sc_flush(ScatterSmem<BUF, RMAX> &S, u64 *out, uint32_t R, bool final)
+{
+    for (uint32_t d = threadIdx.x; d < R; d += blockDim.x) {
+        const uint32_t c = S.cnt[d], dn = S.done[d], base = S.base[d];
+        uint32_t e, nd;
+        if (c - dn > BUF) { /* overflowed: [dn + BUF, c) went straight out */
+            e = dn + BUF;
+            nd = c;
+        } else if (final) {
+            e = nd = c;
+        } else {
+            const uint32_t al = (base + c) & ~3u; /* last sector boundary of the run so far */
+            e = nd = al > base + dn ? al - base : dn;
+        }
+        const u64 *b = S.buf + d * BUF;
+        uint32_t k = dn;
+        if (k < e && ((base + k) & 1u)) {
+            out[base + k] = b[k & (BUF - 1)];
+            k++;
+        }
+        for (; k + 1 < e; k += 2) {
+            const u64 x = b[k & (BUF - 1)], y = b[(k + 1) & (BUF - 1)];
+            *reinterpret_cast<ulonglong2 *>(out + base + k) = make_ulonglong2(x, y);
+        }
+        if (k < e)
+            out[base + k] = b[k & (BUF - 1)];
+        S.done[d] = nd;
+    }
+}
+
+/* pass 1 scatter: per item (one batch), records into digit d0 order; EV events per thread per
+ * sub-tile between flushes */
+template <uint32_t BUF, uint32_t RMAX, int EV>
+__global__ void __launch_bounds__(kPassThreads) k_w_scatter1(hirace_dev_ctx c, const uint4 *__restrict__ ev, WinDev W)
+{
+    extern __shared__ __align__(16) unsigned char s_dyn[];
+    ScatterSmem<BUF, RMAX> &S = *reinterpret_cast<ScatterSmem<BUF, RMAX> *>(s_dyn);
+    if (W.aux[kAuxAbort])
+        return;
+    geom G = make_geom(c);
+    const uint64_t total_threads = (uint64_t)c.grid_blocks * c.block_threads;
+    const uint32_t tid_max = total_threads > 0xffffffffull ? 0xffffffffu : (uint32_t)(total_threads - 1);
+    const uint32_t ni = W.aux[kAuxItems1], R0 = 1u << W.d0b, wmask = (1u << W.wl) - 1u;
+    const bool two = W.d1b != 0;
+    const uint32_t T = blockDim.x;
+    uint32_t bad = 0;
+    for (uint32_t item = blockIdx.x; item < ni; item += gridDim.x) {
+        const uint4 it = W.items1[item];
+        for (uint32_t d = threadIdx.x; d < R0; d += T) {
+            S.cnt[d] = 0;
+            S.done[d] = 0;
+            S.base[d] = W.count1[(uint64_t)d * ni + item];
+        }
+        __syncthreads();
+        const uint32_t key = W.batch_key[it.z];
+        for (uint32_t i0 = it.x; i0 < it.y; i0 += T * EV) {
+            uint4 e[EV];
+#pragma unroll
+            for (int k = 0; k < EV; k++) {
+                const uint32_t i = i0 + k * T + threadIdx.x;
+                e[k] = i < it.y ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
+            }
+#pragma unroll
+            for (int k = 0; k < EV; k++) {
+                if (i0 + k * T + threadIdx.x < it.y) {
+                    const Elems E = elems_of(e[k], key, c, G, tid_max, bad);
+                    for (uint32_t q = 0; q < E.ne; q++) {
+                        const uint64_t idx = E.idx0 + q;
+                        const uint32_t win = (uint32_t)(idx >> W.wl);
+                        sc_put(S, W.rec1, win & (R0 - 1u),
+                               wrec((uint32_t)idx & wmask, E.kind, two ? (win >> W.d0b) : it.z, E.tid));
+                    }
+                }
+            }
+            __syncthreads();
+            sc_flush(S, W.rec1, R0, false);
+            __syncthreads();
+        }
+        sc_flush(S, W.rec1, R0, true);
+        __syncthreads();
+    }
+    (void)bad; /* reported by the count pass */
+}
+
+/* pass 2 scatter: per chunk of the pass-1 output, piece by piece ((d0, batch) segments in
+ * order), records into digit d1 order; the record's f field becomes the batch index */
+template <uint32_t BUF, uint32_t RMAX, int EV>
+__global__ void __launch_bounds__(kPassThreads) k_w_scatter2(WinDev W, const uint32_t *nbp)
+{
+    extern __shared__ __align__(16) unsigned char s_dyn[];
+    ScatterSmem<BUF, RMAX> &S = *reinterpret_cast<ScatterSmem<BUF, RMAX> *>(s_dyn);
+    if (W.aux[kAuxAbort])
+        return;
+    const uint32_t nb = *nbp, ni = W.aux[kAuxItems1], R0 = 1u << W.d0b, R1 = 1u << W.d1b;
+    const uint32_t total1 = W.aux[kAuxTotal1], nc = W.aux[kAuxChunks2];
+    const uint32_t nseg = R0 * nb, T = blockDim.x;
+    for (uint32_t ch = blockIdx.x; ch < nc; ch += gridDim.x) {
+        const uint32_t a = ch * W.p2, b = min(total1, a + W.p2);
+        for (uint32_t d = threadIdx.x; d < R1; d += T) {
+            S.cnt[d] = 0;
+            S.done[d] = 0;
+            S.base[d] = W.count2[(uint64_t)d * nc + ch];
+        }
+        uint32_t lo = 0, hi = nseg; /* last segment j with seg1(j) <= a */
+        while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (seg1(W, mid, nb, ni, R0, total1) <= a)
+                lo = mid;
+            else
+                hi = mid;
+        }
+        __syncthreads();
+        for (uint32_t j = lo; j < nseg; j++) {
+            const uint32_t s0 = max(a, seg1(W, j, nb, ni, R0, total1));
+            if (s0 >= b)
+                break;
+            const uint32_t s1 = min(b, seg1(W, j + 1, nb, ni, R0, total1));
+            if (s1 <= s0)
+                continue;
+            const uint32_t batch = j % nb;
+            for (uint32_t i0 = s0; i0 < s1; i0 += T * EV) {
+                u64 r[EV];
+#pragma unroll
+                for (int k = 0; k < EV; k++) {
+                    const uint32_t i = i0 + k * T + threadIdx.x;
+                    r[k] = i < s1 ? ld_rec(W.rec1 + i) : 0ull;
+                }
+#pragma unroll
+                for (int k = 0; k < EV; k++)
+                    if (i0 + k * T + threadIdx.x < s1) {
+                        const uint32_t lo32 = (uint32_t)r[k];
+                        sc_put(S, W.rec2, (lo32 >> 16) & (R1 - 1u),
+                               ((r[k] >> 32) << 32) | (u64)((lo32 & 0xffffu) | (batch << 16)));
+                    }
+                __syncthreads(); /* also: the next piece (next batch of this d0) lands after this one */
+                sc_flush(S, W.rec2, R1, false);
+                __syncthreads();
+            }
+        }
+        sc_flush(S, W.rec2, R1, true);
         __syncthreads();
     }
 }
@@ -519,22 +705,31 @@ __device__ __forceinline__ void light_step(u64 *sh, bool ok, uint32_t word, uint
     }
 }
 
-__global__ void __launch_bounds__(kLightThreads, 1) k_w_light(hirace_dev_ctx c, WinDev W, const uint32_t *nbp)
+/* Light-window replay.  Dynamic shared memory = [window records: 2^wl x 8 B][record ring:
+ * 2 x kRing x 8 B].  Per window: the window comes in by TMA bulk copy (or is zero-filled when
+ * stale), the window's access records stream through the two-buffer ring by TMA bulk copies
+ * (chunk k+2 is requested as soon as chunk k is consumed), each tile of blockDim records is
+ * processed by the whole CTA, with a __syncthreads where the batch changes, and the window goes
+ * back by TMA bulk copy while the next window starts. */
+__global__ void __launch_bounds__(kLightThreads, 2) k_w_light(hirace_dev_ctx c, WinDev W)
 {
     extern __shared__ __align__(128) unsigned char s_dyn[];
     __shared__ __align__(16) unsigned char s_raw[RAW_TABLE_BYTES];
     __shared__ unsigned long long s_stats[4];
-    __shared__ __align__(8) uint64_t s_mbar;
-    __shared__ uint32_t s_w, s_next;
+    __shared__ __align__(8) uint64_t s_mbar[3]; /* shadow, ring 0, ring 1 */
+    __shared__ uint32_t s_w;
     if (W.aux[kAuxAbort])
         return;
+    const uint32_t wsz = 1u << W.wl, wbytes = wsz * 8u, wmask = wsz - 1u;
     u64 *const sh = reinterpret_cast<u64 *>(s_dyn);
+    u64 *const ring = sh + wsz;
     for (int i = threadIdx.x; i < RAW_TABLE_BYTES / 16; i += blockDim.x)
         reinterpret_cast<uint4 *>(s_raw)[i] = __ldg(reinterpret_cast<const uint4 *>(c.table + 2048) + i);
     if (threadIdx.x < 4)
         s_stats[threadIdx.x] = 0;
     if (threadIdx.x == 0) {
-        mbar_init(&s_mbar, 1);
+        for (int k = 0; k < 3; k++)
+            mbar_init(&s_mbar[k], 1);
         fence_mbar_init();
     }
     __syncthreads();
@@ -542,10 +737,8 @@ __global__ void __launch_bounds__(kLightThreads, 1) k_w_light(hirace_dev_ctx c, 
     const Rec<u64> rec(c);
     const uint32_t lane = threadIdx.x & 31, below = (1u << lane) - 1;
     const uint32_t nl = W.aux[kAuxNLight], cur = *W.cur_gen;
-    const uint32_t wsz = 1u << W.wl, wbytes = wsz * 8u, wmask = wsz - 1u;
-    (void)nbp;
     Counters cnt{0, 0, 0, 0};
-    uint32_t phase = 0;
+    uint32_t ph_sh = 0, ph_ring = 0; /* mbarrier parities (bit k: ring buffer k) */
     for (;;) {
         if (threadIdx.x == 0)
             s_w = atomicAdd(&W.aux[kAuxQueue], 1u);
@@ -557,56 +750,77 @@ __global__ void __launch_bounds__(kLightThreads, 1) k_w_light(hirace_dev_ctx c, 
         const uint32_t beg = W.win_cnt[w], end = W.win_cnt[w + 1];
         u64 *const gw = reinterpret_cast<u64 *>(c.shadow) + ((uint64_t)w << W.wl);
         const bool fresh = W.gen[w] != cur;
-        /* the previous window's bulk store must have read shared memory before it is reused */
-        if (threadIdx.x == 0)
+        const uint32_t a0 = beg & ~1u, aend = (end + 1u) & ~1u; /* 16-byte aligned record range */
+        const uint32_t nch = (aend - a0 + kRing - 1) / kRing;
+        if (threadIdx.x == 0) {
+            /* the previous window's bulk store must have read shared memory before reuse */
             asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            for (uint32_t k = 0; k < 2 && k < nch; k++) {
+                const uint32_t s0 = a0 + k * kRing, m = min(kRing, aend - s0);
+                mbar_arrive_expect_tx(&s_mbar[1 + k], m * 8u);
+                bulk_g2s(ring + k * kRing, W.rec2 + s0, m * 8u, &s_mbar[1 + k]);
+            }
+            if (!fresh) {
+                mbar_arrive_expect_tx(&s_mbar[0], wbytes);
+                for (uint32_t o = 0; o < wbytes; o += 32768u)
+                    bulk_g2s(s_dyn + o, reinterpret_cast<const unsigned char *>(gw) + o, min(32768u, wbytes - o),
+                             &s_mbar[0]);
+            }
+        }
         __syncthreads();
         if (fresh) { /* lazy reset: a stale window is all INIT */
             for (uint32_t q = threadIdx.x; q < wsz / 2; q += blockDim.x)
                 reinterpret_cast<uint4 *>(sh)[q] = make_uint4(0, 0, 0, 0);
-        } else if (threadIdx.x == 0) {
-            mbar_arrive_expect_tx(&s_mbar, wbytes);
-            for (uint32_t o = 0; o < wbytes; o += 32768u)
-                bulk_g2s(s_dyn + o, reinterpret_cast<const unsigned char *>(gw) + o, min(32768u, wbytes - o), &s_mbar);
+        } else {
+            mbar_wait(&s_mbar[0], ph_sh);
+            ph_sh ^= 1u;
         }
-        /* first tile's records in flight while the window arrives */
-        uint32_t i = beg + threadIdx.x;
-        u64 r = i < end ? ld_rec(W.rec2 + i) : 0ull;
-        if (!fresh) {
-            mbar_wait(&s_mbar, phase);
-            phase ^= 1u;
-        }
-        __syncthreads();
-        uint32_t cur_b = (uint32_t)__ldg(W.rec2 + beg) >> 16;
-        for (uint32_t base = beg; base < end; base += blockDim.x, i += blockDim.x) {
-            const u64 rr = r;
-            const bool valid = i < end;
-            r = i + blockDim.x < end ? ld_rec(W.rec2 + i + blockDim.x) : 0ull; /* next tile */
-            const uint32_t lo32 = (uint32_t)rr, my_b = valid ? lo32 >> 16 : 0xffffffffu;
-            const uint32_t tid = (uint32_t)(rr >> 32), kind = (lo32 >> 14) & 3u, word = lo32 & wmask;
-            const uint32_t last = min(end, base + blockDim.x) - 1u;
-            const uint32_t hi_b = (uint32_t)__ldg(W.rec2 + last) >> 16;
-            uint32_t b = cur_b;
-            for (;;) {
-                const Batch B = make_batch<u64>(W.batch_key[b], rec);
-                light_step(sh, valid && my_b == b, word, tid, kind, B, 0, (uint64_t)w << W.wl, c, G, rec, s_raw, cnt,
-                           lane, below);
-                if (b == hi_b)
-                    break;
-                /* every access of batch b in this window is done before batch b' > b starts */
-                if (threadIdx.x == 0)
-                    s_next = 0xffffffffu;
-                __syncthreads();
-                const uint32_t cand = __reduce_min_sync(0xffffffffu, (valid && my_b > b) ? my_b : 0xffffffffu);
-                if (lane == 0 && cand != 0xffffffffu)
-                    atomicMin(&s_next, cand);
-                __syncthreads();
-                b = s_next;
+        uint32_t cur_b = 0xffffffffu;
+        for (uint32_t k = 0; k < nch; k++) {
+            const uint32_t bi = k & 1u;
+            mbar_wait(&s_mbar[1 + bi], (ph_ring >> bi) & 1u);
+            ph_ring ^= 1u << bi;
+            __syncthreads(); /* zero fill (first chunk) / previous chunk done */
+            const uint32_t c0 = a0 + k * kRing;
+            const u64 *const rb = ring + bi * kRing;
+            const uint32_t lo = max(beg, c0), hi = min(end, c0 + kRing);
+            if (cur_b == 0xffffffffu)
+                cur_b = (uint32_t)rb[lo - c0] >> 16;
+            for (uint32_t base = lo; base < hi; base += blockDim.x) {
+                const uint32_t i = base + threadIdx.x;
+                const bool valid = i < hi;
+                const u64 rr = valid ? rb[i - c0] : 0ull;
+                const uint32_t lo32 = (uint32_t)rr, my_b = valid ? lo32 >> 16 : 0xffffffffu;
+                const uint32_t tid = (uint32_t)(rr >> 32), kind = (lo32 >> 14) & 3u, word = lo32 & wmask;
+                const uint32_t hi_b = (uint32_t)rb[min(hi, base + blockDim.x) - 1u - c0] >> 16;
+                uint32_t b = cur_b;
+                for (;;) {
+                    if (__any_sync(0xffffffffu, valid && my_b == b)) { /* warp-uniform: records are batch-sorted */
+                        const Batch B = make_batch<u64>(W.batch_key[b], rec);
+                        light_step(sh, valid && my_b == b, word, tid, kind, B, 0, (uint64_t)w << W.wl, c, G, rec,
+                                   s_raw, cnt, lane, below);
+                    }
+                    if (b == hi_b)
+                        break;
+                    /* every access of batch b in this window is done before a later batch starts
+                     * (the barrier), and the tile is batch-sorted, so the next batch is the one of
+                     * the first record past the le records of batches <= b */
+                    const uint32_t le = (uint32_t)__syncthreads_count(valid && my_b <= b);
+                    b = (uint32_t)rb[base + le - c0] >> 16;
+                }
+                cur_b = hi_b;
             }
-            cur_b = hi_b;
+            __syncthreads(); /* this ring buffer is consumed */
+            if (threadIdx.x == 0 && k + 2 < nch) {
+                const uint32_t s0 = a0 + (k + 2) * kRing, m = min(kRing, aend - s0);
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_arrive_expect_tx(&s_mbar[1 + bi], m * 8u);
+                bulk_g2s(ring + bi * kRing, W.rec2 + s0, m * 8u, &s_mbar[1 + bi]);
+            }
         }
         __syncthreads();
-        /* write the window back (async proxy reads what the generic proxy wrote) */
+        /* write the window back (the async proxy reads what the generic proxy wrote) */
         if (threadIdx.x == 0) {
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             for (uint32_t o = 0; o < wbytes; o += 32768u)
@@ -621,6 +835,24 @@ __global__ void __launch_bounds__(kLightThreads, 1) k_w_light(hirace_dev_ctx c, 
     if (threadIdx.x == 0)
         asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
     flush_stats(c, cnt, s_stats, lane);
+}
+
+/* diagnostics (HIRACE_WIN_VALIDATE): records of every window batch-sorted, per-window counts
+ * consistent; violations counted into aux[kAuxViolations] */
+__global__ void k_w_validate(WinDev W)
+{
+    if (W.aux[kAuxAbort])
+        return;
+    for (uint32_t w = blockIdx.x; w < W.nw; w += gridDim.x) {
+        const uint32_t b0 = W.win_cnt[w], b1 = W.win_cnt[w + 1];
+        if (b1 < b0 && threadIdx.x == 0)
+            atomicAdd(&W.aux[kAuxViolations], 1000000u);
+        for (uint32_t i = b0 + 1 + threadIdx.x; i < b1; i += blockDim.x)
+            if (((uint32_t)W.rec2[i] >> 16) < ((uint32_t)W.rec2[i - 1] >> 16))
+                atomicAdd(&W.aux[kAuxViolations], 1u);
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0 && W.win_cnt[W.nw] != W.aux[kAuxTotal1])
+        atomicAdd(&W.aux[kAuxViolations], 1u << 30);
 }
 
 /* lazy reset: the generation moves on, so every window reads as INIT until replayed */
@@ -654,15 +886,27 @@ __global__ void __launch_bounds__(256) k_w_materialize(hirace_dev_ctx c, WinDev 
     }
 }
 
-size_t light_smem(const WinDev &W) { return (size_t)8u << W.wl; }
+size_t light_smem(const WinDev &W) { return ((size_t)8u << W.wl) + 2u * kRing * 8u; }
 
 } // namespace
 
 const void *window_light_kernel() { return (const void *)k_w_light; }
+int window_light_threads() { return kLightThreads; }
+size_t window_light_smem(uint32_t wl) { return ((size_t)8u << wl) + 2u * kRing * 8u; }
 
 cudaError_t window_init()
 {
-    return cudaFuncSetAttribute(k_w_light, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 << 14);
+    cudaError_t e0;
+#define W_SMEM(fn, bytes)                                                                                            \
+    if ((e0 = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(bytes))) != cudaSuccess)  \
+        return e0;
+    W_SMEM((k_w_scatter1<16, 512, 4>), sizeof(ScatterSmem<16, 512>));
+    W_SMEM((k_w_scatter1<8, 1024, 2>), sizeof(ScatterSmem<8, 1024>));
+    W_SMEM((k_w_scatter2<16, 512, 4>), sizeof(ScatterSmem<16, 512>));
+    W_SMEM((k_w_scatter2<8, 1024, 2>), sizeof(ScatterSmem<8, 1024>));
+#undef W_SMEM
+    return cudaFuncSetAttribute(k_w_light, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)window_light_smem(14));
 }
 
 namespace {
@@ -670,19 +914,14 @@ cudaError_t coop_scan(const hirace_dev_ctx &c, const WinDev &W, uint32_t *a, uin
                       uint32_t extra, uint32_t *total_out, uint32_t *ceil_out, uint32_t ceil_div,
                       const unsigned long long *check_total, uint64_t cap, int sm_count, cudaStream_t st)
 {
-    cudaError_t e = cudaMemsetAsync(W.bar, 0, sizeof(unsigned int), st);
-    if (e != cudaSuccess)
-        return e;
-    int grid = sm_count * 2 < kScanMaxCtas ? sm_count * 2 : kScanMaxCtas;
-    uint32_t *pa = a, *pp = W.partials, *pt = total_out, *pc = ceil_out, *pab = W.aux + kAuxAbort;
-    const uint32_t *pcols = cols;
-    uint32_t r = rows, x = extra, cd = ceil_div ? ceil_div : 1u;
-    uint64_t cp = cap;
-    const unsigned long long *pct = check_total;
-    unsigned int *pb = W.bar, *perr = c.error_flags;
-    void *args[] = {&pa, &r, &pcols, &x, &pp, &pb, &pt, &pc, &cd, &pct, &cp, &pab, &perr};
-    note_launches(1);
-    return cudaLaunchCooperativeKernel((const void *)k_w_scan, dim3(grid), dim3(1024), args, 0, st);
+    const uint32_t G = (uint32_t)(sm_count < kScanMaxCtas ? sm_count : kScanMaxCtas);
+    uint32_t *abort = W.aux + kAuxAbort;
+    note_launches(3);
+    k_w_scan_reduce<<<G, 1024, 0, st>>>(a, rows, cols, extra, G, W.partials, check_total, cap, abort,
+                                        c.error_flags);
+    k_w_scan_partials<<<1, 1024, 0, st>>>(W.partials, G, total_out, ceil_out, ceil_div ? ceil_div : 1u, abort);
+    k_w_scan_apply<<<G, 1024, 0, st>>>(a, rows, cols, extra, G, W.partials, abort);
+    return cudaGetLastError();
 }
 } // namespace
 
@@ -724,7 +963,14 @@ cudaError_t launch_window_check(const hirace_dev_ctx &c, const WinDev &W, const 
     W_TRY(cudaGetLastError());
     W_TRY(coop_scan(c, W, W.count1, 1u << W.d0b, W.aux + kAuxItems1, 0, W.aux + kAuxTotal1, W.aux + kAuxChunks2, W.p2,
                     W.elems, W.elem_cap, sm_count, st));
-    k_w_pass1<true><<<pgrid, kPassThreads, 0, st>>>(c, reinterpret_cast<const uint4 *>(ev), W);
+    if ((1u << W.d0b) <= 512)
+        k_w_scatter1<16, 512, 4><<<pgrid, kPassThreads, sizeof(ScatterSmem<16, 512>), st>>>(
+            c, reinterpret_cast<const uint4 *>(ev), W);
+    else if ((1u << W.d0b) <= kMaxBufDigits)
+        k_w_scatter1<8, 1024, 2><<<pgrid, kPassThreads, sizeof(ScatterSmem<8, 1024>), st>>>(
+            c, reinterpret_cast<const uint4 *>(ev), W);
+    else
+        k_w_pass1<true><<<pgrid, kPassThreads, 0, st>>>(c, reinterpret_cast<const uint4 *>(ev), W);
     W_TRY(cudaGetLastError());
     if (two) {
         note_launches(2);
@@ -732,10 +978,17 @@ cudaError_t launch_window_check(const hirace_dev_ctx &c, const WinDev &W, const 
         W_TRY(cudaGetLastError());
         W_TRY(coop_scan(c, W, W.count2, 1u << W.d1b, W.aux + kAuxChunks2, 0, W.aux + kAuxTotal2, nullptr, 1,
                         nullptr, 0, sm_count, st));
-        k_w_pass2<true><<<pgrid, kPassThreads, 0, st>>>(W, s.nbatches);
+        if ((1u << W.d1b) <= 512)
+            k_w_scatter2<16, 512, 4><<<pgrid, kPassThreads, sizeof(ScatterSmem<16, 512>), st>>>(W, s.nbatches);
+        else if ((1u << W.d1b) <= kMaxBufDigits)
+            k_w_scatter2<8, 1024, 2><<<pgrid, kPassThreads, sizeof(ScatterSmem<8, 1024>), st>>>(W, s.nbatches);
+        else
+            k_w_pass2<true><<<pgrid, kPassThreads, 0, st>>>(W, s.nbatches);
         W_TRY(cudaGetLastError());
     }
     W_TRY(coop_scan(c, W, W.win_cnt, 1, nullptr, W.nw + 1, nullptr, nullptr, 1, nullptr, 0, sm_count, st));
+    if (getenv("HIRACE_WIN_VALIDATE"))
+        k_w_validate<<<sm_count * 4, 256, 0, st>>>(W);
     note_launches(2);
     k_w_classify<<<sm_count * 4, 256, 0, st>>>(W);
     k_w_hseg<<<sm_count, 256, 0, st>>>(W, s.nbatches);
@@ -751,7 +1004,7 @@ cudaError_t launch_window_check(const hirace_dev_ctx &c, const WinDev &W, const 
                                           st));
     }
     note_launches(1);
-    k_w_light<<<W.light_ctas, kLightThreads, light_smem(W), st>>>(c, W, s.nbatches);
+    k_w_light<<<W.light_ctas, kLightThreads, light_smem(W), st>>>(c, W);
     W_TRY(cudaGetLastError());
     if (d_total) { /* report buffer; else stale windows := INIT and the shadow scan */
         W_TRY(launch_collect_reports(c, out, cap, d_total, st));

@@ -52,21 +52,3 @@ def scenario_trace(geom, steps):
 
 def as_dict(keys, cls):
     return {int(k): int(c) for k, c in zip(keys, cls)}
-
-
-def oracle_on_words(trace, words, chunk=1 << 26):
-    """Oracle verdicts for a sample of GLOBAL words at any trace size: the events touching the
-    sampled words (filtered chunk by chunk) carry every racing pair on them, so Oracle-D on that
-    subset is exact for those words.  Returns {word: class}."""
-    import oracle
-    words = np.unique(np.asarray(words, dtype=np.uint64))
-    keep = []
-    ev = trace.events
-    for lo in range(0, ev.shape[0], chunk):
-        part = ev[lo:lo + chunk]
-        w = part["addr"] >> np.uint64(2)
-        sel = ((part["addr"] & tg.SHARED_BIT) == 0) & np.isin(w, words)
-        keep.append(part[sel])
-    sub = np.concatenate(keep) if keep else ev[:0]
-    k, c, _ = oracle.races(sub, trace.block_threads, trace.warp_size)
-    return {int(a): int(b) for a, b in zip(k, c)}

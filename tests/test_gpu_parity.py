@@ -333,40 +333,66 @@ def test_cfg3_full_rmat20_bfs_vs_oracle(racy):
     n, recs = _fused(t, cap=max(1, len(want)) + 16)
     assert n == len(want)
     assert as_dict(recs) == want
+    _both_modes(t, want)
 
 
-def _cfg5_check(t, sample=4000):
-    from tests.helpers import oracle_on_words
-    want = {w: CLS[c] for w, c in t.info["expected"].items()}
-    n, recs = _fused(t, cap=len(want) + 1024)
-    got = as_dict(recs)
-    assert n == len(want) and got == want          # by construction
-    rng = np.random.default_rng(1)
-    reg = t.info["regions"]
-    sample_words = np.concatenate([
-        np.array(list(want)[:200], np.uint64),
-        rng.integers(0, reg["gather"], sample // 4).astype(np.uint64),          # private
-        rng.integers(reg["gather"], reg["hot"], sample // 4).astype(np.uint64),  # gather
-        rng.integers(reg["hot"], reg["hot"] + 64, sample // 4).astype(np.uint64),  # hottest atomics
-        rng.integers(reg["inj"], reg["pat"] + 2048, sample // 4).astype(np.uint64)])
-    sampled = oracle_on_words(t, sample_words)
-    assert {w: got[w] for w in sampled if w in got} == sampled
-    assert all(int(w) not in got or int(w) in sampled for w in sample_words)
+def _oracle_all_cores(t):
+    k, c, _ = oracle.races_parallel(t.events, t.block_threads, t.warp_size)
+    return {int(a): int(b) for a, b in zip(k, c)}
 
 
-def test_cfg5_medium_vs_construction_and_sampled_oracle():
-    # 2^28 tracked words, 8192 blocks x 256 threads, 32 batches: ~1.3e8 events
+def _both_modes(t, want):
+    """The check in both replay strategies (include/hirace.h hirace_replay_mode) == want."""
+    for mode in (hr.REPLAY_WINDOW, hr.REPLAY_BATCH):
+        c = hr.Checker.for_trace(t)
+        c.set_replay_mode(mode)
+        c.reset()
+        d = hr.events_to_device(t.events)
+        cap = len(want) + 1024
+        out = torch.zeros(cap * 16, dtype=torch.uint8, device="cuda")
+        tot = torch.zeros(1, dtype=torch.int64, device="cuda")
+        c.check_device(d, out, cap, tot)
+        torch.cuda.synchronize()
+        assert c.sync() == 0
+        n = int(tot.item())
+        recs = out.cpu().numpy().view(hr.RACE_DTYPE)[:n]
+        assert n == len(want), mode
+        assert as_dict(recs) == want, mode
+        assert c.stats()["checked"] == word_accesses(t)
+        del d, out
+        c.close()
+        torch.cuda.empty_cache()
+
+
+def test_cfg5_medium_vs_oracle_both_modes():
+    # 2^28 tracked words, 8192 blocks x 256 threads, 32 batches: ~1.3e8 events; the whole trace
+    # through the all-core oracle (oracle/oracle_par.c), and the construction
     t = tg.cfg5(grid_blocks=8192, words_log2=28)
     assert t.n > 1e8
-    _cfg5_check(t)
+    want = _oracle_all_cores(t)
+    assert want == {w: CLS[c] for w, c in t.info["expected"].items()}
+    _both_modes(t, want)
 
 
 @pytest.mark.slow
-def test_cfg5_full_1e9_vs_construction_and_sampled_oracle():
-    # BASELINE configs[4] on one GPU: 2^32 tracked words (32 GiB shadow), 1.07e9 events (17 GB)
+def test_cfg5_full_1e9_vs_oracle_both_modes():
+    # BASELINE configs[4] on one GPU: 2^32 tracked words (32 GiB shadow), 1.07e9 events (17 GB);
+    # GPU race set == the oracle's on the WHOLE trace (all host cores, address-sharded)
     t = tg.cfg5()
     assert t.n > 1.07e9
-    _cfg5_check(t)
+    want = _oracle_all_cores(t)
+    assert want == {w: CLS[c] for w, c in t.info["expected"].items()}
+    _both_modes(t, want)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("racy", [False, True])
+def test_cfg3_full_rmat20_cc_vs_oracle(racy):
+    # BASELINE configs[2], connected components (2 label-propagation kernels) on RMAT-20
+    t = tg.cfg3("cc", racy)
+    want = _oracle_all_cores(t)
+    assert bool(want) == racy
+    _both_modes(t, want)
 
 
 # ---- SURVEY §8(f) f2: relaxed read-vs-atomic policy (DESIGN.md reading R2b) ----------------
