@@ -671,6 +671,9 @@ hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_eve
     if (win)
         HR_CUDA(c, launch_window_check(c->dev, c->win, c->scr, d_events, (uint32_t)n, c->sm_count, c->replay_grid, st,
                                        c->shadow_words, d_out, cap, d_n_total));
+    else
+        HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st, c->shadow_words, d_out, cap, d_n_total,
+                                 report_mode(c)));
     if (win && getenv("HIRACE_WIN_VALIDATE")) { /* diagnostics: synchronous */
         uint32_t aux[kAuxCount];
         HR_CUDA(c, cudaStreamSynchronize(st));
@@ -679,9 +682,6 @@ hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_eve
                 aux[kAuxItems1], aux[kAuxTotal1], aux[kAuxChunks2], aux[kAuxNHeavy], aux[kAuxNLight], aux[kAuxAbort],
                 aux[kAuxViolations]);
     }
-    else
-        HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st, c->shadow_words, d_out, cap, d_n_total,
-                                 report_mode(c)));
     if (c->t_stop)
         HR_CUDA(c, cudaEventRecord(c->t_stop, st));
     return HIRACE_OK;
