@@ -118,8 +118,8 @@ hirace_status device_errors(hirace_ctx *c)
     return c->sticky;
 }
 
-constexpr uint64_t kWindowAutoBytes = 1ull << 30; /* AUTO: window-major for shadows >= 1 GiB */
 constexpr uint32_t kWindowPadLog2 = 14;           /* shadow allocation padded to 2^14 records */
+constexpr uint32_t kWindowLog2Default = 12;       /* 32 KB windows: 4 light CTAs per SM (§8)    */
 
 /* does this context replay window-major? (8-byte records, 4-byte elements) */
 bool window_active(const hirace_ctx *c)
@@ -128,7 +128,10 @@ bool window_active(const hirace_ctx *c)
         return false;
     if (c->replay_mode == HIRACE_REPLAY_WINDOW)
         return true;
-    return c->replay_mode == HIRACE_REPLAY_AUTO && c->shadow_words * 8 >= kWindowAutoBytes;
+    /* AUTO: batch-major everywhere (measured faster on every config); the
+     * HIRACE_WINDOW_AUTO_BYTES environment variable re-enables window-major above a size */
+    const char *v = getenv("HIRACE_WINDOW_AUTO_BYTES");
+    return c->replay_mode == HIRACE_REPLAY_AUTO && v && c->shadow_words * 8 >= strtoull(v, nullptr, 10);
 }
 
 /* window geometry + generation array for window size 2^wl records (all windows stale) */
@@ -142,8 +145,8 @@ cudaError_t window_geometry(hirace_ctx *c, uint32_t wl)
     uint32_t wb = 0;
     while ((1ull << wb) < nw)
         wb++;
-    if (wb > 9 + 12)
-        return cudaErrorInvalidValue;
+    if (wb > 20)
+        return cudaErrorInvalidValue; /* two passes of <= 1024 digits */
     if (W.gen)
         cudaFree(W.gen);
     W.gen = nullptr;
@@ -159,7 +162,8 @@ cudaError_t window_geometry(hirace_ctx *c, uint32_t wl)
         return e;
     W.wl = wl;
     W.nw = (uint32_t)nw;
-    W.d0b = wb < 9 ? wb : 9;
+    /* digits: one pass up to 2^9 windows, else two balanced passes of <= 2^10 digits */
+    W.d0b = wb <= 9 ? wb : (wb + 1) / 2;
     W.d1b = wb - W.d0b;
     W.p1 = 1u << 16;
     W.p2 = 1u << 16;
@@ -286,7 +290,7 @@ hirace_status hirace_set_replay_mode(hirace_ctx *c, int mode, uint32_t window_lo
         return HIRACE_E_INVAL;
     HR_CUDA(c, cudaSetDevice(c->device));
     HR_CUDA(c, cudaDeviceSynchronize());
-    const uint32_t wl = window_log2 ? window_log2 : 14u;
+    const uint32_t wl = window_log2 ? window_log2 : kWindowLog2Default;
     if (c->win.gen && wl != c->win_log2) {
         window_free_scratch(c->win);
         HR_CUDA(c, window_geometry(c, wl));
@@ -444,7 +448,7 @@ hirace_status shadow_alloc_impl(const hirace_config *cfg, const hirace_epoch_lim
     d.c_max_g = lim ? lim->max_g : 254u;
     d.c_max_b = lim ? lim->max_b : 1023u;
     d.c_max_w = lim ? lim->max_w : 511u;
-    if (c->rec_bytes == 8 && cfg->granularity_log2 == 2 && (e = window_geometry(c, 14)) != cudaSuccess)
+    if (c->rec_bytes == 8 && cfg->granularity_log2 == 2 && (e = window_geometry(c, kWindowLog2Default)) != cudaSuccess)
         return fail(e);
     if (hirace_shadow_reset(c, nullptr) != HIRACE_OK || cudaDeviceSynchronize() != cudaSuccess) {
         hirace_shadow_free(c);

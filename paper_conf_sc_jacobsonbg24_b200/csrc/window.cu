@@ -48,9 +48,9 @@ namespace hirace_impl {
 namespace {
 
 constexpr int kPassThreads = 512;
-constexpr int kLightThreads = 512;
-constexpr uint32_t kRing = 2048; /* records per ring buffer (16 KB) */
-constexpr uint32_t kMaxD0 = 512, kMaxD1 = 4096;
+constexpr int kLightThreads = 256;
+constexpr uint32_t kRing = 1024; /* records per ring buffer (8 KB) */
+constexpr uint32_t kMaxD0 = 1024, kMaxD1 = 4096;
 using u64 = unsigned long long;
 
 __device__ __forceinline__ u64 wrec(uint32_t word, uint32_t kind, uint32_t f, uint32_t tid)
@@ -436,12 +436,20 @@ __global__ void __launch_bounds__(kPassThreads) k_w_scatter1(hirace_dev_ctx c, c
         }
         __syncthreads();
         const uint32_t key = W.batch_key[it.z];
+        uint4 nx[EV]; /* the next sub-tile's events are in flight while this one is scattered */
+#pragma unroll
+        for (int k = 0; k < EV; k++) {
+            const uint32_t i = it.x + k * T + threadIdx.x;
+            nx[k] = i < it.y ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
+        }
         for (uint32_t i0 = it.x; i0 < it.y; i0 += T * EV) {
             uint4 e[EV];
 #pragma unroll
             for (int k = 0; k < EV; k++) {
-                const uint32_t i = i0 + k * T + threadIdx.x;
-                e[k] = i < it.y ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
+                e[k] = nx[k];
+                const uint32_t i = i0 + T * EV + k * T + threadIdx.x;
+                if (i < it.y)
+                    nx[k] = ld_event(ev + i);
             }
 #pragma unroll
             for (int k = 0; k < EV; k++) {
@@ -501,12 +509,20 @@ __global__ void __launch_bounds__(kPassThreads) k_w_scatter2(WinDev W, const uin
             if (s1 <= s0)
                 continue;
             const uint32_t batch = j % nb;
+            u64 nx[EV]; /* next sub-tile in flight */
+#pragma unroll
+            for (int k = 0; k < EV; k++) {
+                const uint32_t i = s0 + k * T + threadIdx.x;
+                nx[k] = i < s1 ? ld_rec(W.rec1 + i) : 0ull;
+            }
             for (uint32_t i0 = s0; i0 < s1; i0 += T * EV) {
                 u64 r[EV];
 #pragma unroll
                 for (int k = 0; k < EV; k++) {
-                    const uint32_t i = i0 + k * T + threadIdx.x;
-                    r[k] = i < s1 ? ld_rec(W.rec1 + i) : 0ull;
+                    r[k] = nx[k];
+                    const uint32_t i = i0 + T * EV + k * T + threadIdx.x;
+                    if (i < s1)
+                        nx[k] = ld_rec(W.rec1 + i);
                 }
 #pragma unroll
                 for (int k = 0; k < EV; k++)
@@ -711,7 +727,7 @@ __device__ __forceinline__ void light_step(u64 *sh, bool ok, uint32_t word, uint
  * (chunk k+2 is requested as soon as chunk k is consumed), each tile of blockDim records is
  * processed by the whole CTA, with a __syncthreads where the batch changes, and the window goes
  * back by TMA bulk copy while the next window starts. */
-__global__ void __launch_bounds__(kLightThreads, 2) k_w_light(hirace_dev_ctx c, WinDev W)
+__global__ void __launch_bounds__(kLightThreads, 4) k_w_light(hirace_dev_ctx c, WinDev W)
 {
     extern __shared__ __align__(128) unsigned char s_dyn[];
     __shared__ __align__(16) unsigned char s_raw[RAW_TABLE_BYTES];
@@ -723,6 +739,7 @@ __global__ void __launch_bounds__(kLightThreads, 2) k_w_light(hirace_dev_ctx c, 
     const uint32_t wsz = 1u << W.wl, wbytes = wsz * 8u, wmask = wsz - 1u;
     u64 *const sh = reinterpret_cast<u64 *>(s_dyn);
     u64 *const ring = sh + wsz;
+
     for (int i = threadIdx.x; i < RAW_TABLE_BYTES / 16; i += blockDim.x)
         reinterpret_cast<uint4 *>(s_raw)[i] = __ldg(reinterpret_cast<const uint4 *>(c.table + 2048) + i);
     if (threadIdx.x < 4)
@@ -794,11 +811,25 @@ __global__ void __launch_bounds__(kLightThreads, 2) k_w_light(hirace_dev_ctx c, 
                 const uint32_t lo32 = (uint32_t)rr, my_b = valid ? lo32 >> 16 : 0xffffffffu;
                 const uint32_t tid = (uint32_t)(rr >> 32), kind = (lo32 >> 14) & 3u, word = lo32 & wmask;
                 const uint32_t hi_b = (uint32_t)rb[min(hi, base + blockDim.x) - 1u - c0] >> 16;
+                const uint32_t lo_b = (uint32_t)rb[base - c0] >> 16;
+                if (lo_b == hi_b) { /* one batch: concurrent; after the previous tile if the batch moved on */
+                    if (lo_b != cur_b)
+                        __syncthreads();
+                    if (__any_sync(0xffffffffu, valid)) {
+                        const Batch B = make_batch<u64>(W.batch_key[lo_b], rec);
+                        light_step(sh, valid, word, tid, kind, B, 0, (uint64_t)w << W.wl, c, G, rec, s_raw, cnt, lane,
+                                   below);
+                    }
+                    cur_b = hi_b;
+                    continue;
+                }
+                /* several batches: batch steps, a barrier where the batch changes */
+                const bool act = valid;
                 uint32_t b = cur_b;
                 for (;;) {
-                    if (__any_sync(0xffffffffu, valid && my_b == b)) { /* warp-uniform: records are batch-sorted */
+                    if (__any_sync(0xffffffffu, act && my_b == b)) { /* warp-uniform: records are batch-sorted */
                         const Batch B = make_batch<u64>(W.batch_key[b], rec);
-                        light_step(sh, valid && my_b == b, word, tid, kind, B, 0, (uint64_t)w << W.wl, c, G, rec,
+                        light_step(sh, act && my_b == b, word, tid, kind, B, 0, (uint64_t)w << W.wl, c, G, rec,
                                    s_raw, cnt, lane, below);
                     }
                     if (b == hi_b)
@@ -886,13 +917,18 @@ __global__ void __launch_bounds__(256) k_w_materialize(hirace_dev_ctx c, WinDev 
     }
 }
 
-size_t light_smem(const WinDev &W) { return ((size_t)8u << W.wl) + 2u * kRing * 8u; }
+size_t light_smem_of(uint32_t wl)
+{
+    /* window records | record ring */
+    return ((size_t)8u << wl) + 2u * kRing * 8u;
+}
+size_t light_smem(const WinDev &W) { return light_smem_of(W.wl); }
 
 } // namespace
 
 const void *window_light_kernel() { return (const void *)k_w_light; }
 int window_light_threads() { return kLightThreads; }
-size_t window_light_smem(uint32_t wl) { return ((size_t)8u << wl) + 2u * kRing * 8u; }
+size_t window_light_smem(uint32_t wl) { return light_smem_of(wl); }
 
 cudaError_t window_init()
 {

@@ -271,8 +271,12 @@ def test_window_filter_selected_accesses():
     c.close()
 
 
-def test_auto_mode_picks_window_for_large_shadows():
+def test_auto_mode_is_batch_unless_enabled(monkeypatch):
     big = hr.Checker(64, 256, 32, 1 << 28, 0)       # 2 GiB of records
+    assert not big.window_active
+    big.close()
+    monkeypatch.setenv("HIRACE_WINDOW_AUTO_BYTES", str(1 << 30))
+    big = hr.Checker(64, 256, 32, 1 << 28, 0)
     small = hr.Checker(64, 256, 32, 1 << 20, 0)
     assert big.window_active and not small.window_active
     big.close()
