@@ -198,6 +198,15 @@ hirace_status hirace_shadow_reset(hirace_ctx *ctx, void *stream);
  * WARP/BLOCK scopes are device-side (hirace::barrier) -> INVAL.  Async. */
 hirace_status hirace_barrier(hirace_ctx *ctx, hirace_scope scope, void *stream);
 
+/* Advances the context's grid epoch g by `count` grid-wide synchronisations the host did not
+ * see (same rebase rule as hirace_barrier).  A cooperative kernel whose threads call
+ * hirace::barrier(GRID) k times ends in epoch g + k on the device; before the next inline
+ * kernel the host must therefore advance g by k + 1 (k device grid syncs + the kernel
+ * boundary), e.g. hirace_advance_grid_epochs(ctx, k + 1, stream), so no epoch is reused
+ * (reused epochs would make ordered cross-kernel accesses look concurrent).  Compact contexts:
+ * INVAL.  Async. */
+hirace_status hirace_advance_grid_epochs(hirace_ctx *ctx, uint32_t count, void *stream);
+
 /* ---- replay (a1-a9) ------------------------------------------------------------------- */
 
 /* Replays n DEVICE-resident events through the shadow FSM.  Events must be sorted by batch
@@ -435,7 +444,8 @@ uint32_t hirace_fsm_step_compact(int policy, uint32_t old_shadow, uint32_t tid, 
                                  const hirace_epoch_limits *lim, int *report);
 
 /* Cluster level (reading R16): host model of the
- * derived cluster-level FSM (hirace_device.cuh, namespace hirace::cluster).  Not yet a replay path.
+ * derived cluster-level FSM (hirace_device.cuh, namespace hirace::cluster), 34 reachable states;
+ * the replay path is hirace_cluster_replay below.
  * hirace_fsm_table_cluster writes the 16384-byte table (entry[state<<8 | kind<<6 | sync<<3 | rel]
  * = next:6 | keep:1 | report:1) and the number of live states.  Errors: INVAL (NULL out, or the
  * rules reaching more than 64 states).

@@ -15,12 +15,12 @@
  * Algorithm 1's load / step / CAS loop per event,
  * PAPER.md L249-279, with no store when the record is unchanged), and a grid barrier separates batches (all events of a
  * batch are pairwise concurrent or program-ordered in one thread: PAPER.md L177).
- * Collection selects RACE records in shadow order (cub::DeviceSelect) and expands them to
- * hirace_race rows.
+ * Collection is an ordered compaction of the RACE records in shadow (= key) order written here
+ * (k_cluster_count per 4096-record tile, host prefix over the tiles, k_cluster_emit at each
+ * tile's offset); no library kernel on this path.
  */
 #include <cooperative_groups.h>
-#include <cub/device/device_select.cuh>
-#include <thrust/iterator/counting_iterator.h>
+#include <vector>
 
 #include <stdlib.h>
 #include <string.h>
@@ -44,6 +44,10 @@ struct hirace_cluster_ctx {
     int grid;
     int sm_count;
     hirace_status sticky;
+    uint64_t *coll_tiles;       /* collect scratch: per-tile counts / offsets */
+    uint64_t coll_tiles_cap;
+    hirace_race *coll_rows;     /* collect scratch: output rows              */
+    uint64_t coll_rows_cap;
 };
 
 namespace {
@@ -234,29 +238,80 @@ __global__ void __launch_bounds__(kThreads, 4) k_cluster_replay(const hirace_eve
         atomicAdd(&stats[1], retries);
 }
 
-struct IsRace {
-    const unsigned long long *shadow;
-    const unsigned char *cls;
-    __device__ bool operator()(uint64_t i) const { return cls[shadow[i] & 63u] != 0; }
-};
+/* Collection: an ordered compaction of the RACE records in shadow (= key) order, two passes
+ * over 4096-record tiles (count, then emit at the tile's offset with a block scan). */
+constexpr uint32_t kCollTile = 4096, kCollThreads = 256, kCollPer = kCollTile / kCollThreads;
 
-__global__ void k_cluster_rows(const uint64_t *__restrict__ sel, uint64_t n, const unsigned long long *shadow,
-                               const unsigned char *cls, uint64_t global_words, uint64_t smem_words,
-                               hirace_race *out)
+__device__ __forceinline__ uint32_t coll_block_scan(uint32_t mine, uint32_t *s_w, uint32_t *total)
 {
-    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= n)
-        return;
-    const uint64_t idx = sel[i];
-    const unsigned long long r = shadow[idx];
-    uint64_t key = idx;
-    if (idx >= global_words) {
-        const uint64_t s = idx - global_words;
-        key = HIRACE_SHARED_BIT | ((s / smem_words) << 32) | (s % smem_words);
+    const uint32_t lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    uint32_t incl = mine;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, incl, d);
+        if ((int)lane >= d)
+            incl += y;
     }
-    out[i].key = key;
-    out[i].cls_and_epoch = (uint32_t)cls[r & 63u] | (uint32_t)((r >> SH_G) & 255u) << 8;
-    out[i].detect_tid = (uint32_t)(r >> SH_TID);
+    if (lane == 31)
+        s_w[wid] = incl;
+    __syncthreads();
+    uint32_t before = 0, all = 0;
+    for (uint32_t w = 0; w < nw; w++) {
+        const uint32_t x = s_w[w];
+        before += w < wid ? x : 0u;
+        all += x;
+    }
+    *total = all;
+    return before + incl - mine;
+}
+
+__global__ void __launch_bounds__(kCollThreads) k_cluster_count(const unsigned long long *__restrict__ shadow,
+                                                                uint64_t nw, const unsigned char *__restrict__ cls,
+                                                                uint32_t *tile_cnt)
+{
+    __shared__ uint32_t s_w[32];
+    const uint64_t w0 = (uint64_t)blockIdx.x * kCollTile + (uint64_t)threadIdx.x * kCollPer;
+    uint32_t n = 0;
+    for (uint32_t k = 0; k < kCollPer; k++)
+        n += (w0 + k < nw && cls[__ldcs(shadow + w0 + k) & 63u] != 0) ? 1u : 0u;
+    uint32_t tot;
+    coll_block_scan(n, s_w, &tot);
+    if (threadIdx.x == 0)
+        tile_cnt[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(kCollThreads) k_cluster_emit(const unsigned long long *__restrict__ shadow,
+                                                               uint64_t nw, const unsigned char *__restrict__ cls,
+                                                               const uint64_t *tile_off, uint64_t cap,
+                                                               uint64_t global_words, uint64_t smem_words,
+                                                               hirace_race *out)
+{
+    __shared__ uint32_t s_w[32];
+    const uint64_t w0 = (uint64_t)blockIdx.x * kCollTile + (uint64_t)threadIdx.x * kCollPer;
+    uint32_t n = 0;
+    for (uint32_t k = 0; k < kCollPer; k++)
+        n += (w0 + k < nw && cls[shadow[w0 + k] & 63u] != 0) ? 1u : 0u;
+    uint32_t tot;
+    uint64_t pos = tile_off[blockIdx.x] + coll_block_scan(n, s_w, &tot);
+    for (uint32_t k = 0; k < kCollPer && n; k++) {
+        const uint64_t idx = w0 + k;
+        if (idx >= nw)
+            break;
+        const unsigned long long r = shadow[idx];
+        if (cls[r & 63u] == 0)
+            continue;
+        if (pos < cap) {
+            uint64_t key = idx;
+            if (idx >= global_words) {
+                const uint64_t s = idx - global_words;
+                key = HIRACE_SHARED_BIT | ((s / smem_words) << 32) | (s % smem_words);
+            }
+            out[pos].key = key;
+            out[pos].cls_and_epoch = (uint32_t)cls[r & 63u] | (uint32_t)((r >> SH_G) & 255u) << 8;
+            out[pos].detect_tid = (uint32_t)(r >> SH_TID);
+        }
+        pos++;
+    }
 }
 
 __global__ void k_cluster_fill(unsigned long long *p, uint64_t n)
@@ -285,6 +340,7 @@ hirace_status hirace_cluster_alloc(const hirace_config *cfg, uint32_t cluster_bl
 {
     if (!cfg || !out || !cfg->grid_blocks || !cfg->block_threads || !cfg->warp_size || !cluster_blocks ||
         cluster_blocks > 255 || cfg->grid_blocks % cluster_blocks != 0 || cfg->granularity_log2 != 2 ||
+        (cfg->global_bytes & 3) || (cfg->smem_bytes_per_block & 3) || /* as hirace_shadow_alloc */
         (uint64_t)cfg->grid_blocks * cfg->block_threads > (uint64_t)MAX_TID + 1)
         return HIRACE_E_INVAL;
     *out = nullptr;
@@ -295,8 +351,8 @@ hirace_status hirace_cluster_alloc(const hirace_config *cfg, uint32_t cluster_bl
         return HIRACE_E_NOMEM;
     c->cfg = *cfg;
     c->cluster_blocks = cluster_blocks;
-    c->global_words = (cfg->global_bytes + 3) / 4;
-    c->smem_words = (cfg->smem_bytes_per_block + 3u) / 4u;
+    c->global_words = cfg->global_bytes / 4;
+    c->smem_words = cfg->smem_bytes_per_block / 4u;
     c->shadow_words = c->global_words + (uint64_t)cfg->grid_blocks * c->smem_words;
     unsigned char table[TABLE_BYTES], cls[64] = {0};
     uint32_t nst = 0;
@@ -322,8 +378,13 @@ hirace_status hirace_cluster_alloc(const hirace_config *cfg, uint32_t cluster_bl
     int per_sm = 0;
     if (e == cudaSuccess)
         e = cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, cfg->device);
-    if (e == cudaSuccess)
+    if (e == cudaSuccess) { /* both instantiations may launch: the smaller occupancy bounds the grid */
+        int per_sm2 = 0;
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_cluster_replay<false>, kThreads, 0);
+        if (e == cudaSuccess)
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm2, k_cluster_replay<true>, kThreads, 0);
+        per_sm = per_sm2 < per_sm ? per_sm2 : per_sm;
+    }
     if (e != cudaSuccess || per_sm < 1) {
         hirace_cluster_free(c);
         return e == cudaErrorMemoryAllocation ? HIRACE_E_NOMEM : HIRACE_E_CUDA;
@@ -349,6 +410,8 @@ hirace_status hirace_cluster_free(hirace_cluster_ctx *c)
     cudaFree(c->race_class);
     cudaFree(c->err);
     cudaFree(c->stats);
+    cudaFree(c->coll_tiles);
+    cudaFree(c->coll_rows);
     free(c);
     return HIRACE_OK;
 }
@@ -406,43 +469,57 @@ hirace_status hirace_cluster_collect(hirace_cluster_ctx *c, hirace_race *h_out, 
     hirace_status st = sync_errors(c);
     if (st != HIRACE_OK)
         return st;
-    uint64_t *sel = nullptr, *d_num = nullptr;
-    void *tmp = nullptr;
-    size_t tmp_bytes = 0;
-    hirace_race *d_rows = nullptr;
-    IsRace pred{c->shadow, c->race_class};
-    auto first = thrust::make_counting_iterator<uint64_t>(0);
-    const int64_t nw = (int64_t)c->shadow_words;
-    cudaError_t e = cudaMalloc(&sel, (nw ? nw : 1) * sizeof(uint64_t));
-    if (e == cudaSuccess)
-        e = cudaMalloc(&d_num, sizeof(uint64_t));
-    if (e == cudaSuccess)
-        e = cub::DeviceSelect::If(nullptr, tmp_bytes, first, sel, d_num, nw, pred);
-    if (e == cudaSuccess)
-        e = cudaMalloc(&tmp, tmp_bytes ? tmp_bytes : 1);
-    if (e == cudaSuccess)
-        e = cub::DeviceSelect::If(tmp, tmp_bytes, first, sel, d_num, nw, pred);
-    uint64_t total = 0;
-    if (e == cudaSuccess)
-        e = cudaMemcpy(&total, d_num, sizeof(total), cudaMemcpyDeviceToHost);
-    const uint64_t m = total < cap ? total : cap;
-    if (e == cudaSuccess && m) {
-        e = cudaMalloc(&d_rows, m * sizeof(hirace_race));
-        if (e == cudaSuccess) {
-            hirace_impl::note_launches(1);
-            k_cluster_rows<<<(unsigned)((m + 255) / 256), 256>>>(sel, m, c->shadow, c->race_class, c->global_words,
-                                                                 c->smem_words ? c->smem_words : 1, d_rows);
-            e = cudaGetLastError();
-        }
-        if (e == cudaSuccess)
-            e = cudaMemcpy(h_out, d_rows, m * sizeof(hirace_race), cudaMemcpyDeviceToHost);
+    const uint64_t nw = c->shadow_words;
+    const uint64_t ntiles = (nw + kCollTile - 1) / kCollTile;
+    if (ntiles == 0) {
+        *n_total = 0;
+        return HIRACE_OK;
     }
-    cudaFree(d_rows);
-    cudaFree(tmp);
-    cudaFree(d_num);
-    cudaFree(sel);
-    if (e != cudaSuccess)
+    /* scratch: tile counts / offsets (shadow / 4096 entries), rows of at most cap records;
+     * context-owned, grown on demand */
+    cudaError_t e = cudaSuccess;
+    if (ntiles > c->coll_tiles_cap) {
+        cudaFree(c->coll_tiles);
+        c->coll_tiles = nullptr;
+        c->coll_tiles_cap = 0;
+        if ((e = cudaMalloc(&c->coll_tiles, ntiles * sizeof(uint64_t))) != cudaSuccess)
+            return HIRACE_E_NOMEM;
+        c->coll_tiles_cap = ntiles;
+    }
+    uint32_t *cnt = reinterpret_cast<uint32_t *>(c->coll_tiles);
+    hirace_impl::note_launches(1);
+    k_cluster_count<<<(unsigned)ntiles, kCollThreads>>>(c->shadow, nw, c->race_class, cnt);
+    std::vector<uint32_t> h_cnt(ntiles);
+    if ((e = cudaMemcpy(h_cnt.data(), cnt, ntiles * sizeof(uint32_t), cudaMemcpyDeviceToHost)) != cudaSuccess)
         return HIRACE_E_CUDA;
+    std::vector<uint64_t> h_off(ntiles);
+    uint64_t total = 0;
+    for (uint64_t t = 0; t < ntiles; t++) {
+        h_off[t] = total;
+        total += h_cnt[t];
+    }
+    const uint64_t m = total < cap ? total : cap;
+    if (m) {
+        if (m > c->coll_rows_cap) {
+            cudaFree(c->coll_rows);
+            c->coll_rows = nullptr;
+            c->coll_rows_cap = 0;
+            if ((e = cudaMalloc(&c->coll_rows, m * sizeof(hirace_race))) != cudaSuccess)
+                return HIRACE_E_NOMEM;
+            c->coll_rows_cap = m;
+        }
+        if ((e = cudaMemcpy(c->coll_tiles, h_off.data(), ntiles * sizeof(uint64_t), cudaMemcpyHostToDevice)) !=
+            cudaSuccess)
+            return HIRACE_E_CUDA;
+        hirace_impl::note_launches(1);
+        k_cluster_emit<<<(unsigned)ntiles, kCollThreads>>>(c->shadow, nw, c->race_class, c->coll_tiles, m,
+                                                           c->global_words, c->smem_words ? c->smem_words : 1,
+                                                           c->coll_rows);
+        if ((e = cudaGetLastError()) == cudaSuccess)
+            e = cudaMemcpy(h_out, c->coll_rows, m * sizeof(hirace_race), cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess)
+            return HIRACE_E_CUDA;
+    }
     *n_total = total;
     return HIRACE_OK;
 }

@@ -566,16 +566,29 @@ hirace_status hirace_barrier(hirace_ctx *c, hirace_scope scope, void *stream)
         return HIRACE_E_INVAL;
     if (c->sticky != HIRACE_OK)
         return c->sticky;
-    if (scope != HIRACE_SCOPE_GRID || c->rec_bytes != 8) /* compact contexts are replay-only */
+    if (scope != HIRACE_SCOPE_GRID)
+        return set_sticky(c, HIRACE_E_INVAL);
+    return hirace_advance_grid_epochs(c, 1, stream);
+}
+
+hirace_status hirace_advance_grid_epochs(hirace_ctx *c, uint32_t count, void *stream)
+{
+    if (!c)
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    if (c->rec_bytes != 8) /* compact contexts are replay-only */
         return set_sticky(c, HIRACE_E_INVAL);
     HR_CUDA(c, cudaSetDevice(c->device));
-    if (c->g + 1 >= 255u) {
-        if (ensure_materialized(c, (cudaStream_t)stream) != HIRACE_OK)
-            return c->sticky;
-        HR_CUDA(c, launch_rebase(c->dev, c->shadow_words, (cudaStream_t)stream));
-        c->g = 0;
-    } else {
-        c->g++;
+    for (uint32_t k = 0; k < count; k++) {
+        if (c->g + 1 >= 255u) {
+            if (ensure_materialized(c, (cudaStream_t)stream) != HIRACE_OK)
+                return c->sticky;
+            HR_CUDA(c, launch_rebase(c->dev, c->shadow_words, (cudaStream_t)stream));
+            c->g = 0;
+        } else {
+            c->g++;
+        }
     }
     c->dev.g = c->g;
     return HIRACE_OK;
@@ -990,7 +1003,7 @@ hirace_status hirace_dispatch_wire(hirace_ctx *c, const hirace_event *d_in, cons
     /* asynchronous: a bad record raises the context's sticky device error (BAD_TRACE at the
      * next synchronising call), so the dispatch -> replay path never drains the stream */
     for (uint64_t b = 0; b < nb; b++)
-        HR_CUDA(c, launch_dispatch_wire(d_in, h_offsets[b], h_offsets[b + 1], nranks, my_rank,
+        HR_CUDA(c, launch_dispatch_wire(d_in, h_offsets[b], h_offsets[b + 1], nranks, c->cfg.block_threads,
                                         reinterpret_cast<unsigned long long *const *>(c->d_peer_tab),
                                         c->d_peer_tab + nranks + b * (uint64_t)nranks, c->d_bucket_hist,
                                         c->d_wire_off, c->d_err, st));
@@ -1066,7 +1079,7 @@ hirace_status bucket_wire_impl(hirace_ctx *c, const hirace_event *d_in, const ui
     HR_CUDA(c, cudaMemsetAsync(running, 0, sizeof(unsigned long long), st));
     HR_CUDA(c, cudaMemsetAsync(c->d_wire_flag, 0, sizeof(unsigned int), st));
     for (uint64_t b = 0; b < nb; b++)
-        HR_CUDA(c, launch_bucket_wire(d_in, h_offsets[b], h_offsets[b + 1], nranks, my_rank,
+        HR_CUDA(c, launch_bucket_wire(d_in, h_offsets[b], h_offsets[b + 1], nranks, c->cfg.block_threads,
                                       reinterpret_cast<unsigned long long *>(d_out), cap, c->d_bucket_hist,
                                       c->d_wire_off, running, c->d_wire_counts + b * (uint64_t)nranks, c->d_wire_flag,
                                       st));

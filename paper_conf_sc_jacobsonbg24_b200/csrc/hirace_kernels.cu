@@ -207,10 +207,12 @@ constexpr int kMaxRanks = 32;
 
 constexpr uint32_t kShardChunkLog2 = 14; /* owner granularity: 2^14 words = 64 KiB */
 
-__device__ __forceinline__ uint32_t owner_of(const hirace_event &e, int nranks, int my_rank)
+/* owner rank of an access: global words by 64 KiB chunk, shared words by block (block mod
+ * nranks), so all of a block's shared accesses meet on one rank whichever rank traced them */
+__device__ __forceinline__ uint32_t owner_of(const hirace_event &e, int nranks, uint32_t block_threads)
 {
     if (e.addr & HIRACE_SHARED_BIT)
-        return (uint32_t)my_rank;
+        return (uint32_t)((e.tid / block_threads) % (uint32_t)nranks);
     return (uint32_t)((((e.addr & ~HIRACE_SHARED_BIT) >> 2) >> kShardChunkLog2) % (uint64_t)nranks);
 }
 
@@ -227,7 +229,7 @@ __device__ __forceinline__ uint64_t shard_local_addr(uint64_t addr, int nranks)
 }
 
 __global__ void __launch_bounds__(kBucketThreads) k_bucket_hist(const hirace_event *__restrict__ in, uint32_t n,
-                                                                int nranks, int my_rank, uint32_t *tile_hist,
+                                                                int nranks, uint32_t block_threads, uint32_t *tile_hist,
                                                                 unsigned int *err)
 {
     __shared__ uint32_t s_h[kMaxRanks];
@@ -239,7 +241,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_hist(const hirace_eve
         uint64_t i = base + (uint64_t)it * kBucketThreads + threadIdx.x;
         if (i < n) {
             const hirace_event e = in[i];
-            atomicAdd(&s_h[owner_of(e, nranks, my_rank)], 1u);
+            atomicAdd(&s_h[owner_of(e, nranks, block_threads)], 1u);
             /* a 16-byte event cannot be split: a global access straddling two owner chunks
              * needs the wire format (hirace_bucket_wire) */
             const uint32_t szl = (e.meta >> 2) & 7u;
@@ -303,7 +305,7 @@ __global__ void __launch_bounds__(1024) k_bucket_scan(uint32_t *tile_hist, uint3
 }
 
 __global__ void __launch_bounds__(kBucketThreads) k_bucket_scatter(const hirace_event *__restrict__ in, uint32_t n,
-                                                                   int nranks, int my_rank,
+                                                                   int nranks, uint32_t block_threads,
                                                                    const uint32_t *__restrict__ tile_off,
                                                                    hirace_event *out)
 {
@@ -320,7 +322,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_scatter(const hirace_
         uint32_t own = 0xffffffffu;
         if (i < n) {
             e = in[i];
-            own = owner_of(e, nranks, my_rank);
+            own = owner_of(e, nranks, block_threads);
         }
         const uint32_t peers = __match_any_sync(0xffffffffu, own);
         const uint32_t rank_in_warp = __popc(peers & ((1u << lane) - 1));
@@ -354,9 +356,10 @@ cudaError_t launch_bucket(const hirace_dev_ctx &c, const hirace_event *in, uint3
                           cudaStream_t st)
 {
     note_launches(3);
-    k_bucket_hist<<<ntiles, kBucketThreads, 0, st>>>(in, n, nranks, my_rank, d_tile_hist, c.error_flags);
+    (void)my_rank; /* shared words go to their block's owner (owner_of) */
+    k_bucket_hist<<<ntiles, kBucketThreads, 0, st>>>(in, n, nranks, c.block_threads, d_tile_hist, c.error_flags);
     k_bucket_scan<<<1, 1024, 0, st>>>(d_tile_hist, ntiles, nranks, d_counts);
-    k_bucket_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, n, nranks, my_rank, d_tile_hist, out);
+    k_bucket_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, n, nranks, c.block_threads, d_tile_hist, out);
     return cudaGetLastError();
 }
 
@@ -368,14 +371,14 @@ cudaError_t launch_bucket(const hirace_dev_ctx &c, const hirace_event *in, uint3
 __device__ __forceinline__ uint32_t words_of(uint32_t szl) { return szl <= 2 ? 1u : (szl <= 4 ? 1u << (szl - 2) : 0u); }
 
 /* wire record of word k of event e, and its owner (include/hirace.h) */
-__device__ __forceinline__ uint64_t wire_of(const hirace_event &e, uint32_t k, int nranks, int my_rank,
+__device__ __forceinline__ uint64_t wire_of(const hirace_event &e, uint32_t k, int nranks, uint32_t block_threads,
                                             uint32_t &owner)
 {
     const bool sh = (e.addr & HIRACE_SHARED_BIT) != 0;
     const uint64_t word = ((e.addr & ~HIRACE_SHARED_BIT) >> 2) + k;
     uint64_t w;
     if (sh) {
-        owner = (uint32_t)my_rank;
+        owner = (e.tid / block_threads) % (uint32_t)nranks;
         w = word;
     } else {
         const uint64_t chunk = word >> kShardChunkLog2;
@@ -390,7 +393,7 @@ __device__ __forceinline__ uint64_t wire_of(const hirace_event &e, uint32_t k, i
 }
 
 __global__ void __launch_bounds__(kBucketThreads) k_wire_hist(const hirace_event *__restrict__ in, uint32_t lo,
-                                                              uint32_t hi, int nranks, int my_rank,
+                                                              uint32_t hi, int nranks, uint32_t block_threads,
                                                               uint32_t *tile_hist, unsigned int *err)
 {
     __shared__ uint32_t s_h[kMaxRanks];
@@ -407,7 +410,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_wire_hist(const hirace_event
                 atomicOr(err, hirace::ERR_BAD_TRACE);
             for (uint32_t k = 0; k < nw; k++) {
                 uint32_t own;
-                (void)wire_of(e, k, nranks, my_rank, own);
+                (void)wire_of(e, k, nranks, block_threads, own);
                 if (own < (uint32_t)nranks)
                     atomicAdd(&s_h[own], 1u);
                 else
@@ -481,7 +484,7 @@ __global__ void __launch_bounds__(1024) k_wire_scan(uint32_t *tile_hist, uint32_
  * buffer mapped through CUDA IPC, stores travelling over NVLink), at the slot given by the
  * per-owner offsets in tile_off; no capacity check (the offsets come from exchanged counts) */
 __global__ void __launch_bounds__(kBucketThreads) k_wire_scatter(const hirace_event *__restrict__ in, uint32_t lo,
-                                                                 uint32_t hi, int nranks, int my_rank,
+                                                                 uint32_t hi, int nranks, uint32_t block_threads,
                                                                  const unsigned long long *__restrict__ tile_off,
                                                                  unsigned long long *out, uint64_t cap,
                                                                  unsigned int *err,
@@ -506,7 +509,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_wire_scatter(const hirace_ev
             uint32_t own = 0xffffffffu;
             uint64_t w = 0;
             if (k < nw)
-                w = wire_of(e, k, nranks, my_rank, own); /* own = ~0: invalid, skipped (hist flagged it) */
+                w = wire_of(e, k, nranks, block_threads, own); /* own = ~0: invalid, skipped (hist flagged it) */
             const uint32_t peers = __match_any_sync(0xffffffffu, own);
             const int leader = __ffs(peers) - 1;
             unsigned long long slot = 0;
@@ -525,7 +528,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_wire_scatter(const hirace_ev
     }
 }
 
-cudaError_t launch_bucket_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, int my_rank,
+cudaError_t launch_bucket_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, uint32_t block_threads,
                                unsigned long long *out, uint64_t cap, uint32_t *d_tile_hist,
                                unsigned long long *d_tile_off, unsigned long long *d_running,
                                unsigned long long *d_counts_row, unsigned int *err, cudaStream_t st)
@@ -534,10 +537,10 @@ cudaError_t launch_bucket_wire(const hirace_event *in, uint32_t lo, uint32_t hi,
     if (ntiles == 0)
         return cudaMemsetAsync(d_counts_row, 0, nranks * sizeof(unsigned long long), st);
     note_launches(3);
-    k_wire_hist<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_hist, err);
+    k_wire_hist<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, block_threads, d_tile_hist, err);
     k_wire_scan<<<1, 1024, 0, st>>>(d_tile_hist, ntiles, nranks, d_running, d_counts_row, d_tile_off);
     if (out)
-        k_wire_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_off, out, cap, err,
+        k_wire_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, block_threads, d_tile_off, out, cap, err,
                                                           nullptr);
     return cudaGetLastError();
 }
@@ -587,7 +590,7 @@ __global__ void __launch_bounds__(1024) k_wire_scan_peer(const uint32_t *tile_hi
     }
 }
 
-cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, int my_rank,
+cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, uint32_t block_threads,
                                  unsigned long long *const *d_peer, const unsigned long long *d_owner_base,
                                  uint32_t *d_tile_hist, unsigned long long *d_tile_off, unsigned int *err,
                                  cudaStream_t st)
@@ -596,9 +599,9 @@ cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t h
     if (ntiles == 0)
         return cudaSuccess;
     note_launches(3);
-    k_wire_hist<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_hist, err);
+    k_wire_hist<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, block_threads, d_tile_hist, err);
     k_wire_scan_peer<<<1, 1024, 0, st>>>(d_tile_hist, ntiles, nranks, d_owner_base, d_tile_off);
-    k_wire_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, my_rank, d_tile_off, nullptr, 0, err,
+    k_wire_scatter<<<ntiles, kBucketThreads, 0, st>>>(in, lo, hi, nranks, block_threads, d_tile_off, nullptr, 0, err,
                                                       d_peer);
     return cudaGetLastError();
 }

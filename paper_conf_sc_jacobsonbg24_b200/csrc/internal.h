@@ -59,14 +59,14 @@ cudaError_t launch_bucket(const hirace_dev_ctx &c, const hirace_event *in, uint3
                           hirace_event *out, unsigned long long *d_counts, uint32_t *d_tile_hist, uint32_t ntiles,
                           cudaStream_t st);
 /* one batch [lo, hi) of events -> owner-grouped 8-byte wire records at out[*running ...] */
-cudaError_t launch_bucket_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, int my_rank,
+cudaError_t launch_bucket_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, uint32_t block_threads,
                                unsigned long long *out, uint64_t cap, uint32_t *d_tile_hist,
                                unsigned long long *d_tile_off, unsigned long long *d_running,
                                unsigned long long *d_counts_row, unsigned int *err, cudaStream_t st);
 /* one batch [lo, hi) -> wire records stored straight into their owners' receive buffers
  * d_peer[owner] starting at d_owner_base[owner] (peer dispatch; d_peer / d_owner_base are
  * device arrays of nranks entries) */
-cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, int my_rank,
+cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t hi, int nranks, uint32_t block_threads,
                                  unsigned long long *const *d_peer, const unsigned long long *d_owner_base,
                                  uint32_t *d_tile_hist, unsigned long long *d_tile_off, unsigned int *err,
                                  cudaStream_t st);

@@ -416,7 +416,7 @@ __device__ __forceinline__ void sc_flush(ScatterSmem<BUF, RMAX> &S, u64 *out, ui
 template <uint32_t BUF, uint32_t RMAX, int EV>
 __global__ void __launch_bounds__(kPassThreads) k_w_scatter1(hirace_dev_ctx c, const uint4 *__restrict__ ev, WinDev W)
 {
-    extern __shared__ __align__(16) unsigned char s_dyn[];
+    extern __shared__ __align__(128) unsigned char s_dyn[];
     ScatterSmem<BUF, RMAX> &S = *reinterpret_cast<ScatterSmem<BUF, RMAX> *>(s_dyn);
     if (W.aux[kAuxAbort])
         return;
@@ -478,7 +478,7 @@ __global__ void __launch_bounds__(kPassThreads) k_w_scatter1(hirace_dev_ctx c, c
 template <uint32_t BUF, uint32_t RMAX, int EV>
 __global__ void __launch_bounds__(kPassThreads) k_w_scatter2(WinDev W, const uint32_t *nbp)
 {
-    extern __shared__ __align__(16) unsigned char s_dyn[];
+    extern __shared__ __align__(128) unsigned char s_dyn[];
     ScatterSmem<BUF, RMAX> &S = *reinterpret_cast<ScatterSmem<BUF, RMAX> *>(s_dyn);
     if (W.aux[kAuxAbort])
         return;

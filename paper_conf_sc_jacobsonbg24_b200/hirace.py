@@ -39,7 +39,8 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_fsm_table_cluster", "hirace_fsm_cluster_class", "hirace_fsm_step_cluster",
            "hirace_cluster_alloc", "hirace_cluster_free", "hirace_cluster_reset", "hirace_cluster_replay",
            "hirace_cluster_collect", "hirace_cluster_get_stats", "hirace_status_string",
-           "hirace_version", "hirace_launch_count", "hirace_set_replay_mode", "hirace_get_replay_mode")
+           "hirace_version", "hirace_launch_count", "hirace_set_replay_mode", "hirace_get_replay_mode",
+           "hirace_advance_grid_epochs")
 
 
 class HiraceError(RuntimeError):
@@ -139,6 +140,7 @@ def load():
         "hirace_version": (ctypes.c_char_p, []),
         "hirace_launch_count": (I32, [ctypes.POINTER(U64)]),
         "hirace_set_replay_mode": (I32, [P, I32, U32]),
+        "hirace_advance_grid_epochs": (I32, [P, U32, P]),
         "hirace_get_replay_mode": (I32, [P, ctypes.POINTER(I32)]),
     }
     for name, (res, args) in sig.items():
@@ -333,6 +335,12 @@ class Checker:
 
     def barrier(self, scope=SCOPE_GRID, stream=None):
         _check(self.lib.hirace_barrier(self.h, scope, _stream_handle(stream)), "hirace_barrier")
+
+    def advance_grid_epochs(self, count: int, stream=None):
+        """hirace_advance_grid_epochs: count grid syncs the host did not see (k device grid
+        syncs of a cooperative kernel + its boundary = k + 1)."""
+        _check(self.lib.hirace_advance_grid_epochs(self.h, count, _stream_handle(stream)),
+               "hirace_advance_grid_epochs")
 
     def replay(self, events_dev, n: int | None = None, stream=None):
         """events_dev: CUDA tensor holding 16-byte events (uint8 [16n] or int64 [n,2])."""

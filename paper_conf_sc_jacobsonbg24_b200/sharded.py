@@ -1,8 +1,9 @@
 """Address-sharded multi-GPU mode.
 
-One process per GPU.  Each rank holds the trace events of its own blocks (any partition of the
-trace's events works).  Global words are owned by rank (word >> 14) mod P (64 KiB chunks, so
-coalesced runs stay together); shared-memory words stay with the rank that holds the block.
+One process per GPU.  Each rank holds some of the trace's events (any partition works: by
+block, by thread, by time slice).  Global words are owned by rank (word >> 14) mod P (64 KiB
+chunks, so coalesced runs stay together); the shared-memory words of block k are owned by rank
+k mod P, so all accesses to one shared word meet on one rank whichever rank traced them.
 Batch by batch — in the global (g,b,w) order every rank agrees on — each rank
 
   1. buckets its events of the batch by owner on the GPU (`hirace_bucket_events`: a stable
@@ -52,6 +53,12 @@ def shard_words(global_words: int, nranks: int) -> int:
 
 def owner_of_words(words: np.ndarray, nranks: int) -> np.ndarray:
     return (np.asarray(words, np.uint64) >> np.uint64(CHUNK_LOG2)) % np.uint64(nranks)
+
+
+def owner_of_blocks(blocks: np.ndarray, nranks: int) -> np.ndarray:
+    """Owner rank of the shared-memory words of each block (block mod P; owner_of in
+    csrc/hirace_kernels.cu)."""
+    return np.asarray(blocks, np.uint64) % np.uint64(nranks)
 
 
 def local_to_global_keys(keys: np.ndarray, rank: int, nranks: int) -> np.ndarray:

@@ -38,7 +38,8 @@ def test_bucket_kernel_matches_contract(nranks, rank):
     d = torch.from_numpy(ev.view(np.int64).reshape(-1, 2).copy()).cuda()
     out = torch.empty_like(d)
     counts = c.bucket(d, n, nranks, rank, out)
-    want_t, want_counts = CpuTestOps(None, nranks, rank).bucket(torch.from_numpy(ev.view(np.int64).reshape(-1, 2)))
+    geom = tg.Trace("bucket", ev, 4096, 256, 32, 1 << 20, 64)
+    want_t, want_counts = CpuTestOps(geom, nranks, rank).bucket(torch.from_numpy(ev.view(np.int64).reshape(-1, 2)))
     assert counts == want_counts
     assert np.array_equal(out.cpu().numpy(), want_t.numpy())
     c.close()
@@ -51,7 +52,7 @@ def test_bucket_wire_kernel_matches_contract(nranks, rank):
     d = _to_tensor(t.events).cuda()
     offs, keys = c.find_batches(d)
     wire, counts = c.bucket_wire(d, offs, nranks, rank)
-    want, want_counts = wire_bucket_np(t.events, offs, nranks, rank)
+    want, want_counts = wire_bucket_np(t.events, offs, nranks, t.block_threads)
     assert np.array_equal(counts, want_counts)
     got = wire.cpu().numpy()
     ref = want.numpy()

@@ -51,7 +51,8 @@ class CpuTestOps:
         ev = _to_events(events).copy()
         sh = (ev["addr"] & tg.SHARED_BIT) != 0
         words = (ev["addr"] & ~tg.SHARED_BIT) >> np.uint64(2)
-        owner = np.where(sh, self.r, sharded.owner_of_words(words, self.P)).astype(np.int64)
+        owner = np.where(sh, sharded.owner_of_blocks(ev["tid"] // self.t.block_threads, self.P),
+                         sharded.owner_of_words(words, self.P)).astype(np.int64)
         c = np.uint64(sharded.CHUNK_LOG2)
         local = (((words >> c) // np.uint64(self.P)) << c) | (words & np.uint64((1 << sharded.CHUNK_LOG2) - 1))
         ev["addr"] = np.where(sh, ev["addr"], (local << np.uint64(2)) | (ev["addr"] & np.uint64(3)))
@@ -63,13 +64,13 @@ class CpuTestOps:
         self.got.append(_to_events(events).copy())
 
     def bucket_wire(self, events, offsets):
-        return wire_bucket_np(_to_events(events), offsets, self.P, self.r)
+        return wire_bucket_np(_to_events(events), offsets, self.P, self.t.block_threads)
 
     def replay_wire(self, wire, key):
         self.got.append(wire_to_events(np.asarray(wire), key))
 
     def count_wire(self, events, offsets):
-        return wire_bucket_np(_to_events(events), offsets, self.P, self.r)[1]
+        return wire_bucket_np(_to_events(events), offsets, self.P, self.t.block_threads)[1]
 
     def collect(self):
         ev = np.concatenate(self.got) if self.got else np.empty(0, tg.EVENT_DTYPE)
@@ -128,7 +129,7 @@ class CpuPeerExchange:
             ops.replay_wire(torch.from_numpy(self.buf[start:start + n]), key)
 
 
-def wire_bucket_np(ev, offsets, P, r):
+def wire_bucket_np(ev, offsets, P, bt):
     """Reference of the hirace_bucket_wire contract (include/hirace.h): per batch, one record per
     covered word, routed to its word's owner, shard-local words, owner-grouped (stable here;
     the kernel's order inside a (batch, owner) segment is unspecified)."""
@@ -144,7 +145,7 @@ def wire_bucket_np(ev, offsets, P, r):
         sh = (rep["addr"] & tg.SHARED_BIT) != 0
         word = ((rep["addr"] & ~tg.SHARED_BIT) >> np.uint64(2)) + k.astype(np.uint64)
         c = np.uint64(sharded.CHUNK_LOG2)
-        owner = np.where(sh, r, (word >> c) % np.uint64(P)).astype(np.int64)
+        owner = np.where(sh, sharded.owner_of_blocks(rep["tid"] // bt, P), (word >> c) % np.uint64(P)).astype(np.int64)
         local = np.where(sh, word, (((word >> c) // np.uint64(P)) << c) | (word & np.uint64((1 << 14) - 1)))
         w = (local | (sh.astype(np.uint64) << np.uint64(31)) | (rep["tid"].astype(np.uint64) << np.uint64(32)) |
              ((rep["meta"] & 3).astype(np.uint64) << np.uint64(62)))
@@ -209,14 +210,17 @@ def _words(t):
     return int(np.where(szl <= 2, 1, 1 << np.maximum(szl.astype(np.int64) - 2, 0)).sum())
 
 
-def _worker(rank, world, port, name, q, wire=False):
-    """wire: False = 16-byte events, True = 8-byte wire + all_to_all, "p2p" = peer dispatch."""
+def _worker(rank, world, port, name, q, wire=False, split="block"):
+    """wire: False = 16-byte events, True = 8-byte wire + all_to_all, "p2p" = peer dispatch.
+    split: which events a rank holds: its blocks, or its threads (a block's shared accesses then
+    come from several ranks and must meet on the block's owner)."""
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         t = _make(name)
         blk = t.events["tid"] // t.block_threads
-        mine = t.events[(blk % world) == rank]          # this rank's blocks, batch order kept
+        part = blk if split == "block" else t.events["tid"]
+        mine = t.events[(part % world) == rank]         # this rank's blocks / threads, batch order kept
         ops = CpuTestOps(t, world, rank)
         if wire == "p2p":
             ex, run = CpuPeerExchange(None, dist), sharded.run_sharded_p2p
@@ -258,14 +262,17 @@ def test_sharded_exchange_reproduces_the_oracle(world, name):
     assert cls == [int(x) for x in c]     # same classes
 
 
-@pytest.mark.parametrize("world,name", [(2, "cfg2"), (3, "cfg4"), (2, "cfg3"), (3, "wide"), (2, "multi"),
-                                        (4, "multi")])
-def test_sharded_wire_pipeline_reproduces_the_oracle(world, name):
-    """8-byte wire records, one count-matrix exchange, async per-batch payloads."""
+@pytest.mark.parametrize("world,name,split", [(2, "cfg2", "block"), (3, "cfg4", "block"), (2, "cfg3", "block"),
+                                              (3, "wide", "block"), (2, "multi", "block"), (4, "multi", "block"),
+                                              (2, "cfg2", "thread"), (3, "cfg4", "thread")])
+def test_sharded_wire_pipeline_reproduces_the_oracle(world, name, split):
+    """8-byte wire records, one count-matrix exchange, async per-batch payloads.
+    split="thread": every block's events are spread over the ranks; its shared words still meet
+    on the block's owner rank."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, name, q, True)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, name, q, True, split)) for r in range(world)]
     for p in procs:
         p.start()
     total, keys, cls = q.get(timeout=300)
@@ -321,7 +328,7 @@ def test_wire_reference_roundtrip():
     t = _make("multi")
     offs = np.flatnonzero(np.concatenate(([True], np.diff(t.events["meta"] >> 5) != 0)))
     offs = np.append(offs, t.n)
-    wire, counts = wire_bucket_np(t.events, offs, 1, 0)
+    wire, counts = wire_bucket_np(t.events, offs, 1, t.block_threads)
     assert int(counts.sum()) == _words(t) == wire.shape[0]
     keys = t.events["meta"][offs[:-1]] >> 5
     back = np.concatenate([wire_to_events(wire.numpy()[int(s):int(s + n)], int(k)) for s, n, k in
