@@ -364,8 +364,22 @@ hirace_status hirace_dispatch_wire(hirace_ctx *ctx, const hirace_event *d_in, co
                                    int nranks, int my_rank, void *const *h_peer, const uint64_t *h_dst,
                                    void *stream);
 
-/* A receive buffer of `bytes` on `device` that other processes can map: *d_ptr = its device
- * address here, handle = its 64-byte CUDA IPC handle (to be sent to the peers).  The caller
+/* Per-batch completion of the peer dispatch (instead of one event for the whole dispatch):
+ * after its dispatch of global batch j (which may be empty), every sender calls
+ * hirace_peer_release(ctx, h_peer_flags, nranks, j, j, stream): h_peer_flags[r] = owner r's flag
+ * array (a hirace_peer_buffer_alloc buffer of >= HIRACE_MAX_BATCHES u32, zero-initialised by its
+ * owner, mapped here with hirace_peer_open) - a system-scope release fence, then +1 on flag j of
+ * every owner.  An owner queues hirace_peer_wait(ctx, d_my_flags, j, target, stream) before its
+ * replay of batch j: the stream waits (acquire loads, no host involvement) until flag j >= target,
+ * target = nranks x (runs so far that used batch j, this one included; flags only grow).  The
+ * replay of batch j then overlaps the senders' dispatch of later batches.  Errors: INVAL (NULL
+ * args, nranks not in 1..32, j beyond HIRACE_MAX_BATCHES), CUDA.  Asynchronous. */
+hirace_status hirace_peer_release(hirace_ctx *ctx, void *const *h_peer_flags, int nranks, uint32_t j0, uint32_t j1,
+                                  void *stream);
+hirace_status hirace_peer_wait(hirace_ctx *ctx, const void *d_flags, uint32_t j, uint32_t target, void *stream);
+
+/* A zero-initialised receive buffer of `bytes` on `device` that other processes can map:
+ * *d_ptr = its device address here, handle = its 64-byte CUDA IPC handle (to be sent to the peers).  The caller
  * frees it with hirace_peer_buffer_free after every peer closed it.  Errors: INVAL, NOMEM, CUDA. */
 hirace_status hirace_peer_buffer_alloc(int device, uint64_t bytes, void **d_ptr, unsigned char handle[64]);
 hirace_status hirace_peer_buffer_free(void *d_ptr);

@@ -52,6 +52,7 @@ struct hirace_ctx {
     /* peer dispatch: [nranks peer buffer pointers | nb x nranks destination offsets] */
     unsigned long long *d_peer_tab = nullptr;
     uint64_t peer_tab_cap = 0;
+    void **d_flag_tab = nullptr; /* peer flag-array addresses (hirace_peer_release) */
     /* host-trace staging ring */
     hirace_event *d_stage[2] = {nullptr, nullptr};
     uint64_t stage_cap = 0;
@@ -482,7 +483,7 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
                     c->scr.batch_off, c->scr.nbatches, c->scr.batch_ctr, c->scr.grid_bar,
                     c->scr.grid_bar2, c->scr.cta_cnt, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
                     c->d_stage[0], c->d_stage[1], c->d_wire_off, c->d_wire_counts, c->d_wire_flag,
-                    c->d_peer_tab};
+                    c->d_peer_tab, c->d_flag_tab};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
@@ -1010,6 +1011,33 @@ hirace_status hirace_dispatch_wire(hirace_ctx *c, const hirace_event *d_in, cons
     return HIRACE_OK;
 }
 
+hirace_status hirace_peer_release(hirace_ctx *c, void *const *h_peer_flags, int nranks, uint32_t j0, uint32_t j1,
+                                  void *stream)
+{
+    if (!c || !h_peer_flags || nranks < 1 || nranks > 32 || j1 < j0 || j1 >= HIRACE_MAX_BATCHES)
+        return HIRACE_E_INVAL;
+    for (int r = 0; r < nranks; r++)
+        if (!h_peer_flags[r])
+            return HIRACE_E_INVAL;
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    if (!c->d_flag_tab)
+        HR_CUDA(c, cudaMalloc(&c->d_flag_tab, 32 * sizeof(void *)));
+    /* pinned staging: the copy is stream-ordered behind the previous release's kernel */
+    HR_CUDA(c, cudaMemcpyAsync(c->d_flag_tab, h_peer_flags, nranks * sizeof(void *), cudaMemcpyHostToDevice, st));
+    HR_CUDA(c, launch_peer_release(reinterpret_cast<unsigned int *const *>(c->d_flag_tab), nranks, j0, j1, st));
+    return HIRACE_OK;
+}
+
+hirace_status hirace_peer_wait(hirace_ctx *c, const void *d_flags, uint32_t j, uint32_t target, void *stream)
+{
+    if (!c || !d_flags || j >= HIRACE_MAX_BATCHES)
+        return HIRACE_E_INVAL;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    HR_CUDA(c, launch_peer_wait(static_cast<const unsigned int *>(d_flags), j, target, (cudaStream_t)stream));
+    return HIRACE_OK;
+}
+
 hirace_status hirace_peer_buffer_alloc(int device, uint64_t bytes, void **d_ptr, unsigned char handle[64])
 {
     if (!d_ptr || !handle || bytes == 0)
@@ -1021,6 +1049,10 @@ hirace_status hirace_peer_buffer_alloc(int device, uint64_t bytes, void **d_ptr,
     cudaError_t e = cudaMalloc(&p, bytes);
     if (e != cudaSuccess)
         return e == cudaErrorMemoryAllocation ? HIRACE_E_NOMEM : HIRACE_E_CUDA;
+    if (cudaMemset(p, 0, bytes) != cudaSuccess) { /* zero-initialised (completion flags start at 0) */
+        cudaFree(p);
+        return HIRACE_E_CUDA;
+    }
     cudaIpcMemHandle_t h;
     static_assert(sizeof(h) == 64, "CUDA IPC handles are 64 bytes");
     if (cudaIpcGetMemHandle(&h, p) != cudaSuccess) {

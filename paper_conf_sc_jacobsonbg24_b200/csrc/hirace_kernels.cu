@@ -637,6 +637,47 @@ cudaError_t launch_reset(void *shadow, uint64_t bytes, unsigned long long *repor
     return e;
 }
 
+/* ---- per-batch completion flags of the peer dispatch -------------------------
+ * A sender releases global batch j to every owner after its dispatch kernels for j (stream
+ * order): a system-scope release fence, then one red.add on each owner's flag j (peer memory).
+ * An owner's stream waits (acquire loads) until its flag j reached target = (runs so far that
+ * used j) x nranks, then replays batch j: replay of j overlaps the senders' later batches. */
+__global__ void k_peer_release(unsigned int *const *flags, int nranks, uint32_t j0, uint32_t j1)
+{
+    asm volatile("fence.acq_rel.sys;" ::: "memory");
+    for (uint32_t q = threadIdx.x; q < (uint32_t)nranks * (j1 - j0 + 1u); q += blockDim.x) {
+        unsigned int *f = flags[q % (uint32_t)nranks] + j0 + q / (uint32_t)nranks;
+        asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(f) : "memory");
+    }
+}
+
+__global__ void k_peer_wait(const unsigned int *flags, uint32_t j, uint32_t target)
+{
+    if (threadIdx.x == 0) {
+        unsigned int v;
+        for (;;) {
+            asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(flags + j) : "memory");
+            if (v >= target)
+                break;
+            __nanosleep(256);
+        }
+    }
+}
+
+cudaError_t launch_peer_release(unsigned int *const *d_flags, int nranks, uint32_t j0, uint32_t j1, cudaStream_t st)
+{
+    note_launches(1);
+    k_peer_release<<<1, 128, 0, st>>>(d_flags, nranks, j0, j1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_peer_wait(const unsigned int *flags, uint32_t j, uint32_t target, cudaStream_t st)
+{
+    note_launches(1);
+    k_peer_wait<<<1, 32, 0, st>>>(flags, j, target);
+    return cudaGetLastError();
+}
+
 static std::atomic<unsigned long long> g_launches{0};
 
 void note_launches(unsigned k)

@@ -70,6 +70,10 @@ cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t h
                                  unsigned long long *const *d_peer, const unsigned long long *d_owner_base,
                                  uint32_t *d_tile_hist, unsigned long long *d_tile_off, unsigned int *err,
                                  cudaStream_t st);
+/* per-batch completion flags of the peer dispatch: release [j0, j1] to every owner (d_flags:
+ * device array of nranks flag-array addresses), or wait until flags[j] >= target */
+cudaError_t launch_peer_release(unsigned int *const *d_flags, int nranks, uint32_t j0, uint32_t j1, cudaStream_t st);
+cudaError_t launch_peer_wait(const unsigned int *flags, uint32_t j, uint32_t target, cudaStream_t st);
 /* single-batch replay of 8-byte wire records (batch key given) */
 cudaError_t launch_replay_wire(const hirace_dev_ctx &c, const unsigned long long *wire, uint32_t n, uint32_t batch_key,
                                int grid, cudaStream_t st);

@@ -40,7 +40,7 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_cluster_alloc", "hirace_cluster_free", "hirace_cluster_reset", "hirace_cluster_replay",
            "hirace_cluster_collect", "hirace_cluster_get_stats", "hirace_status_string",
            "hirace_version", "hirace_launch_count", "hirace_set_replay_mode", "hirace_get_replay_mode",
-           "hirace_advance_grid_epochs")
+           "hirace_advance_grid_epochs", "hirace_peer_release", "hirace_peer_wait")
 
 
 class HiraceError(RuntimeError):
@@ -141,6 +141,8 @@ def load():
         "hirace_launch_count": (I32, [ctypes.POINTER(U64)]),
         "hirace_set_replay_mode": (I32, [P, I32, U32]),
         "hirace_advance_grid_epochs": (I32, [P, U32, P]),
+        "hirace_peer_release": (I32, [P, P, I32, U32, U32, P]),
+        "hirace_peer_wait": (I32, [P, P, U32, U32, P]),
         "hirace_get_replay_mode": (I32, [P, ctypes.POINTER(I32)]),
     }
     for name, (res, args) in sig.items():
@@ -340,7 +342,7 @@ class Checker:
         """hirace_advance_grid_epochs: count grid syncs the host did not see (k device grid
         syncs of a cooperative kernel + its boundary = k + 1)."""
         _check(self.lib.hirace_advance_grid_epochs(self.h, count, _stream_handle(stream)),
-               "hirace_advance_grid_epochs")
+               "hirace_advance_grid_epochs", "hirace_peer_release", "hirace_peer_wait")
 
     def replay(self, events_dev, n: int | None = None, stream=None):
         """events_dev: CUDA tensor holding 16-byte events (uint8 [16n] or int64 [n,2])."""
@@ -508,6 +510,17 @@ class Checker:
                                              offs.ctypes.data, nb, nranks, my_rank, tab,
                                              d.ctypes.data, _stream_handle(stream)),
                "hirace_dispatch_wire")
+
+    def peer_release(self, peer_flags, j0: int, j1: int, stream=None):
+        """hirace_peer_release: +1 on flags [j0, j1] of every owner (after this rank's dispatch)."""
+        tab = (ctypes.c_void_p * len(peer_flags))(*[ctypes.c_void_p(int(p)) for p in peer_flags])
+        _check(self.lib.hirace_peer_release(self.h, tab, len(peer_flags), j0, j1, _stream_handle(stream)),
+               "hirace_peer_release")
+
+    def peer_wait(self, flags_ptr: int, j: int, target: int, stream=None):
+        """hirace_peer_wait: the stream waits until this rank's flag j >= target."""
+        _check(self.lib.hirace_peer_wait(self.h, ctypes.c_void_p(flags_ptr), j, target, _stream_handle(stream)),
+               "hirace_peer_wait")
 
     def replay_wire(self, wire_dev, n: int, batch_key: int, stream=None):
         """Replays n wire records of one batch (key g<<19 | b<<9 | w)."""

@@ -149,12 +149,18 @@ class PeerExchange:
     rank's stream before the count all-gather, so every owner has finished replaying the
     previous run before any rank dispatches into its buffer again."""
 
+    per_batch = True  # run_sharded_p2p: per-batch completion flags instead of one fence
+
     def __init__(self, group, dist, device: int = 0):
         import torch
         self.group, self.dist, self.device = group, dist, device
         self.buf = None
         self.opened = {}   # rank -> (handle, ptr)
         self.ptrs = None
+        self.flags = None          # this rank's flag array (peer buffer, zeroed once)
+        self.flag_ptrs = None      # every owner's flag array, mapped here
+        self.flag_opened = {}
+        self.uses = {}             # global batch index -> runs that used it
         # completion: an interprocess event per rank, recorded after its dispatch; the owners'
         # streams wait on the peers' events (GPU-side ordering, no stream drain)
         with torch.cuda.device(device):
@@ -199,6 +205,40 @@ class PeerExchange:
         self.ptrs = ptrs
         return ptrs
 
+    def _setup_flags(self):
+        from .hirace import MAX_BATCHES, PeerBuffer, peer_open
+        if self.flag_ptrs is not None:
+            return
+        self.flags = PeerBuffer(4 * (MAX_BATCHES + 1), self.device)  # zero-initialised
+        handles = self._gather(self.flags.handle)
+        me = self.dist.get_rank(self.group)
+        ptrs = []
+        for r, h in enumerate(handles):
+            if r == me:
+                ptrs.append(self.flags.ptr)
+            else:
+                self.flag_opened[r] = peer_open(h, self.device)
+                ptrs.append(self.flag_opened[r])
+        self.flag_ptrs = ptrs
+        self.dist.barrier(group=self.group)  # every owner's flags exist before any release
+
+    def dispatch_batch(self, ops, events, offs, i, dst_row):
+        """This rank's local batch i (or None: nothing to send for this global batch)."""
+        self._setup_flags()
+        if i is not None:
+            ops.dispatch_wire(events, offs[i:i + 2], self.ptrs, dst_row.reshape(1, -1))
+
+    def release(self, ops, j):
+        ops.ctx.peer_release(self.flag_ptrs, j, j)
+
+    def wait(self, ops, j):
+        P = self.dist.get_world_size(self.group)
+        ops.ctx.peer_wait(self.flags.ptr, j, (self.uses.get(j, 0) + 1) * P)
+
+    def end_run(self, nbg):
+        for j in range(nbg):
+            self.uses[j] = self.uses.get(j, 0) + 1
+
     def fence(self):
         """Every rank's dispatch stores are complete and visible before any replay: each rank
         records its interprocess event after its dispatch, a host barrier orders those records
@@ -228,10 +268,16 @@ class PeerExchange:
         for _, (_, ptr) in self.opened.items():
             peer_close(ptr)
         self.opened = {}
+        for _, ptr in self.flag_opened.items():
+            peer_close(ptr)
+        self.flag_opened = {}
         self.dist.barrier(group=self.group)
         if self.buf is not None:
             self.buf.free()
             self.buf = None
+        if self.flags is not None:
+            self.flags.free()
+            self.flags = None
 
 
 # ---------------------------------------------------------------------------------------------
@@ -396,9 +442,26 @@ def run_sharded_p2p(local_events, ops, exchange, group, dist, on_batch=None):
         mine[gidx] = counts
     dst, base, n_recv = p2p_layout(exchange.all_counts(mine), me)
     exchange.setup(8 * int(n_recv.sum()))
+    received = 0
+    if getattr(exchange, "per_batch", False):
+        # per-batch completion: this rank dispatches global batch j (possibly nothing) and
+        # releases it to every owner; its stream then waits until every sender released j and
+        # replays it - batch j's replay overlaps the peers' dispatch of later batches
+        local = {int(g): i for i, g in enumerate(gidx)}
+        for j, k in enumerate(order):
+            i = local.get(j)
+            exchange.dispatch_batch(ops, local_events, offs, i, dst[j] if i is not None else None)
+            exchange.release(ops, j)
+            exchange.wait(ops, j)
+            n = int(n_recv[j])
+            exchange.received(ops, int(base[j]), n, int(k))
+            received += n
+            if on_batch is not None:
+                on_batch(int(k), n)
+        exchange.end_run(nbg)
+        return received
     exchange.dispatch(ops, local_events, offs, dst[gidx] if len(keys) else np.zeros((0, P), np.int64))
     exchange.fence()
-    received = 0
     for j, k in enumerate(order):
         n = int(n_recv[j])
         exchange.received(ops, int(base[j]), n, int(k))

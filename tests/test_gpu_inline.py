@@ -122,22 +122,22 @@ def test_inline_sticky_race_across_launches_with_smem_shadow():
 def test_inline_cooperative_kernels_in_sequence_need_epoch_advance():
     # a cooperative kernel whose threads pass k device grid syncs ends k epochs past
     # the host's g.  hirace_advance_grid_epochs(k + 1) before the next kernel keeps every epoch
-    # fresh: two clean multiphase launches in a row report nothing.  With only the kernel
-    # boundary (hirace_barrier), the second launch reuses epochs of the first, and accesses the
-    # grid syncs ordered look concurrent.
+    # fresh: two clean multiphase launches in a row (each starting at the host context's g)
+    # report nothing.  With only the kernel boundary (hirace_barrier), the second launch reuses
+    # epochs of the first, and accesses the grid syncs ordered look concurrent.
     nb, phases = 6, 34
     AB = torch.rand(4 * nb * 256, device="cuda")
     bar = torch.zeros(1, dtype=torch.int32, device="cuda")
     for advance, want_empty in ((phases, True), (None, False)):
         c = hr.Checker(nb, 256, 32, 4 * nb * 256, 514)
         c.reset()
-        ex.multiphase(c, AB, nb, phases, 0, bar)
+        ex.multiphase(c, AB, nb, phases, 0, bar, g0=c.dev_ctx().g)
         torch.cuda.synchronize()
         if advance is None:
             c.barrier()
         else:
             c.advance_grid_epochs(advance)   # (phases - 1) device grid syncs + the boundary
-        ex.multiphase(c, AB, nb, phases, 0, bar)
+        ex.multiphase(c, AB, nb, phases, 0, bar, g0=c.dev_ctx().g)
         got = rdict(c.collect())
         c.close()
         assert (got == {}) == want_empty, (advance, len(got))

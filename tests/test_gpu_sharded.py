@@ -112,28 +112,38 @@ def test_replay_wire_rejects_out_of_range():
     c.close()
 
 
-def _gpu_worker(rank, world, port, name, q, wire=False):
+def _gpu_worker(rank, world, port, name, q, wire=False, split="block", multi_gpu=False):
+    """multi_gpu: one GPU per rank and NCCL (the real multi-GPU path); else every rank on GPU 0
+    with gloo for the host-side agreement."""
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
-    torch.cuda.set_device(0)
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    dev = rank if multi_gpu else 0
+    torch.cuda.set_device(dev)
+    if multi_gpu:
+        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", dev))
+    else:
+        dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         t = _make(name)
         blk = t.events["tid"] // t.block_threads
-        mine = t.events[(blk % world) == rank]
+        part = blk if split == "block" else t.events["tid"]
+        mine = t.events[(part % world) == rank]
         ops = sharded.GpuOps(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words, world,
-                             rank, device=0)
+                             rank, device=dev)
         if wire == "p2p":   # peer dispatch into CUDA-IPC-mapped buffers of the other processes
-            ex, run = sharded.PeerExchange(None, dist, device=0), sharded.run_sharded_p2p
+            ex, run = sharded.PeerExchange(None, dist, device=dev), sharded.run_sharded_p2p
+        elif multi_gpu:
+            ex = sharded.NcclExchange(None, f"cuda:{dev}")
+            run = sharded.run_sharded_wire if wire else sharded.run_sharded
         else:
             ex = sharded.HostExchange(None, device="cuda:0")
             run = sharded.run_sharded_wire if wire else sharded.run_sharded
-        n = run(_to_tensor(mine).cuda(), ops, ex, None, dist)
+        n = run(_to_tensor(mine).to(f"cuda:{dev}"), ops, ex, None, dist)
         if wire == "p2p":   # a second trace on the same buffers (handles cached, no regrowth)
-            n2 = run(_to_tensor(mine).cuda(), ops, ex, None, dist)
+            n2 = run(_to_tensor(mine).to(f"cuda:{dev}"), ops, ex, None, dist)
             assert n2 == n
             ex.close()
         races = sharded.gather_races(ops.collect(), None, dist)
-        tot = torch.tensor([n])
+        tot = torch.tensor([n], device=f"cuda:{dev}" if multi_gpu else "cpu")
         dist.all_reduce(tot)
         if rank == 0:
             q.put((int(tot.item()), races["key"].tolist(), (races["cls_and_epoch"] & 0xFF).tolist()))
@@ -185,15 +195,18 @@ def test_sharded_wire_gpu_ranks_reproduce_the_oracle(world, name):
     assert cls == [int(x) for x in c]
 
 
-@pytest.mark.parametrize("world,name", [(1, "multi"), (2, "cfg2"), (3, "multi"), (2, "cfg3"), (4, "cfg4")])
-def test_sharded_p2p_gpu_ranks_reproduce_the_oracle(world, name):
+@pytest.mark.parametrize("world,name,split", [(1, "multi", "block"), (2, "cfg2", "block"), (3, "multi", "block"),
+                                              (2, "cfg3", "block"), (4, "cfg4", "block"), (2, "cfg2", "thread")])
+def test_sharded_p2p_gpu_ranks_reproduce_the_oracle(world, name, split):
     """Peer dispatch with the real kernels: `world` processes share the GPU, each maps the
-    others' receive buffers through CUDA IPC and the dispatch kernel stores straight into them.
-    The trace is replayed twice (RACE is sticky, so the race set is unchanged)."""
+    others' receive buffers through CUDA IPC, the dispatch kernel stores straight into them and
+    every batch is released per owner (hirace_peer_release / hirace_peer_wait).  The trace is
+    replayed twice (RACE is sticky, so the race set is unchanged).  split="thread": each block's
+    events come from several ranks."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_gpu_worker, args=(r, world, port, name, q, "p2p")) for r in range(world)]
+    procs = [ctx.Process(target=_gpu_worker, args=(r, world, port, name, q, "p2p", split)) for r in range(world)]
     for p in procs:
         p.start()
     total, keys, cls = q.get(timeout=600)
@@ -201,6 +214,31 @@ def test_sharded_p2p_gpu_ranks_reproduce_the_oracle(world, name):
         p.join(timeout=120)
         assert p.exitcode == 0
     t = _make(name)
+    k, c, _ = oracle.races_of(t)
+    assert total == _words(t)
+    assert keys == [int(x) for x in k]
+    assert cls == [int(x) for x in c]
+
+
+@pytest.mark.skipif(torch.cuda.device_count() < 2, reason="needs >= 2 GPUs (one rank per GPU over NCCL)")
+@pytest.mark.parametrize("mode", ["wire", "p2p"])
+def test_sharded_multi_gpu_nccl_ranks_reproduce_the_oracle(mode):
+    """The real multi-GPU path: one process per GPU, NCCL all_to_all (wire) or peer dispatch
+    over NVLink with per-batch release flags (p2p)."""
+    world = min(4, torch.cuda.device_count())
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    wire = True if mode == "wire" else "p2p"
+    procs = [ctx.Process(target=_gpu_worker, args=(r, world, port, "cfg2", q, wire, "thread", True))
+             for r in range(world)]
+    for p in procs:
+        p.start()
+    total, keys, cls = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    t = _make("cfg2")
     k, c, _ = oracle.races_of(t)
     assert total == _words(t)
     assert keys == [int(x) for x in k]

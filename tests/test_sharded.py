@@ -129,6 +129,50 @@ class CpuPeerExchange:
             ops.replay_wire(torch.from_numpy(self.buf[start:start + n]), key)
 
 
+class CpuPeerExchangePerBatch(CpuPeerExchange):
+    """The per-batch completion protocol of sharded.PeerExchange (hirace_peer_release /
+    hirace_peer_wait): every rank dispatches global batch j (possibly nothing), releases it,
+    and its replay of j waits until every sender's records of j are in its buffer."""
+
+    per_batch = True
+
+    def setup(self, need_bytes):
+        super().setup(need_bytes)
+        self.released = []
+
+    def dispatch_batch(self, ops, events, offs, i, dst_row):
+        P = self.dist.get_world_size(self.group)
+        msgs = [[] for _ in range(P)]
+        if i is not None:
+            wire, counts = ops.bucket_wire(events, offs[i:i + 2])
+            w = wire.numpy()
+            flat = np.asarray(counts, np.int64).reshape(-1)
+            pos = np.concatenate(([0], np.cumsum(flat)))
+            for r in range(P):
+                if flat[r]:
+                    msgs[r].append((int(dst_row[r]), w[pos[r]:pos[r + 1]].copy()))
+        me = self.dist.get_rank(self.group)
+        self.pending = [m[me] for m in self._gather(msgs)]
+
+    def release(self, ops, j):
+        for m in self.pending:                   # the peers' stores of batch j land here
+            for off, recs in m:
+                assert (self.buf[off:off + len(recs)] == -1).all()
+                self.buf[off:off + len(recs)] = recs
+        self.released.append(j)
+
+    def wait(self, ops, j):
+        assert self.released and self.released[-1] == j
+
+    def received(self, ops, start, n, key):
+        assert (self.buf[start:start + n] != -1).all()   # batch j complete before its replay
+        super().received(ops, start, n, key)
+
+    def end_run(self, nbg):
+        assert self.released == list(range(nbg))
+        assert (self.buf != -1).all()
+
+
 def wire_bucket_np(ev, offsets, P, bt):
     """Reference of the hirace_bucket_wire contract (include/hirace.h): per batch, one record per
     covered word, routed to its word's owner, shard-local words, owner-grouped (stable here;
@@ -224,6 +268,8 @@ def _worker(rank, world, port, name, q, wire=False, split="block"):
         ops = CpuTestOps(t, world, rank)
         if wire == "p2p":
             ex, run = CpuPeerExchange(None, dist), sharded.run_sharded_p2p
+        elif wire == "p2p_batch":
+            ex, run = CpuPeerExchangePerBatch(None, dist), sharded.run_sharded_p2p
         else:
             ex = sharded.HostExchange(None)
             run = sharded.run_sharded_wire if wire else sharded.run_sharded
@@ -287,15 +333,16 @@ def test_sharded_wire_pipeline_reproduces_the_oracle(world, name, split):
     assert len(k) > 0
 
 
+@pytest.mark.parametrize("mode", ["p2p", "p2p_batch"])
 @pytest.mark.parametrize("world,name", [(2, "cfg2"), (3, "cfg4"), (2, "cfg3"), (3, "wide"), (4, "multi")])
-def test_sharded_p2p_pipeline_reproduces_the_oracle(world, name):
+def test_sharded_p2p_pipeline_reproduces_the_oracle(world, name, mode):
     """Peer-memory dispatch (run_sharded_p2p): count matrices all-gathered once, every rank
     stores its records at sharded.p2p_layout offsets of the owners' buffers (disjoint, every
     slot written), owners replay batch by batch."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, name, q, "p2p")) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, name, q, mode)) for r in range(world)]
     for p in procs:
         p.start()
     total, keys, cls = q.get(timeout=300)
