@@ -342,7 +342,7 @@ class Checker:
         """hirace_advance_grid_epochs: count grid syncs the host did not see (k device grid
         syncs of a cooperative kernel + its boundary = k + 1)."""
         _check(self.lib.hirace_advance_grid_epochs(self.h, count, _stream_handle(stream)),
-               "hirace_advance_grid_epochs", "hirace_peer_release", "hirace_peer_wait")
+               "hirace_advance_grid_epochs")
 
     def replay(self, events_dev, n: int | None = None, stream=None):
         """events_dev: CUDA tensor holding 16-byte events (uint8 [16n] or int64 [n,2])."""
