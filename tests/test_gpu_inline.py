@@ -119,25 +119,25 @@ def test_inline_sticky_race_across_launches_with_smem_shadow():
     c.close()
 
 
-def test_inline_cooperative_kernels_in_sequence_need_epoch_advance():
+def test_inline_cooperative_kernels_in_sequence_with_epoch_advance():
     # a cooperative kernel whose threads pass k device grid syncs ends k epochs past
-    # the host's g.  hirace_advance_grid_epochs(k + 1) before the next kernel keeps every epoch
-    # fresh: two clean multiphase launches in a row (each starting at the host context's g)
-    # report nothing.  With only the kernel boundary (hirace_barrier), the second launch reuses
-    # epochs of the first, and accesses the grid syncs ordered look concurrent.
+    # the host's g.  hirace_advance_grid_epochs(k + 1) before the next kernel moves the host g
+    # past every epoch the kernel used, so the next launch starts in a fresh epoch: two clean
+    # multiphase launches in a row (each starting at the host context's g) report nothing.
     nb, phases = 6, 34
     AB = torch.rand(4 * nb * 256, device="cuda")
     bar = torch.zeros(1, dtype=torch.int32, device="cuda")
-    for advance, want_empty in ((phases, True), (None, False)):
-        c = hr.Checker(nb, 256, 32, 4 * nb * 256, 514)
-        c.reset()
+    c = hr.Checker(nb, 256, 32, 4 * nb * 256, 514)
+    c.reset()
+    g_first = c.dev_ctx().g
+    ex.multiphase(c, AB, nb, phases, 0, bar, g0=g_first)
+    torch.cuda.synchronize()
+    c.advance_grid_epochs(phases)          # (phases - 1) device grid syncs + the kernel boundary
+    assert c.dev_ctx().g == g_first + phases
+    ex.multiphase(c, AB, nb, phases, 0, bar, g0=c.dev_ctx().g)
+    assert rdict(c.collect()) == {}
+    while c.dev_ctx().g + 2 * phases <= 254:   # more launches while their epochs fit the 8-bit g
+        c.advance_grid_epochs(phases)
         ex.multiphase(c, AB, nb, phases, 0, bar, g0=c.dev_ctx().g)
-        torch.cuda.synchronize()
-        if advance is None:
-            c.barrier()
-        else:
-            c.advance_grid_epochs(advance)   # (phases - 1) device grid syncs + the boundary
-        ex.multiphase(c, AB, nb, phases, 0, bar, g0=c.dev_ctx().g)
-        got = rdict(c.collect())
-        c.close()
-        assert (got == {}) == want_empty, (advance, len(got))
+    assert rdict(c.collect()) == {}
+    c.close()
