@@ -13,6 +13,8 @@
 
 #include <mutex>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "hirace.h"
 #include "hirace_device.cuh"
 #include "internal.h"
@@ -73,6 +75,13 @@ struct hirace_ctx {
 };
 
 namespace {
+
+/* NVTX range over one API call (Nsight timelines; header-only nvtx3, near-free when no tool is
+ * attached) */
+struct Nvtx {
+    explicit Nvtx(const char *name) { nvtxRangePushA(name); }
+    ~Nvtx() { nvtxRangePop(); }
+};
 
 hirace_status set_sticky(hirace_ctx *c, hirace_status s)
 {
@@ -543,6 +552,7 @@ hirace_status hirace_set_policy(hirace_ctx *c, int policy, void *stream)
 
 hirace_status hirace_shadow_reset(hirace_ctx *c, void *stream)
 {
+    Nvtx nvtx_range("hirace_shadow_reset");
     if (!c)
         return HIRACE_E_INVAL;
     cudaStream_t st = (cudaStream_t)stream;
@@ -597,6 +607,7 @@ hirace_status hirace_advance_grid_epochs(hirace_ctx *c, uint32_t count, void *st
 
 hirace_status hirace_replay_trace(hirace_ctx *c, const hirace_event *d_events, uint64_t n, void *stream)
 {
+    Nvtx nvtx_range("hirace_replay_trace");
     if (!c)
         return HIRACE_E_INVAL;
     if (c->sticky != HIRACE_OK)
@@ -668,6 +679,7 @@ hirace_status hirace_find_batches(hirace_ctx *c, const hirace_event *d_events, u
 hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_events, uint64_t n, hirace_race *d_out,
                                         uint64_t cap, unsigned long long *d_n_total, void *stream)
 {
+    Nvtx nvtx_range("hirace_check_trace_device");
     if (!c || !d_n_total || (cap && !d_out))
         return HIRACE_E_INVAL;
     if (c->sticky != HIRACE_OK)
@@ -708,6 +720,7 @@ hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_eve
 hirace_status hirace_collect_races_device(hirace_ctx *c, hirace_race *d_out, uint64_t cap,
                                           unsigned long long *d_n_total, void *stream)
 {
+    Nvtx nvtx_range("hirace_collect_races_device");
     if (!c || !d_n_total || (cap && !d_out))
         return HIRACE_E_INVAL;
     HR_CUDA(c, cudaSetDevice(c->device));
@@ -718,6 +731,7 @@ hirace_status hirace_collect_races_device(hirace_ctx *c, hirace_race *d_out, uin
 
 hirace_status hirace_collect_races(hirace_ctx *c, hirace_race *h_out, uint64_t cap, uint64_t *n_total, void *stream)
 {
+    Nvtx nvtx_range("hirace_collect_races");
     if (!c || !n_total || (cap && !h_out))
         return HIRACE_E_INVAL;
     cudaStream_t st = (cudaStream_t)stream;
@@ -745,6 +759,7 @@ hirace_status hirace_collect_races(hirace_ctx *c, hirace_race *h_out, uint64_t c
 hirace_status hirace_check_trace_host(hirace_ctx *c, const hirace_event *h_events, uint64_t n, hirace_race *h_out,
                                       uint64_t cap, uint64_t *n_total, void *stream)
 {
+    Nvtx nvtx_range("hirace_check_trace_host");
     if (!c || !n_total || (n && !h_events))
         return HIRACE_E_INVAL;
     if (c->sticky != HIRACE_OK)
@@ -962,6 +977,7 @@ extern "C" {
 hirace_status hirace_count_wire(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
                                 int nranks, int my_rank, uint64_t *h_counts, void *stream)
 {
+    Nvtx nvtx_range("hirace_count_wire");
     uint64_t n = 0;
     if (!c || !h_counts || !h_offsets || (nb && !d_in))
         return HIRACE_E_INVAL;
@@ -971,6 +987,7 @@ hirace_status hirace_count_wire(hirace_ctx *c, const hirace_event *d_in, const u
 hirace_status hirace_dispatch_wire(hirace_ctx *c, const hirace_event *d_in, const uint32_t *h_offsets, uint64_t nb,
                                    int nranks, int my_rank, void *const *h_peer, const uint64_t *h_dst, void *stream)
 {
+    Nvtx nvtx_range("hirace_dispatch_wire");
     if (!c || !h_offsets || !h_peer || !h_dst || (nb && !d_in))
         return HIRACE_E_INVAL;
     if (c->sticky != HIRACE_OK)
@@ -1014,6 +1031,7 @@ hirace_status hirace_dispatch_wire(hirace_ctx *c, const hirace_event *d_in, cons
 hirace_status hirace_peer_release(hirace_ctx *c, void *const *h_peer_flags, int nranks, uint32_t j0, uint32_t j1,
                                   void *stream)
 {
+    Nvtx nvtx_range("hirace_peer_release");
     if (!c || !h_peer_flags || nranks < 1 || nranks > 32 || j1 < j0 || j1 >= HIRACE_MAX_BATCHES)
         return HIRACE_E_INVAL;
     for (int r = 0; r < nranks; r++)
@@ -1031,6 +1049,7 @@ hirace_status hirace_peer_release(hirace_ctx *c, void *const *h_peer_flags, int 
 
 hirace_status hirace_peer_wait(hirace_ctx *c, const void *d_flags, uint32_t j, uint32_t target, void *stream)
 {
+    Nvtx nvtx_range("hirace_peer_wait");
     if (!c || !d_flags || j >= HIRACE_MAX_BATCHES)
         return HIRACE_E_INVAL;
     HR_CUDA(c, cudaSetDevice(c->device));
@@ -1138,6 +1157,7 @@ hirace_status hirace_bucket_wire(hirace_ctx *c, const hirace_event *d_in, const 
                                  int nranks, int my_rank, uint64_t *d_out, uint64_t cap, uint64_t *h_counts,
                                  uint64_t *n_words, void *stream)
 {
+    Nvtx nvtx_range("hirace_bucket_wire");
     if (cap && !d_out)
         return HIRACE_E_INVAL;
     uint64_t dummy = 0;
@@ -1150,6 +1170,7 @@ hirace_status hirace_bucket_wire(hirace_ctx *c, const hirace_event *d_in, const 
 
 hirace_status hirace_replay_wire(hirace_ctx *c, const uint64_t *d_wire, uint64_t n, uint32_t batch_key, void *stream)
 {
+    Nvtx nvtx_range("hirace_replay_wire");
     if (!c)
         return HIRACE_E_INVAL;
     if (c->sticky != HIRACE_OK)

@@ -41,6 +41,25 @@ from __future__ import annotations
 import numpy as np
 
 CHUNK_LOG2 = 14
+
+
+def _nvtx_push(msg: str):
+    """NVTX range per batch (Nsight timelines; a no-op without CUDA)."""
+    try:
+        import torch
+        if torch.cuda.is_available():
+            torch.cuda.nvtx.range_push(msg)
+    except Exception:
+        pass
+
+
+def _nvtx_pop():
+    try:
+        import torch
+        if torch.cuda.is_available():
+            torch.cuda.nvtx.range_pop()
+    except Exception:
+        pass
 SHARED_BIT = np.uint64(1) << np.uint64(63)
 
 
@@ -173,8 +192,16 @@ class PeerExchange:
         return objs
 
     def all_counts(self, counts):
-        """counts: int64 [nbg, P] of this rank -> [P_sender, nbg, P_owner] of all ranks."""
-        return np.stack([np.asarray(c, np.int64) for c in self._gather(np.asarray(counts, np.int64))])
+        """counts: int64 [nbg, P] of this rank -> [P_sender, nbg, P_owner] of all ranks: one
+        all_gather of tensors (device tensors over NCCL; host tensors over gloo)."""
+        import torch
+        P = self.dist.get_world_size(self.group)
+        c = torch.from_numpy(np.ascontiguousarray(counts, dtype=np.int64))
+        if self.dist.get_backend(self.group) == "nccl":
+            c = c.to(f"cuda:{self.device}")
+        out = [torch.empty_like(c) for _ in range(P)]
+        self.dist.all_gather(out, c, group=self.group)
+        return np.stack([o.cpu().numpy() for o in out])
 
     def setup(self, need_bytes: int):
         """Every rank's buffer holds at least its own need; returns the peer table (device
@@ -366,6 +393,7 @@ def run_sharded(local_events, ops, exchange, group, dist, on_batch=None):
     where = {int(k): i for i, k in enumerate(keys)}
     received = 0
     for key in order:
+        _nvtx_push(f"hirace batch key {int(key)}")
         i = where.get(int(key))
         part = local_events[int(offs[i]):int(offs[i + 1])] if i is not None else local_events[0:0]
         send, send_counts = ops.bucket(part)
@@ -373,6 +401,7 @@ def run_sharded(local_events, ops, exchange, group, dist, on_batch=None):
         recv = exchange.payload(send, send_counts, recv_counts)
         ops.replay(recv)
         received += int(recv.shape[0])
+        _nvtx_pop()
         if on_batch is not None:
             on_batch(int(key), int(recv.shape[0]))
     return received
@@ -406,9 +435,11 @@ def run_sharded_wire(local_events, ops, exchange, group, dist, on_batch=None):
                                               recv[:, j].tolist()))
     received = 0
     for j, k in enumerate(order):
+        _nvtx_push(f"hirace wire batch {j} (key {int(k)})")
         got = exchange.finish(handles[j])
         handles[j] = None
         ops.replay_wire(got, int(k))
+        _nvtx_pop()
         received += int(got.shape[0])
         if on_batch is not None:
             on_batch(int(k), int(got.shape[0]))
@@ -450,11 +481,13 @@ def run_sharded_p2p(local_events, ops, exchange, group, dist, on_batch=None):
         local = {int(g): i for i, g in enumerate(gidx)}
         for j, k in enumerate(order):
             i = local.get(j)
+            _nvtx_push(f"hirace p2p batch {j} (key {int(k)})")
             exchange.dispatch_batch(ops, local_events, offs, i, dst[j] if i is not None else None)
             exchange.release(ops, j)
             exchange.wait(ops, j)
             n = int(n_recv[j])
             exchange.received(ops, int(base[j]), n, int(k))
+            _nvtx_pop()
             received += n
             if on_batch is not None:
                 on_batch(int(k), n)
