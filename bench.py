@@ -305,6 +305,25 @@ def measure_slowdown(dev: int, reps: int = 5) -> dict:
         return tot / reps
 
     out = {}
+    for agg in (False, True):  # per-thread hooks, then warp-aggregated hooks (HIRACE_INLINE_AGGREGATE)
+        ex.use_aggregated_hooks(agg)
+        r = _slowdown_programs(dev, reps, timed)
+        if not agg:
+            out.update(r)
+        else:
+            for k, v in r.items():
+                out[k]["slowdown_warp_aggregated"] = v["slowdown"]
+    ex.use_aggregated_hooks(False)
+    return out
+
+
+def _slowdown_programs(dev: int, reps: int, timed) -> dict:
+    import torch
+
+    import paper_conf_sc_jacobsonbg24_b200 as hr
+    import tracegen as tg
+    from paper_conf_sc_jacobsonbg24_b200 import examples as ex
+    out = {}
     n, steps = 512, 8
     c = hr.Checker(1024, 256, 32, 2 * n * n, 324, device=dev)
     buf = torch.rand(2 * n * n, device=f"cuda:{dev}")

@@ -17,6 +17,7 @@ LIBDIR = os.path.join(PKG, "lib")
 SO = os.path.join(LIBDIR, "libhirace.so")
 EXDIR = os.path.join(PKG, "examples")
 EXSO = os.path.join(LIBDIR, "libhirace_examples.so")
+EXSO_AGG = os.path.join(LIBDIR, "libhirace_examples_agg.so")  # inline hooks with warp aggregation
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -41,9 +42,9 @@ def stale(so, srcs) -> bool:
     return any(os.path.getmtime(p) > t for p in srcs + headers())
 
 
-def _nvcc(so, srcs, verbose):
+def _nvcc(so, srcs, verbose, defines=()):
     cmd = [NVCC, *ARCH, "-lineinfo", "-O3", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "-shared",
-           "-I", INCLUDE, "-I", CSRC, "-o", so + ".tmp", *srcs]
+           *[f"-D{d}" for d in defines], "-I", INCLUDE, "-I", CSRC, "-o", so + ".tmp", *srcs]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     subprocess.check_call(cmd)
@@ -57,6 +58,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         _nvcc(SO, sources(), verbose)
     if force or stale(EXSO, ex_sources()):
         _nvcc(EXSO, ex_sources(), verbose)
+    if force or stale(EXSO_AGG, ex_sources()):
+        _nvcc(EXSO_AGG, ex_sources(), verbose, defines=("HIRACE_INLINE_AGGREGATE=1",))
     return SO
 
 

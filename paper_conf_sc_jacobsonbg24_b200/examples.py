@@ -9,16 +9,26 @@ import os
 
 from .hirace import DevCtx, _stream_handle
 
-_LIB = os.path.join(os.path.dirname(os.path.abspath(__file__)), "lib", "libhirace_examples.so")
-_lib = None
+_LIBDIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "lib")
+_SO = {False: os.path.join(_LIBDIR, "libhirace_examples.so"),       # per-thread inline hooks
+       True: os.path.join(_LIBDIR, "libhirace_examples_agg.so")}    # warp-aggregated (HIRACE_INLINE_AGGREGATE)
+_libs = {}
+_aggregate = False
+
+
+def use_aggregated_hooks(flag: bool):
+    """Selects the build of the native programs whose hooks aggregate same-element accesses of a
+    warp (hirace::on_access_warp) instead of checking thread by thread."""
+    global _aggregate
+    _aggregate = bool(flag)
 
 
 def load():
-    global _lib
-    if _lib is None:
-        if not os.path.exists(_LIB):
-            raise RuntimeError(f"{_LIB} missing: python -m paper_conf_sc_jacobsonbg24_b200.build")
-        lib = ctypes.CDLL(_LIB)
+    if _aggregate not in _libs:
+        so = _SO[_aggregate]
+        if not os.path.exists(so):
+            raise RuntimeError(f"{so} missing: python -m paper_conf_sc_jacobsonbg24_b200.build")
+        lib = ctypes.CDLL(so)
         P, I, U = ctypes.c_void_p, ctypes.c_int, ctypes.c_uint
         lib.hx_stencil.argtypes = [P, P, I, I, I, U, I, P]
         lib.hx_reduce.argtypes = [P, P, I, I, I, U, I, P]
@@ -26,8 +36,8 @@ def load():
         lib.hx_bfs.argtypes = [P, P, P, P, I, I, U, ctypes.POINTER(I), P]
         for f in (lib.hx_stencil, lib.hx_reduce, lib.hx_multiphase, lib.hx_bfs):
             f.restype = I
-        _lib = lib
-    return _lib
+        _libs[_aggregate] = lib
+    return _libs[_aggregate]
 
 
 def _ctx(checker, base_ptr):
@@ -78,4 +88,4 @@ def bfs(checker, base, nindex, nlist, dist, V: int, racy: bool, g0: int = 0, str
     return levels.value
 
 
-__all__ = ["stencil", "reduce", "multiphase", "bfs", "load", "DevCtx"]
+__all__ = ["stencil", "reduce", "multiphase", "bfs", "load", "use_aggregated_hooks", "DevCtx"]

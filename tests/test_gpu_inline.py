@@ -19,6 +19,15 @@ import paper_conf_sc_jacobsonbg24_b200 as hr  # noqa: E402
 from paper_conf_sc_jacobsonbg24_b200 import examples as ex  # noqa: E402
 
 
+@pytest.fixture(autouse=True, params=[False, True], ids=["thread_hooks", "warp_hooks"])
+def hooks(request):
+    """Every inline test runs with the per-thread hooks and with the warp-aggregated ones
+    (hirace::on_access_warp, libhirace_examples_agg.so)."""
+    ex.use_aggregated_hooks(request.param)
+    yield request.param
+    ex.use_aggregated_hooks(False)
+
+
 def odict(t):
     k, c, _ = oracle.races_of(t)
     return {int(a): int(b) for a, b in zip(k, c)}
