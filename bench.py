@@ -521,6 +521,9 @@ def measure_single(args, config: int, variant: str, K: int, W: int, dev: int, cl
     if args.replay_mode != "auto":
         c.set_replay_mode({"batch": hr.REPLAY_BATCH, "window": hr.REPLAY_WINDOW}[args.replay_mode], args.window_log2)
     window = c.window_active
+    epoch = args.reset_mode == "epoch" and not window and c.rec_bytes == 8
+    if epoch:
+        c.set_reset_mode(hr.RESET_EPOCH)
     d_ev = hr.events_to_device(trace.events, f"cuda:{dev}")
     cap = 1 << 20
     d_out = torch.empty(cap * 16, dtype=torch.uint8, device=f"cuda:{dev}")
@@ -590,13 +593,28 @@ def measure_single(args, config: int, variant: str, K: int, W: int, dev: int, cl
         except Exception as exc:  # capture unsupported: the eager timing stands
             print(f"bench: CUDA graph step unavailable ({exc}); eager timing", file=sys.stderr)
     st = c.stats()
+    reset = {"mode": "window-lazy" if window else ("epoch" if epoch else "full")}
+    if epoch:
+        # epoch reset: a rebase sweep of the whole shadow every floor(255 / epochs per check)
+        # checks; its cost, amortised, is added to the measured step (reading R19)
+        gmax = int((trace.events["meta"][-1] >> 24) & 255) if trace.n else 0
+        per_sweep = max(1, 255 // (gmax + 1))
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        c.barrier(stream=stream)         # normalises the shadow: one forced rebase sweep
+        e1.record(stream)
+        torch.cuda.synchronize()
+        sweep_ms = e0.elapsed_time(e1)
+        ms += K * sweep_ms / per_sweep
+        reset.update(sweep_ms=sweep_ms, checks_per_sweep=per_sweep, amortized_ms_per_step=sweep_ms / per_sweep,
+                     note="amortised sweep added to ms_per_step")
     peak, peak_kind = peaks()
     bpa = bytes_per_access(c.rec_bytes)
     ms_per_step = ms / K
     achieved = bpa * n_acc / (kern_ms / 1e3) / 1e9
     key = f"cfg{config}_{variant}" + ("_compact" if args.compact else "")
     res = {"config": config, "variant": variant, "trace": trace.name, "events": int(trace.n), "accesses": n_acc,
-           "replay": "window-major" if window else "batch-major",
+           "replay": "window-major" if window else "batch-major", "reset": reset,
            "value": n_acc * K / (ms / 1e3), "ms_per_step": ms_per_step, "step_mode": step_mode,
            "eager_ms_per_step": eager_ms / K, "launches_per_step": launches_per_step,
            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
@@ -666,7 +684,9 @@ def main():
     ap.add_argument("--no-graph", action="store_true", help="time the eager step instead of its CUDA graph")
     ap.add_argument("--replay-mode", default="auto", choices=["auto", "batch", "window"],
                     help="hirace_set_replay_mode: batch-major k_replay or window-major (auto: window for >= 1 GiB)")
-    ap.add_argument("--window-log2", type=int, default=0, help="records per window (log2; 0 = 14)")
+    ap.add_argument("--window-log2", type=int, default=0, help="records per window (log2; 0 = 12)")
+    ap.add_argument("--reset-mode", default="epoch", choices=["epoch", "full"],
+                    help="hirace_set_reset_mode: epoch (O(flagged) reset, amortised sweeps counted) or full memset")
     ap.add_argument("--compact", action="store_true",
                     help="compact 4-byte shadow records (hirace_shadow_alloc_compact, SURVEY §8(f) f1)")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p", "host"],
@@ -744,7 +764,7 @@ def main():
             r, _ = measure_single(args, cfg, "racy", min(K, 20), W, dev, None)
             per_config[f"config{cfg}"] = {k: r[k] for k in ("trace", "events", "value", "ms_per_step", "step_mode",
                                                             "roofline", "roofline_step", "flagged_words",
-                                                            "launches_per_step")}
+                                                            "launches_per_step", "replay", "reset")}
     slow = None if (args.no_slowdown or rank != 0) else measure_slowdown(dev)
     clocks.stop()
     if rank != 0:
@@ -765,6 +785,7 @@ def main():
         "cpu_baseline": cpu, "e2e": e2e,
         "gpu_launches": res["launches_per_step"] * K,
         "step_mode": res["step_mode"], "eager_ms_per_step": res["eager_ms_per_step"],
+        "replay": res["replay"], "reset": res["reset"],
         "clocks": clocks.summary(),
         "check": {"flagged_words": res["flagged_words"], "expected_flagged": res["expected_flagged"],
                   "per_step": st},  # stats are per step (reset clears them)

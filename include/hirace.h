@@ -149,6 +149,9 @@ typedef struct {
     unsigned int f_active, f_tid_mask, f_tid_match, f_spaces;
     unsigned long long f_glo, f_ghi;
     unsigned int f_smem_words, f_pad;
+    /* epoch reset (hirace_set_reset_mode): device word holding the grid-epoch offset the
+     * replay adds to every trace g (records store g + offset); NULL = 0                     */
+    const unsigned int *g_base;
 } hirace_dev_ctx;
 
 /* ---- lifecycle (a11: shadow alloc/init, "Initially, all State values are set
@@ -190,6 +193,23 @@ hirace_status hirace_shadow_free(hirace_ctx *ctx);
 
 /* Sets every shadow record to INIT, clears reports, stats and sticky errors; g := 0. Async. */
 hirace_status hirace_shadow_reset(hirace_ctx *ctx, void *stream);
+
+/* How hirace_shadow_reset returns the shadow to all-INIT (reading R19).
+ * FULL (default): every record is rewritten (a memset of the shadow: 32 GiB on config 5).
+ * EPOCH: O(flagged words) - the next check's grid epochs start past every epoch used since the
+ * last sweep (the replay adds an offset to the trace's g), so a record left by an earlier
+ * check has a different g and reads as INIT by the FSM's own rule (a different grid epoch
+ * restarts a record, reading R4); only the RACE records (sticky) are cleared, from the report
+ * buffer.  A full sweep still happens when the report buffer overflowed, and a rebase sweep
+ * (records of the current check keep their epochs minus the offset, older ones become INIT)
+ * when the offset plus a trace's largest g would pass 254 - once per ~254 / (epochs per
+ * check) checks.  Race sets and classes are identical in both modes; the g in reported
+ * cls_and_epoch is the trace's g in both.  EPOCH applies to the batch-major replay of 8-byte
+ * records; inline hooks, wire replay and hirace_barrier first normalise the shadow (a rebase
+ * sweep).  INVAL for compact contexts or window-major mode, or an unknown mode.  Waits for the
+ * device, then resets the shadow. */
+typedef enum { HIRACE_RESET_FULL = 0, HIRACE_RESET_EPOCH = 1 } hirace_reset_mode;
+hirace_status hirace_set_reset_mode(hirace_ctx *ctx, int mode);
 
 /* Host barrier hook.  Only HIRACE_SCOPE_GRID is meaningful on the host: a kernel boundary /
  * grid sync advances the context's grid epoch g used by inline hooks.  When g

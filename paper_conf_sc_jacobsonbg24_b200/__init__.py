@@ -5,7 +5,7 @@ The compute path is libhirace.so (sm_100a CUDA kernels behind the C-ABI in inclu
 """
 from .hirace import (ATOMIC_BLOCK, ATOMIC_GRID, EVENT_DTYPE, RACE_DTYPE, READ, WRITE, Checker, ClusterChecker,  # noqa: F401
                      HiraceError, POLICY_RELAXED_READ_ATOMIC, POLICY_STRICT, REPLAY_AUTO, REPLAY_BATCH,
-                     REPLAY_WINDOW, events_to_device, launch_count, fsm_step,
+                     REPLAY_WINDOW, RESET_EPOCH, RESET_FULL, events_to_device, launch_count, fsm_step,
                      fsm_cluster_class, fsm_step_cluster, fsm_step_compact, fsm_table,
                      fsm_table_cluster, load, races_to_dict, trace_epoch_limits)
 
@@ -13,4 +13,4 @@ __all__ = ["Checker", "ClusterChecker", "HiraceError", "EVENT_DTYPE", "RACE_DTYP
            "fsm_table", "fsm_table_cluster", "fsm_step_cluster", "fsm_cluster_class", "trace_epoch_limits",
            "load", "races_to_dict", "READ", "WRITE", "ATOMIC_BLOCK", "ATOMIC_GRID",
            "POLICY_STRICT", "POLICY_RELAXED_READ_ATOMIC", "REPLAY_AUTO", "REPLAY_BATCH", "REPLAY_WINDOW",
-           "launch_count"]
+           "RESET_FULL", "RESET_EPOCH", "launch_count"]

@@ -20,6 +20,9 @@
 namespace hirace_impl {
 
 constexpr int kCollectPerThread = 16; /* consecutive words per thread per tile */
+
+/* epoch reset: records hold g + offset; collected rows carry the trace's g */
+__device__ __forceinline__ uint32_t gsub(const hirace_dev_ctx &c) { return c.g_base ? *c.g_base : 0u; }
 static_assert(kCollectTile == 256 * kCollectPerThread, "collect tile = 256 threads x 16 words");
 
 /* flagged-word count of the 16 words of this thread in tile t; words kept in v (16-byte
@@ -188,7 +191,7 @@ __device__ __forceinline__ void collect_phase(const hirace_dev_ctx &c, uint64_t 
                                 const uint64_t blk = sidx / smem_words;
                                 rr.key = HIRACE_SHARED_BIT | (blk << 32) | (sidx - blk * smem_words);
                             }
-                            rr.cls_and_epoch = hirace::race_class(hirace::st_of(o)) | (rec.g(o) << 8);
+                            rr.cls_and_epoch = hirace::race_class(hirace::st_of(o)) | (((rec.g(o) - gsub(c)) & 255u) << 8);
                             rr.detect_tid = rec.tid(o);
                             out[pos] = rr;
                         }
@@ -286,7 +289,7 @@ __device__ __forceinline__ bool collect_phase_small(const hirace_dev_ctx &c, uin
                     const uint64_t blk = sidx / smem_words;
                     rr.key = HIRACE_SHARED_BIT | (blk << 32) | (sidx - blk * smem_words);
                 }
-                rr.cls_and_epoch = hirace::race_class(hirace::st_of(v[k])) | (rec.g(v[k]) << 8);
+                rr.cls_and_epoch = hirace::race_class(hirace::st_of(v[k])) | (((rec.g(v[k]) - gsub(c)) & 255u) << 8);
                 rr.detect_tid = rec.tid(v[k]);
                 out[at] = rr;
             }
@@ -366,7 +369,7 @@ __device__ __forceinline__ void collect_reports_cta(const hirace_dev_ctx &c, hir
         if (pos < cap) {
             hirace_race rr;
             rr.key = key;
-            rr.cls_and_epoch = hirace::race_class(hirace::st_of(o)) | (rec.g(o) << 8);
+            rr.cls_and_epoch = hirace::race_class(hirace::st_of(o)) | (((rec.g(o) - gsub(c)) & 255u) << 8);
             rr.detect_tid = rec.tid(o);
             out[pos] = rr;
         }

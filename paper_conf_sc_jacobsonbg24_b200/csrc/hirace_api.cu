@@ -69,6 +69,8 @@ struct hirace_ctx {
     hirace_event *d_trace = nullptr; /* whole-trace staging for hirace_check_trace_host */
     uint64_t trace_cap = 0;
     bool lazy = false;            /* a lazy reset left stale windows behind */
+    int reset_mode = HIRACE_RESET_FULL;
+    unsigned int *d_gepoch = nullptr; /* epoch reset: {gbase, gnext} (device) */
     uint32_t g = 0;
     cudaEvent_t t_start = nullptr, t_stop = nullptr;
     hirace_status sticky = HIRACE_OK;
@@ -257,6 +259,16 @@ cudaError_t window_scratch(hirace_ctx *c, uint64_t n)
     return cudaSuccess;
 }
 
+/* epoch reset: bring the shadow back to offset 0 (records keep the trace's g) before a path
+ * that does not add the offset (inline hooks, wire replay, hirace_barrier) */
+hirace_status ensure_epoch_normal(hirace_ctx *c, cudaStream_t st)
+{
+    if (c->reset_mode != HIRACE_RESET_EPOCH)
+        return HIRACE_OK;
+    HR_CUDA(c, launch_epoch_prep(c->dev, c->shadow_words, c->d_gepoch, nullptr, nullptr, nullptr, 1, c->sm_count, st));
+    return HIRACE_OK;
+}
+
 /* stale windows := INIT before a path that reads or writes the shadow directly */
 hirace_status ensure_materialized(hirace_ctx *c, cudaStream_t st)
 {
@@ -307,12 +319,40 @@ hirace_status hirace_set_replay_mode(hirace_ctx *c, int mode, uint32_t window_lo
     }
     c->replay_mode = mode;
     c->lazy = false;
+    if (window_active(c)) { /* window-major has its own (lazy) reset */
+        c->reset_mode = HIRACE_RESET_FULL;
+        c->dev.g_base = nullptr;
+    }
     /* the mode change starts from an all-INIT shadow (full reset: every window current) */
     HR_CUDA(c, launch_reset(c->d_shadow, c->shadow_words * c->rec_bytes, c->d_report_count, c->d_stats, c->d_err,
                             c->sm_count, nullptr));
     HR_CUDA(c, cudaDeviceSynchronize());
     c->g = 0;
     c->dev.g = 0;
+    c->sticky = HIRACE_OK;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_set_reset_mode(hirace_ctx *c, int mode)
+{
+    if (!c || (mode != HIRACE_RESET_FULL && mode != HIRACE_RESET_EPOCH))
+        return HIRACE_E_INVAL;
+    if (mode == HIRACE_RESET_EPOCH && (c->rec_bytes != 8 || window_active(c)))
+        return HIRACE_E_INVAL;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    HR_CUDA(c, cudaDeviceSynchronize());
+    if (mode == HIRACE_RESET_EPOCH) {
+        if (!c->d_gepoch)
+            HR_CUDA(c, cudaMalloc(&c->d_gepoch, 4 * sizeof(unsigned int)));
+        HR_CUDA(c, cudaMemset(c->d_gepoch, 0, 4 * sizeof(unsigned int)));
+        c->dev.g_base = c->d_gepoch;
+    } else {
+        c->dev.g_base = nullptr;
+    }
+    c->reset_mode = mode;
+    HR_CUDA(c, launch_reset(c->d_shadow, c->shadow_words * c->rec_bytes, c->d_report_count, c->d_stats, c->d_err,
+                            c->sm_count, nullptr));
+    HR_CUDA(c, cudaDeviceSynchronize());
     c->sticky = HIRACE_OK;
     return HIRACE_OK;
 }
@@ -452,6 +492,7 @@ hirace_status shadow_alloc_impl(const hirace_config *cfg, const hirace_epoch_lim
     d.f_ghi = ~0ull;
     d.f_smem_words = d.smem_words;
     d.f_pad = 0;
+    d.g_base = nullptr;
     d.c_sh_b = lay.sh_b;
     d.c_sh_w = lay.sh_w;
     d.c_sh_t = lay.sh_t;
@@ -492,7 +533,7 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
                     c->scr.batch_off, c->scr.nbatches, c->scr.batch_ctr, c->scr.grid_bar,
                     c->scr.grid_bar2, c->scr.cta_cnt, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
                     c->d_stage[0], c->d_stage[1], c->d_wire_off, c->d_wire_counts, c->d_wire_flag,
-                    c->d_peer_tab, c->d_flag_tab};
+                    c->d_peer_tab, c->d_flag_tab, c->d_gepoch};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
@@ -560,6 +601,9 @@ hirace_status hirace_shadow_reset(hirace_ctx *c, void *stream)
     if (window_active(c)) { /* lazy: the generation moves on, windows read as INIT (O(1)) */
         HR_CUDA(c, launch_lazy_reset(c->dev, c->win, st));
         c->lazy = true;
+    } else if (c->reset_mode == HIRACE_RESET_EPOCH) { /* O(flagged): epochs move on */
+        HR_CUDA(c, launch_epoch_reset(c->dev, c->shadow_words, c->d_gepoch, c->sm_count, st));
+        c->lazy = false;
     } else {
         HR_CUDA(c, launch_reset(c->d_shadow, c->shadow_words * c->rec_bytes, c->d_report_count, c->d_stats, c->d_err,
                                 c->sm_count, st));
@@ -591,6 +635,8 @@ hirace_status hirace_advance_grid_epochs(hirace_ctx *c, uint32_t count, void *st
     if (c->rec_bytes != 8) /* compact contexts are replay-only */
         return set_sticky(c, HIRACE_E_INVAL);
     HR_CUDA(c, cudaSetDevice(c->device));
+    if (count && ensure_epoch_normal(c, (cudaStream_t)stream) != HIRACE_OK)
+        return c->sticky;
     for (uint32_t k = 0; k < count; k++) {
         if (c->g + 1 >= 255u) {
             if (ensure_materialized(c, (cudaStream_t)stream) != HIRACE_OK)
@@ -624,6 +670,9 @@ hirace_status hirace_replay_trace(hirace_ctx *c, const hirace_event *d_events, u
     else if (ensure_materialized(c, st) != HIRACE_OK)
         return c->sticky;
     HR_CUDA(c, launch_find_batches(d_events, (uint32_t)n, c->scr, c->d_err, c->sm_count, st));
+    if (!win && c->reset_mode == HIRACE_RESET_EPOCH)
+        HR_CUDA(c, launch_epoch_prep(c->dev, c->shadow_words, c->d_gepoch, d_events, c->scr.batch_off,
+                                     c->scr.nbatches, 0, c->sm_count, st));
     if (c->t_start)
         HR_CUDA(c, cudaEventRecord(c->t_start, st));
     if (win)
@@ -696,6 +745,9 @@ hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_eve
     else if (ensure_materialized(c, st) != HIRACE_OK)
         return c->sticky;
     HR_CUDA(c, launch_find_batches(d_events, (uint32_t)n, c->scr, c->d_err, c->sm_count, st));
+    if (!win && c->reset_mode == HIRACE_RESET_EPOCH)
+        HR_CUDA(c, launch_epoch_prep(c->dev, c->shadow_words, c->d_gepoch, d_events, c->scr.batch_off,
+                                     c->scr.nbatches, 0, c->sm_count, st));
     if (c->t_start)
         HR_CUDA(c, cudaEventRecord(c->t_start, st));
     if (win)
@@ -861,9 +913,9 @@ hirace_status hirace_get_dev_ctx(hirace_ctx *c, const void *global_base, hirace_
 {
     if (!c || !out || c->rec_bytes != 8) /* inline hooks use the 8-byte record */
         return HIRACE_E_INVAL;
-    if (c->lazy) { /* inline hooks update the shadow in place: no stale windows */
+    if (c->lazy || c->reset_mode == HIRACE_RESET_EPOCH) { /* inline hooks use the trace's epochs */
         HR_CUDA(c, cudaSetDevice(c->device));
-        if (ensure_materialized(c, nullptr) != HIRACE_OK)
+        if (ensure_materialized(c, nullptr) != HIRACE_OK || ensure_epoch_normal(c, nullptr) != HIRACE_OK)
             return c->sticky;
     }
     *out = c->dev;
@@ -1181,7 +1233,7 @@ hirace_status hirace_replay_wire(hirace_ctx *c, const uint64_t *d_wire, uint64_t
         return set_sticky(c, HIRACE_E_INVAL);
     cudaStream_t st = (cudaStream_t)stream;
     HR_CUDA(c, cudaSetDevice(c->device));
-    if (ensure_materialized(c, st) != HIRACE_OK)
+    if (ensure_materialized(c, st) != HIRACE_OK || ensure_epoch_normal(c, st) != HIRACE_OK)
         return c->sticky;
     if (c->t_start)
         HR_CUDA(c, cudaEventRecord(c->t_start, st));

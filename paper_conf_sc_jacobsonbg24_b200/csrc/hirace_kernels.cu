@@ -637,6 +637,109 @@ cudaError_t launch_reset(void *shadow, uint64_t bytes, unsigned long long *repor
     return e;
 }
 
+/* ---- epoch reset (include/hirace.h hirace_set_reset_mode EPOCH; reading R19) -----
+ * gep[0] = gbase (offset the replay adds to the trace's g), gep[1] = gnext (first epoch no
+ * record of this check uses).  A reset clears the RACE records listed in the report buffer
+ * (every RACE record was reported when it entered RACE) and moves gbase to gnext; when the
+ * buffer overflowed it sweeps the whole shadow and starts over at 0. */
+__global__ void __launch_bounds__(256) k_epoch_reset(hirace_dev_ctx c, uint64_t shadow_words)
+{
+    const unsigned long long nrep = *c.report_count;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    const uint64_t i0 = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (nrep <= c.report_capacity) {
+        for (uint64_t i = i0; i < nrep; i += stride) {
+            const uint64_t key = c.reports[i].key;
+            uint64_t idx = key;
+            if (key & HIRACE_SHARED_BIT)
+                idx = c.global_words + ((key >> 32) & 0x7fffffffull) * c.smem_words + (key & 0xffffffffull);
+            if (idx < shadow_words)
+                c.shadow[idx] = 0ull;
+        }
+    } else {
+        for (uint64_t i = i0; i < shadow_words; i += stride)
+            __stcs(c.shadow + i, 0ull);
+    }
+}
+
+__global__ void k_epoch_reset_fin(hirace_dev_ctx c, unsigned int *gep)
+{
+    if (threadIdx.x < 4)
+        c.stats[threadIdx.x] = 0;
+    if (threadIdx.x == 0) {
+        const bool covered = *c.report_count <= c.report_capacity;
+        gep[0] = covered ? gep[1] : 0u;
+        gep[1] = gep[0];
+        *c.report_count = 0;
+        *c.error_flags = 0;
+    }
+}
+
+/* raw g of the last batch (batches are sorted by key, g in the top bits) */
+__device__ __forceinline__ uint32_t last_batch_g(const hirace_event *ev, const uint32_t *off, const uint32_t *nbp)
+{
+    if (!ev || !nbp)
+        return 0u;
+    const uint32_t nb = *nbp;
+    return nb ? (__ldg(&ev[off[nb - 1]].meta) >> 24) : 0u;
+}
+
+/* Before a replay: when gbase + the trace's largest g would pass 254 (or force), rebase: records
+ * of this check (g >= gbase) keep their epochs minus gbase, older ones become INIT. */
+__global__ void __launch_bounds__(256) k_epoch_prep(hirace_dev_ctx c, uint64_t shadow_words, const unsigned int *gep,
+                                                    const hirace_event *ev, const uint32_t *off, const uint32_t *nbp,
+                                                    int force)
+{
+    const uint32_t gbase = gep[0], gmax = last_batch_g(ev, off, nbp);
+    if (!force && gbase + gmax <= 254u)
+        return;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < shadow_words; i += stride) {
+        const unsigned long long r = c.shadow[i];
+        if (r == 0ull)
+            continue;
+        const uint32_t g = (uint32_t)(r >> SH_G) & 255u;
+        const unsigned long long n =
+            g >= gbase ? ((r & ~(255ull << SH_G)) | ((unsigned long long)(g - gbase) << SH_G)) : 0ull;
+        if (n != r)
+            c.shadow[i] = n;
+    }
+}
+
+__global__ void k_epoch_prep_fin(unsigned int *gep, const hirace_event *ev, const uint32_t *off, const uint32_t *nbp,
+                                 int force)
+{
+    if (threadIdx.x != 0)
+        return;
+    const uint32_t gmax = last_batch_g(ev, off, nbp);
+    if (force || gep[0] + gmax > 254u) {
+        gep[1] = gep[1] > gep[0] ? gep[1] - gep[0] : 0u;
+        gep[0] = 0;
+    }
+    const uint32_t need = gep[0] + gmax + 1u;
+    if (need > gep[1])
+        gep[1] = need;
+}
+
+cudaError_t launch_epoch_reset(const hirace_dev_ctx &c, uint64_t shadow_words, unsigned int *gep, int sm_count,
+                               cudaStream_t st)
+{
+    note_launches(2);
+    k_epoch_reset<<<sm_count * 8, 256, 0, st>>>(c, shadow_words);
+    k_epoch_reset_fin<<<1, 32, 0, st>>>(c, gep);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_epoch_prep(const hirace_dev_ctx &c, uint64_t shadow_words, unsigned int *gep,
+                              const hirace_event *ev, const uint32_t *off, const uint32_t *nbp, int force,
+                              int sm_count, cudaStream_t st)
+{
+    note_launches(2);
+    k_epoch_prep<<<sm_count * 8, 256, 0, st>>>(c, shadow_words, gep, ev, off, nbp, force);
+    k_epoch_prep_fin<<<1, 32, 0, st>>>(gep, ev, off, nbp, force);
+    return cudaGetLastError();
+}
+
 /* ---- per-batch completion flags of the peer dispatch -------------------------
  * A sender releases global batch j to every owner after its dispatch kernels for j (stream
  * order): a system-scope release fence, then one red.add on each owner's flag j (peer memory).

@@ -70,6 +70,13 @@ cudaError_t launch_dispatch_wire(const hirace_event *in, uint32_t lo, uint32_t h
                                  unsigned long long *const *d_peer, const unsigned long long *d_owner_base,
                                  uint32_t *d_tile_hist, unsigned long long *d_tile_off, unsigned int *err,
                                  cudaStream_t st);
+/* epoch reset (hirace_set_reset_mode EPOCH): O(flagged) reset, and the pre-replay rebase
+ * check (force: always rebase, e.g. before inline hooks); gep = device {gbase, gnext} */
+cudaError_t launch_epoch_reset(const hirace_dev_ctx &c, uint64_t shadow_words, unsigned int *gep, int sm_count,
+                               cudaStream_t st);
+cudaError_t launch_epoch_prep(const hirace_dev_ctx &c, uint64_t shadow_words, unsigned int *gep,
+                              const hirace_event *ev, const uint32_t *off, const uint32_t *nbp, int force,
+                              int sm_count, cudaStream_t st);
 /* per-batch completion flags of the peer dispatch: release [j0, j1] to every owner (d_flags:
  * device array of nranks flag-array addresses), or wait until flags[j] >= target */
 cudaError_t launch_peer_release(unsigned int *const *d_flags, int nranks, uint32_t j0, uint32_t j1, cudaStream_t st);

@@ -77,7 +77,7 @@ __device__ __noinline__ uint4 chunk_multiword(const hirace_dev_ctx c, const geom
         const uint32_t cls = commit_groups<R>(shadow + my, o, lead ? peers : 0u, e.z, e.w & 3u, G, raw, B, rec, cnt,
                                               rtid, true);
         if (__any_sync(FULL, cls != 0))
-            append_reports(c, cls, key_of(G, e, k, gran), B.g, rtid, lane);
+            append_reports(c, cls, key_of(G, e, k, gran), B.graw, rtid, lane);
     }
     return make_uint4(cnt.checked, cnt.retry, cnt.cas, cnt.nowrite);
 }
@@ -191,8 +191,9 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
     uint4 e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
     uint4 e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
+    const uint32_t gb = c.g_base ? *c.g_base : 0u; /* epoch reset: offset of this check's epochs */
     for (uint32_t bi = 0; bi < nb; bi++) {
-        const Batch B = make_batch<R>(__ldg(&ev[bstart].w) >> 5, rec);
+        const Batch B = make_batch<R>(__ldg(&ev[bstart].w) >> 5, rec, gb);
         const uint32_t keysz = B.key << 3; /* (meta >> 2) - keysz = size_log2 for this batch */
         if (B.g == 255u)
             bad = 1; /* reserved for retired RACE records (R7) */

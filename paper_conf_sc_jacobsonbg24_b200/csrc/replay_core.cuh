@@ -28,15 +28,18 @@ constexpr uint64_t NONE = ~0ull;
 constexpr int kMinBlocks = HIRACE_REPLAY_MINB;
 
 struct Batch {
-    uint32_t key, g, b, w, ep; /* ep = epochs in record layout */
+    uint32_t key, g, b, w, ep; /* ep = epochs in record layout; g = trace g + epoch offset */
+    uint32_t graw;             /* the trace's g (reports carry it)                          */
     bool fit;                  /* epochs within the record layout's fields (compact limits) */
 };
 
-template <typename R> __device__ __forceinline__ Batch make_batch(uint32_t key, const Rec<R> &rec)
+/* gb: the epoch-reset offset (hirace_set_reset_mode EPOCH) added to the trace's g */
+template <typename R> __device__ __forceinline__ Batch make_batch(uint32_t key, const Rec<R> &rec, uint32_t gb = 0)
 {
     Batch B;
     B.key = key;
-    B.g = key >> 19;
+    B.graw = key >> 19;
+    B.g = B.graw + gb;
     B.b = (key >> 9) & 1023u;
     B.w = key & 511u;
     B.ep = rec.ep(B.g, B.b, B.w);
@@ -247,7 +250,7 @@ __device__ __forceinline__ void chunk_finish(const Lane &cur, R o, const Issued<
     }
     /* a7 */
     if (__any_sync(FULL, cls != 0))
-        append_reports(c, cls, key_of_idx(cur, c, G), B.g, rtid, lane);
+        append_reports(c, cls, key_of_idx(cur, c, G), B.graw, rtid, lane);
 }
 
 /* One 32-event chunk (one event per lane) after decode: a4 load, a5 transition, a6 CAS, a3

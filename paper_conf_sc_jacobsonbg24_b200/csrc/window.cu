@@ -717,7 +717,7 @@ __device__ __forceinline__ void light_step(u64 *sh, bool ok, uint32_t word, uint
         L.tid = tid;
         L.kind = kind;
         L.ok = true;
-        append_reports(c, cls, key_of_idx(L, c, G), B.g, rtid, lane);
+        append_reports(c, cls, key_of_idx(L, c, G), B.graw, rtid, lane);
     }
 }
 

@@ -27,6 +27,7 @@ STATUS = {0: "HIRACE_OK", -1: "HIRACE_E_INVAL", -2: "HIRACE_E_NOMEM", -3: "HIRAC
 
 POLICY_STRICT, POLICY_RELAXED_READ_ATOMIC = 0, 1
 REPLAY_AUTO, REPLAY_BATCH, REPLAY_WINDOW = 0, 1, 2
+RESET_FULL, RESET_EPOCH = 0, 1
 
 # every symbol include/hirace.h declares (checked by tests/test_abi.py against the header)
 EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_free", "hirace_shadow_reset", "hirace_barrier",
@@ -40,7 +41,7 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_cluster_alloc", "hirace_cluster_free", "hirace_cluster_reset", "hirace_cluster_replay",
            "hirace_cluster_collect", "hirace_cluster_get_stats", "hirace_status_string",
            "hirace_version", "hirace_launch_count", "hirace_set_replay_mode", "hirace_get_replay_mode",
-           "hirace_advance_grid_epochs", "hirace_peer_release", "hirace_peer_wait")
+           "hirace_advance_grid_epochs", "hirace_peer_release", "hirace_peer_wait", "hirace_set_reset_mode")
 
 
 class HiraceError(RuntimeError):
@@ -70,7 +71,7 @@ class DevCtx(ctypes.Structure):
                 ("c_max_b", ctypes.c_uint32), ("c_max_w", ctypes.c_uint32), ("gran_log2", ctypes.c_uint32),
                 ("f_active", ctypes.c_uint32), ("f_tid_mask", ctypes.c_uint32), ("f_tid_match", ctypes.c_uint32),
                 ("f_spaces", ctypes.c_uint32), ("f_glo", ctypes.c_uint64), ("f_ghi", ctypes.c_uint64),
-                ("f_smem_words", ctypes.c_uint32), ("f_pad", ctypes.c_uint32)]
+                ("f_smem_words", ctypes.c_uint32), ("f_pad", ctypes.c_uint32), ("g_base", ctypes.c_void_p)]
 
 
 class EpochLimits(ctypes.Structure):
@@ -143,6 +144,7 @@ def load():
         "hirace_advance_grid_epochs": (I32, [P, U32, P]),
         "hirace_peer_release": (I32, [P, P, I32, U32, U32, P]),
         "hirace_peer_wait": (I32, [P, P, U32, U32, P]),
+        "hirace_set_reset_mode": (I32, [P, I32]),
         "hirace_get_replay_mode": (I32, [P, ctypes.POINTER(I32)]),
     }
     for name, (res, args) in sig.items():
@@ -430,6 +432,10 @@ class Checker:
     def set_replay_mode(self, mode: int, window_log2: int = 0):
         """REPLAY_AUTO / REPLAY_BATCH / REPLAY_WINDOW (include/hirace.h); resets the shadow."""
         _check(self.lib.hirace_set_replay_mode(self.h, mode, window_log2), "hirace_set_replay_mode")
+
+    def set_reset_mode(self, mode: int):
+        """RESET_FULL / RESET_EPOCH (include/hirace.h hirace_set_reset_mode)."""
+        _check(self.lib.hirace_set_reset_mode(self.h, mode), "hirace_set_reset_mode")
 
     @property
     def window_active(self) -> bool:
