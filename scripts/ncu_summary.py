@@ -7,7 +7,9 @@ WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "smsp__issue_active.avg.pct", "launch__registers_per_thread", "sm__warps_active.avg.pct",
         "lts__throughput.avg.pct", "smsp__inst_executed.sum", "launch__grid_size", "launch__occupancy_limit",
         "l1tex__t_requests_pipe_lsu_mem_global_op_atom.sum", "lts__t_sectors_srcunit_tex_op_read.sum",
-        "dram__throughput.avg.pct"]
+        "dram__throughput.avg.pct", "lts__t_sector_hit_rate.pct", "lts__t_sector_op_read_hit_rate.pct",
+        "lts__t_sector_op_atom_hit_rate.pct", "lts__t_sectors_op_atom.sum", "lts__t_requests_op_atom.sum",
+        "l1tex__t_sector_hit_rate.pct", "lts__t_sectors.sum", "dram__bytes.sum.per_second"]
 
 
 def main(path):
