@@ -385,13 +385,18 @@ def run_sharded_bench(args, world, rank, local_rank):
     dev = local_rank % torch.cuda.device_count()
     torch.cuda.set_device(dev)
     shared_gpu = world > torch.cuda.device_count()  # several ranks per GPU: NCCL cannot run there
+    if shared_gpu and args.transport == "nccl":
+        # NCCL needs one GPU per rank; ranks sharing a GPU (functional runs on a 1-GPU pool) take
+        # the peer-dispatch path, its control plane over gloo (the records still go peer to peer)
+        args.transport = "p2p"
+        print("bench: ranks share a GPU, NCCL unavailable: --transport p2p over gloo", file=sys.stderr)
     if args.transport == "nccl" or (args.transport == "p2p" and not shared_gpu):
         dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
         ex = sharded.NcclExchange(None, f"cuda:{dev}") if args.transport == "nccl" else \
             sharded.PeerExchange(None, dist, device=dev)
     elif args.transport == "p2p":  # control plane over gloo; the records still go peer to peer
         dist.init_process_group("gloo")
-        ex = sharded.PeerExchange(None, dist, device=dev)
+        ex = sharded.PeerExchange(None, dist, device=dev, per_batch=False)
     else:
         dist.init_process_group("gloo")
         ex = sharded.HostExchange(None, device=f"cuda:{dev}")

@@ -168,10 +168,12 @@ class PeerExchange:
     rank's stream before the count all-gather, so every owner has finished replaying the
     previous run before any rank dispatches into its buffer again."""
 
-    per_batch = True  # run_sharded_p2p: per-batch completion flags instead of one fence
-
-    def __init__(self, group, dist, device: int = 0):
+    def __init__(self, group, dist, device: int = 0, per_batch: bool = True):
+        """per_batch: run_sharded_p2p completes batch by batch with device flags (one GPU per
+        rank); False: one fence after the whole dispatch (ranks time-sliced on one GPU, where a
+        spinning wait only burns the other ranks' time slices)."""
         import torch
+        self.per_batch = per_batch
         self.group, self.dist, self.device = group, dist, device
         self.buf = None
         self.opened = {}   # rank -> (handle, ptr)
