@@ -12,6 +12,10 @@ two share no code.
   brute.py    literal O(n^2) pairwise enumeration of C1, for tiny traces.
   races_cluster / brute.races_cluster: the definition with a thread-block-cluster level
               (reading R16); class CLUSTER = 4.
+  races_masked / brute.races_masked: the definition with partial-mask __syncwarp(mask)
+              (reading R20; C1.1''/C1.2'' in
+              oracle_d.c): the oracle by forward knowledge propagation along the sync log, the
+              brute force by per-lane vector clocks.
 
 Pins (tests/test_oracle_pins.py): brute force on random tiny traces, the paper's listings
 (closed forms, tests/golden/), configs 1/2/4 closed forms, read-only invariants.
@@ -58,6 +62,10 @@ def _load():
         lib.oracle_races_par.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                          ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
                                          ctypes.c_int, ctypes.c_uint32, ctypes.c_int, ctypes.c_int]
+        lib.oracle_races_masked.restype = ctypes.c_int64
+        lib.oracle_races_masked.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
+                                            ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p,
+                                            ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int]
         lib.oracle_races_cluster.restype = ctypes.c_int64
         lib.oracle_races_cluster.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32,
                                              ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
@@ -149,4 +157,39 @@ def races_cluster(events: np.ndarray, block_threads: int, warp_size: int, cluste
 
 def races_cluster_dict(trace) -> dict:
     k, c, _ = races_cluster(trace.events, trace.block_threads, trace.warp_size, trace.cluster_blocks)
+    return {int(a): int(b) for a, b in zip(k, c)}
+
+
+class BadSyncLog(ValueError):
+    """oracle_races_masked returned -4: malformed partial-sync log, or an access after a partial
+    sync its lane is not in."""
+
+
+def races_masked(events: np.ndarray, block_threads: int, warp_size: int, syncs, policy: int = 0):
+    """Oracle-D with partial-mask warp syncs (C1.1''/C1.2'' in oracle_d.c; 4-byte words).
+    syncs: tracegen.SYNC_DTYPE log (None/empty = none).  Returns (keys, cls, gstar) by key."""
+    lib = _load()
+    ev = np.ascontiguousarray(events)
+    n = int(ev.shape[0])
+    sy = np.ascontiguousarray(syncs) if syncs is not None else None
+    ns = 0 if sy is None else int(sy.shape[0])
+    cap = max(1024, n)
+    while True:
+        keys = np.empty(cap, np.uint64)
+        cls = np.empty(cap, np.uint8)
+        gs = np.empty(cap, np.uint8)
+        r = lib.oracle_races_masked(ev.ctypes.data if n else None, n, block_threads, warp_size,
+                                    sy.ctypes.data if ns else None, ns, keys.ctypes.data, cls.ctypes.data,
+                                    gs.ctypes.data, cap, policy)
+        if r == -4:
+            raise BadSyncLog("malformed partial-sync log or an access outside its sync's mask")
+        if r < 0:
+            raise RuntimeError(f"oracle_races_masked failed ({r})")
+        if r <= cap:
+            return keys[:r], cls[:r], gs[:r]
+        cap = int(r)
+
+
+def races_masked_dict(trace, policy: int = 0) -> dict:
+    k, c, _ = races_masked(trace.events, trace.block_threads, trace.warp_size, trace.warp_syncs, policy)
     return {int(a): int(b) for a, b in zip(k, c)}

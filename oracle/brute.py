@@ -169,3 +169,79 @@ def races_cluster(events, block_threads, warp_size, cluster_blocks):
         in_b = [p for p in in_c if p[2] == bstar]
         out[key] = (BLOCK if any(p[3] == BLOCK for p in in_b) else WARP, gstar)
     return out
+
+
+# ---------------------------------------------------------------------------------------------
+# Partial-mask __syncwarp(mask) ("a bounded history of sub-warp
+# synchronizations (essentially a warp-level vector clock)"; reading R20).  The pair
+# loop of C1 with same-warp concurrency decided by textbook vector clocks: every lane holds a
+# vector V (V[i] = the latest sync number of lane i it knows of); a sync of mask M joins the
+# vectors of its lanes and stamps V[i] = s for i in M; e1 (lane i, after sync w1) happens
+# before e2 (lane j, after sync w2) iff V_j after w2 has V[i] > w1.  Unlisted numbers are
+# full-mask syncs.  (oracle_d.c decides the same relation by forward knowledge propagation.)
+# ---------------------------------------------------------------------------------------------
+
+
+def warp_vector_clocks(listed: dict, smax: int, lanes: int) -> dict:
+    """{s: V after sync s} for s = 1..smax; listed = {s: mask} of one warp in one (g, b)."""
+    cur = [[0] * lanes for _ in range(lanes)]
+    out = {}
+    for s in range(1, smax + 1):
+        m = listed.get(s, (1 << lanes) - 1)
+        members = [l for l in range(lanes) if (m >> l) & 1]
+        j = [max(cur[l][i] for l in members) for i in range(lanes)]
+        for i in members:
+            j[i] = s
+        for l in members:
+            cur[l] = list(j)
+        out[s] = j
+    return out
+
+
+def races_masked(events, syncs, block_threads, warp_size, policy=0):
+    """{key: (class, g*)} with C1.2'' same-warp concurrency (4-byte words)."""
+    acc = accesses(events, block_threads, warp_size)
+    wpb = -(-block_threads // warp_size)
+    fam = {}
+    for s in (syncs if syncs is not None else []):
+        meta = int(s["meta"])
+        fam.setdefault((meta >> 24 & 255, meta >> 14 & 1023, int(s["warp"])), {})[meta >> 5 & 511] = int(s["mask"])
+    clocks = {}
+
+    def vc(a):
+        key = (a[3], a[4], a[6] * wpb + a[7])
+        if key not in fam or a[5] == 0:
+            return None
+        if key not in clocks:
+            smax = max(max(fam[key]), max(x[5] for x in acc if (x[3], x[4], x[6] * wpb + x[7]) == key))
+            clocks[key] = warp_vector_clocks(fam[key], smax, warp_size)
+        return clocks[key][a[5]]
+
+    def lane(a):
+        return (a[1] % block_threads) % warp_size
+
+    def conc(a, c):
+        family = (a[3], a[4], a[6] * wpb + a[7])
+        same = a[1] != c[1] and family == (c[3], c[4], c[6] * wpb + c[7])
+        if not same or family not in fam:
+            return concurrent(a, c)
+        x, y = (a, c) if a[5] <= c[5] else (c, a)
+        return x[5] == y[5] or vc(y)[lane(x)] <= x[5]
+
+    pairs = {}
+    for i in range(len(acc)):
+        for j in range(i + 1, len(acc)):
+            a, c = acc[i], acc[j]
+            if a[0] == c[0] and conflict(a, c, policy) and conc(a, c):
+                pairs.setdefault(a[0], []).append((a[3], a[4], level(a, c)))
+    out = {}
+    for key, ps in pairs.items():
+        gstar = min(p[0] for p in ps)
+        in_g = [p for p in ps if p[0] == gstar]
+        if any(p[2] == GRID for p in in_g):
+            out[key] = (GRID, gstar)
+            continue
+        bstar = min(p[1] for p in in_g)
+        in_b = [p for p in in_g if p[1] == bstar]
+        out[key] = (BLOCK if any(p[2] == BLOCK for p in in_b) else WARP, gstar)
+    return out

@@ -140,14 +140,129 @@ static int masks_push(masks_t *s, uint8_t v)
  * by C1.2/C1.3 and is reported so a test can pin it).
  * out_g receives g* (the grid epoch of the first racing pair).
  */
-int64_t oracle_races_gran(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
+/*
+ * ---------------------------------------------------------------------------------------------
+ * Partial-mask warp synchronisation ("masked warp
+ * synchronization primitives may be used to implement non-hierarchical barrier points";
+ * DESIGN.md reading R20).
+ *
+ *   C1.1''  Inside one block epoch (g, b) a warp's synchronisations -- full-mask __syncwarp /
+ *           votes and partial __syncwarp(mask) -- are numbered 1, 2, ... in a linear order that
+ *           respects every lane's program order.  An access's w is the number of the last sync
+ *           its lane passed (0 = none).  The log lists the partial syncs (warp = block *
+ *           warps_per_block + warp, mask over lanes, g, b, w); unlisted numbers are full-mask.
+ *   C1.2''  Two accesses of different lanes of one warp in one (g, b), w1 <= w2:
+ *           e1 happens before e2  <=>  w1 < w2 and a chain of syncs s_1 < ... < s_m exists with
+ *           w1 < s_1, s_m <= w2, lane1 in M(s_1), lane2 in M(s_m), and consecutive syncs of the
+ *           chain sharing a lane (M(s_k) & M(s_k+1) != 0) -- the transitive closure of program
+ *           order and sync rendezvous.  Concurrent <=> not ordered.  Evaluated literally: the set
+ *           of lanes that know of e1 starts as {lane1} and absorbs M(s) for every s in
+ *           (w1, w2] whose mask meets it.  With only full masks this is "w1 == w2" (C1.2).
+ *   Everything else (other warps, blocks, epochs, conflict, class) is C1.2-C1.6 unchanged.
+ * ---------------------------------------------------------------------------------------------
+ */
+typedef struct {
+    uint32_t warp, mask, meta, pad;
+} oracle_sync; /* tracegen.SYNC_DTYPE; meta = w:9 << 5 | b:10 << 14 | g:8 << 24 */
+
+static uint64_t sync_key(uint32_t g, uint32_t b, uint32_t warp)
+{
+    return ((uint64_t)g << 50) | ((uint64_t)b << 40) | warp;
+}
+static uint64_t sync_key_of(const oracle_sync *s)
+{
+    return sync_key((s->meta >> 24) & 255, (s->meta >> 14) & 1023, s->warp);
+}
+
+/* the log entries of warp `warp` in (g, b): [*lo, *hi) of the sorted log */
+static void sync_family(const oracle_sync *sy, uint64_t nsync, uint32_t g, uint32_t b, uint32_t warp, uint64_t *lo,
+                        uint64_t *hi)
+{
+    const uint64_t k = sync_key(g, b, warp);
+    uint64_t a = 0, z = nsync;
+    while (a < z) {
+        uint64_t m = (a + z) / 2;
+        if (sync_key_of(&sy[m]) < k)
+            a = m + 1;
+        else
+            z = m;
+    }
+    *lo = a;
+    while (a < nsync && sync_key_of(&sy[a]) == k)
+        a++;
+    *hi = a;
+}
+
+/* M(s): the listed mask of sync number s, or all lanes (unlisted = full-mask sync) */
+static uint32_t sync_mask(const oracle_sync *f, uint64_t nf, uint32_t s, int *listed)
+{
+    for (uint64_t i = 0; i < nf; i++)
+        if (((f[i].meta >> 5) & 511) == s) {
+            *listed = 1;
+            return f[i].mask;
+        }
+    *listed = 0;
+    return 0xffffffffu;
+}
+
+/* C1.2'': does the access of lane i after sync w1 happen before the access of lane j after
+ * sync w2 (w1 < w2)? */
+static int masked_ordered(const oracle_sync *f, uint64_t nf, uint32_t i, uint32_t w1, uint32_t j, uint32_t w2)
+{
+    uint32_t know = 1u << i;
+    for (uint32_t s = w1 + 1; s <= w2; s++) {
+        int listed;
+        const uint32_t m = sync_mask(f, nf, s, &listed);
+        if (m & know)
+            know |= m;
+    }
+    return (know >> j) & 1u;
+}
+
+/* WARP level of one (key, g, block, b, warp) group with a partial-sync log: a conflicting
+ * concurrent pair of accesses of different threads?  acc[0..m) sorted by (w, tid).  Returns 1 /
+ * 0, or -4 when an access claims a partial sync its lane is not in. */
+static int masked_warp_race(const access_t *acc, uint64_t m, const oracle_sync *f, uint64_t nf, uint32_t block_threads,
+                            uint32_t warp_size, int policy)
+{
+    for (uint64_t x = 0; x < m; x++) {
+        const uint32_t lx = (acc[x].tid % block_threads) % warp_size;
+        int listed;
+        const uint32_t mx = acc[x].w ? sync_mask(f, nf, acc[x].w, &listed) : 0xffffffffu;
+        if (!((mx >> lx) & 1u))
+            return -4;
+    }
+    for (uint64_t x = 0; x < m; x++)
+        for (uint64_t y = x + 1; y < m; y++) {
+            if (acc[x].tid == acc[y].tid || !conflict(acc[x].kind, acc[y].kind, 1, policy))
+                continue;
+            const uint32_t lx = (acc[x].tid % block_threads) % warp_size;
+            const uint32_t ly = (acc[y].tid % block_threads) % warp_size;
+            if (acc[x].w == acc[y].w || !masked_ordered(f, nf, lx, acc[x].w, ly, acc[y].w))
+                return 1;
+        }
+    return 0;
+}
+
+static int64_t races_core(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
                           uint64_t *out_key, uint8_t *out_cls, uint8_t *out_g, uint64_t cap, int policy,
-                          uint32_t gran_log2)
+                          uint32_t gran_log2, const oracle_sync *sy, uint64_t nsync)
 {
     if (policy != 0 && policy != 1)
         return -1;
-    if (block_threads == 0 || warp_size == 0 || (n && !ev) || gran_log2 > 2)
+    if (block_threads == 0 || warp_size == 0 || (n && !ev) || gran_log2 > 2 || (nsync && !sy))
         return -1;
+    if (nsync && (warp_size > 32 || gran_log2 != 2))
+        return -1;
+    for (uint64_t i = 0; i < nsync; i++) { /* C1.1'': a sorted log of real partial syncs */
+        const uint32_t w = (sy[i].meta >> 5) & 511;
+        if (w == 0 || sy[i].mask == 0 || (warp_size < 32 && (sy[i].mask >> warp_size)) || (sy[i].meta & 31))
+            return -4;
+        if (i && !(sync_key_of(&sy[i - 1]) < sync_key_of(&sy[i]) ||
+                   (sync_key_of(&sy[i - 1]) == sync_key_of(&sy[i]) && ((sy[i - 1].meta >> 5) & 511) < w)))
+            return -4;
+    }
+    const uint32_t wpb = (block_threads + warp_size - 1) / warp_size;
     /* C1.1: expand to element-level accesses; an element ("granule") is 1 << gran_log2 bytes
      * (per-element shadow; reading R8: 4-byte words by default, bytes
      * or half-words for arrays of such elements) */
@@ -232,8 +347,20 @@ int64_t oracle_races_gran(const oracle_event *ev, uint64_t n, uint32_t block_thr
                             wmask |= (uint8_t)(1u << acc[we].kind), we++;
                         if (masks_push(&warps, wmask))
                             err = -1;
-                        /* WARP level: groups = threads of (block, b, warp, w) */
-                        for (uint64_t xs = ws; xs < we;) {
+                        /* WARP level: groups = threads of (block, b, warp, w); with partial
+                         * syncs in this (g, b) of this warp, the pairs of C1.2'' */
+                        uint64_t flo = 0, fhi = 0;
+                        if (nsync)
+                            sync_family(sy, nsync, g, b, blk * wpb + wp, &flo, &fhi);
+                        if (fhi > flo) {
+                            const int r = masked_warp_race(acc + ws, we - ws, sy + flo, fhi - flo, block_threads,
+                                                           warp_size, policy);
+                            if (r < 0)
+                                err = r;
+                            else if (r)
+                                warp_race = 1;
+                        }
+                        for (uint64_t xs = ws; fhi == flo && xs < we;) {
                             uint32_t w = acc[xs].w;
                             uint64_t xe = xs;
                             while (xe < we && acc[xe].w == w)
@@ -294,6 +421,23 @@ int64_t oracle_races_gran(const oracle_event *ev, uint64_t n, uint32_t block_thr
     free(threads.m);
     free(acc);
     return err ? err : nflag;
+}
+
+int64_t oracle_races_gran(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
+                          uint64_t *out_key, uint8_t *out_cls, uint8_t *out_g, uint64_t cap, int policy,
+                          uint32_t gran_log2)
+{
+    return races_core(ev, n, block_threads, warp_size, out_key, out_cls, out_g, cap, policy, gran_log2, NULL, 0);
+}
+
+/* C1 with the partial-mask warp syncs of C1.1''/C1.2'' (4-byte words).  Returns as
+ * oracle_races_gran, plus -4: malformed log, or an access after a partial sync its lane is not
+ * in. */
+int64_t oracle_races_masked(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
+                            const oracle_sync *syncs, uint64_t nsync, uint64_t *out_key, uint8_t *out_cls,
+                            uint8_t *out_g, uint64_t cap, int policy)
+{
+    return races_core(ev, n, block_threads, warp_size, out_key, out_cls, out_g, cap, policy, 2, syncs, nsync);
 }
 
 int64_t oracle_races_policy(const oracle_event *ev, uint64_t n, uint32_t block_threads, uint32_t warp_size,
