@@ -45,7 +45,10 @@ typedef enum {
     HIRACE_E_REPORT_OVERFLOW = -5,/* reserved: collection never loses races (shadow scan)     */
     HIRACE_E_BAD_TRACE = -6,      /* replay input not sorted by (g,b,w), tid/address out of
                                      range, access size > 16 B, or > HIRACE_MAX_BATCHES batches */
-    HIRACE_E_COMM = -7            /* sharded mode exchange failure (set by the Python layer)   */
+    HIRACE_E_COMM = -7,           /* sharded mode exchange failure (set by the Python layer)   */
+    HIRACE_E_HISTORY_OVERFLOW = -8/* the sub-warp access history (hirace_set_warp_syncs) was
+                                     full: some masked-warp accesses were not compared with
+                                     their lanes' history, races among them may be missed   */
 } hirace_status;
 
 /* Access kinds: the paper's 4 memory access types. */
@@ -491,6 +494,53 @@ uint32_t hirace_fsm_cluster_class(uint32_t state);
 uint64_t hirace_fsm_step_cluster(uint64_t old_shadow, uint32_t tid, uint32_t kind, uint32_t g, uint32_t c, uint32_t b,
                                  uint32_t w, uint32_t block_threads, uint32_t warp_size, uint32_t cluster_blocks,
                                  int *report);
+
+/* ---- partial-mask warp synchronisation ------------------
+ * "masked warp synchronization primitives may be used to implement non-hierarchical barrier
+ * points, which are not amenable to representation within HiRace's FSM.  In these cases,
+ * HiRace ... tracks a bounded history of sub-warp synchronizations (essentially a warp-level
+ * vector clock) and opportunistically prunes the history" (R20).
+ *
+ * Trace convention.  Inside one block epoch (g, b) each warp numbers its synchronisations --
+ * full-mask __syncwarp / votes and partial __syncwarp(mask) alike -- 1, 2, 3, ... in a linear
+ * order consistent with every lane's program order.  An event's w is the number of the LAST warp
+ * sync its lane passed (0 = none), so traces without partial masks keep their meaning (w =
+ * full-warp syncs since the last b).  The partial syncs are listed in a log of
+ * hirace_warp_sync records sorted by (g, b, warp, w), strictly increasing; numbers not listed
+ * are full-mask syncs.
+ *   warp  global warp id = block * ceil(block_threads / warp_size) + warp in block
+ *   mask  the participating lanes (bit i = lane i), non-zero, lanes < warp_size
+ *   meta  w:9 << 5 | b:10 << 14 | g:8 << 24  (the event meta layout with kind = size = 0)
+ * An access of lane j after sync w1 happens before an access of lane i != j after sync w2 > w1
+ * iff a chain of syncs w1 < s_1 < ... < s_m <= w2 links lane j to lane i (consecutive syncs
+ * share a lane); every other ordering is the three-level one. */
+typedef struct {
+    uint32_t warp;
+    uint32_t mask;
+    uint32_t meta;
+    uint32_t pad; /* 0 */
+} hirace_warp_sync;
+
+/* Sets the partial-sync log for the following hirace_replay_trace / hirace_check_trace_*
+ * calls of ctx (until replaced; n == 0 removes it).  d_syncs: DEVICE array of n records (read
+ * during this call only; the context keeps its own derived copy).  The library derives, per
+ * (g, b, warp) family, the warp vector clock after every listed sync (one warp per family),
+ * and allocates a sub-warp access history of history_slots slots (rounded up to a power of two;
+ * 0 = 65,536; 272 B each): one slot per word that masked-family accesses touch in a block epoch,
+ * holding per lane and access class (read / atomic / write) the last sync number.  The replay
+ * then runs the per-access FSM as usual with w read as the sync number, and additionally
+ * compares each access of a family at a listed sync with its lanes' history against the vector
+ * clock: a conflicting access not ordered before it is a race of the FSM state's level (WARP
+ * while one warp touched the word in the block epoch, else BLOCK / GRID; R20).
+ * Replay-only and batch-major: while a log is set, window-major mode replays batch-major, and
+ * the wire / sharded entry points and inline hooks return HIRACE_E_INVAL.  The history is
+ * cleared by hirace_shadow_reset.  Synchronises `stream`.
+ * Errors: INVAL (NULL ctx / n && !d_syncs, warp_size > 32, granularity_log2 != 2), BAD_TRACE
+ * (unsorted or duplicate records, w == 0, mask 0 or beyond warp_size, warp id beyond the grid;
+ * sticky), NOMEM, CUDA.  During replay: an access after a listed sync whose mask lacks its lane
+ * -> sticky BAD_TRACE; a full history -> sticky HIRACE_E_HISTORY_OVERFLOW. */
+hirace_status hirace_set_warp_syncs(hirace_ctx *ctx, const hirace_warp_sync *d_syncs, uint64_t n,
+                                    uint64_t history_slots, void *stream);
 
 /* ---- cluster-level replay (reading R16) ----------------------------
  * A context whose hierarchy has a thread-block-cluster level between the block and the grid:

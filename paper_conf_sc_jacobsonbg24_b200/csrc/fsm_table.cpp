@@ -42,6 +42,7 @@
 
 #include "hirace.h"
 #include "hirace_device.cuh"
+#include "internal.h"
 
 namespace {
 
@@ -426,6 +427,22 @@ int states(CD *out, int cap)
 } // namespace clus
 
 } // namespace
+
+namespace hirace_impl {
+/* masked replay (subwarp.cu): a race the sub-warp history finds has the level of the state the
+ * FSM reached -- one warp (T, W) -> RACE_W, >= 2 warps (B) -> RACE_B, >= 2 blocks (G) -> RACE_G */
+void fsm_race_of(int policy, unsigned char out[32])
+{
+    for (int s = 0; s < 32; s++) {
+        Group g = G_NONE;
+        if (s < (int)hirace::ST_COUNT)
+            g = policy == 1 ? relaxed::kR[s].grp : kStates[s].grp;
+        out[s] = (unsigned char)(g == G_T || g == G_W ? hirace::ST_RACE_W
+                                                       : g == G_B ? hirace::ST_RACE_B
+                                                                  : g == G_G ? hirace::ST_RACE_G : s);
+    }
+}
+} // namespace hirace_impl
 
 extern "C" hirace_status hirace_fsm_table_policy(int policy, unsigned char out[2048])
 {

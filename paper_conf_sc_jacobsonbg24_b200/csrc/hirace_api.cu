@@ -73,6 +73,10 @@ struct hirace_ctx {
     unsigned int *d_gepoch = nullptr; /* epoch reset: {gbase, gnext} (device) */
     uint32_t g = 0;
     cudaEvent_t t_start = nullptr, t_stop = nullptr;
+    /* partial-mask warp syncs (hirace_set_warp_syncs) */
+    WsDev ws{};
+    uint64_t ws_n = 0, ws_slots = 0;
+    int masked_grid = 0;
     hirace_status sticky = HIRACE_OK;
 };
 
@@ -127,6 +131,8 @@ hirace_status device_errors(hirace_ctx *c)
         set_sticky(c, HIRACE_E_CLOCK_OVERFLOW);
     if (flags & ERR_CAPACITY)
         set_sticky(c, HIRACE_E_NOMEM);
+    if (flags & ERR_HISTORY)
+        set_sticky(c, HIRACE_E_HISTORY_OVERFLOW);
     return c->sticky;
 }
 
@@ -136,8 +142,8 @@ constexpr uint32_t kWindowLog2Default = 12;       /* 32 KB windows: 4 light CTAs
 /* does this context replay window-major? (8-byte records, 4-byte elements) */
 bool window_active(const hirace_ctx *c)
 {
-    if (c->rec_bytes != 8 || c->cfg.granularity_log2 != 2 || !c->win.gen)
-        return false;
+    if (c->rec_bytes != 8 || c->cfg.granularity_log2 != 2 || !c->win.gen || c->ws_n)
+        return false; /* (a partial-sync log replays batch-major) */
     if (c->replay_mode == HIRACE_REPLAY_WINDOW)
         return true;
     /* AUTO: batch-major everywhere (measured faster on every config); the
@@ -298,9 +304,84 @@ hirace_status collect_into(hirace_ctx *c, hirace_race *d_out, uint64_t cap, unsi
     return HIRACE_OK;
 }
 
+/* masked replay launch: the policy-dependent tables are refreshed from the context */
+cudaError_t launch_masked(hirace_ctx *c, const hirace_event *d_events, cudaStream_t st)
+{
+    WsDev W = c->ws;
+    const bool relaxed = c->policy == HIRACE_POLICY_RELAXED_READ_ATOMIC;
+    /* classes R 0, A 1, X 2 inside one block (C1.3): strict R-A, R-X, A-X, X-X; relaxed only X */
+    W.confl[0] = relaxed ? 4u : 6u;
+    W.confl[1] = relaxed ? 4u : 5u;
+    W.confl[2] = 7u;
+    fsm_race_of(c->policy, W.race_of);
+    return launch_replay_masked(c->dev, W, d_events, c->scr, c->masked_grid, st);
+}
+
+void ws_free(hirace_ctx *c)
+{
+    void *ptrs[] = {c->ws.fam_key, c->ws.fam_lo, c->ws.nfam, c->ws.sync_w, c->ws.sync_mask, c->ws.vrow, c->ws.hist};
+    for (void *p : ptrs)
+        if (p)
+            cudaFree(p);
+    c->ws = WsDev{};
+    c->ws_n = 0;
+    c->ws_slots = 0;
+}
+
 } // namespace
 
 extern "C" {
+
+hirace_status hirace_set_warp_syncs(hirace_ctx *c, const hirace_warp_sync *d_syncs, uint64_t n, uint64_t history_slots,
+                                    void *stream)
+{
+    Nvtx nvtx_range("hirace_set_warp_syncs");
+    if (!c || (n && !d_syncs) || n >= (1ull << 31) || history_slots > (1ull << 32))
+        return HIRACE_E_INVAL;
+    if (n && (c->cfg.warp_size > 32 || c->cfg.granularity_log2 != 2))
+        return HIRACE_E_INVAL;
+    if (c->sticky != HIRACE_OK)
+        return c->sticky;
+    cudaStream_t st = (cudaStream_t)stream;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    if (ensure_materialized(c, st) != HIRACE_OK) /* from here on: batch-major, shadow explicit */
+        return c->sticky;
+    HR_CUDA(c, cudaStreamSynchronize(st));
+    ws_free(c);
+    if (n == 0)
+        return HIRACE_OK;
+    uint64_t slots = 64;
+    while (slots < (history_slots ? history_slots : 65536ull))
+        slots <<= 1;
+    WsDev &W = c->ws;
+    cudaError_t e;
+    if ((e = cudaMalloc(&W.fam_key, n * sizeof(unsigned long long))) != cudaSuccess ||
+        (e = cudaMalloc(&W.fam_lo, (n + 1) * sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&W.nfam, sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&W.sync_w, n * sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&W.sync_mask, n * sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&W.vrow, n * 32 * sizeof(unsigned short))) != cudaSuccess ||
+        (e = cudaMalloc(&W.hist, slots * kSlotWords * sizeof(unsigned long long))) != cudaSuccess) {
+        ws_free(c);
+        return from_cuda(c, e);
+    }
+    W.slots_mask = slots - 1;
+    W.wpb = (c->cfg.block_threads + c->cfg.warp_size - 1) / c->cfg.warp_size;
+    c->ws_slots = slots;
+    if (!c->masked_grid)
+        c->masked_grid = masked_max_grid(c->device);
+    HR_CUDA(c, cudaMemsetAsync(W.hist, 0xff, slots * kSlotWords * sizeof(unsigned long long), st));
+    HR_CUDA(c, launch_ws_prepare(d_syncs, (uint32_t)n, c->cfg.grid_blocks * W.wpb, c->cfg.warp_size, W, c->d_err,
+                                 c->sm_count, st));
+    HR_CUDA(c, cudaStreamSynchronize(st));
+    hirace_status s = device_errors(c);
+    if (s != HIRACE_OK) {
+        ws_free(c);
+        return s;
+    }
+    c->ws_n = n;
+    return HIRACE_OK;
+}
 
 const char *hirace_version(void) { return "hirace-b200 0.2 (sm_100a)"; }
 
@@ -384,6 +465,7 @@ const char *hirace_status_string(hirace_status s)
     case HIRACE_E_REPORT_OVERFLOW: return "report overflow";
     case HIRACE_E_BAD_TRACE: return "bad trace";
     case HIRACE_E_COMM: return "communication error";
+    case HIRACE_E_HISTORY_OVERFLOW: return "sub-warp history full: masked-warp accesses not all compared";
     }
     return "unknown";
 }
@@ -533,7 +615,8 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
                     c->scr.batch_off, c->scr.nbatches, c->scr.batch_ctr, c->scr.grid_bar,
                     c->scr.grid_bar2, c->scr.cta_cnt, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
                     c->d_stage[0], c->d_stage[1], c->d_wire_off, c->d_wire_counts, c->d_wire_flag,
-                    c->d_peer_tab, c->d_flag_tab, c->d_gepoch};
+                    c->d_peer_tab, c->d_flag_tab, c->d_gepoch, c->ws.fam_key, c->ws.fam_lo, c->ws.nfam,
+                    c->ws.sync_w, c->ws.sync_mask, c->ws.vrow, c->ws.hist};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
@@ -609,6 +692,8 @@ hirace_status hirace_shadow_reset(hirace_ctx *c, void *stream)
                                 c->sm_count, st));
         c->lazy = false;
     }
+    if (c->ws.hist) /* the sub-warp history belongs to the check */
+        HR_CUDA(c, cudaMemsetAsync(c->ws.hist, 0xff, c->ws_slots * kSlotWords * sizeof(unsigned long long), st));
     c->g = 0;
     c->dev.g = 0;
     c->sticky = HIRACE_OK;
@@ -678,6 +763,8 @@ hirace_status hirace_replay_trace(hirace_ctx *c, const hirace_event *d_events, u
     if (win)
         HR_CUDA(c, launch_window_check(c->dev, c->win, c->scr, d_events, (uint32_t)n, c->sm_count, c->replay_grid, st,
                                        c->shadow_words, nullptr, 0, nullptr));
+    else if (c->ws_n)
+        HR_CUDA(c, launch_masked(c, d_events, st));
     else
         HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st));
     if (c->t_stop)
@@ -753,7 +840,11 @@ hirace_status hirace_check_trace_device(hirace_ctx *c, const hirace_event *d_eve
     if (win)
         HR_CUDA(c, launch_window_check(c->dev, c->win, c->scr, d_events, (uint32_t)n, c->sm_count, c->replay_grid, st,
                                        c->shadow_words, d_out, cap, d_n_total));
-    else
+    else if (c->ws_n) {
+        HR_CUDA(c, launch_masked(c, d_events, st));
+        if (collect_into(c, d_out, cap, d_n_total, st) != HIRACE_OK)
+            return c->sticky;
+    } else
         HR_CUDA(c, launch_replay(c->dev, d_events, c->scr, c->replay_grid, st, c->shadow_words, d_out, cap, d_n_total,
                                  report_mode(c)));
     if (win && getenv("HIRACE_WIN_VALIDATE")) { /* diagnostics: synchronous */
@@ -911,7 +1002,7 @@ hirace_status hirace_sync(hirace_ctx *c)
 
 hirace_status hirace_get_dev_ctx(hirace_ctx *c, const void *global_base, hirace_dev_ctx *out)
 {
-    if (!c || !out || c->rec_bytes != 8) /* inline hooks use the 8-byte record */
+    if (!c || !out || c->rec_bytes != 8 || c->ws_n) /* inline hooks: 8-byte record, no sync log */
         return HIRACE_E_INVAL;
     if (c->lazy || c->reset_mode == HIRACE_RESET_EPOCH) { /* inline hooks use the trace's epochs */
         HR_CUDA(c, cudaSetDevice(c->device));
@@ -928,7 +1019,7 @@ hirace_status hirace_bucket_events(hirace_ctx *c, const hirace_event *d_in, uint
                                    hirace_event *d_out, uint64_t *h_counts, void *stream)
 {
     if (!c || !h_counts || nranks < 1 || nranks > 32 || my_rank < 0 || my_rank >= nranks || n >= 0xffffffffull ||
-        (n && (!d_in || !d_out)) || c->cfg.granularity_log2 != 2)
+        (n && (!d_in || !d_out)) || c->cfg.granularity_log2 != 2 || c->ws_n)
         return HIRACE_E_INVAL;
     if (c->sticky != HIRACE_OK)
         return c->sticky;
@@ -1008,7 +1099,7 @@ hirace_status wire_args_ok(hirace_ctx *c, const uint32_t *h_offsets, uint64_t nb
                            uint32_t *maxlen)
 {
     if (nranks < 1 || nranks > 32 || my_rank < 0 || my_rank >= nranks || nb > HIRACE_MAX_BATCHES ||
-        c->cfg.granularity_log2 != 2)
+        c->cfg.granularity_log2 != 2 || c->ws_n)
         return HIRACE_E_INVAL;
     const uint64_t threads = (uint64_t)c->cfg.grid_blocks * c->cfg.block_threads;
     if (threads > HIRACE_WIRE_MAX_TIDS || (uint64_t)c->dev.smem_words > HIRACE_WIRE_MAX_WORDS)
@@ -1223,7 +1314,7 @@ hirace_status hirace_bucket_wire(hirace_ctx *c, const hirace_event *d_in, const 
 hirace_status hirace_replay_wire(hirace_ctx *c, const uint64_t *d_wire, uint64_t n, uint32_t batch_key, void *stream)
 {
     Nvtx nvtx_range("hirace_replay_wire");
-    if (!c)
+    if (!c || c->ws_n)
         return HIRACE_E_INVAL;
     if (c->sticky != HIRACE_OK)
         return c->sticky;

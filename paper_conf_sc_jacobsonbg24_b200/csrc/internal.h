@@ -122,6 +122,7 @@ constexpr int kScanMaxCtas = 1024;
 constexpr int kBarSlots = 8;
 constexpr uint32_t kWinHeavyCap = 64;
 constexpr uint32_t ERR_CAPACITY = 8u; /* window path: more element accesses than rec1/rec2 hold */
+constexpr uint32_t ERR_HISTORY = 16u; /* masked replay: the sub-warp history table was full     */
 /* the whole window-major check: partition, heavy + light replay, then (d_total != null) the
  * collect into out / d_total */
 cudaError_t launch_window_check(const hirace_dev_ctx &c, const WinDev &W, const Scratch &s, const hirace_event *ev,
@@ -137,6 +138,31 @@ const void *window_light_kernel();
 int window_light_threads();
 size_t window_light_smem(uint32_t wl);
 cudaError_t window_init();
+/* ---- partial-mask warp syncs (subwarp.cu; hirace_set_warp_syncs, R20) ----------
+ * Families = (g, b, warp) with listed syncs, sorted by key g<<50 | b<<40 | warp; sync_w / mask
+ * / vrow per listed sync (vrow: the warp vector clock after it, 32 u16); hist: open-addressing
+ * table of kSlotWords-word slots [key, owner, 32 lane words]. */
+constexpr uint32_t kSlotWords = 34;
+struct WsDev {
+    unsigned long long *fam_key;
+    uint32_t *fam_lo;        /* [nfam + 1] first listed sync of each family */
+    uint32_t *nfam;
+    uint32_t *sync_w, *sync_mask;
+    unsigned short *vrow;
+    unsigned long long *hist;
+    unsigned long long slots_mask;
+    uint32_t wpb;            /* warps per block */
+    uint32_t confl[3];       /* per access class (R, A, X): classes it conflicts with in a block */
+    unsigned char race_of[32]; /* FSM state -> the RACE state of its level (policy's table) */
+};
+cudaError_t launch_ws_prepare(const hirace_warp_sync *d_syncs, uint32_t n, uint32_t total_warps, uint32_t warp_size,
+                              const WsDev &W, unsigned int *err, int sm_count, cudaStream_t st);
+cudaError_t launch_replay_masked(const hirace_dev_ctx &c, const WsDev &W, const hirace_event *ev, const Scratch &s,
+                                 int grid, cudaStream_t st);
+int masked_max_grid(int device);
+/* fsm_table.cpp: per state, the RACE state of its hierarchy level under `policy` */
+void fsm_race_of(int policy, unsigned char out[32]);
+
 /* process-wide count of kernels the library has launched (hirace_launch_count) */
 void note_launches(unsigned k);
 unsigned long long launch_count();

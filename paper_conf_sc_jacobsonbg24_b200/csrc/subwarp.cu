@@ -1,0 +1,462 @@
+/*
+ * subwarp.cu — partial-mask warp synchronisation ("HiRace
+ * tracks a bounded history of sub-warp synchronizations (essentially a warp-level vector clock)
+ * and opportunistically prunes the history"; reading R20; include/hirace.h
+ * hirace_set_warp_syncs).
+ *
+ * Split of the work.  A __syncwarp(mask) orders lanes of one warp only, so every relation the
+ * three-level FSM decides across warps, blocks and epochs stays exact.  Only the WARP-level
+ * question changes: inside one block epoch two accesses of different lanes are no longer
+ * "concurrent iff same w".  The replay therefore
+ *   1. runs the FSM with w read as the warp's sync number (event w = last sync its lane passed):
+ *      equal numbers are truly concurrent (same-batch pairs, exact), different numbers are
+ *      treated as ordered -- which misses exactly the pairs a partial mask left unordered;
+ *   2. catches those pairs with a per-word sub-warp history: per lane and access class (read,
+ *      atomic, write) the last sync number at which that lane accessed the word in this block
+ *      epoch ("pruned" to one number per lane and class: the latest is the one most likely to
+ *      be unordered, since e1 -> e2 iff V_e2[lane(e1)] > w1 is monotone in w1), compared with the
+ *      warp vector clock V after the accessing lane's last sync;
+ *   3. on such a race, turns the FSM's next state into the RACE state of its level (T/W ->
+ *      RACE_W, B -> RACE_B, G -> RACE_G), storing the detecting accessor, so the class rules
+ *      (C1.6) and the sticky upgrades work unchanged.
+ * The history of a word belongs to the first warp that uses it in the block epoch; another warp
+ * with partial syncs touching the same word in the same (g, b) makes every race of either warp a
+ * BLOCK race the FSM finds by itself (a conflicting same-warp pair always conflicts with one of
+ * the other warp's accesses), so its accesses skip the history.
+ *
+ * Kernels: k_ws_families (one CTA: log validation, (g,b,warp) families by a block scan),
+ * k_ws_clocks (one warp per family: the vector clock after every listed sync, joins of 32
+ * columns in shared memory), k_replay_masked (persistent cooperative replay, one event per
+ * thread per step, contiguous warp shares, grid barrier between batches).
+ */
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "hirace_device.cuh"
+#include "internal.h"
+#include "kernel_common.cuh"
+#include "record.cuh"
+#include "replay_core.cuh"
+
+namespace hirace_impl {
+
+using namespace hirace;
+
+namespace {
+
+constexpr int kFamThreads = 1024;
+constexpr int kClockWarps = 8;
+constexpr int kMaskedThreads = 256;
+constexpr uint32_t kProbes = 64;
+constexpr unsigned long long kEmpty = ~0ull;
+
+__device__ __forceinline__ unsigned long long fam_key(uint32_t g, uint32_t b, uint32_t warp)
+{
+    return ((unsigned long long)g << 50) | ((unsigned long long)b << 40) | warp;
+}
+
+/* Validation + families: one CTA walks the log in 1024-record tiles, flags family heads and
+ * numbers them with a block scan. */
+__global__ void __launch_bounds__(kFamThreads)
+    k_ws_families(const hirace_warp_sync *__restrict__ s, uint32_t n, uint32_t total_warps, uint32_t warp_size,
+                  WsDev W, unsigned int *err)
+{
+    __shared__ uint32_t sc[kFamThreads];
+    __shared__ uint32_t s_base;
+    const uint32_t t = threadIdx.x;
+    if (t == 0)
+        s_base = 0;
+    __syncthreads();
+    for (uint32_t base = 0; base < n; base += kFamThreads) {
+        const uint32_t i = base + t;
+        uint32_t head = 0;
+        unsigned long long key = 0;
+        if (i < n) {
+            const hirace_warp_sync x = s[i];
+            const uint32_t w = (x.meta >> 5) & 511u;
+            key = fam_key(x.meta >> 24, (x.meta >> 14) & 1023u, x.warp);
+            bool ok = w >= 1 && x.mask != 0 && (warp_size >= 32 || (x.mask >> warp_size) == 0) &&
+                      x.warp < total_warps && (x.meta & 31u) == 0 && x.pad == 0;
+            if (i == 0) {
+                head = 1;
+            } else {
+                const hirace_warp_sync y = s[i - 1];
+                const unsigned long long pk = fam_key(y.meta >> 24, (y.meta >> 14) & 1023u, y.warp);
+                head = key != pk;
+                ok = ok && (key > pk || (key == pk && w > ((y.meta >> 5) & 511u)));
+            }
+            if (!ok)
+                atomicOr(err, ERR_BAD_TRACE);
+            W.sync_w[i] = w;
+            W.sync_mask[i] = x.mask;
+        }
+        sc[t] = head;
+        __syncthreads();
+        for (uint32_t d = 1; d < kFamThreads; d <<= 1) { /* inclusive Hillis-Steele scan */
+            const uint32_t v = t >= d ? sc[t - d] : 0u;
+            __syncthreads();
+            sc[t] += v;
+            __syncthreads();
+        }
+        if (head) {
+            const uint32_t f = s_base + sc[t] - 1;
+            W.fam_key[f] = key;
+            W.fam_lo[f] = i;
+        }
+        __syncthreads();
+        if (t == kFamThreads - 1)
+            s_base += sc[t];
+        __syncthreads();
+    }
+    if (t == 0) {
+        *W.nfam = s_base;
+        W.fam_lo[s_base] = n;
+    }
+}
+
+/* Warp vector clocks: one warp per family, lane i owns column i of the 32 x 32 matrix
+ * V[l][i] = the largest sync number of lane i that lane l knows of.  An unlisted number before a
+ * listed sync is a full-mask sync: everyone knows everything up to it.  A listed sync s of mask M
+ * joins the rows of M and stamps V[.][i] = s for i in M; the joined row is the clock after s. */
+__global__ void __launch_bounds__(kClockWarps * 32) k_ws_clocks(WsDev W)
+{
+    __shared__ unsigned short V[kClockWarps][32][33];
+    const uint32_t lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+    const uint32_t nfam = *W.nfam;
+    for (uint32_t f = blockIdx.x * kClockWarps + wl; f < nfam; f += gridDim.x * kClockWarps) {
+        for (int l = 0; l < 32; l++)
+            V[wl][l][lane] = 0;
+        uint32_t prev = 0;
+        const uint32_t lo = W.fam_lo[f], hi = W.fam_lo[f + 1];
+        for (uint32_t s = lo; s < hi; s++) {
+            const uint32_t ws = W.sync_w[s], m = W.sync_mask[s];
+            __syncwarp();
+            if (ws - 1 > prev)
+                for (int l = 0; l < 32; l++)
+                    V[wl][l][lane] = (unsigned short)(ws - 1);
+            __syncwarp();
+            uint32_t j = 0;
+            for (uint32_t r = m; r; r &= r - 1)
+                j = max(j, (uint32_t)V[wl][__ffs(r) - 1][lane]);
+            const uint32_t v = ((m >> lane) & 1u) ? ws : j;
+            __syncwarp();
+            for (uint32_t r = m; r; r &= r - 1)
+                V[wl][__ffs(r) - 1][lane] = (unsigned short)v;
+            W.vrow[(size_t)s * 32 + lane] = (unsigned short)v;
+            prev = ws;
+        }
+        __syncwarp();
+    }
+}
+
+__device__ __forceinline__ unsigned long long ld_rel64(const unsigned long long *p)
+{
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ unsigned long long mix64(unsigned long long x)
+{
+    x ^= x >> 33;
+    x *= 0xff51afd7ed558ccdull;
+    x ^= x >> 33;
+    x *= 0xc4ceb9fe1a85ec53ull;
+    return x ^ (x >> 33);
+}
+
+/* History slot of `key` owned by `owner` (valid:1 | g:8 | b:10 | warp:40 <<...), or null when
+ * another warp owns the word in this block epoch or the table is full (*full = 1).  Slot =
+ * [key, owner, 32 lane words]. */
+__device__ unsigned long long *hist_slot(const WsDev &W, unsigned long long key, unsigned long long owner,
+                                         uint32_t &full)
+{
+    unsigned long long h = mix64(key) & W.slots_mask;
+    for (uint32_t p = 0; p < kProbes; p++, h = (h + 1) & W.slots_mask) {
+        unsigned long long *s = W.hist + h * kSlotWords;
+        unsigned long long k = ld_rel64(s);
+        if (k == kEmpty) {
+            k = atomicCAS(s, kEmpty, key);
+            if (k == kEmpty)
+                k = key;
+        }
+        if (k != key)
+            continue;
+        unsigned long long ow = ld_rel64(s + 1);
+        for (;;) {
+            if (ow == owner)
+                return s;
+            if ((ow >> 40) == (owner >> 40))
+                return nullptr; /* same (g, b), another warp: its races are BLOCK races anyway */
+            const unsigned long long prev = atomicCAS(s + 1, ow, owner);
+            if (prev == ow)
+                return s;
+            ow = prev;
+        }
+    }
+    full = 1;
+    return nullptr;
+}
+
+/* lane word: stamp (1 | g:8 | b:10) << 30 | per class c (0 R, 1 A, 2 X) at bits 10c: present:1
+ * (bit 9) | w:9 */
+__device__ __forceinline__ bool side_check(const unsigned long long *slot, uint32_t lane, uint32_t lanes,
+                                           uint32_t stamp, uint32_t confl, uint32_t w2, const unsigned short *V)
+{
+    for (uint32_t i = 0; i < lanes; i++) {
+        if (i == lane)
+            continue;
+        const unsigned long long v = ld_rel64(slot + 2 + i);
+        if ((uint32_t)(v >> 30) != stamp)
+            continue;
+        const uint32_t vi = V[i];
+        for (uint32_t cm = confl; cm; cm &= cm - 1) {
+            const uint32_t c = __ffs(cm) - 1;
+            const uint32_t f = (uint32_t)(v >> (10 * c)) & 1023u;
+            if ((f & 512u) && (f & 511u) < w2 && vi <= (f & 511u))
+                return true;
+        }
+    }
+    return false;
+}
+
+__device__ __forceinline__ void side_update(unsigned long long *p, uint32_t stamp, uint32_t cls, uint32_t w2)
+{
+    unsigned long long v = ld_rel64(p);
+    for (;;) {
+        unsigned long long nv = (uint32_t)(v >> 30) == stamp ? v : ((unsigned long long)stamp << 30);
+        const uint32_t f = (uint32_t)(nv >> (10 * cls)) & 1023u;
+        if ((f & 512u) && (f & 511u) >= w2 && nv == v)
+            return;
+        nv = (nv & ~(1023ull << (10 * cls))) | ((unsigned long long)(512u | w2) << (10 * cls));
+        const unsigned long long prev = atomicCAS(p, v, nv);
+        if (prev == v)
+            return;
+        v = prev;
+    }
+}
+
+/* first index in [lo, hi) with a[i] >= x */
+template <typename T> __device__ __forceinline__ uint32_t lower_bound(const T *a, uint32_t lo, uint32_t hi, T x)
+{
+    while (lo < hi) {
+        const uint32_t m = (lo + hi) >> 1;
+        if (a[m] < x)
+            lo = m + 1;
+        else
+            hi = m;
+    }
+    return lo;
+}
+
+template <bool P2, typename R>
+__global__ void __launch_bounds__(kMaskedThreads)
+    k_replay_masked(hirace_dev_ctx c, WsDev W, const uint4 *__restrict__ ev, const uint32_t *__restrict__ off,
+                    const uint32_t *__restrict__ nbp, unsigned int *bar)
+{
+    __shared__ __align__(16) unsigned char s_table[2048 + RAW_TABLE_BYTES];
+    __shared__ unsigned long long s_stats[4];
+    const uint32_t lane = threadIdx.x & 31;
+    for (int i = threadIdx.x; i < (2048 + RAW_TABLE_BYTES) / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(s_table)[i] = __ldg(reinterpret_cast<const uint4 *>(c.table) + i);
+    if (threadIdx.x < 4)
+        s_stats[threadIdx.x] = 0;
+    __syncthreads();
+
+    geom G = make_geom(c);
+    G.pow2 = P2;
+    const Rec<R> rec(c);
+    const unsigned char *const raw = s_table + 2048;
+    R *const shadow = shadow_as<R>(c);
+    const uint32_t nb = *nbp;
+    const uint32_t nfam = *W.nfam;
+    const uint64_t total_threads = (uint64_t)c.grid_blocks * c.block_threads;
+    const uint32_t tid_max = total_threads > 0xffffffffull ? 0xffffffffu : (uint32_t)(total_threads - 1);
+    const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    const uint32_t gb = c.g_base ? *c.g_base : 0u;
+    const uint32_t gran = c.gran_log2;
+    const uint32_t lanes = c.warp_size;
+    unsigned int bar_epoch = 0;
+    Counters cnt{0, 0, 0, 0};
+    uint32_t bad = 0, clk = 0, full = 0;
+
+    for (uint32_t bi = 0; bi < nb; bi++) {
+        const uint32_t bstart = __ldg(&off[bi]), bend = __ldg(&off[bi + 1]);
+        const Batch B = make_batch<R>(__ldg(&ev[bstart].w) >> 5, rec, gb);
+        if (B.g == 255u)
+            bad = 1;
+        if (!B.fit)
+            clk = 1;
+        uint32_t i, iend;
+        warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
+        for (; B.fit && i < iend; i += 32) {
+            const uint4 e = ld_event(ev + i);
+            const uint32_t tid = e.z, meta = e.w, kind = meta & 3u, szl = (meta >> 2) & 7u;
+            const bool sh = (int)e.y < 0;
+            const uint64_t offb = (((uint64_t)(e.y & 0x7fffffffu)) << 32) | e.x;
+            const uint64_t word = offb >> gran;
+            const uint32_t nw = szl <= gran ? 1u : (1u << (szl - gran));
+            const uint64_t lim = sh ? c.smem_words : c.global_words;
+            if ((meta >> 5) != B.key || szl > 4 || tid > tid_max || word + nw > lim) {
+                bad = 1;
+                continue;
+            }
+            if (c.f_active && !((tid & c.f_tid_mask) == c.f_tid_match &&
+                                (sh ? (c.f_spaces & 2u) != 0
+                                    : ((c.f_spaces & 1u) != 0 && word >= c.f_glo && word < c.f_ghi))))
+                continue;
+            uint32_t blk, wib;
+            coords(tid, G, &blk, &wib);
+            const uint32_t lt = tid - blk * G.bt;
+            const uint32_t ln = lt - wib * lanes;
+            /* the family of this warp in (g, b) and the listed sync this access follows */
+            bool chk = false, upd = false;
+            uint32_t row = 0;
+            unsigned long long owner = 0;
+            if (nfam) {
+                const uint32_t gw = blk * W.wpb + wib;
+                const unsigned long long fk = fam_key(B.graw, B.b, gw);
+                const uint32_t f = lower_bound<unsigned long long>(W.fam_key, 0, nfam, fk);
+                if (f < nfam && W.fam_key[f] == fk) {
+                    const uint32_t lo = W.fam_lo[f], hi = W.fam_lo[f + 1];
+                    const uint32_t r = lower_bound<uint32_t>(W.sync_w, lo, hi, B.w);
+                    if (r < hi && W.sync_w[r] == B.w) {
+                        if (!((W.sync_mask[r] >> ln) & 1u)) {
+                            bad = 1;
+                            continue;
+                        }
+                        chk = true;
+                        row = r;
+                    }
+                    upd = B.w < W.sync_w[hi - 1];
+                    owner = (1ull << 63) | ((unsigned long long)B.g << 50) | ((unsigned long long)B.b << 40) | gw;
+                }
+            }
+            const uint32_t cls = kind == HIRACE_READ ? 0u : (kind == HIRACE_WRITE ? 2u : 1u);
+            const uint32_t stamp = (1u << 18) | (B.g << 10) | B.b;
+            for (uint32_t k = 0; k < nw; k++) {
+                const uint64_t wk = word + k;
+                const uint64_t idx = sh ? c.global_words + (uint64_t)blk * c.smem_words + wk : wk;
+                const uint64_t key = sh ? (HIRACE_SHARED_BIT | ((uint64_t)blk << 32) | wk) : wk;
+                bool side = false;
+                if (chk || upd) {
+                    unsigned long long *slot = hist_slot(W, key, owner, full);
+                    if (slot) {
+                        if (chk)
+                            side = side_check(slot, ln, lanes, stamp, W.confl[cls], B.w, W.vrow + (size_t)row * 32);
+                        if (upd)
+                            side_update(slot + 2 + ln, stamp, cls, B.w);
+                    }
+                }
+                /* a4-a6 with the side verdict folded into the transition */
+                R *p = shadow + idx;
+                R o = Rec<R>::load(p);
+                cnt.checked++;
+                bool first = true;
+                for (;;) {
+                    uint32_t ent = raw[((uint32_t)(o & 31u) << 7) | rec.label(o, tid, kind, B.ep, G)];
+                    if (side) {
+                        const uint32_t ns = W.race_of[ent & E_STATE];
+                        if (ns != (ent & E_STATE))
+                            ent = ns | E_REPORT; /* store the detecting accessor */
+                    }
+                    const R n = rec.next(o, ent, tid, B.ep);
+                    if (n == o)
+                        break;
+                    cnt.cas += first ? 1u : 0u;
+                    cnt.retry += first ? 0u : 1u;
+                    first = false;
+                    const R prev = Rec<R>::cas(p, o, n);
+                    if (prev == o) {
+                        const uint32_t cn = race_class(st_of(n)), co = race_class(st_of(o));
+                        if ((ent & E_REPORT) && cn > co) {
+                            const unsigned long long pos = atomicAdd(c.report_count, 1ull);
+                            if (pos < c.report_capacity) {
+                                hirace_race rr;
+                                rr.key = key;
+                                rr.cls_and_epoch = cn | (B.graw << 8);
+                                rr.detect_tid = tid;
+                                c.reports[pos] = rr;
+                            }
+                        }
+                        break;
+                    }
+                    o = prev;
+                }
+            }
+        }
+        if (bi + 1 < nb)
+            grid_sync(bar, gridDim.x, bar_epoch);
+    }
+    if (bad)
+        atomicOr(c.error_flags, ERR_BAD_TRACE);
+    if (clk)
+        atomicOr(c.error_flags, ERR_CLOCK);
+    if (full)
+        atomicOr(c.error_flags, ERR_HISTORY);
+    __syncwarp();
+    flush_stats(c, cnt, s_stats, lane);
+}
+
+bool pow2_geom(const hirace_dev_ctx &c)
+{
+    return (c.block_threads & (c.block_threads - 1)) == 0 && (c.warp_size & (c.warp_size - 1)) == 0;
+}
+
+const void *masked_kernel(const hirace_dev_ctx &c)
+{
+    const bool p2 = pow2_geom(c);
+    if (c.rec_bytes == 4)
+        return p2 ? (const void *)k_replay_masked<true, unsigned int> : (const void *)k_replay_masked<false, unsigned int>;
+    return p2 ? (const void *)k_replay_masked<true, unsigned long long>
+              : (const void *)k_replay_masked<false, unsigned long long>;
+}
+
+} // namespace
+
+cudaError_t launch_ws_prepare(const hirace_warp_sync *d_syncs, uint32_t n, uint32_t total_warps, uint32_t warp_size,
+                              const WsDev &W, unsigned int *err, int sm_count, cudaStream_t st)
+{
+    note_launches(2);
+    k_ws_families<<<1, kFamThreads, 0, st>>>(d_syncs, n, total_warps, warp_size, W, err);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess)
+        return e;
+    const uint32_t blocks = (n + kClockWarps - 1) / kClockWarps;
+    const uint32_t grid = blocks < (uint32_t)(8 * sm_count) ? (blocks ? blocks : 1u) : (uint32_t)(8 * sm_count);
+    k_ws_clocks<<<grid, kClockWarps * 32, 0, st>>>(W);
+    return cudaGetLastError();
+}
+
+int masked_max_grid(int device)
+{
+    int sms = 0, occ = 1 << 30;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    const void *fns[] = {(const void *)k_replay_masked<true, unsigned long long>,
+                         (const void *)k_replay_masked<false, unsigned long long>,
+                         (const void *)k_replay_masked<true, unsigned int>,
+                         (const void *)k_replay_masked<false, unsigned int>};
+    for (const void *f : fns) {
+        int o = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, f, kMaskedThreads, 0);
+        occ = o < occ ? o : occ;
+    }
+    return sms * (occ < 1 ? 1 : occ);
+}
+
+cudaError_t launch_replay_masked(const hirace_dev_ctx &c, const WsDev &W, const hirace_event *ev, const Scratch &s,
+                                 int grid, cudaStream_t st)
+{
+    hirace_dev_ctx cc = c;
+    WsDev ww = W;
+    const uint4 *evp = reinterpret_cast<const uint4 *>(ev);
+    const uint32_t *offp = s.batch_off;
+    const uint32_t *nbp = s.nbatches;
+    unsigned int *barp = s.grid_bar;
+    void *args[] = {&cc, &ww, &evp, &offp, &nbp, &barp};
+    note_launches(1);
+    return cudaLaunchCooperativeKernel(masked_kernel(c), dim3(grid), dim3(kMaskedThreads), args, 0, st);
+}
+
+} // namespace hirace_impl

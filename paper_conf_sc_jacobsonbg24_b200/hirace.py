@@ -15,6 +15,7 @@ SO_PATH = os.environ.get("HIRACE_LIB") or os.path.join(_PKG, "lib", "libhirace.s
 
 EVENT_DTYPE = np.dtype([("addr", "<u8"), ("tid", "<u4"), ("meta", "<u4")])
 RACE_DTYPE = np.dtype([("key", "<u8"), ("cls_and_epoch", "<u4"), ("detect_tid", "<u4")])
+WARP_SYNC_DTYPE = np.dtype([("warp", "<u4"), ("mask", "<u4"), ("meta", "<u4"), ("pad", "<u4")])  # hirace_warp_sync
 
 READ, WRITE, ATOMIC_BLOCK, ATOMIC_GRID = 0, 1, 2, 3
 SCOPE_WARP, SCOPE_BLOCK, SCOPE_GRID = 1, 2, 3
@@ -23,7 +24,7 @@ MAX_BATCHES = 32767
 
 STATUS = {0: "HIRACE_OK", -1: "HIRACE_E_INVAL", -2: "HIRACE_E_NOMEM", -3: "HIRACE_E_CUDA",
           -4: "HIRACE_E_CLOCK_OVERFLOW", -5: "HIRACE_E_REPORT_OVERFLOW", -6: "HIRACE_E_BAD_TRACE",
-          -7: "HIRACE_E_COMM"}
+          -7: "HIRACE_E_COMM", -8: "HIRACE_E_HISTORY_OVERFLOW"}
 
 POLICY_STRICT, POLICY_RELAXED_READ_ATOMIC = 0, 1
 REPLAY_AUTO, REPLAY_BATCH, REPLAY_WINDOW = 0, 1, 2
@@ -41,7 +42,8 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_cluster_alloc", "hirace_cluster_free", "hirace_cluster_reset", "hirace_cluster_replay",
            "hirace_cluster_collect", "hirace_cluster_get_stats", "hirace_status_string",
            "hirace_version", "hirace_launch_count", "hirace_set_replay_mode", "hirace_get_replay_mode",
-           "hirace_advance_grid_epochs", "hirace_peer_release", "hirace_peer_wait", "hirace_set_reset_mode")
+           "hirace_advance_grid_epochs", "hirace_peer_release", "hirace_peer_wait", "hirace_set_reset_mode",
+           "hirace_set_warp_syncs")
 
 
 class HiraceError(RuntimeError):
@@ -146,6 +148,7 @@ def load():
         "hirace_peer_wait": (I32, [P, P, U32, U32, P]),
         "hirace_set_reset_mode": (I32, [P, I32]),
         "hirace_get_replay_mode": (I32, [P, ctypes.POINTER(I32)]),
+        "hirace_set_warp_syncs": (I32, [P, P, U64, U64, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -299,12 +302,37 @@ class Checker:
             self.set_policy(policy)
 
     @classmethod
-    def for_trace(cls, trace, report_capacity: int = 0, device: int = 0, policy: int = 0, compact: bool = False):
-        """compact=True: 4-byte records sized by the trace's own epoch maxima."""
+    def for_trace(cls, trace, report_capacity: int = 0, device: int = 0, policy: int = 0, compact: bool = False,
+                  history_slots: int = 0):
+        """compact=True: 4-byte records sized by the trace's own epoch maxima.  A trace with a
+        partial-mask warp-sync log (trace.warp_syncs) gets it set (hirace_set_warp_syncs)."""
         lim = trace_epoch_limits(trace.events) if compact else None
-        return cls(trace.grid_blocks, trace.block_threads, trace.warp_size, trace.global_words, trace.smem_words,
-                   report_capacity, device, policy, compact=lim,
-                   granularity_log2=getattr(trace, "granularity_log2", 2))
+        c = cls(trace.grid_blocks, trace.block_threads, trace.warp_size, trace.global_words, trace.smem_words,
+                report_capacity, device, policy, compact=lim,
+                granularity_log2=getattr(trace, "granularity_log2", 2))
+        syncs = getattr(trace, "warp_syncs", None)
+        if syncs is not None and len(syncs):
+            c.set_warp_syncs(syncs, history_slots)
+        return c
+
+    def set_warp_syncs(self, syncs, history_slots: int = 0, stream=None):
+        """hirace_set_warp_syncs: syncs = WARP_SYNC_DTYPE numpy array (copied to the device for
+        the call) or a CUDA tensor of 16-byte records; empty / None removes the log."""
+        import torch
+        if syncs is None or len(syncs) == 0:
+            _check(self.lib.hirace_set_warp_syncs(self.h, None, 0, 0, _stream_handle(stream)),
+                   "hirace_set_warp_syncs")
+            return
+        if isinstance(syncs, np.ndarray):
+            arr = np.ascontiguousarray(syncs)
+            assert arr.dtype.itemsize == 16
+            dev = torch.from_numpy(arr.view(np.uint8).reshape(-1)).to(f"cuda:{self.device}")
+            n = arr.shape[0]
+        else:
+            dev = syncs
+            n = dev.numel() * dev.element_size() // 16
+        _check(self.lib.hirace_set_warp_syncs(self.h, ctypes.c_void_p(dev.data_ptr()), n, history_slots,
+                                              _stream_handle(stream)), "hirace_set_warp_syncs")
 
     def set_filter(self, tid_mask: int = 0, tid_match: int = 0, spaces: int = 3, global_lo: int = 0,
                    global_hi: int = (1 << 64) - 1):
