@@ -71,6 +71,8 @@ def make_trace(config: int, variant: str, nranks: int = 1, rank: int = 0):
         return tg.cfg4("B" if variant == "racy" else None)
     if config == 5:
         return tg.cfg5(nranks=nranks, rank=rank)
+    if config == 6:  # partial-mask __syncwarp: tiled_partition<8> reduction, 1M threads
+        return tg.tiled_reduce(4096, 256, 8, 4, "half_mask" if variant == "racy" else None)
     raise SystemExit(f"unknown config {config}")
 
 
@@ -624,7 +626,8 @@ def measure_single(args, config: int, variant: str, K: int, W: int, dev: int, cl
            "eager_ms_per_step": eager_ms / K, "launches_per_step": launches_per_step,
            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                         "traffic": load_traffic(key), "traffic_key": key,
-                        "kernel": "k_replay (incl. fused collect)", "kernel_ms": kern_ms,
+                        "kernel": ("k_replay_masked + collect" if trace.warp_syncs is not None
+                                   else "k_replay (incl. fused collect)"), "kernel_ms": kern_ms,
                         "kernel_share": kern_ms / ms_per_step, "bytes_per_access": bpa, "peak_kind": peak_kind},
            "roofline_step": {"bound": "hbm", "achieved": bpa * n_acc / (ms_per_step / 1e3) / 1e9, "peak": peak,
                              "unit": "GB/s", "frac": bpa * n_acc / (ms_per_step / 1e3) / 1e9 / peak,
@@ -763,7 +766,7 @@ def main():
     del trace, ctx
     per_config = {}
     if not args.no_per_config and world == 1:
-        for cfg in (2, 3, 4):
+        for cfg in (2, 3, 4, 6):
             if cfg == args.config:
                 continue
             r, _ = measure_single(args, cfg, "racy", min(K, 20), W, dev, None)

@@ -526,7 +526,7 @@ typedef struct {
  * during this call only; the context keeps its own derived copy).  The library derives, per
  * (g, b, warp) family, the warp vector clock after every listed sync (one warp per family),
  * and allocates a sub-warp access history of history_slots slots (rounded up to a power of two;
- * 0 = 65,536; 272 B each): one slot per word that masked-family accesses touch in a block epoch,
+ * 0 = 65,536; 288 B each): one slot per word that masked-family accesses touch in a block epoch,
  * holding per lane and access class (read / atomic / write) the last sync number.  The replay
  * then runs the per-access FSM as usual with w read as the sync number, and additionally
  * compares each access of a family at a listed sync with its lanes' history against the vector

@@ -319,7 +319,8 @@ cudaError_t launch_masked(hirace_ctx *c, const hirace_event *d_events, cudaStrea
 
 void ws_free(hirace_ctx *c)
 {
-    void *ptrs[] = {c->ws.fam_key, c->ws.fam_lo, c->ws.nfam, c->ws.sync_w, c->ws.sync_mask, c->ws.vrow, c->ws.hist};
+    void *ptrs[] = {c->ws.fam_key, c->ws.fam_lo, c->ws.nfam, c->ws.sync_w, c->ws.sync_mask, c->ws.sync_fam,
+                    c->ws.vrow, c->ws.fhash, c->ws.hist};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
@@ -353,6 +354,9 @@ hirace_status hirace_set_warp_syncs(hirace_ctx *c, const hirace_warp_sync *d_syn
     uint64_t slots = 64;
     while (slots < (history_slots ? history_slots : 65536ull))
         slots <<= 1;
+    uint64_t fh_slots = 64;
+    while (fh_slots < 4 * n) /* listed syncs + family records (<= n) at most half full */
+        fh_slots <<= 1;
     WsDev &W = c->ws;
     cudaError_t e;
     if ((e = cudaMalloc(&W.fam_key, n * sizeof(unsigned long long))) != cudaSuccess ||
@@ -360,17 +364,22 @@ hirace_status hirace_set_warp_syncs(hirace_ctx *c, const hirace_warp_sync *d_syn
         (e = cudaMalloc(&W.nfam, sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&W.sync_w, n * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&W.sync_mask, n * sizeof(uint32_t))) != cudaSuccess ||
+        (e = cudaMalloc(&W.sync_fam, n * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&W.vrow, n * 32 * sizeof(unsigned short))) != cudaSuccess ||
+        (e = cudaMalloc(&W.fhash, fh_slots * sizeof(uint4))) != cudaSuccess ||
         (e = cudaMalloc(&W.hist, slots * kSlotWords * sizeof(unsigned long long))) != cudaSuccess) {
         ws_free(c);
         return from_cuda(c, e);
     }
     W.slots_mask = slots - 1;
+    W.fh_mask = fh_slots - 1;
+    W.nsync = (uint32_t)n;
     W.wpb = (c->cfg.block_threads + c->cfg.warp_size - 1) / c->cfg.warp_size;
     c->ws_slots = slots;
     if (!c->masked_grid)
         c->masked_grid = masked_max_grid(c->device);
     HR_CUDA(c, cudaMemsetAsync(W.hist, 0xff, slots * kSlotWords * sizeof(unsigned long long), st));
+    HR_CUDA(c, cudaMemsetAsync(W.fhash, 0xff, fh_slots * sizeof(uint4), st));
     HR_CUDA(c, launch_ws_prepare(d_syncs, (uint32_t)n, c->cfg.grid_blocks * W.wpb, c->cfg.warp_size, W, c->d_err,
                                  c->sm_count, st));
     HR_CUDA(c, cudaStreamSynchronize(st));
@@ -616,7 +625,7 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
                     c->scr.grid_bar2, c->scr.cta_cnt, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
                     c->d_stage[0], c->d_stage[1], c->d_wire_off, c->d_wire_counts, c->d_wire_flag,
                     c->d_peer_tab, c->d_flag_tab, c->d_gepoch, c->ws.fam_key, c->ws.fam_lo, c->ws.nfam,
-                    c->ws.sync_w, c->ws.sync_mask, c->ws.vrow, c->ws.hist};
+                    c->ws.sync_w, c->ws.sync_mask, c->ws.sync_fam, c->ws.vrow, c->ws.fhash, c->ws.hist};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);

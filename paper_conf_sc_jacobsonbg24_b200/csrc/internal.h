@@ -141,14 +141,17 @@ cudaError_t window_init();
 /* ---- partial-mask warp syncs (subwarp.cu; hirace_set_warp_syncs, R20) ----------
  * Families = (g, b, warp) with listed syncs, sorted by key g<<50 | b<<40 | warp; sync_w / mask
  * / vrow per listed sync (vrow: the warp vector clock after it, 32 u16); hist: open-addressing
- * table of kSlotWords-word slots [key, owner, 32 lane words]. */
-constexpr uint32_t kSlotWords = 34;
+ * table of kSlotWords-word slots [key, owner, presence, -, 32 lane words] (subwarp.cu). */
+constexpr uint32_t kSlotWords = 36;
 struct WsDev {
     unsigned long long *fam_key;
     uint32_t *fam_lo;        /* [nfam + 1] first listed sync of each family */
     uint32_t *nfam;
-    uint32_t *sync_w, *sync_mask;
+    uint32_t *sync_w, *sync_mask, *sync_fam;
     unsigned short *vrow;
+    uint4 *fhash;            /* (family, w) lookup: {key lo, key hi, row, smax}; 2x(n + families) */
+    unsigned long long fh_mask;
+    uint32_t nsync;
     unsigned long long *hist;
     unsigned long long slots_mask;
     uint32_t wpb;            /* warps per block */

@@ -47,7 +47,7 @@ namespace {
 constexpr int kFamThreads = 1024;
 constexpr int kClockWarps = 8;
 constexpr int kMaskedThreads = 256;
-constexpr uint32_t kProbes = 64;
+constexpr uint32_t kProbes = 4096; /* linear probing; a full table ends the search */
 constexpr unsigned long long kEmpty = ~0ull;
 
 __device__ __forceinline__ unsigned long long fam_key(uint32_t g, uint32_t b, uint32_t warp)
@@ -98,6 +98,8 @@ __global__ void __launch_bounds__(kFamThreads)
             sc[t] += v;
             __syncthreads();
         }
+        if (i < n)
+            W.sync_fam[i] = s_base + sc[t] - 1;
         if (head) {
             const uint32_t f = s_base + sc[t] - 1;
             W.fam_key[f] = key;
@@ -149,11 +151,11 @@ __global__ void __launch_bounds__(kClockWarps * 32) k_ws_clocks(WsDev W)
     }
 }
 
-__device__ __forceinline__ unsigned long long ld_rel64(const unsigned long long *p)
+/* lookup key of (family, sync number w): g:8 << 51 | b:10 << 41 | w:9 << 32 | warp:32 (w = 0: the
+ * family record) */
+__device__ __forceinline__ unsigned long long sync_hkey(uint32_t g, uint32_t b, uint32_t w, uint32_t warp)
 {
-    unsigned long long v;
-    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
+    return ((unsigned long long)g << 51) | ((unsigned long long)b << 41) | ((unsigned long long)w << 32) | warp;
 }
 
 __device__ __forceinline__ unsigned long long mix64(unsigned long long x)
@@ -165,16 +167,52 @@ __device__ __forceinline__ unsigned long long mix64(unsigned long long x)
     return x ^ (x >> 33);
 }
 
+__device__ void fh_insert(const WsDev &W, unsigned long long hk, uint32_t row, uint32_t smax)
+{
+    for (unsigned long long h = mix64(hk) & W.fh_mask;; h = (h + 1) & W.fh_mask) {
+        unsigned long long *e = reinterpret_cast<unsigned long long *>(W.fhash + h);
+        if (atomicCAS(e, kEmpty, hk) == kEmpty) {
+            W.fhash[h].z = row;
+            W.fhash[h].w = smax;
+            return;
+        }
+    }
+}
+
+/* One lookup table for the replay: (family, w) of every listed sync -> {row, smax}, and
+ * (family, 0) -> {~0, smax} (smax = the family's last listed sync number).  Half full at most. */
+__global__ void k_ws_hash(WsDev W, uint32_t n)
+{
+    for (uint32_t s = blockIdx.x * blockDim.x + threadIdx.x; s < n; s += gridDim.x * blockDim.x) {
+        const uint32_t f = W.sync_fam[s];
+        const unsigned long long fk = W.fam_key[f];
+        const uint32_t g = (uint32_t)(fk >> 50), b = (uint32_t)(fk >> 40) & 1023u, warp = (uint32_t)fk;
+        const uint32_t smax = W.sync_w[W.fam_lo[f + 1] - 1];
+        fh_insert(W, sync_hkey(g, b, W.sync_w[s], warp), s, smax);
+        if (s == W.fam_lo[f])
+            fh_insert(W, sync_hkey(g, b, 0, warp), ~0u, smax);
+    }
+}
+
+__device__ __forceinline__ uint4 fh_find(const WsDev &W, unsigned long long hk)
+{
+    for (unsigned long long h = mix64(hk) & W.fh_mask;; h = (h + 1) & W.fh_mask) {
+        const uint4 e = __ldg(W.fhash + h);
+        const unsigned long long k = ((unsigned long long)e.y << 32) | e.x;
+        if (k == hk || k == kEmpty)
+            return k == hk ? e : make_uint4(0xffffffffu, 0xffffffffu, 0xffffffffu, 0);
+    }
+}
+
 /* History slot of `key` owned by `owner` (valid:1 | g:8 | b:10 | warp:40 <<...), or null when
- * another warp owns the word in this block epoch or the table is full (*full = 1).  Slot =
- * [key, owner, 32 lane words]. */
+ * another warp owns the word in this block epoch or the table is full (*full = 1). */
 __device__ unsigned long long *hist_slot(const WsDev &W, unsigned long long key, unsigned long long owner,
                                          uint32_t &full)
 {
     unsigned long long h = mix64(key) & W.slots_mask;
     for (uint32_t p = 0; p < kProbes; p++, h = (h + 1) & W.slots_mask) {
         unsigned long long *s = W.hist + h * kSlotWords;
-        unsigned long long k = ld_rel64(s);
+        unsigned long long k = __ldcg(s);
         if (k == kEmpty) {
             k = atomicCAS(s, kEmpty, key);
             if (k == kEmpty)
@@ -182,7 +220,7 @@ __device__ unsigned long long *hist_slot(const WsDev &W, unsigned long long key,
         }
         if (k != key)
             continue;
-        unsigned long long ow = ld_rel64(s + 1);
+        unsigned long long ow = __ldcg(s + 1);
         for (;;) {
             if (ow == owner)
                 return s;
@@ -198,31 +236,62 @@ __device__ unsigned long long *hist_slot(const WsDev &W, unsigned long long key,
     return nullptr;
 }
 
-/* lane word: stamp (1 | g:8 | b:10) << 30 | per class c (0 R, 1 A, 2 X) at bits 10c: present:1
- * (bit 9) | w:9 */
-__device__ __forceinline__ bool side_check(const unsigned long long *slot, uint32_t lane, uint32_t lanes,
-                                           uint32_t stamp, uint32_t confl, uint32_t w2, const unsigned short *V)
+/* Slot = [key, owner, presence, -, 32 lane words] (288 B, 32-B aligned).  presence = stamp << 32
+ * | mask of the lanes with an entry in the owner's block epoch; lane word = stamp (1 | g:8 | b:10)
+ * << 30 | per class c (0 R, 1 A, 2 X) at bits 10c: present:1 (bit 9) | w:9.  Only the lanes of the
+ * presence mask are read (independent L2 loads), so a word touched by a few lanes costs a few
+ * sectors.  Returns the race verdict; sets this lane's presence bit (upd). */
+__device__ __forceinline__ bool side_check(unsigned long long *slot, uint32_t lane, uint32_t stamp, uint32_t confl,
+                                           uint32_t w2, const unsigned short *V, bool chk, bool upd)
 {
-    for (uint32_t i = 0; i < lanes; i++) {
-        if (i == lane)
-            continue;
-        const unsigned long long v = ld_rel64(slot + 2 + i);
-        if ((uint32_t)(v >> 30) != stamp)
-            continue;
-        const uint32_t vi = V[i];
-        for (uint32_t cm = confl; cm; cm &= cm - 1) {
-            const uint32_t c = __ffs(cm) - 1;
-            const uint32_t f = (uint32_t)(v >> (10 * c)) & 1023u;
-            if ((f & 512u) && (f & 511u) < w2 && vi <= (f & 511u))
-                return true;
+    unsigned long long pr = __ldcg(slot + 2);
+    const bool cur = (uint32_t)(pr >> 32) == stamp;
+    uint32_t others = cur ? ((uint32_t)pr & ~(1u << lane)) : 0u;
+    if (upd && (!cur || !(((uint32_t)pr >> lane) & 1u))) { /* register this lane */
+        for (;;) {
+            const unsigned long long np = ((unsigned long long)stamp << 32) |
+                                          ((uint32_t)(pr >> 32) == stamp ? (uint32_t)pr : 0u) | (1u << lane);
+            const unsigned long long prev = atomicCAS(slot + 2, pr, np);
+            if (prev == pr)
+                break;
+            pr = prev;
+            if ((uint32_t)(pr >> 32) == stamp)
+                others = (uint32_t)pr & ~(1u << lane);
         }
     }
-    return false;
+    if (!chk)
+        return false;
+    bool race = false;
+    while (others) {
+        uint32_t idx[4];
+        unsigned long long x[4];
+        int m = 0;
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            idx[j] = others ? (uint32_t)(__ffs(others) - 1) : 32u;
+            others &= others - 1;
+            x[j] = idx[j] < 32 ? __ldcg(slot + 4 + idx[j]) : 0ull;
+            m += idx[j] < 32;
+        }
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            if (j >= m || (uint32_t)(x[j] >> 30) != stamp)
+                continue;
+            const uint32_t vi = __ldg(V + idx[j]);
+            for (uint32_t cm = confl; cm; cm &= cm - 1) {
+                const uint32_t c = __ffs(cm) - 1;
+                const uint32_t f = (uint32_t)(x[j] >> (10 * c)) & 1023u;
+                race |= (f & 512u) && (f & 511u) < w2 && vi <= (f & 511u);
+            }
+        }
+    }
+    return race;
 }
 
+/* this lane's class entry := max(entry, w2) in the current block epoch (v: last seen value) */
 __device__ __forceinline__ void side_update(unsigned long long *p, uint32_t stamp, uint32_t cls, uint32_t w2)
 {
-    unsigned long long v = ld_rel64(p);
+    unsigned long long v = __ldcg(p);
     for (;;) {
         unsigned long long nv = (uint32_t)(v >> 30) == stamp ? v : ((unsigned long long)stamp << 30);
         const uint32_t f = (uint32_t)(nv >> (10 * cls)) & 1023u;
@@ -236,21 +305,8 @@ __device__ __forceinline__ void side_update(unsigned long long *p, uint32_t stam
     }
 }
 
-/* first index in [lo, hi) with a[i] >= x */
-template <typename T> __device__ __forceinline__ uint32_t lower_bound(const T *a, uint32_t lo, uint32_t hi, T x)
-{
-    while (lo < hi) {
-        const uint32_t m = (lo + hi) >> 1;
-        if (a[m] < x)
-            lo = m + 1;
-        else
-            hi = m;
-    }
-    return lo;
-}
-
 template <bool P2, typename R>
-__global__ void __launch_bounds__(kMaskedThreads)
+__global__ void __launch_bounds__(kMaskedThreads, 4)
     k_replay_masked(hirace_dev_ctx c, WsDev W, const uint4 *__restrict__ ev, const uint32_t *__restrict__ off,
                     const uint32_t *__restrict__ nbp, unsigned int *bar)
 {
@@ -269,14 +325,12 @@ __global__ void __launch_bounds__(kMaskedThreads)
     const unsigned char *const raw = s_table + 2048;
     R *const shadow = shadow_as<R>(c);
     const uint32_t nb = *nbp;
-    const uint32_t nfam = *W.nfam;
     const uint64_t total_threads = (uint64_t)c.grid_blocks * c.block_threads;
     const uint32_t tid_max = total_threads > 0xffffffffull ? 0xffffffffu : (uint32_t)(total_threads - 1);
     const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
     const uint32_t gb = c.g_base ? *c.g_base : 0u;
     const uint32_t gran = c.gran_log2;
-    const uint32_t lanes = c.warp_size;
     unsigned int bar_epoch = 0;
     Counters cnt{0, 0, 0, 0};
     uint32_t bad = 0, clk = 0, full = 0;
@@ -309,27 +363,27 @@ __global__ void __launch_bounds__(kMaskedThreads)
             uint32_t blk, wib;
             coords(tid, G, &blk, &wib);
             const uint32_t lt = tid - blk * G.bt;
-            const uint32_t ln = lt - wib * lanes;
+            const uint32_t ln = lt - wib * c.warp_size;
             /* the family of this warp in (g, b) and the listed sync this access follows */
             bool chk = false, upd = false;
             uint32_t row = 0;
             unsigned long long owner = 0;
-            if (nfam) {
+            if (W.nsync) {
                 const uint32_t gw = blk * W.wpb + wib;
-                const unsigned long long fk = fam_key(B.graw, B.b, gw);
-                const uint32_t f = lower_bound<unsigned long long>(W.fam_key, 0, nfam, fk);
-                if (f < nfam && W.fam_key[f] == fk) {
-                    const uint32_t lo = W.fam_lo[f], hi = W.fam_lo[f + 1];
-                    const uint32_t r = lower_bound<uint32_t>(W.sync_w, lo, hi, B.w);
-                    if (r < hi && W.sync_w[r] == B.w) {
-                        if (!((W.sync_mask[r] >> ln) & 1u)) {
-                            bad = 1;
-                            continue;
-                        }
-                        chk = true;
-                        row = r;
+                /* w == 0 (no sync passed yet) finds the family record {~0, smax} */
+                uint4 fe = fh_find(W, sync_hkey(B.graw, B.b, B.w, gw));
+                if (fe.z != 0xffffffffu) {
+                    if (!((__ldg(W.sync_mask + fe.z) >> ln) & 1u)) {
+                        bad = 1;
+                        continue;
                     }
-                    upd = B.w < W.sync_w[hi - 1];
+                    chk = true;
+                    row = fe.z;
+                } else if (B.w && fe.x == 0xffffffffu && fe.y == 0xffffffffu) {
+                    fe = fh_find(W, sync_hkey(B.graw, B.b, 0, gw));
+                }
+                if (fe.x != 0xffffffffu || fe.y != 0xffffffffu) {
+                    upd = B.w < fe.w;
                     owner = (1ull << 63) | ((unsigned long long)B.g << 50) | ((unsigned long long)B.b << 40) | gw;
                 }
             }
@@ -339,19 +393,18 @@ __global__ void __launch_bounds__(kMaskedThreads)
                 const uint64_t wk = word + k;
                 const uint64_t idx = sh ? c.global_words + (uint64_t)blk * c.smem_words + wk : wk;
                 const uint64_t key = sh ? (HIRACE_SHARED_BIT | ((uint64_t)blk << 32) | wk) : wk;
+                /* a4 first: its latency overlaps the history work (a stale value costs a retry) */
+                R *p = shadow + idx;
+                R o = Rec<R>::load(p);
                 bool side = false;
                 if (chk || upd) {
                     unsigned long long *slot = hist_slot(W, key, owner, full);
                     if (slot) {
-                        if (chk)
-                            side = side_check(slot, ln, lanes, stamp, W.confl[cls], B.w, W.vrow + (size_t)row * 32);
+                        side = side_check(slot, ln, stamp, W.confl[cls], B.w, W.vrow + (size_t)row * 32, chk, upd);
                         if (upd)
-                            side_update(slot + 2 + ln, stamp, cls, B.w);
+                            side_update(slot + 4 + ln, stamp, cls, B.w);
                     }
                 }
-                /* a4-a6 with the side verdict folded into the transition */
-                R *p = shadow + idx;
-                R o = Rec<R>::load(p);
                 cnt.checked++;
                 bool first = true;
                 for (;;) {
@@ -418,7 +471,7 @@ const void *masked_kernel(const hirace_dev_ctx &c)
 cudaError_t launch_ws_prepare(const hirace_warp_sync *d_syncs, uint32_t n, uint32_t total_warps, uint32_t warp_size,
                               const WsDev &W, unsigned int *err, int sm_count, cudaStream_t st)
 {
-    note_launches(2);
+    note_launches(1);
     k_ws_families<<<1, kFamThreads, 0, st>>>(d_syncs, n, total_warps, warp_size, W, err);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess)
@@ -426,6 +479,11 @@ cudaError_t launch_ws_prepare(const hirace_warp_sync *d_syncs, uint32_t n, uint3
     const uint32_t blocks = (n + kClockWarps - 1) / kClockWarps;
     const uint32_t grid = blocks < (uint32_t)(8 * sm_count) ? (blocks ? blocks : 1u) : (uint32_t)(8 * sm_count);
     k_ws_clocks<<<grid, kClockWarps * 32, 0, st>>>(W);
+    if ((e = cudaGetLastError()) != cudaSuccess)
+        return e;
+    note_launches(2);
+    const uint32_t hb = (n + 255) / 256;
+    k_ws_hash<<<hb < (uint32_t)(8 * sm_count) ? hb : (uint32_t)(8 * sm_count), 256, 0, st>>>(W, n);
     return cudaGetLastError();
 }
 

@@ -312,7 +312,7 @@ class Checker:
                 granularity_log2=getattr(trace, "granularity_log2", 2))
         syncs = getattr(trace, "warp_syncs", None)
         if syncs is not None and len(syncs):
-            c.set_warp_syncs(syncs, history_slots)
+            c.set_warp_syncs(syncs, history_slots or trace.info.get("history_slots", 0))
         return c
 
     def set_warp_syncs(self, syncs, history_slots: int = 0, stream=None):
