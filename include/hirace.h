@@ -60,7 +60,8 @@ typedef enum {
 } hirace_kind;
 
 /* Barrier scopes.  GRID = grid-wide sync or kernel boundary. */
-typedef enum { HIRACE_SCOPE_WARP = 1, HIRACE_SCOPE_BLOCK = 2, HIRACE_SCOPE_GRID = 3 } hirace_scope;
+typedef enum { HIRACE_SCOPE_WARP = 1, HIRACE_SCOPE_BLOCK = 2, HIRACE_SCOPE_GRID = 3,
+               HIRACE_SCOPE_CLUSTER = 4 /* barrier.cluster / cluster.sync(): cluster contexts only */ } hirace_scope;
 
 /* Race class = the coarsest hierarchy level of the first racing epoch (R6). */
 typedef enum { HIRACE_RACE_WARP = 1, HIRACE_RACE_BLOCK = 2, HIRACE_RACE_GRID = 3 } hirace_race_class;
@@ -575,6 +576,28 @@ hirace_status hirace_cluster_reset(hirace_cluster_ctx *ctx, void *stream);
 hirace_status hirace_cluster_replay(hirace_cluster_ctx *ctx, const hirace_event *d_events, uint64_t n, void *stream);
 hirace_status hirace_cluster_collect(hirace_cluster_ctx *ctx, hirace_race *h_out, uint64_t cap, uint64_t *n_total);
 hirace_status hirace_cluster_get_stats(hirace_cluster_ctx *ctx, uint64_t *checked, uint64_t *cas_retries);
+
+/* Inline hooks for a cluster context (the paper's wrapper, with the cluster level
+ * of R16): device context handed by value to instrumented cluster kernels; the device side is
+ * hirace::cluster::thread_init / on_access / barrier in include/hirace_device.cuh.  DSMEM
+ * accesses are recognised from the generic address (an address another block of the cluster
+ * maps through cluster.map_shared_rank / __cluster_map_shared_rank).  All pointers are device
+ * pointers owned by the cluster context; g = grid epoch of the launch (0 here: the caller sets
+ * it per launch, <= 254, one per kernel boundary).  Results: hirace_cluster_collect.
+ * Errors (inline): out-of-range thread ids / epochs set the context's range flag (BAD_TRACE at
+ * the next collect) and stop checking in that thread. */
+typedef struct {
+    unsigned long long *shadow;  /* [global_words | grid_blocks * smem_words] cluster records */
+    const unsigned char *table;  /* 16 KB cluster FSM table (hirace_fsm_table_cluster)       */
+    unsigned int *error_flags;   /* bit0 bad trace, bit1 range                               */
+    unsigned long long *stats;   /* [checked word accesses, CAS retries]                     */
+    const void *global_base;     /* tracked global base (may be NULL)                        */
+    unsigned long long global_words;
+    unsigned int smem_words, grid_blocks, block_threads, warp_size, cluster_blocks;
+    unsigned int g;
+} hirace_cluster_dev_ctx;
+hirace_status hirace_cluster_get_dev_ctx(hirace_cluster_ctx *ctx, const void *global_base,
+                                         hirace_cluster_dev_ctx *out);
 
 const char *hirace_status_string(hirace_status s);
 

@@ -538,4 +538,23 @@ hirace_status hirace_cluster_get_stats(hirace_cluster_ctx *c, uint64_t *checked,
     return HIRACE_OK;
 }
 
+hirace_status hirace_cluster_get_dev_ctx(hirace_cluster_ctx *c, const void *global_base, hirace_cluster_dev_ctx *out)
+{
+    if (!c || !out)
+        return HIRACE_E_INVAL;
+    out->shadow = c->shadow;
+    out->table = c->table;
+    out->error_flags = c->err;
+    out->stats = c->stats;
+    out->global_base = global_base;
+    out->global_words = c->global_words;
+    out->smem_words = (unsigned int)c->smem_words;
+    out->grid_blocks = c->cfg.grid_blocks;
+    out->block_threads = c->cfg.block_threads;
+    out->warp_size = c->cfg.warp_size;
+    out->cluster_blocks = c->cluster_blocks;
+    out->g = 0;
+    return HIRACE_OK;
+}
+
 } /* extern "C" */

@@ -34,7 +34,10 @@ def load():
         lib.hx_reduce.argtypes = [P, P, I, I, I, U, I, P]
         lib.hx_multiphase.argtypes = [P, P, I, I, I, I, I, P, U, I, P]
         lib.hx_bfs.argtypes = [P, P, P, P, I, I, U, ctypes.POINTER(I), P]
-        for f in (lib.hx_stencil, lib.hx_reduce, lib.hx_multiphase, lib.hx_bfs):
+        lib.hx_cluster_halo.argtypes = [P, P, I, I, I, I, P]
+        lib.hx_cluster_hist.argtypes = [P, P, I, I, I, I, I, I, P]
+        for f in (lib.hx_stencil, lib.hx_reduce, lib.hx_multiphase, lib.hx_bfs, lib.hx_cluster_halo,
+                  lib.hx_cluster_hist):
             f.restype = I
         _libs[_aggregate] = lib
     return _libs[_aggregate]
@@ -89,3 +92,22 @@ def bfs(checker, base, nindex, nlist, dist, V: int, racy: bool, g0: int = 0, str
 
 
 __all__ = ["stencil", "reduce", "multiphase", "bfs", "load", "use_aggregated_hooks", "DevCtx"]
+
+
+def cluster_halo(checker, out, nclusters: int, cluster_blocks: int, block_threads: int, sync: str, stream=None):
+    """DSMEM halo (tracegen.cluster_halo) under the cluster inline hooks; checker: ClusterChecker
+    or None (uninstrumented); out: CUDA float32 tensor of nclusters*cluster_blocks*block_threads.
+    sync: "cluster", "block" or "none"."""
+    d, p = _ctx(checker, out.data_ptr())
+    mode = {"none": 0, "cluster": 1, "block": 2}[sync]
+    _ok(load().hx_cluster_halo(p, ctypes.c_void_p(out.data_ptr()), nclusters, cluster_blocks, block_threads, mode,
+                               _stream_handle(stream)), "hx_cluster_halo")
+
+
+def cluster_hist(checker, out, nclusters: int, cluster_blocks: int, block_threads: int, bins: int,
+                 block_scope: bool, drop: int | None, stream=None):
+    """DSMEM histogram (tracegen.cluster_histogram); out: CUDA int32 tensor of nclusters*bins (the
+    tracked global base)."""
+    d, p = _ctx(checker, out.data_ptr())
+    _ok(load().hx_cluster_hist(p, ctypes.c_void_p(out.data_ptr()), nclusters, cluster_blocks, block_threads, bins,
+                               int(block_scope), int(drop or 0), _stream_handle(stream)), "hx_cluster_hist")

@@ -43,7 +43,7 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_cluster_collect", "hirace_cluster_get_stats", "hirace_status_string",
            "hirace_version", "hirace_launch_count", "hirace_set_replay_mode", "hirace_get_replay_mode",
            "hirace_advance_grid_epochs", "hirace_peer_release", "hirace_peer_wait", "hirace_set_reset_mode",
-           "hirace_set_warp_syncs")
+           "hirace_set_warp_syncs", "hirace_cluster_get_dev_ctx")
 
 
 class HiraceError(RuntimeError):
@@ -74,6 +74,14 @@ class DevCtx(ctypes.Structure):
                 ("f_active", ctypes.c_uint32), ("f_tid_mask", ctypes.c_uint32), ("f_tid_match", ctypes.c_uint32),
                 ("f_spaces", ctypes.c_uint32), ("f_glo", ctypes.c_uint64), ("f_ghi", ctypes.c_uint64),
                 ("f_smem_words", ctypes.c_uint32), ("f_pad", ctypes.c_uint32), ("g_base", ctypes.c_void_p)]
+
+
+class ClusterDevCtx(ctypes.Structure):
+    """hirace_cluster_dev_ctx (include/hirace.h): handed by value to instrumented cluster kernels."""
+    _fields_ = [("shadow", ctypes.c_void_p), ("table", ctypes.c_void_p), ("error_flags", ctypes.c_void_p),
+                ("stats", ctypes.c_void_p), ("global_base", ctypes.c_void_p), ("global_words", ctypes.c_uint64),
+                ("smem_words", ctypes.c_uint32), ("grid_blocks", ctypes.c_uint32), ("block_threads", ctypes.c_uint32),
+                ("warp_size", ctypes.c_uint32), ("cluster_blocks", ctypes.c_uint32), ("g", ctypes.c_uint32)]
 
 
 class EpochLimits(ctypes.Structure):
@@ -149,6 +157,7 @@ def load():
         "hirace_set_reset_mode": (I32, [P, I32]),
         "hirace_get_replay_mode": (I32, [P, ctypes.POINTER(I32)]),
         "hirace_set_warp_syncs": (I32, [P, P, U64, U64, P]),
+        "hirace_cluster_get_dev_ctx": (I32, [P, P, ctypes.POINTER(ClusterDevCtx)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -321,7 +330,7 @@ class Checker:
         import torch
         if syncs is None or len(syncs) == 0:
             _check(self.lib.hirace_set_warp_syncs(self.h, None, 0, 0, _stream_handle(stream)),
-                   "hirace_set_warp_syncs")
+                   "hirace_set_warp_syncs", "hirace_cluster_get_dev_ctx")
             return
         if isinstance(syncs, np.ndarray):
             arr = np.ascontiguousarray(syncs)
@@ -644,6 +653,13 @@ class ClusterChecker:
             if total.value <= cap:
                 return out[: total.value]
             cap = int(total.value)
+
+    def dev_ctx(self, global_base: int = 0) -> ClusterDevCtx:
+        """hirace_cluster_get_dev_ctx: the device context of the cluster inline hooks."""
+        d = ClusterDevCtx()
+        _check(self.lib.hirace_cluster_get_dev_ctx(self.h, ctypes.c_void_p(global_base), ctypes.byref(d)),
+               "hirace_cluster_get_dev_ctx")
+        return d
 
     def stats(self):
         a, b = ctypes.c_uint64(0), ctypes.c_uint64(0)

@@ -77,3 +77,22 @@ def test_ctypes_structs_match_the_c_header(tmp_path):
     assert [int(x) for x in out[:3]] == [ctypes.sizeof(hb.Config), ctypes.sizeof(hb.DevCtx),
                                         ctypes.sizeof(hb.EpochLimits)]
     assert [int(x) for x in out[3:]] == [getattr(hb.DevCtx, f).offset for f in fields]
+
+
+def test_cluster_dev_ctx_mirror_matches_the_c_header(tmp_path):
+    import ctypes
+    import subprocess
+
+    from paper_conf_sc_jacobsonbg24_b200 import hirace as hb
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    fields = [f for f, _ in hb.ClusterDevCtx._fields_]
+    src = tmp_path / "csz.c"
+    src.write_text("#include <stdio.h>\n#include <stddef.h>\n#include \"hirace.h\"\nint main(){\n"
+                   "printf(\"%zu %zu\\n\", sizeof(hirace_cluster_dev_ctx), sizeof(hirace_warp_sync));\n"
+                   + "".join(f"printf(\"%zu\\n\", offsetof(hirace_cluster_dev_ctx, {f}));\n" for f in fields)
+                   + "return 0;}\n")
+    exe = tmp_path / "csz"
+    subprocess.check_call(["gcc", "-I", os.path.join(root, "include"), str(src), "-o", str(exe)])
+    out = [int(x) for x in subprocess.check_output([str(exe)], text=True).split()]
+    assert out[:2] == [ctypes.sizeof(hb.ClusterDevCtx), hb.WARP_SYNC_DTYPE.itemsize]
+    assert out[2:] == [getattr(hb.ClusterDevCtx, f).offset for f in fields]
