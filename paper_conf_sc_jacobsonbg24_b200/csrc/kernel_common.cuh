@@ -7,6 +7,10 @@
 
 #include "hirace.h"
 
+#ifndef HIRACE_BAR_ACQLOAD
+#define HIRACE_BAR_ACQLOAD 1
+#endif
+
 namespace hirace_impl {
 
 /* batch key (g,b,w) of event p = meta >> 5 */
@@ -36,7 +40,13 @@ __device__ __forceinline__ void grid_sync(unsigned int *bar, unsigned int nctas,
             __nanosleep(HIRACE_BAR_SLEEP);
 #endif
         }
+#if HIRACE_BAR_ACQLOAD
+        /* one acquire load of the counter: it reads the last arrival's value, so it synchronises
+         * with every red.release of the release sequence (instead of a full acq_rel fence) */
+        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
+#else
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
+#endif
     }
     __syncthreads();
 }

@@ -33,6 +33,13 @@
 #include "record.cuh"
 #include "replay_core.cuh"
 
+#ifndef HIRACE_HOIST_OFFSETS
+#define HIRACE_HOIST_OFFSETS 0
+#endif
+#ifndef HIRACE_HOIST_KEY
+#define HIRACE_HOIST_KEY 1
+#endif
+
 namespace hirace_impl {
 
 using namespace hirace;
@@ -192,8 +199,21 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     uint4 e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
     uint4 e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
     const uint32_t gb = c.g_base ? *c.g_base : 0u; /* epoch reset: offset of this check's epochs */
+    /* the batch key is read before the barrier that precedes the batch (its load latency is
+     * off the post-barrier critical path) */
+    uint32_t key_next = nb ? __ldg(&ev[bstart].w) >> 5 : 0u;
     for (uint32_t bi = 0; bi < nb; bi++) {
-        const Batch B = make_batch<R>(__ldg(&ev[bstart].w) >> 5, rec, gb);
+#if !HIRACE_HOIST_KEY
+        key_next = __ldg(&ev[bstart].w) >> 5;
+#endif
+        const Batch B = make_batch<R>(key_next, rec, gb);
+#if HIRACE_HOIST_OFFSETS
+        uint32_t nstart = 0, nend = 0; /* next batch's bounds, requested while this one runs */
+        if (bi + 1 < nb) {
+            nstart = __ldg(&off[bi + 1]);
+            nend = __ldg(&off[bi + 2]);
+        }
+#endif
         const uint32_t keysz = B.key << 3; /* (meta >> 2) - keysz = size_log2 for this batch */
         if (B.g == 255u)
             bad = 1; /* reserved for retired RACE records (R7) */
@@ -209,8 +229,16 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
             process_decoded<R>(cur, B, c, G, rec, raw, tab_s, cnt, lane, below);
         }
         if (bi + 1 < nb) {
+#if HIRACE_HOIST_OFFSETS
+            bstart = nstart;
+            bend = nend;
+#else
             bstart = __ldg(&off[bi + 1]);
             bend = __ldg(&off[bi + 2]);
+#endif
+#if HIRACE_HOIST_KEY
+            key_next = __ldg(&ev[bstart].w) >> 5;
+#endif
             warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
             e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
             e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);

@@ -330,7 +330,7 @@ class Checker:
         import torch
         if syncs is None or len(syncs) == 0:
             _check(self.lib.hirace_set_warp_syncs(self.h, None, 0, 0, _stream_handle(stream)),
-                   "hirace_set_warp_syncs", "hirace_cluster_get_dev_ctx")
+                   "hirace_set_warp_syncs")
             return
         if isinstance(syncs, np.ndarray):
             arr = np.ascontiguousarray(syncs)

@@ -1,0 +1,13 @@
+#!/bin/bash
+OUT=gpurun_out; mkdir -p $OUT
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+timeout 600 python -m pytest tests/test_gpu_masked.py -q -x -k "epoch_reset or removing" > $OUT/pytest_masked_fix.log 2>&1; echo "rc=$?" >> $OUT/pytest_masked_fix.log
+for so in build/variants/*.so; do
+  v=$(basename $so .so); [ "$v" = base ] && continue
+  HIRACE_LIB=$PWD/$so timeout 600 python -m pytest tests/test_gpu_parity.py tests/test_gpu_epoch.py -x -q -k "not full and not cfg5" > $OUT/pytest_$v.log 2>&1
+  echo "pytest exit $?" >> $OUT/pytest_$v.log
+done
+REPS=2 CFGS="2 4 3" timeout 2400 bash scripts/ab4.sh > /dev/null 2>&1
+cp $OUT/ab_summary.txt $OUT/ab_summary_234.txt
+REPS=1 CFGS="5" timeout 1800 bash scripts/ab4.sh > /dev/null 2>&1
+cp $OUT/ab_summary.txt $OUT/ab_summary_5.txt
