@@ -6,5 +6,5 @@ for so in build/variants/*.so; do
   HIRACE_LIB=$PWD/$so timeout 600 python -m pytest tests/test_gpu_parity.py tests/test_gpu_epoch.py tests/test_gpu_edges.py -x -q -k "not full and not cfg5" > $OUT/pytest_$v.log 2>&1
   echo "pytest exit $?" >> $OUT/pytest_$v.log
 done
-REPS=2 CFGS="2 4" timeout 2400 bash scripts/ab4.sh > /dev/null 2>&1
-cp $OUT/ab_summary.txt $OUT/ab_summary_hier.txt
+REPS=2 CFGS="${CFGS:-2 4 3}" timeout 2400 bash scripts/ab4.sh > /dev/null 2>&1
+cp $OUT/ab_summary.txt $OUT/ab_summary_${TAG:-x}.txt
