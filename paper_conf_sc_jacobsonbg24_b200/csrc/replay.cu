@@ -33,9 +33,6 @@
 #include "record.cuh"
 #include "replay_core.cuh"
 
-#ifndef HIRACE_TMA_EVENTS
-#define HIRACE_TMA_EVENTS 0
-#endif
 
 namespace hirace_impl {
 
@@ -146,15 +143,6 @@ __device__ __forceinline__ Lane decode(const uint4 &e, bool valid_in, uint32_t k
     return L;
 }
 
-#if HIRACE_TMA_EVENTS
-constexpr int kTmaSlots = 4;
-/* one 32-event chunk (m events) into a ring slot by the TMA engine, completing on mb */
-__device__ __forceinline__ void tma_chunk(uint4 *dst, uint64_t *mb, const uint4 *src, uint32_t m)
-{
-    mbar_arrive_expect_tx(mb, m * 16u);
-    bulk_g2s(dst, src, m * 16u, mb);
-}
-#endif
 
 /* out of line so the collect's registers do not raise the replay loop's allocation */
 template <typename R>
@@ -181,19 +169,6 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
         reinterpret_cast<uint4 *>(s_table)[i] = __ldg(reinterpret_cast<const uint4 *>(c.table) + i);
     if (threadIdx.x < 4)
         s_stats[threadIdx.x] = 0;
-#if HIRACE_TMA_EVENTS
-    /* a1 by the TMA engine: per warp a ring of kTmaSlots 32-event chunks in shared memory, filled
-     * by 1-D bulk copies (lane 0) that complete on one mbarrier per slot */
-    __shared__ __align__(128) uint4 s_ring[kReplayThreads / 32][kTmaSlots][32];
-    __shared__ __align__(8) uint64_t s_mb[kReplayThreads / 32][kTmaSlots];
-    const uint32_t wl = threadIdx.x >> 5;
-    if (lane == 0) {
-        for (int k = 0; k < kTmaSlots; k++)
-            mbar_init(&s_mb[wl][k], 1);
-        fence_mbar_init();
-    }
-    uint32_t qi = 0, qc = 0; /* chunks issued / consumed by this warp */
-#endif
 
     geom G = make_geom(c);
     G.pow2 = P2; /* compile-time geometry mode: shifts (P2) or fast division */
@@ -216,14 +191,8 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
     __syncthreads();
     uint32_t i, iend; /* this warp's contiguous share of the batch: events [i - lane, iend) */
     warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
-#if HIRACE_TMA_EVENTS
-    if (lane == 0) /* the first chunks of the first batch */
-        for (uint32_t s0 = i; s0 < iend && s0 < i + 32 * (kTmaSlots - 1); s0 += 32, qi++)
-            tma_chunk(&s_ring[wl][qi % kTmaSlots][0], &s_mb[wl][qi % kTmaSlots], ev + s0, min(32u, iend - s0));
-#else
     uint4 e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
     uint4 e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
-#endif
     const uint32_t gb = c.g_base ? *c.g_base : 0u; /* epoch reset: offset of this check's epochs */
     /* the batch key is read before the barrier that precedes the batch (its load latency is
      * off the post-barrier critical path) */
@@ -237,22 +206,9 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
             clk = 1; /* compact record: epochs beyond the declared limits; batch not checked */
 
         for (; i - lane < iend; i += 32) {
-#if HIRACE_TMA_EVENTS
-            const uint32_t ahead = i - lane + 32 * (kTmaSlots - 1); /* refill the slot read last */
-            if (lane == 0 && ahead < iend) {
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                tma_chunk(&s_ring[wl][qi % kTmaSlots][0], &s_mb[wl][qi % kTmaSlots], ev + ahead, min(32u, iend - ahead));
-                qi++;
-            }
-            mbar_wait(&s_mb[wl][qc % kTmaSlots], (qc / kTmaSlots) & 1u);
-            const uint4 e = i < iend ? s_ring[wl][qc % kTmaSlots][lane] : make_uint4(0, 0, 0, 0);
-            qc++;
-            __syncwarp();
-#else
             const uint4 e = e0;
             e0 = e1; /* a1: keep the next chunks' events in flight */
             ld_event_if(ev + i + 64, i + 64 < iend, e1);
-#endif
             const bool valid = i < iend && B.fit;
             const Lane cur = decode<W32, R>(e, valid, keysz, B, tid_max, c, G, raw, cnt, bad, lane);
             process_decoded<R>(cur, B, c, G, rec, raw, tab_s, cnt, lane, below);
@@ -262,18 +218,8 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
             bend = __ldg(&off[bi + 2]);
             key_next = __ldg(&ev[bstart].w) >> 5;
             warp_share(bstart, bend, warp_global, nwarps, lane, i, iend);
-#if HIRACE_TMA_EVENTS
-            __syncwarp();
-            if (lane == 0) {
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                for (uint32_t s0 = i; s0 < iend && s0 < i + 32 * (kTmaSlots - 1); s0 += 32, qi++)
-                    tma_chunk(&s_ring[wl][qi % kTmaSlots][0], &s_mb[wl][qi % kTmaSlots], ev + s0,
-                              min(32u, iend - s0));
-            }
-#else
             e0 = i < iend ? ld_event(ev + i) : make_uint4(0, 0, 0, 0);
             e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
-#endif
 #ifdef HIRACE_BARRIER_TRACE
             __syncthreads();
             if (threadIdx.x == 0 && bi < 128 && blockIdx.x < 2048)
