@@ -265,6 +265,54 @@ def host_cpu() -> dict:
     return {"cpu_model": model, "nproc": os.cpu_count()}
 
 
+def random_rmw_count(trace, d_ev) -> int:
+    """Config 5: accesses to its two randomly addressed regions (the uniform gather over 2^30
+    words and the one-word-per-thread fillers; tracegen.cfg5 regions), counted on the device."""
+    import torch
+    reg = trace.info["regions"]
+    T = trace.grid_blocks * trace.block_threads
+    lo1, hi1 = reg["gather"], reg["hot"]          # [W/2, 3W/4)
+    lo2, hi2 = reg["inj"], reg["inj"] + T
+    addr = d_ev.view(torch.int64).view(-1, 2)[:, 0]
+    n = 0
+    for a in range(0, addr.numel(), 1 << 27):
+        w = (addr[a:a + (1 << 27)] & ((1 << 62) - 1)) >> 2
+        n += int(((w >= lo1) & (w < hi1)).sum()) + int(((w >= lo2) & (w < hi2)).sum())
+    return n
+
+
+def random_roofline(n_random: int, kern_ms: float, dev: int) -> dict:
+    """The resource config 5 is bound by: scattered first-touch load+CAS pairs into an HBM-sized
+    shadow.  Peak = the same-process microbenchmark rate of random 8-byte
+    load+CAS pairs over an 8 GiB word array (config 5's gather region), cold L2; achieved = the
+    replay's random-region accesses per second of k_replay (which moves the streaming 2/3 of the
+    trace at the same time)."""
+    import torch
+
+    from paper_conf_sc_jacobsonbg24_b200 import hirace as h
+    dv = f"cuda:{dev}"
+    words = torch.zeros(1 << 30, dtype=torch.int64, device=dv)
+    gen = torch.Generator(device=dv)
+    gen.manual_seed(20241117)
+    m = min(n_random, 320 * 10**6)
+    idx = torch.randint(0, 1 << 30, (m,), generator=gen, device=dv, dtype=torch.int64)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dv)
+    best = 0.0
+    for _ in range(2):
+        flush.fill_(1)
+        torch.cuda.synchronize()
+        ms = h.microbench_indexed(words.data_ptr(), idx.data_ptr(), m, 3, 8, device=dev)
+        best = max(best, m / (ms * 1e-3))
+    del words, idx, flush
+    torch.cuda.empty_cache()
+    ach = n_random / (kern_ms / 1e3)
+    return {"bound": "dram_random_rmw", "achieved": ach, "peak": best, "unit": "load+CAS pairs/s", "frac": ach / best,
+            "random_accesses": n_random,
+            "peak_kind": "measured (hirace_microbench_indexed op 3, 3.2e8 random words of 8 GiB, 8 CTAs/SM)",
+            "note": "achieved counts only the gather + filler accesses; the kernel moves the coalesced "
+                    "private accesses, the hot atomics and the 16-B events in the same time"}
+
+
 def l2_roofline(st: dict, n_acc: int, kern_ms: float, rec_bytes: int, dev: int) -> dict:
     """the L2-atomic roofline of this workload, from microbenchmarks run in the same
     process on L2-resident words (coalesced, the replay's access shape): every access is one
@@ -756,9 +804,21 @@ def main():
         except Exception as exc:  # diagnostics only; never fails the bench line
             l2 = {"error": str(exc)}
     rec_bytes = c.rec_bytes
+    n_random = None
+    if rank == 0 and args.config == 5 and "regions" in trace.info:
+        try:
+            n_random = random_rmw_count(trace, ctx["d_ev"])
+        except Exception as exc:  # diagnostics only
+            print(f"bench: random-region count failed ({exc})", file=sys.stderr)
     c.close()
     ctx["d_ev"] = None
     torch.cuda.empty_cache()
+    rnd = None
+    if n_random:
+        try:
+            rnd = random_roofline(n_random, kern_ms, dev)
+        except Exception as exc:  # diagnostics only
+            rnd = {"error": str(exc)}
     cpu = None
     if not args.no_cpu_baseline and world == 1 and rank == 0:
         cpu = cpu_baseline(trace, 20.0)
@@ -790,6 +850,7 @@ def main():
         "scaling": "strong" if args.config == 5 else "weak", "vs_baseline": None,
         "dtype": "u64" if rec_bytes == 8 else "u32", "data": "synthetic", "config": cb,
         "roofline": roof, "roofline_step": res["roofline_step"], "roofline_l2": l2,
+        "roofline_dram_random": rnd,
         "cpu_baseline": cpu, "e2e": e2e,
         "gpu_launches": res["launches_per_step"] * K,
         "step_mode": res["step_mode"], "eager_ms_per_step": res["eager_ms_per_step"],
