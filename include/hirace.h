@@ -527,8 +527,9 @@ typedef struct {
  * during this call only; the context keeps its own derived copy).  The library derives, per
  * (g, b, warp) family, the warp vector clock after every listed sync (one warp per family),
  * and allocates a sub-warp access history of history_slots slots (rounded up to a power of two;
- * 0 = 65,536; 288 B each): one slot per word that masked-family accesses touch in a block epoch,
- * holding per lane and access class (read / atomic / write) the last sync number.  The replay
+ * 0 = 65,536; 64 B each, plus a pool of slots/8 spill blocks of 256 B): one slot per word that
+ * masked-family accesses touch in a block epoch, holding for up to five (lane, access class)
+ * pairs the last sync number (read / atomic / write), more pairs in a spill block.  The replay
  * then runs the per-access FSM as usual with w read as the sync number, and additionally
  * compares each access of a family at a listed sync with its lanes' history against the vector
  * clock: a conflicting access not ordered before it is a race of the FSM state's level (WARP

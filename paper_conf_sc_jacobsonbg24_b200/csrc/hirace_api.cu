@@ -317,10 +317,21 @@ cudaError_t launch_masked(hirace_ctx *c, const hirace_event *d_events, cudaStrea
     return launch_replay_masked(c->dev, W, d_events, c->scr, c->masked_grid, st);
 }
 
+/* empty history: every slot free, no spill block handed out, the pool's lane words stale */
+cudaError_t ws_clear(hirace_ctx *c, cudaStream_t st)
+{
+    cudaError_t e = cudaMemsetAsync(c->ws.hist, 0xff, c->ws_slots * kSlotWords * sizeof(unsigned long long), st);
+    if (e == cudaSuccess)
+        e = cudaMemsetAsync(c->ws.spill, 0xff, c->ws.nspill * 32 * sizeof(unsigned long long), st);
+    if (e == cudaSuccess)
+        e = cudaMemsetAsync(c->ws.spill_count, 0, sizeof(unsigned long long), st);
+    return e;
+}
+
 void ws_free(hirace_ctx *c)
 {
     void *ptrs[] = {c->ws.fam_key, c->ws.fam_lo, c->ws.nfam, c->ws.sync_w, c->ws.sync_mask, c->ws.sync_fam,
-                    c->ws.vrow, c->ws.fhash, c->ws.hist};
+                    c->ws.vrow, c->ws.fhash, c->ws.hist, c->ws.spill, c->ws.spill_count};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
@@ -367,18 +378,21 @@ hirace_status hirace_set_warp_syncs(hirace_ctx *c, const hirace_warp_sync *d_syn
         (e = cudaMalloc(&W.sync_fam, n * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&W.vrow, n * 32 * sizeof(unsigned short))) != cudaSuccess ||
         (e = cudaMalloc(&W.fhash, fh_slots * sizeof(uint4))) != cudaSuccess ||
-        (e = cudaMalloc(&W.hist, slots * kSlotWords * sizeof(unsigned long long))) != cudaSuccess) {
+        (e = cudaMalloc(&W.hist, slots * kSlotWords * sizeof(unsigned long long))) != cudaSuccess ||
+        (e = cudaMalloc(&W.spill, (slots / 8) * 32 * sizeof(unsigned long long))) != cudaSuccess ||
+        (e = cudaMalloc(&W.spill_count, sizeof(unsigned long long))) != cudaSuccess) {
         ws_free(c);
         return from_cuda(c, e);
     }
     W.slots_mask = slots - 1;
+    W.nspill = slots / 8;
     W.fh_mask = fh_slots - 1;
     W.nsync = (uint32_t)n;
     W.wpb = (c->cfg.block_threads + c->cfg.warp_size - 1) / c->cfg.warp_size;
     c->ws_slots = slots;
     if (!c->masked_grid)
         c->masked_grid = masked_max_grid(c->device);
-    HR_CUDA(c, cudaMemsetAsync(W.hist, 0xff, slots * kSlotWords * sizeof(unsigned long long), st));
+    HR_CUDA(c, ws_clear(c, st));
     HR_CUDA(c, cudaMemsetAsync(W.fhash, 0xff, fh_slots * sizeof(uint4), st));
     HR_CUDA(c, launch_ws_prepare(d_syncs, (uint32_t)n, c->cfg.grid_blocks * W.wpb, c->cfg.warp_size, W, c->d_err,
                                  c->sm_count, st));
@@ -625,7 +639,8 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
                     c->scr.grid_bar2, c->scr.cta_cnt, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
                     c->d_stage[0], c->d_stage[1], c->d_wire_off, c->d_wire_counts, c->d_wire_flag,
                     c->d_peer_tab, c->d_flag_tab, c->d_gepoch, c->ws.fam_key, c->ws.fam_lo, c->ws.nfam,
-                    c->ws.sync_w, c->ws.sync_mask, c->ws.sync_fam, c->ws.vrow, c->ws.fhash, c->ws.hist};
+                    c->ws.sync_w, c->ws.sync_mask, c->ws.sync_fam, c->ws.vrow, c->ws.fhash, c->ws.hist,
+                    c->ws.spill, c->ws.spill_count};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
@@ -702,7 +717,7 @@ hirace_status hirace_shadow_reset(hirace_ctx *c, void *stream)
         c->lazy = false;
     }
     if (c->ws.hist) /* the sub-warp history belongs to the check */
-        HR_CUDA(c, cudaMemsetAsync(c->ws.hist, 0xff, c->ws_slots * kSlotWords * sizeof(unsigned long long), st));
+        HR_CUDA(c, ws_clear(c, st));
     c->g = 0;
     c->dev.g = 0;
     c->sticky = HIRACE_OK;

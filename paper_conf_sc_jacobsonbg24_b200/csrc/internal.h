@@ -141,8 +141,9 @@ cudaError_t window_init();
 /* ---- partial-mask warp syncs (subwarp.cu; hirace_set_warp_syncs, R20) ----------
  * Families = (g, b, warp) with listed syncs, sorted by key g<<50 | b<<40 | warp; sync_w / mask
  * / vrow per listed sync (vrow: the warp vector clock after it, 32 u16); hist: open-addressing
- * table of kSlotWords-word slots [key, owner, presence, -, 32 lane words] (subwarp.cu). */
-constexpr uint32_t kSlotWords = 36;
+ * table of kSlotWords-word slots [key, owner, spill, 5 entries] plus a pool of 32-lane spill
+ * blocks (subwarp.cu). */
+constexpr uint32_t kSlotWords = 8;
 struct WsDev {
     unsigned long long *fam_key;
     uint32_t *fam_lo;        /* [nfam + 1] first listed sync of each family */
@@ -154,6 +155,9 @@ struct WsDev {
     uint32_t nsync;
     unsigned long long *hist;
     unsigned long long slots_mask;
+    unsigned long long *spill;        /* nspill blocks of 32 lane words                  */
+    unsigned long long *spill_count;  /* blocks handed out in this check                 */
+    unsigned long long nspill;
     uint32_t wpb;            /* warps per block */
     uint32_t confl[3];       /* per access class (R, A, X): classes it conflicts with in a block */
     unsigned char race_of[32]; /* FSM state -> the RACE state of its level (policy's table) */

@@ -223,3 +223,43 @@ def test_window_mode_replays_batch_major_with_a_log():
         assert _gpu(t, checker=c)[0] == _want(t)
     finally:
         c.close()
+
+
+def _broadcast_trace(nwords, lanes_mask, writer_lane):
+    """one warp of 32 lanes: every lane reads words 0..nwords-1 (w = 0); a partial sync of
+    lanes_mask; writer_lane writes every word (w = 1).  Readers outside the mask race with the
+    write; the 32 (lane, read) pairs per word overflow a slot's five entries into a spill block."""
+    import numpy as np
+    rows = [(wd, False, ln, tg.READ, 0, 0, 0) for wd in range(nwords) for ln in range(32)]
+    rows += [(wd, False, writer_lane, tg.WRITE, 1, 0, 0) for wd in range(nwords)]
+    ev = np.empty(len(rows), dtype=tg.EVENT_DTYPE)
+    a = np.array(rows, dtype=np.int64)
+    ev["addr"] = a[:, 0].astype(np.uint64) << np.uint64(2)
+    ev["tid"] = a[:, 2]
+    ev["meta"] = tg.pack_meta(a[:, 3], 2, a[:, 4], a[:, 5], a[:, 6])
+    sy = tg.make_syncs([0], [lanes_mask], [1], [0], [0])
+    return tg.Trace("bcast", tg.sort_by_batch(ev), 1, 32, 32, nwords, 0, warp_syncs=sy)
+
+
+@pytest.mark.parametrize("mask,writer,expect_race", [(0x0000FFFF, 0, True), (0xFFFFFFFE, 31, True),
+                                                     (0xFFFFFFFF, 0, False)])
+def test_spilled_history_is_exact(mask, writer, expect_race):
+    """32 readers per word exceed the slot's five (lane, class) entries: the spill block keeps the
+    history exact (the writer after a sync of `mask`; a race iff some reader is outside it)"""
+    t = _broadcast_trace(64, mask, writer)
+    want = _want(t)
+    assert bool(want) == expect_race
+    for shuffle in (None, 1, 2):
+        ts = t if shuffle is None else _with(t, tg._shuffle_within_batches(t.events, shuffle))
+        assert _gpu(ts)[0] == want
+
+
+def test_spill_pool_overflow_is_reported():
+    t = _broadcast_trace(256, 0x0000FFFF, 0)
+    c = hr.Checker.for_trace(t, history_slots=64)  # 64 slots -> 8 spill blocks for 256 words
+    try:
+        with pytest.raises(hr.HiraceError) as e:
+            _gpu(t, checker=c)
+        assert e.value.status == -8
+    finally:
+        c.close()
