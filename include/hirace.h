@@ -544,6 +544,33 @@ typedef struct {
 hirace_status hirace_set_warp_syncs(hirace_ctx *ctx, const hirace_warp_sync *d_syncs, uint64_t n,
                                     uint64_t history_slots, void *stream);
 
+/* Partial-mask syncs in the INLINE hooks (the paper's setting): the
+ * sub-warp history of an instrumented kernel (device pointers owned by the context; the same
+ * 64-B bounded-history slots and spill pool as the replay), passed by value next to the
+ * hirace_dev_ctx.  Device side (include/hirace_device.cuh, namespace hirace::ws): a per-warp
+ * vector clock in a caller-provided __shared__ buffer (ws_smem_bytes(blockDim)),
+ * thread_init_ws, syncwarp (call right after every __syncwarp(mask) / tile.sync(), also the
+ * full-mask ones), barrier_ws (after __syncthreads / at a grid sync), on_access_ws.  The sync
+ * numbering is the order in which the warp reaches its syncs (an atomic per-warp counter), so
+ * any schedule gives the relation of R20. */
+typedef struct {
+    unsigned long long *hist;        /* slots_mask + 1 slots of 8 words                       */
+    unsigned long long slots_mask;
+    unsigned long long *spill;       /* nspill blocks of 32 lane words                        */
+    unsigned long long *spill_count;
+    unsigned long long nspill;
+    unsigned int confl[3];           /* per class (R, A, X): the classes it conflicts with    */
+    unsigned char race_of[32];       /* FSM state -> RACE state of its level                   */
+} hirace_ws_ctx;
+
+/* Allocates (first call) the context's inline sub-warp history with history_slots slots (power
+ * of two, 0 = 65,536) and writes its device handle.  The conflict and level tables follow the
+ * context's policy at the time of the call.  Cleared by hirace_shadow_reset.  Synchronous.
+ * Errors: INVAL (NULL args, compact record, warp_size > 32, granularity_log2 != 2), NOMEM, CUDA.
+ * During the kernel: a full history -> sticky HIRACE_E_HISTORY_OVERFLOW, a warp sync number
+ * beyond 511 -> sticky HIRACE_E_CLOCK_OVERFLOW. */
+hirace_status hirace_inline_warp_syncs(hirace_ctx *ctx, uint64_t history_slots, hirace_ws_ctx *out);
+
 /* ---- cluster-level replay (reading R16) ----------------------------
  * A context whose hierarchy has a thread-block-cluster level between the block and the grid:
  * blocks [k*cluster_blocks, (k+1)*cluster_blocks) form cluster k (cluster_blocks must divide

@@ -76,6 +76,8 @@ struct hirace_ctx {
     /* partial-mask warp syncs (hirace_set_warp_syncs) */
     WsDev ws{};
     uint64_t ws_n = 0, ws_slots = 0;
+    hirace_ws_ctx iws{};        /* inline hooks' sub-warp history (hirace_inline_warp_syncs) */
+    uint64_t iws_slots = 0;
     int masked_grid = 0;
     hirace_status sticky = HIRACE_OK;
 };
@@ -304,34 +306,45 @@ hirace_status collect_into(hirace_ctx *c, hirace_race *d_out, uint64_t cap, unsi
     return HIRACE_OK;
 }
 
+/* classes R 0, A 1, X 2 inside one block (C1.3): strict R-A, R-X, A-X, X-X conflict; relaxed only
+ * pairs with X; and the FSM state -> RACE-of-its-level table of the policy */
+void ws_policy_tables(int policy, hirace_ws_ctx &H)
+{
+    const bool relaxed = policy == HIRACE_POLICY_RELAXED_READ_ATOMIC;
+    H.confl[0] = relaxed ? 4u : 6u;
+    H.confl[1] = relaxed ? 4u : 5u;
+    H.confl[2] = 7u;
+    fsm_race_of(policy, H.race_of);
+}
+
 /* masked replay launch: the policy-dependent tables are refreshed from the context */
 cudaError_t launch_masked(hirace_ctx *c, const hirace_event *d_events, cudaStream_t st)
 {
     WsDev W = c->ws;
-    const bool relaxed = c->policy == HIRACE_POLICY_RELAXED_READ_ATOMIC;
-    /* classes R 0, A 1, X 2 inside one block (C1.3): strict R-A, R-X, A-X, X-X; relaxed only X */
-    W.confl[0] = relaxed ? 4u : 6u;
-    W.confl[1] = relaxed ? 4u : 5u;
-    W.confl[2] = 7u;
-    fsm_race_of(c->policy, W.race_of);
+    ws_policy_tables(c->policy, W.H);
     return launch_replay_masked(c->dev, W, d_events, c->scr, c->masked_grid, st);
 }
 
 /* empty history: every slot free, no spill block handed out, the pool's lane words stale */
+cudaError_t hist_clear(const hirace_ws_ctx &H, uint64_t slots, cudaStream_t st)
+{
+    cudaError_t e = cudaMemsetAsync(H.hist, 0xff, slots * kSlotWords * sizeof(unsigned long long), st);
+    if (e == cudaSuccess)
+        e = cudaMemsetAsync(H.spill, 0xff, H.nspill * 32 * sizeof(unsigned long long), st);
+    if (e == cudaSuccess)
+        e = cudaMemsetAsync(H.spill_count, 0, sizeof(unsigned long long), st);
+    return e;
+}
+
 cudaError_t ws_clear(hirace_ctx *c, cudaStream_t st)
 {
-    cudaError_t e = cudaMemsetAsync(c->ws.hist, 0xff, c->ws_slots * kSlotWords * sizeof(unsigned long long), st);
-    if (e == cudaSuccess)
-        e = cudaMemsetAsync(c->ws.spill, 0xff, c->ws.nspill * 32 * sizeof(unsigned long long), st);
-    if (e == cudaSuccess)
-        e = cudaMemsetAsync(c->ws.spill_count, 0, sizeof(unsigned long long), st);
-    return e;
+    return hist_clear(c->ws.H, c->ws_slots, st);
 }
 
 void ws_free(hirace_ctx *c)
 {
     void *ptrs[] = {c->ws.fam_key, c->ws.fam_lo, c->ws.nfam, c->ws.sync_w, c->ws.sync_mask, c->ws.sync_fam,
-                    c->ws.vrow, c->ws.fhash, c->ws.hist, c->ws.spill, c->ws.spill_count};
+                    c->ws.vrow, c->ws.fhash, c->ws.H.hist, c->ws.H.spill, c->ws.H.spill_count};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
@@ -378,14 +391,14 @@ hirace_status hirace_set_warp_syncs(hirace_ctx *c, const hirace_warp_sync *d_syn
         (e = cudaMalloc(&W.sync_fam, n * sizeof(uint32_t))) != cudaSuccess ||
         (e = cudaMalloc(&W.vrow, n * 32 * sizeof(unsigned short))) != cudaSuccess ||
         (e = cudaMalloc(&W.fhash, fh_slots * sizeof(uint4))) != cudaSuccess ||
-        (e = cudaMalloc(&W.hist, slots * kSlotWords * sizeof(unsigned long long))) != cudaSuccess ||
-        (e = cudaMalloc(&W.spill, (slots / 8) * 32 * sizeof(unsigned long long))) != cudaSuccess ||
-        (e = cudaMalloc(&W.spill_count, sizeof(unsigned long long))) != cudaSuccess) {
+        (e = cudaMalloc(&W.H.hist, slots * kSlotWords * sizeof(unsigned long long))) != cudaSuccess ||
+        (e = cudaMalloc(&W.H.spill, (slots / 8) * 32 * sizeof(unsigned long long))) != cudaSuccess ||
+        (e = cudaMalloc(&W.H.spill_count, sizeof(unsigned long long))) != cudaSuccess) {
         ws_free(c);
         return from_cuda(c, e);
     }
-    W.slots_mask = slots - 1;
-    W.nspill = slots / 8;
+    W.H.slots_mask = slots - 1;
+    W.H.nspill = slots / 8;
     W.fh_mask = fh_slots - 1;
     W.nsync = (uint32_t)n;
     W.wpb = (c->cfg.block_threads + c->cfg.warp_size - 1) / c->cfg.warp_size;
@@ -403,6 +416,39 @@ hirace_status hirace_set_warp_syncs(hirace_ctx *c, const hirace_warp_sync *d_syn
         return s;
     }
     c->ws_n = n;
+    return HIRACE_OK;
+}
+
+hirace_status hirace_inline_warp_syncs(hirace_ctx *c, uint64_t history_slots, hirace_ws_ctx *out)
+{
+    if (!c || !out || c->rec_bytes != 8 || c->cfg.warp_size > 32 || c->cfg.granularity_log2 != 2 ||
+        history_slots > (1ull << 32))
+        return HIRACE_E_INVAL;
+    HR_CUDA(c, cudaSetDevice(c->device));
+    if (!c->iws.hist) {
+        uint64_t slots = 64;
+        while (slots < (history_slots ? history_slots : 65536ull))
+            slots <<= 1;
+        hirace_ws_ctx &H = c->iws;
+        cudaError_t e;
+        if ((e = cudaMalloc(&H.hist, slots * kSlotWords * sizeof(unsigned long long))) != cudaSuccess ||
+            (e = cudaMalloc(&H.spill, (slots / 8) * 32 * sizeof(unsigned long long))) != cudaSuccess ||
+            (e = cudaMalloc(&H.spill_count, sizeof(unsigned long long))) != cudaSuccess) {
+            void *ptrs[] = {H.hist, H.spill, H.spill_count};
+            for (void *p : ptrs)
+                if (p)
+                    cudaFree(p);
+            H = hirace_ws_ctx{};
+            return from_cuda(c, e);
+        }
+        H.slots_mask = slots - 1;
+        H.nspill = slots / 8;
+        c->iws_slots = slots;
+        HR_CUDA(c, hist_clear(H, slots, nullptr));
+        HR_CUDA(c, cudaDeviceSynchronize());
+    }
+    ws_policy_tables(c->policy, c->iws);
+    *out = c->iws;
     return HIRACE_OK;
 }
 
@@ -639,8 +685,8 @@ hirace_status hirace_shadow_free(hirace_ctx *c)
                     c->scr.grid_bar2, c->scr.cta_cnt, c->d_collect, c->d_total, c->d_bucket_hist, c->d_bucket_counts,
                     c->d_stage[0], c->d_stage[1], c->d_wire_off, c->d_wire_counts, c->d_wire_flag,
                     c->d_peer_tab, c->d_flag_tab, c->d_gepoch, c->ws.fam_key, c->ws.fam_lo, c->ws.nfam,
-                    c->ws.sync_w, c->ws.sync_mask, c->ws.sync_fam, c->ws.vrow, c->ws.fhash, c->ws.hist,
-                    c->ws.spill, c->ws.spill_count};
+                    c->ws.sync_w, c->ws.sync_mask, c->ws.sync_fam, c->ws.vrow, c->ws.fhash, c->ws.H.hist,
+                    c->ws.H.spill, c->ws.H.spill_count, c->iws.hist, c->iws.spill, c->iws.spill_count};
     for (void *p : ptrs)
         if (p)
             cudaFree(p);
@@ -716,8 +762,10 @@ hirace_status hirace_shadow_reset(hirace_ctx *c, void *stream)
                                 c->sm_count, st));
         c->lazy = false;
     }
-    if (c->ws.hist) /* the sub-warp history belongs to the check */
+    if (c->ws.H.hist) /* the sub-warp histories belong to the check */
         HR_CUDA(c, ws_clear(c, st));
+    if (c->iws.hist)
+        HR_CUDA(c, hist_clear(c->iws, c->iws_slots, st));
     c->g = 0;
     c->dev.g = 0;
     c->sticky = HIRACE_OK;

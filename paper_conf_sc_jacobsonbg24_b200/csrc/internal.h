@@ -6,6 +6,7 @@
 #include <stdint.h>
 
 #include "hirace.h"
+#include "hirace_device.cuh"
 
 namespace hirace_impl {
 
@@ -143,7 +144,7 @@ cudaError_t window_init();
  * / vrow per listed sync (vrow: the warp vector clock after it, 32 u16); hist: open-addressing
  * table of kSlotWords-word slots [key, owner, spill, 5 entries] plus a pool of 32-lane spill
  * blocks (subwarp.cu). */
-constexpr uint32_t kSlotWords = 8;
+constexpr uint32_t kSlotWords = 8; /* = hirace::ws::kSlotWords (checked in subwarp.cu) */
 struct WsDev {
     unsigned long long *fam_key;
     uint32_t *fam_lo;        /* [nfam + 1] first listed sync of each family */
@@ -153,14 +154,8 @@ struct WsDev {
     uint4 *fhash;            /* (family, w) lookup: {key lo, key hi, row, smax}; 2x(n + families) */
     unsigned long long fh_mask;
     uint32_t nsync;
-    unsigned long long *hist;
-    unsigned long long slots_mask;
-    unsigned long long *spill;        /* nspill blocks of 32 lane words                  */
-    unsigned long long *spill_count;  /* blocks handed out in this check                 */
-    unsigned long long nspill;
+    hirace_ws_ctx H;          /* the sub-warp history (hirace_device.cuh hirace::ws)     */
     uint32_t wpb;            /* warps per block */
-    uint32_t confl[3];       /* per access class (R, A, X): classes it conflicts with in a block */
-    unsigned char race_of[32]; /* FSM state -> the RACE state of its level (policy's table) */
 };
 cudaError_t launch_ws_prepare(const hirace_warp_sync *d_syncs, uint32_t n, uint32_t total_warps, uint32_t warp_size,
                               const WsDev &W, unsigned int *err, int sm_count, cudaStream_t st);

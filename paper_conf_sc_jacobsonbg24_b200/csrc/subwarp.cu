@@ -47,8 +47,9 @@ namespace {
 constexpr int kFamThreads = 1024;
 constexpr int kClockWarps = 8;
 constexpr int kMaskedThreads = 256;
-constexpr uint32_t kProbes = 4096; /* linear probing; a full table ends the search */
-constexpr unsigned long long kEmpty = ~0ull;
+static_assert(kSlotWords == ws::kSlotWords, "history slot layout");
+using ws::kEmpty;
+using ws::mix64;
 
 __device__ __forceinline__ unsigned long long fam_key(uint32_t g, uint32_t b, uint32_t warp)
 {
@@ -158,14 +159,6 @@ __device__ __forceinline__ unsigned long long sync_hkey(uint32_t g, uint32_t b, 
     return ((unsigned long long)g << 51) | ((unsigned long long)b << 41) | ((unsigned long long)w << 32) | warp;
 }
 
-__device__ __forceinline__ unsigned long long mix64(unsigned long long x)
-{
-    x ^= x >> 33;
-    x *= 0xff51afd7ed558ccdull;
-    x ^= x >> 33;
-    x *= 0xc4ceb9fe1a85ec53ull;
-    return x ^ (x >> 33);
-}
 
 __device__ void fh_insert(const WsDev &W, unsigned long long hk, uint32_t row, uint32_t smax)
 {
@@ -202,154 +195,6 @@ __device__ __forceinline__ uint4 fh_find(const WsDev &W, unsigned long long hk)
         if (k == hk || k == kEmpty)
             return k == hk ? e : make_uint4(0xffffffffu, 0xffffffffu, 0xffffffffu, 0);
     }
-}
-
-/* History slot of `key` owned by `owner` (valid:1 | g:8 | b:10 | warp:40 <<...), or null when
- * another warp owns the word in this block epoch or the table is full (*full = 1).  The whole
- * 64-B slot is read with the probe (one round trip); v[1..3] return its spill word and entries. */
-__device__ unsigned long long *hist_slot(const WsDev &W, unsigned long long key, unsigned long long owner,
-                                         uint32_t &full, ulonglong2 v[4])
-{
-    unsigned long long h = mix64(key) & W.slots_mask;
-    for (uint32_t p = 0; p < kProbes; p++, h = (h + 1) & W.slots_mask) {
-        unsigned long long *s = W.hist + h * kSlotWords;
-        const ulonglong2 *sv = reinterpret_cast<const ulonglong2 *>(s);
-#pragma unroll
-        for (int j = 0; j < 4; j++)
-            v[j] = __ldcg(sv + j);
-        unsigned long long k = v[0].x;
-        if (k == kEmpty) {
-            k = atomicCAS(s, kEmpty, key);
-            if (k == kEmpty)
-                k = key;
-        }
-        if (k != key)
-            continue;
-        unsigned long long ow = v[0].y;
-        for (;;) {
-            if (ow == owner)
-                return s;
-            if ((ow >> 40) == (owner >> 40))
-                return nullptr; /* same (g, b), another warp: its races are BLOCK races anyway */
-            const unsigned long long prev = atomicCAS(s + 1, ow, owner);
-            if (prev == ow)
-                return s;
-            ow = prev;
-        }
-    }
-    full = 1;
-    return nullptr;
-}
-
-/* Slot = 64 B (one L2 line pair, 64-B aligned): [key, owner, spill, 5 entries].  Entry =
- * stamp (1 | g:8 | b:10) << 32 | lane << 16 | class << 12 | w (class 0 R, 1 A, 2 X): the last sync
- * number at which `lane` touched the word with that class in the owner's block epoch; an entry
- * with another stamp is free.  The paper's bounded history: five (lane, class)
- * pairs fit the slot (a tiled reduction word is touched by two or three); more spill to a
- * 32-lane block from a pool (spill = its index, ~0 = none; lane word = stamp << 30 | per class c
- * at bits 10c: present:1 | w:9), so the history stays exact.  An entry's pair never moves within
- * a block epoch (entries are freed only by a new stamp), so a pair is in the slot or in the spill
- * block, and a check reads both. */
-__device__ __forceinline__ uint64_t ent_make(uint32_t stamp, uint32_t lane, uint32_t cls, uint32_t w)
-{
-    return ((uint64_t)stamp << 32) | (lane << 16) | (cls << 12) | w;
-}
-
-__device__ __forceinline__ bool spill_check(const unsigned long long *blk, uint32_t lane, uint32_t stamp, uint32_t confl,
-                                            uint32_t w2, const unsigned short *V)
-{
-    bool race = false;
-    for (uint32_t q = 0; q < 32; q += 2) {
-        const ulonglong2 a = __ldcg(reinterpret_cast<const ulonglong2 *>(blk + q));
-#pragma unroll
-        for (int j = 0; j < 2; j++) {
-            const uint32_t i = q + j;
-            const unsigned long long x = j ? a.y : a.x;
-            if (i == lane || (uint32_t)(x >> 30) != stamp)
-                continue;
-            const uint32_t vi = __ldg(V + i);
-            for (uint32_t cm = confl; cm; cm &= cm - 1) {
-                const uint32_t c = __ffs(cm) - 1;
-                const uint32_t f = (uint32_t)(x >> (10 * c)) & 1023u;
-                race |= (f & 512u) && (f & 511u) < w2 && vi <= (f & 511u);
-            }
-        }
-    }
-    return race;
-}
-
-/* a spill lane word's class entry := max(entry, w2) in the current block epoch */
-__device__ __forceinline__ void spill_update(unsigned long long *p, uint32_t stamp, uint32_t cls, uint32_t w2)
-{
-    unsigned long long v = __ldcg(p);
-    for (;;) {
-        unsigned long long nv = (uint32_t)(v >> 30) == stamp ? v : ((unsigned long long)stamp << 30);
-        const uint32_t f = (uint32_t)(nv >> (10 * cls)) & 1023u;
-        if ((f & 512u) && (f & 511u) >= w2 && nv == v)
-            return;
-        nv = (nv & ~(1023ull << (10 * cls))) | ((unsigned long long)(512u | w2) << (10 * cls));
-        const unsigned long long prev = atomicCAS(p, v, nv);
-        if (prev == v)
-            return;
-        v = prev;
-    }
-}
-
-/* The history step of one access (lane, class cls, after sync w2): with chk, is a conflicting
- * access of another lane in this block epoch not ordered before it (V = the clock after w2)?
- * With upd, record (lane, cls, w2). */
-__device__ __forceinline__ bool side_step(const WsDev &W, unsigned long long *slot, const ulonglong2 v[4],
-                                          uint32_t lane, uint32_t stamp, uint32_t cls, uint32_t confl, uint32_t w2,
-                                          const unsigned short *V, bool chk, bool upd, uint32_t &full)
-{
-    unsigned long long sp = v[1].x;
-    unsigned long long e[5] = {v[1].y, v[2].x, v[2].y, v[3].x, v[3].y};
-    bool race = false;
-    if (chk) {
-#pragma unroll
-        for (int k = 0; k < 5; k++) {
-            const uint32_t el = (uint32_t)(e[k] >> 16) & 31u, ec = (uint32_t)(e[k] >> 12) & 3u, ew = (uint32_t)e[k] & 511u;
-            if ((uint32_t)(e[k] >> 32) == stamp && el != lane && ((confl >> ec) & 1u) && ew < w2 && __ldg(V + el) <= ew)
-                race = true;
-        }
-        if (sp != kEmpty)
-            race |= spill_check(W.spill + sp * 32, lane, stamp, confl, w2, V);
-    }
-    if (!upd)
-        return race;
-    for (;;) {
-        int own = -1, fr = -1;
-#pragma unroll
-        for (int k = 0; k < 5; k++) {
-            if ((uint32_t)(e[k] >> 32) == stamp) {
-                if (((uint32_t)(e[k] >> 16) & 31u) == lane && ((uint32_t)(e[k] >> 12) & 3u) == cls)
-                    own = k;
-            } else if (fr < 0) {
-                fr = k;
-            }
-        }
-        const int k = own >= 0 ? own : fr;
-        if (k < 0)
-            break; /* slot full: spill */
-        if (own >= 0 && ((uint32_t)e[k] & 511u) >= w2)
-            return race;
-        const unsigned long long nv = ent_make(stamp, lane, cls, w2);
-        const unsigned long long prev = atomicCAS(slot + 3 + k, e[k], nv);
-        if (prev == e[k])
-            return race;
-        e[k] = prev;
-    }
-    if (sp == kEmpty) {
-        const unsigned long long idx = atomicAdd(W.spill_count, 1ull);
-        if (idx >= W.nspill) {
-            full = 1;
-            return race;
-        }
-        const unsigned long long prev = atomicCAS(slot + 2, kEmpty, idx);
-        sp = prev == kEmpty ? idx : prev;
-    }
-    spill_update(W.spill + sp * 32 + lane, stamp, cls, w2);
-    return race;
 }
 
 #ifndef HIRACE_MASKED_MINB
@@ -449,17 +294,17 @@ __global__ void __launch_bounds__(kMaskedThreads, HIRACE_MASKED_MINB)
                 bool side = false;
                 if (chk || upd) {
                     ulonglong2 sv[4];
-                    unsigned long long *slot = hist_slot(W, key, owner, full, sv);
+                    unsigned long long *slot = ws::hist_slot(W.H, key, owner, full, sv);
                     if (slot)
-                        side = side_step(W, slot, sv, ln, stamp, cls, W.confl[cls], B.w, W.vrow + (size_t)row * 32,
-                                         chk, upd, full);
+                        side = ws::side_step(W.H, slot, sv, ln, stamp, cls, W.H.confl[cls], B.w,
+                                             W.vrow + (size_t)row * 32, chk, upd, B.w, full);
                 }
                 cnt.checked++;
                 bool first = true;
                 for (;;) {
                     uint32_t ent = raw[((uint32_t)(o & 31u) << 7) | rec.label(o, tid, kind, B.ep, G)];
                     if (side) {
-                        const uint32_t ns = W.race_of[ent & E_STATE];
+                        const uint32_t ns = W.H.race_of[ent & E_STATE];
                         if (ns != (ent & E_STATE))
                             ent = ns | E_REPORT; /* store the detecting accessor */
                     }

@@ -35,9 +35,10 @@ def load():
         lib.hx_multiphase.argtypes = [P, P, I, I, I, I, I, P, U, I, P]
         lib.hx_bfs.argtypes = [P, P, P, P, I, I, U, ctypes.POINTER(I), P]
         lib.hx_cluster_halo.argtypes = [P, P, I, I, I, I, P]
+        lib.hx_tiled.argtypes = [P, P, P, I, I, I, I, I, P]
         lib.hx_cluster_hist.argtypes = [P, P, I, I, I, I, I, I, P]
         for f in (lib.hx_stencil, lib.hx_reduce, lib.hx_multiphase, lib.hx_bfs, lib.hx_cluster_halo,
-                  lib.hx_cluster_hist):
+                  lib.hx_cluster_hist, lib.hx_tiled):
             f.restype = I
         _libs[_aggregate] = lib
     return _libs[_aggregate]
@@ -111,3 +112,19 @@ def cluster_hist(checker, out, nclusters: int, cluster_blocks: int, block_thread
     d, p = _ctx(checker, out.data_ptr())
     _ok(load().hx_cluster_hist(p, ctypes.c_void_p(out.data_ptr()), nclusters, cluster_blocks, block_threads, bins,
                                int(block_scope), int(drop or 0), _stream_handle(stream)), "hx_cluster_hist")
+
+
+def tiled(checker, out, grid: int, block_threads: int, tile: int, rounds: int, racy: str | None,
+          history_slots: int = 0, stream=None):
+    """tiled_partition<tile> reduction (tracegen.tiled_reduce's program) under the inline hooks with
+    partial-mask syncs; checker None = uninstrumented.  out: CUDA float32 tensor of
+    grid*block_threads/tile (the tracked global base).  racy: None, "half_mask" or "pair"."""
+    mode = {None: 0, "half_mask": 1, "pair": 2}[racy]
+    if checker is None:
+        p = w = None
+    else:
+        d = checker.dev_ctx(out.data_ptr())
+        ws = checker.inline_ws(history_slots)
+        p, w = ctypes.byref(d), ctypes.byref(ws)
+    _ok(load().hx_tiled(p, w, ctypes.c_void_p(out.data_ptr()), grid, block_threads, tile, rounds, mode,
+                        _stream_handle(stream)), "hx_tiled")

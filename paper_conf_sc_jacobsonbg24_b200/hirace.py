@@ -43,7 +43,7 @@ EXPORTS = ("hirace_shadow_alloc", "hirace_shadow_alloc_compact", "hirace_shadow_
            "hirace_cluster_collect", "hirace_cluster_get_stats", "hirace_status_string",
            "hirace_version", "hirace_launch_count", "hirace_set_replay_mode", "hirace_get_replay_mode",
            "hirace_advance_grid_epochs", "hirace_peer_release", "hirace_peer_wait", "hirace_set_reset_mode",
-           "hirace_set_warp_syncs", "hirace_cluster_get_dev_ctx")
+           "hirace_set_warp_syncs", "hirace_cluster_get_dev_ctx", "hirace_inline_warp_syncs")
 
 
 class HiraceError(RuntimeError):
@@ -82,6 +82,13 @@ class ClusterDevCtx(ctypes.Structure):
                 ("stats", ctypes.c_void_p), ("global_base", ctypes.c_void_p), ("global_words", ctypes.c_uint64),
                 ("smem_words", ctypes.c_uint32), ("grid_blocks", ctypes.c_uint32), ("block_threads", ctypes.c_uint32),
                 ("warp_size", ctypes.c_uint32), ("cluster_blocks", ctypes.c_uint32), ("g", ctypes.c_uint32)]
+
+
+class WsCtx(ctypes.Structure):
+    """hirace_ws_ctx (include/hirace.h): the inline hooks' sub-warp history."""
+    _fields_ = [("hist", ctypes.c_void_p), ("slots_mask", ctypes.c_uint64), ("spill", ctypes.c_void_p),
+                ("spill_count", ctypes.c_void_p), ("nspill", ctypes.c_uint64), ("confl", ctypes.c_uint32 * 3),
+                ("race_of", ctypes.c_uint8 * 32)]
 
 
 class EpochLimits(ctypes.Structure):
@@ -158,6 +165,7 @@ def load():
         "hirace_get_replay_mode": (I32, [P, ctypes.POINTER(I32)]),
         "hirace_set_warp_syncs": (I32, [P, P, U64, U64, P]),
         "hirace_cluster_get_dev_ctx": (I32, [P, P, ctypes.POINTER(ClusterDevCtx)]),
+        "hirace_inline_warp_syncs": (I32, [P, U64, ctypes.POINTER(WsCtx)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -498,6 +506,13 @@ class Checker:
         _check(self.lib.hirace_get_dev_ctx(self.h, ctypes.c_void_p(global_base), ctypes.byref(d)),
                "hirace_get_dev_ctx")
         return d
+
+    def inline_ws(self, history_slots: int = 0) -> WsCtx:
+        """hirace_inline_warp_syncs: the sub-warp history handle for inline hooks with
+        partial-mask syncs (hirace::ws::*)."""
+        w = WsCtx()
+        _check(self.lib.hirace_inline_warp_syncs(self.h, history_slots, ctypes.byref(w)), "hirace_inline_warp_syncs")
+        return w
 
     def bucket(self, events_dev, n: int, nranks: int, my_rank: int, out_dev, stream=None) -> list[int]:
         counts = (ctypes.c_uint64 * nranks)()

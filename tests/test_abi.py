@@ -96,3 +96,22 @@ def test_cluster_dev_ctx_mirror_matches_the_c_header(tmp_path):
     out = [int(x) for x in subprocess.check_output([str(exe)], text=True).split()]
     assert out[:2] == [ctypes.sizeof(hb.ClusterDevCtx), hb.WARP_SYNC_DTYPE.itemsize]
     assert out[2:] == [getattr(hb.ClusterDevCtx, f).offset for f in fields]
+
+
+def test_ws_ctx_mirror_matches_the_c_header(tmp_path):
+    import ctypes
+    import subprocess
+
+    from paper_conf_sc_jacobsonbg24_b200 import hirace as hb
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    fields = [f for f, _ in hb.WsCtx._fields_]
+    src = tmp_path / "wsz.c"
+    src.write_text("#include <stdio.h>\n#include <stddef.h>\n#include \"hirace.h\"\nint main(){\n"
+                   "printf(\"%zu\\n\", sizeof(hirace_ws_ctx));\n"
+                   + "".join(f"printf(\"%zu\\n\", offsetof(hirace_ws_ctx, {f}));\n" for f in fields)
+                   + "return 0;}\n")
+    exe = tmp_path / "wsz"
+    subprocess.check_call(["gcc", "-I", os.path.join(root, "include"), str(src), "-o", str(exe)])
+    out = [int(x) for x in subprocess.check_output([str(exe)], text=True).split()]
+    assert out[0] == ctypes.sizeof(hb.WsCtx)
+    assert out[1:] == [getattr(hb.WsCtx, f).offset for f in fields]
