@@ -417,6 +417,16 @@ def _slowdown_programs(dev: int, reps: int, timed) -> dict:
                 lambda: (reset_dist(), c.reset()))
     out["cfg3_bfs_rmat18_clean"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat}
     c.close()
+    # partial-mask syncs (config 6's program, inline sub-warp hooks): tiled_partition<8> reduction
+    nb, bs, tile = 4096, 256, 8
+    c = hr.Checker(nb, bs, 32, nb * bs // tile, bs, device=dev)
+    o = torch.zeros(nb * bs // tile, device=f"cuda:{dev}")
+    c.inline_ws(2 * nb * bs)
+    nat = timed(lambda: ex.tiled(None, o, nb, bs, tile, 4, "half_mask"))
+    ins = timed(lambda: ex.tiled(c, o, nb, bs, tile, 4, "half_mask"), c.reset)
+    out["cfg6_tiled_masked_racy"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat,
+                                     "hooks": "hirace::ws (partial-mask syncs)"}
+    c.close()
     return out
 
 
