@@ -534,8 +534,10 @@ typedef struct {
  * compares each access of a family at a listed sync with its lanes' history against the vector
  * clock: a conflicting access not ordered before it is a race of the FSM state's level (WARP
  * while one warp touched the word in the block epoch, else BLOCK / GRID; R20).
- * Replay-only and batch-major: while a log is set, window-major mode replays batch-major, and
- * the wire / sharded entry points and inline hooks return HIRACE_E_INVAL.  The history is
+ * The log drives the replay (batch-major: while a log is set, window-major mode replays
+ * batch-major, and the wire / sharded entry points and hirace_get_dev_ctx return
+ * HIRACE_E_INVAL); instrumented kernels take partial syncs live through
+ * hirace_inline_warp_syncs instead.  The history is
  * cleared by hirace_shadow_reset.  Synchronises `stream`.
  * Errors: INVAL (NULL ctx / n && !d_syncs, warp_size > 32, granularity_log2 != 2), BAD_TRACE
  * (unsorted or duplicate records, w == 0, mask 0 or beyond warp_size, warp id beyond the grid;
