@@ -424,8 +424,10 @@ def _slowdown_programs(dev: int, reps: int, timed) -> dict:
     c.inline_ws(2 * nb * bs)
     nat = timed(lambda: ex.tiled(None, o, nb, bs, tile, 4, "half_mask"))
     ins = timed(lambda: ex.tiled(c, o, nb, bs, tile, 4, "half_mask"), c.reset)
+    ins_g = timed(lambda: ex.tiled(c, o, nb, bs, tile, 4, "half_mask", smem_tracking=False), c.reset)
     out["cfg6_tiled_masked_racy"] = {"native_ms": nat, "instrumented_ms": ins, "slowdown": ins / nat,
-                                     "hooks": "hirace::ws (partial-mask syncs)"}
+                                     "slowdown_global_history": ins_g / nat,
+                                     "hooks": "hirace::ws (partial-mask syncs), shared-word history in smem"}
     c.close()
     return out
 

@@ -35,7 +35,7 @@ def load():
         lib.hx_multiphase.argtypes = [P, P, I, I, I, I, I, P, U, I, P]
         lib.hx_bfs.argtypes = [P, P, P, P, I, I, U, ctypes.POINTER(I), P]
         lib.hx_cluster_halo.argtypes = [P, P, I, I, I, I, P]
-        lib.hx_tiled.argtypes = [P, P, P, I, I, I, I, I, P]
+        lib.hx_tiled.argtypes = [P, P, P, I, I, I, I, I, I, P]
         lib.hx_cluster_hist.argtypes = [P, P, I, I, I, I, I, I, P]
         for f in (lib.hx_stencil, lib.hx_reduce, lib.hx_multiphase, lib.hx_bfs, lib.hx_cluster_halo,
                   lib.hx_cluster_hist, lib.hx_tiled):
@@ -115,10 +115,12 @@ def cluster_hist(checker, out, nclusters: int, cluster_blocks: int, block_thread
 
 
 def tiled(checker, out, grid: int, block_threads: int, tile: int, rounds: int, racy: str | None,
-          history_slots: int = 0, stream=None):
+          history_slots: int = 0, smem_tracking: bool = True, stream=None):
     """tiled_partition<tile> reduction (tracegen.tiled_reduce's program) under the inline hooks with
     partial-mask syncs; checker None = uninstrumented.  out: CUDA float32 tensor of
-    grid*block_threads/tile (the tracked global base).  racy: None, "half_mask" or "pair"."""
+    grid*block_threads/tile (the tracked global base).  racy: None, "half_mask" or "pair".
+    smem_tracking: the shared words' history slots and FSM records in shared memory (else in the
+    context's global table and shadow)."""
     mode = {None: 0, "half_mask": 1, "pair": 2}[racy]
     if checker is None:
         p = w = None
@@ -127,4 +129,4 @@ def tiled(checker, out, grid: int, block_threads: int, tile: int, rounds: int, r
         ws = checker.inline_ws(history_slots)
         p, w = ctypes.byref(d), ctypes.byref(ws)
     _ok(load().hx_tiled(p, w, ctypes.c_void_p(out.data_ptr()), grid, block_threads, tile, rounds, mode,
-                        _stream_handle(stream)), "hx_tiled")
+                        int(smem_tracking), _stream_handle(stream)), "hx_tiled")

@@ -19,25 +19,26 @@ import paper_conf_sc_jacobsonbg24_b200 as hr  # noqa: E402
 from paper_conf_sc_jacobsonbg24_b200 import examples as ex  # noqa: E402
 
 
-def _run(t, tile, rounds, racy, history_slots=0):
+def _run(t, tile, rounds, racy, history_slots=0, smem_tracking=True):
     c = hr.Checker(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words)
     try:
         out = torch.zeros(t.global_words, dtype=torch.float32, device="cuda")
         ex.tiled(c, out, t.grid_blocks, t.block_threads, tile, rounds, racy,
-                 history_slots or t.info.get("history_slots", 0))
+                 history_slots or t.info.get("history_slots", 0), smem_tracking)
         torch.cuda.synchronize()
         return hr.races_to_dict(c.collect())
     finally:
         c.close()
 
 
+@pytest.mark.parametrize("smem_tracking", [True, False])
 @pytest.mark.parametrize("racy", [None, "half_mask", "pair"])
 @pytest.mark.parametrize("nb,bs,tile,rounds", [(2, 64, 4, 2), (8, 128, 8, 3), (16, 256, 16, 2), (4, 64, 32, 2),
                                                (64, 256, 8, 2)])
-def test_inline_tiled_reduction(racy, nb, bs, tile, rounds):
+def test_inline_tiled_reduction(racy, nb, bs, tile, rounds, smem_tracking):
     t = tg.tiled_reduce(nb, bs, tile, rounds, racy)
     want = oracle.races_masked_dict(t)
-    assert _run(t, tile, rounds, racy) == want
+    assert _run(t, tile, rounds, racy, smem_tracking=smem_tracking) == want
     assert (len(want) == 0) == (racy is None)
 
 
@@ -53,7 +54,7 @@ def test_inline_history_overflow_is_reported():
     c = hr.Checker(t.grid_blocks, t.block_threads, t.warp_size, t.global_words, t.smem_words)
     try:
         out = torch.zeros(t.global_words, dtype=torch.float32, device="cuda")
-        ex.tiled(c, out, t.grid_blocks, t.block_threads, 8, 1, None, history_slots=64)
+        ex.tiled(c, out, t.grid_blocks, t.block_threads, 8, 1, None, history_slots=64, smem_tracking=False)
         torch.cuda.synchronize()
         with pytest.raises(hr.HiraceError) as e:
             c.collect()
