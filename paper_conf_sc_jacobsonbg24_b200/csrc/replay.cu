@@ -41,6 +41,7 @@ using namespace hirace;
 #ifdef HIRACE_BARRIER_TRACE
 /* diagnostics build only: per (batch, CTA) globaltimer at arrival and after release */
 __device__ unsigned long long g_bar_trace[128 * 2048 * 2];
+__device__ unsigned int g_bar_smid[2048];
 __device__ __forceinline__ unsigned long long gtimer()
 {
     unsigned long long t;
@@ -222,8 +223,12 @@ __global__ void __launch_bounds__(kReplayThreads, kMinBlocks)
             e1 = i + 32 < iend ? ld_event(ev + i + 32) : make_uint4(0, 0, 0, 0);
 #ifdef HIRACE_BARRIER_TRACE
             __syncthreads();
-            if (threadIdx.x == 0 && bi < 128 && blockIdx.x < 2048)
+            if (threadIdx.x == 0 && bi < 128 && blockIdx.x < 2048) {
                 g_bar_trace[(bi * 2048 + blockIdx.x) * 2] = gtimer();
+                unsigned int sm;
+                asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+                g_bar_smid[blockIdx.x] = sm;
+            }
 #endif
             grid_sync(bar, gridDim.x, bar_epoch);
 #ifdef HIRACE_BARRIER_TRACE
@@ -353,6 +358,10 @@ const void *replay_kernel(const hirace_dev_ctx &c, bool w32)
 extern "C" int hirace_debug_barrier_trace(unsigned long long *host, uint64_t n)
 {
     return (int)cudaMemcpyFromSymbol(host, g_bar_trace, n * sizeof(unsigned long long));
+}
+extern "C" int hirace_debug_barrier_smid(unsigned int *host, uint64_t n)
+{
+    return (int)cudaMemcpyFromSymbol(host, g_bar_smid, n * sizeof(unsigned int));
 }
 #endif
 

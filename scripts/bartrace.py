@@ -50,3 +50,18 @@ if len(ranks) > 2:
           f"(min {off.min():.3f}, max {off.max():.3f})")
     mean_rank = ranks.mean(axis=0)
     print("latest 10 CTAs on average:", np.argsort(-mean_rank)[:10].tolist())
+
+# per-SM view: an SM's arrival = its last CTA's; is the spread between SMs or inside an SM?
+lib.hirace_debug_barrier_smid.argtypes = [ctypes.c_void_p, ctypes.c_uint64]
+smid = np.zeros(2048, np.uint32)
+lib.hirace_debug_barrier_smid(smid.ctypes.data, smid.size)
+smid = smid[:grid]
+for b in range(min(nb - 1, 12)):
+    arr = buf[b, :grid, 0]
+    per_sm = {}
+    for i in range(grid):
+        per_sm.setdefault(int(smid[i]), []).append(int(arr[i]))
+    last = np.array([max(v) for v in per_sm.values()], dtype=np.int64)
+    first = np.array([min(v) for v in per_sm.values()], dtype=np.int64)
+    print(f"batch {b}: {len(per_sm)} SMs; SM finish spread {(last.max() - last.min()) / 1e3:6.2f} us "
+          f"(p50 {(np.median(last) - last.min()) / 1e3:5.2f}); intra-SM CTA gap p50 {np.median(last - first) / 1e3:5.2f} us")
