@@ -122,3 +122,35 @@ def test_malformed_logs_are_rejected(bad):
         sy["mask"][0] = 1 << t.warp_size
     with pytest.raises(oracle.BadSyncLog):
         oracle.races_masked(t.events, t.block_threads, t.warp_size, sy)
+
+
+def _lane_in_listed_mask(t):
+    """every access after a listed (partial) sync comes from a lane of that sync's mask"""
+    m = t.events["meta"]
+    w, b, g = (m >> 5) & 511, (m >> 14) & 1023, m >> 24
+    tid = t.events["tid"].astype(np.int64)
+    wpb = -(-t.block_threads // t.warp_size)
+    warp = (tid // t.block_threads) * wpb + (tid % t.block_threads) // t.warp_size
+    lane = (tid % t.block_threads) % t.warp_size
+    sy = t.warp_syncs
+    listed = {(int(s["meta"]) >> 24, (int(s["meta"]) >> 14) & 1023, int(s["warp"]), (int(s["meta"]) >> 5) & 511):
+              int(s["mask"]) for s in sy}
+    for i in range(t.n):
+        k = (int(g[i]), int(b[i]), int(warp[i]), int(w[i]))
+        if k in listed:
+            assert (listed[k] >> int(lane[i])) & 1, (t.name, i)
+
+
+def test_generators_emit_well_formed_logs():
+    """tracegen side of R20: logs sorted by (g, b, warp, w), strictly increasing, non-empty masks
+    inside the warp, and accesses only after syncs their lane took part in"""
+    traces = [tg.random_tiny_masked(s) for s in range(200)]
+    traces += [tg.tiled_reduce(4, 64, tl, 2, r) for tl in (4, 8, 32) for r in (None, "half_mask", "pair")]
+    for t in traces:
+        sy = t.warp_syncs
+        key = [(int(s["meta"]) >> 24, (int(s["meta"]) >> 14) & 1023, int(s["warp"]), (int(s["meta"]) >> 5) & 511)
+               for s in sy]
+        assert key == sorted(key) and len(set(key)) == len(key), t.name
+        assert all(k[3] >= 1 for k in key)
+        assert all(0 < int(s["mask"]) < (1 << t.warp_size) for s in sy)
+        _lane_in_listed_mask(t)
