@@ -263,3 +263,11 @@ def test_spill_pool_overflow_is_reported():
         assert e.value.status == -8
     finally:
         c.close()
+
+
+def test_random_masked_programs_with_wide_accesses():
+    """8/16-byte accesses: the masked replay checks every covered word (k_replay_masked's word loop)"""
+    for seed in range(300):
+        t = tg.random_tiny_masked(seed, wide=True)
+        assert _gpu(t)[0] == _want(t), t.name
+        assert _gpu(t, compact=True)[0] == _want(t), t.name

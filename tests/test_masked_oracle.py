@@ -154,3 +154,12 @@ def test_generators_emit_well_formed_logs():
         assert all(k[3] >= 1 for k in key)
         assert all(0 < int(s["mask"]) < (1 << t.warp_size) for s in sy)
         _lane_in_listed_mask(t)
+
+
+def test_wide_accesses_oracle_equals_brute_force():
+    """8- and 16-byte accesses cover 2 / 4 words (C1.1), each checked with the partial syncs"""
+    for seed in range(600):
+        t = tg.random_tiny_masked(seed, wide=True)
+        k, c, g = oracle.races_masked(t.events, t.block_threads, t.warp_size, t.warp_syncs)
+        got = {int(a): (int(b), int(x)) for a, b, x in zip(k, c, g)}
+        assert got == brute.races_masked(t.events, t.warp_syncs, t.block_threads, t.warp_size), t.name
