@@ -271,3 +271,19 @@ def test_random_masked_programs_with_wide_accesses():
         t = tg.random_tiny_masked(seed, wide=True)
         assert _gpu(t)[0] == _want(t), t.name
         assert _gpu(t, compact=True)[0] == _want(t), t.name
+
+
+def test_masked_replay_with_selective_tracking():
+    """hirace_set_filter (f4) on the masked path: with shared memory deselected the verdict equals
+    the oracle's on the global accesses alone (the partial syncs still order them)"""
+    import numpy as np
+    for seed in range(200):
+        t = tg.random_tiny_masked(seed)
+        c = hr.Checker.for_trace(t)
+        try:
+            c.set_filter(0, 0, 1)  # global memory only
+            got = _gpu(t, checker=c)[0]
+        finally:
+            c.close()
+        glob = (t.events["addr"] >> np.uint64(63)) == 0
+        assert got == _want(_with(t, t.events[glob])), t.name
