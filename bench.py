@@ -494,6 +494,8 @@ def run_sharded_bench(args, world, rank, local_rank):
     flagged = int(d_total.item())
     dist.barrier()
     torch.cuda.synchronize()
+    from paper_conf_sc_jacobsonbg24_b200 import hirace as _hb
+    l0 = _hb.launch_count()
     w0 = time.time()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record()
@@ -502,6 +504,7 @@ def run_sharded_bench(args, world, rank, local_rank):
     e1.record()
     torch.cuda.synchronize()
     w1 = time.time()
+    launches = _hb.launch_count() - l0
     dist.barrier()
     clocks.mark(w0, w1)
     clocks.stop()
@@ -509,9 +512,13 @@ def run_sharded_bench(args, world, rank, local_rank):
     fl = torch.tensor([flagged], dtype=torch.int64)
     if nccl:
         ms, fl = ms.cuda(), fl.cuda()
+    nl = torch.tensor([launches], dtype=torch.int64)
+    if nccl:
+        nl = nl.cuda()
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     dist.all_reduce(fl)
-    ms, flagged = float(ms.item()), int(fl.item())
+    dist.all_reduce(nl)  # the library's kernels launched in the timed region, all ranks
+    ms, flagged, launches = float(ms.item()), int(fl.item()), int(nl.item())
     # e2e: every step copies this rank's events from pinned host memory to the device, runs the
     # sharded step and reads the flagged words back (D2H); max over ranks of the wall time
     e2e = None
@@ -567,12 +574,13 @@ def run_sharded_bench(args, world, rank, local_rank):
                             "frac": BYTES_PER_ACCESS * n_total / world / (per_step / 1e3) / 1e9 / peak,
                             "traffic": None, "kernel": "whole sharded step per GPU", "peak_kind": peak_kind},
                "cpu_baseline": None,  # the oracle is timed on rank 0 at N=1 only
-               "e2e": e2e, "gpu_launches": None, "clocks": clocks.summary(),
+               "e2e": e2e, "gpu_launches": launches, "clocks": clocks.summary(),
                "check": {"flagged_words": flagged, "expected": len(t.info["expected"])}}
-        print(json.dumps(out), flush=True)
     if isinstance(ex, sharded.PeerExchange):
         ex.close()
     dist.destroy_process_group()
+    if rank == 0:  # last, after NCCL's teardown log lines
+        print(json.dumps(out), flush=True)
 
 
 def measure_single(args, config: int, variant: str, K: int, W: int, dev: int, clocks=None, keep=False):
@@ -875,9 +883,9 @@ def main():
         "shadow_overhead": {"bytes_per_tracked_word": rec_bytes, "ratio_to_tracked_bytes": rec_bytes / 4,
                             "iguard_ratio_context": 4.0},
     }
-    print(json.dumps(out), flush=True)
     if world > 1:
         dist.destroy_process_group()
+    print(json.dumps(out), flush=True)  # last, after any NCCL teardown log lines
 
 
 if __name__ == "__main__":
